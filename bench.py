@@ -1,0 +1,469 @@
+"""Benchmark of the B200 Cas-OFFinder hot path (bench contract: one JSON line on rank 0).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl ours|reference]
+
+One *step* = one pass of the whole hot path over the synthetic genome: for every chunk
+(whole chromosome) the finder, the comparer and the device hit sort (SURVEY.md §8(a)
+rows a3-a7 on the device; a1 pack and a2 H2D are outside ``value`` because the inputs
+are resident in HBM, and inside ``e2e``).  ``value`` = genome bases of the whole job /
+max-over-ranks device time; comparisons/s are reported beside it.  Multi-GPU: chunks
+are LPT-sharded over ranks (no collective on the data path), strong scaling.
+
+``e2e`` runs the same search through the public API from pinned HOST planes every step:
+cof_load_chunk (H2D) -> find -> compare -> sort -> cof_collect (D2H + decorate) ->
+cof_merge.  ``--impl reference`` times the CPU oracle (the only other program that
+computes this path) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_socc_jinv23_b200 import synth  # noqa: E402
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.thread.join(timeout=2)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nme, v in zip(names, parts[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nme)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- workload
+def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
+    """Synthetic workload + the device state the timed step runs on: resident planes of
+    every chunk, one plan_dev per chunk (its counters), shared item buffers, per-chunk
+    hit buffers sized from a first (untimed) pass."""
+    import torch
+    from paper_conf_socc_jinv23_b200 import cof, search
+
+    wl = synth.make_workload(name, scale=scale, threads=max(1, min(16, os.cpu_count() or 1)))
+    L = wl.cfg.L
+    all_chunks = search.plan_chunks([len(s) for s in wl.seqs], L, None)
+    chunks = all_chunks if chunks is None else chunks
+    st = type("State", (), {})()
+    st.device = device or torch.device("cuda", torch.cuda.current_device())
+    st.stream = torch.cuda.current_stream(st.device)
+    st.chunks = chunks
+    st.plan = cof.cof_plan_create(wl.cfg.pattern, wl.guides, wl.thresholds)
+    nbytes = cof.cof_plan_device_bytes(st.plan)
+    st.host = search.HostGenome(wl.seqs, chunks)
+    st.d_planes, st.d_chunks, st.plan_devs = [], [], []
+    for i, ch in enumerate(chunks):
+        d = st.host.planes[i].to(st.device, non_blocking=True)
+        st.d_planes.append(d)
+        st.d_chunks.append(cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, d[0], d[1], d[2]))
+        pd = torch.empty(nbytes + 256, dtype=torch.uint8, device=st.device)
+        cof.cof_plan_upload(st.plan, pd, st.stream)
+        st.plan_devs.append(pd)
+    max_owned = max(ch.n_owned for ch in chunks)
+    st.items = torch.empty((2, max_owned), dtype=torch.int32, device=st.device)
+    st.find_ws = torch.empty(cof.cof_find_workspace_bytes(max_owned), dtype=torch.uint8, device=st.device)
+    # first pass with host counts: exact item / hit counts per chunk
+    st.counts = []
+    tmp_cap = 1 << 20
+    tmp_hits = torch.empty(tmp_cap, dtype=torch.int64, device=st.device)
+    for i, ch in enumerate(chunks):
+        nf, nr = cof.cof_find_pam(st.plan, st.plan_devs[i], st.d_chunks[i], st.find_ws, st.items[0], st.items[1],
+                                  max_owned, st.stream)
+        try:
+            nh = cof.cof_compare(st.plan, st.plan_devs[i], st.d_chunks[i], st.items[0], nf, st.items[1], nr,
+                                 tmp_hits, tmp_cap, st.stream)
+        except cof.CofError as e:
+            if e.status != cof.COF_E_CAPACITY:
+                raise
+            nh = cof.cof_read_counts(st.plan, st.plan_devs[i], st.stream)[2]
+        st.counts.append((nf, nr, nh))
+    del tmp_hits
+    st.caps = [max(1024, int(c[2] * 1.1) + 1024) for c in st.counts]
+    st.hits = [torch.empty(c, dtype=torch.int64, device=st.device) for c in st.caps]
+    st.tmp = torch.empty(max(st.caps), dtype=torch.int64, device=st.device)
+    st.sort_ws = torch.empty(cof.cof_sort_workspace_bytes(max(st.caps)), dtype=torch.uint8, device=st.device)
+    st.max_owned = max_owned
+    torch.cuda.synchronize(st.device)
+    return wl, st
+
+
+def run_device_pipeline(wl, st, collect=False, events=None):
+    """One step on the device: per chunk find -> compare -> sort, counts kept on the
+    device (no host round trip between kernels).  ``events``: list to append
+    (start, end) CUDA event pairs bracketing each comparer launch.  With ``collect``
+    returns the merged, decorated hit array (cof_collect + cof_merge)."""
+    import torch
+    from paper_conf_socc_jinv23_b200 import cof, search
+
+    ON = cof.COF_COUNT_ON_DEVICE
+    s = st.stream
+    for i in range(len(st.chunks)):
+        dch, pd = st.d_chunks[i], st.plan_devs[i]
+        cof.cof_find_pam(st.plan, pd, dch, st.find_ws, st.items[0], st.items[1], st.max_owned, s, sync=False)
+        if events is not None:
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+        cof.cof_compare(st.plan, pd, dch, st.items[0], ON, st.items[1], ON, st.hits[i], st.caps[i], s, sync=False)
+        if events is not None:
+            e1.record(s)
+            events.append((e0, e1))
+        cof.cof_sort_hits(st.plan, pd, dch, st.hits[i], st.tmp, st.caps[i], ON, st.sort_ws, s)
+    if not collect:
+        return None
+    out = []
+    for i in range(len(st.chunks)):
+        nf, nr, nh = cof.cof_read_counts(st.plan, st.plan_devs[i], s)
+        if nh > st.caps[i]:
+            raise RuntimeError(f"chunk {i}: {nh} hits exceed capacity {st.caps[i]}")
+        out.append(cof.cof_collect(st.plan, st.host.chunk_struct(i), st.hits[i], nh, s))
+    return search.merge_hit_lists(out)
+
+
+def step_counts(st):
+    from paper_conf_socc_jinv23_b200 import cof
+    tot = [0, 0, 0]
+    for i in range(len(st.chunks)):
+        c = cof.cof_read_counts(st.plan, st.plan_devs[i], st.stream)
+        if c[2] > st.caps[i]:
+            raise RuntimeError(f"chunk {i}: {c[2]} hits exceed capacity {st.caps[i]}")
+        for k in range(3):
+            tot[k] += c[k]
+    return tot
+
+
+def run_e2e_step(wl, st, searcher):
+    """Public-API end-to-end step from pinned host planes; returns (hits, h2d, d2h bytes)."""
+    hits = searcher.search_host(st.host)
+    h2d = st.host.bytes
+    d2h = len(hits) * 8 + 16 * len(st.chunks)
+    return hits, h2d, d2h
+
+
+# ----------------------------------------------------------------------------- oracle arm
+def oracle_sample(wl, target_s: float, threads: int):
+    """Bounded sample for the CPU oracle: the first B window starts after the leading
+    telomere of every chromosome in turn, B calibrated to ~target_s of CPU time."""
+    from oracle import oracle as orc
+    cfg = wl.cfg
+    c = int(np.argmax([len(s) for s in wl.seqs]))
+    s0 = 1_000_000 if len(wl.seqs[c]) > 3_000_000 else 0
+    probe = 20_000
+    t = time.perf_counter()
+    orc.search([wl.seqs[c]], cfg.pattern, wl.guides, wl.thresholds, ranges=[(s0, s0 + probe)], threads=threads)
+    dt = max(time.perf_counter() - t, 1e-3)
+    n = int(min(len(wl.seqs[c]) - s0 - cfg.L, max(probe, probe * target_s / dt)))
+    return c, s0, n
+
+
+def run_oracle(wl, c, s0, n, threads):
+    from oracle import oracle as orc
+    cfg = wl.cfg
+    t = time.perf_counter()
+    h = orc.search([wl.seqs[c]], cfg.pattern, wl.guides, wl.thresholds, ranges=[(s0, s0 + n)], threads=threads)
+    return time.perf_counter() - t, len(h)
+
+
+def items_per_base_estimate(st, wl):
+    tot_items = sum(c[0] + c[1] for c in st.counts)
+    return tot_items / max(1, sum(ch.n_owned for ch in st.chunks))
+
+
+# ----------------------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C5")
+    ap.add_argument("--scale", type=float, default=1.0)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--comparer", default="table", choices=["table", "popc"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    cfgname = args.config
+    metric = "genome Gbases/s (and guide x site comparisons/s)"
+
+    if args.impl == "reference":
+        if rank != 0:
+            return 0
+        return main_reference(args, cfgname, metric)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_socc_jinv23_b200 import cof, search
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    cof.cof_set_comparer(args.comparer)
+    cfg = synth.config(cfgname, args.scale)
+    L = cfg.L
+    all_chunks = search.plan_chunks([l for _, l in cfg.genome.chroms], L, None)
+    shards = search.shard_lpt(all_chunks, world)
+    mine = shards[rank]
+    wl, st = prepare_workload(cfgname, args.scale, chunks=mine, device=dev)
+    genome_bases = wl.total_bases
+    my_items = sum(c[0] + c[1] for c in st.counts)
+    comps_mine = my_items * len(wl.guides)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for _ in range(max(args.warmup, 3)):
+        run_device_pipeline(wl, st)
+    torch.cuda.synchronize(dev)
+    barrier()
+    torch.cuda.synchronize(dev)
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    events = []
+    launches0 = cof.cof_launch_count()
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t_start.record(st.stream)
+    for _ in range(args.steps):
+        run_device_pipeline(wl, st, events=events)
+    t_end.record(st.stream)
+    torch.cuda.synchronize(dev)
+    launches = cof.cof_launch_count() - launches0
+    clk = clocks.stop()
+    barrier()
+    ms_total = t_start.elapsed_time(t_end)
+    cmp_ms = sum(a.elapsed_time(b) for a, b in events)
+    totals = step_counts(st)   # verifies capacities
+
+    # max over ranks
+    t = torch.tensor([ms_total, cmp_ms, float(comps_mine), float(totals[2]), float(my_items)],
+                     dtype=torch.float64, device=dev)
+    if world > 1:
+        tmax = t.clone()
+        dist.all_reduce(tmax[:2], op=dist.ReduceOp.MAX)
+        tsum = t.clone()
+        dist.all_reduce(tsum[2:], op=dist.ReduceOp.SUM)
+        ms_total, cmp_ms_max = float(tmax[0]), float(tmax[1])
+        comps_all, hits_all, items_all = float(tsum[2]), float(tsum[3]), float(tsum[4])
+    else:
+        cmp_ms_max = cmp_ms
+        comps_all, hits_all, items_all = float(comps_mine), float(totals[2]), float(my_items)
+    ms_step = ms_total / args.steps
+    gbases = genome_bases / (ms_step * 1e-3) / 1e9
+    comps_s = comps_all / (ms_step * 1e-3)
+
+    # roofline of the dominant kernel (comparer): comparisons/s vs the ALU/LDS roof
+    peaks, peak_src = _peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    n_sm = torch.cuda.get_device_properties(dev).multi_processor_count
+    roof = comparer_roof(st.plan, n_sm, sm_max, args.comparer)
+    cmp_rate = comps_mine * args.steps / (cmp_ms * 1e-3) if cmp_ms > 0 else 0.0
+    n_cmp_launch = len(events)
+
+    e2e = None
+    if not args.no_e2e:
+        e2e = measure_e2e(wl, st, dev, args, world, genome_bases)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        threads = len(os.sched_getaffinity(0))
+        c, s0, n = oracle_sample(wl, 12.0, threads)
+        dt, nh = run_oracle(wl, c, s0, n, threads)
+        ipb = items_per_base_estimate(st, wl)
+        cpu = {"value": n / dt / 1e9, "unit": "Gbases/s", "cores": threads, "kind": "oracle",
+               "comparisons_per_s": n * ipb * len(wl.guides) / dt,
+               "sample": f"{n} window starts of {wl.names[c]} from offset {s0}, both strands, all "
+                         f"{len(wl.guides)} guides ({dt:.1f} s, {nh} hits)"}
+
+    if rank == 0:
+        line = {
+            "metric": metric, "value": round(gbases, 4), "unit": "Gbases/s", "n_gpus": world,
+            "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": round(ms_step, 4),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32 bit-planes",
+            "data": "synthetic (seeded hg38-shaped genome, synth.py)",
+            "comparisons_per_s": comps_s, "hits_per_step": int(hits_all), "items_per_step": int(items_all),
+            "config": {"workload": cfgname, "description": cfg.description, "genome_bases": genome_bases,
+                       "chromosomes": len(wl.seqs), "guides": len(wl.guides), "threshold": cfg.threshold,
+                       "pattern": cfg.pattern, "chunking": "whole chromosome per chunk",
+                       "parallelism": f"chromosome LPT shards over {world} GPU(s)",
+                       "comparer": args.comparer,
+                       "l2": "inputs larger than L2 (1.16 GB planes + item lists), no flush"},
+            "roofline": {"bound": "alu", "kernel": f"cof_comparer_{args.comparer}",
+                         "achieved": cmp_rate, "peak": roof["peak"], "unit": "comparisons/s",
+                         "frac": cmp_rate / roof["peak"] if roof["peak"] else None, "traffic": None,
+                         "peak_basis": roof["basis"], "launches": n_cmp_launch,
+                         "share_of_step": cmp_ms_max / ms_total if ms_total else None},
+            "gpu_launches": int(launches // args.steps) if args.steps else 0,
+            "gpu_launches_timed_region": int(launches),
+            "clocks": clk,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+            "peaks_source": peak_src,
+        }
+        print(json.dumps(line))
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def comparer_roof(plan, n_sm, sm_mhz, impl):
+    """Peak comparisons/s of the comparer's binding pipe.
+    popc: 1 POPC per comparison, POPC = 16/clk/SM (measured, tools/microbench_pipes.cu).
+    table: per item and 32-guide block, the minimal carry-save tree (FA/HA count from
+    gen_csa for this plan's pair count) + 6-step borrow chain + 1 mask op, all LOP3 on
+    the 64/clk/SM ALU pipe; co-bound by shared memory: NP 64-bit lookups per item and
+    block = 2*NP wavefronts per 32 items x 32 guides at 1 wavefront/clk/SM."""
+    clk = sm_mhz * 1e6
+    if impl == "popc":
+        return {"peak": 16 * n_sm * clk, "basis": "POPC pipe 16/clk/SM x SMs x max SM clock"}
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "gen_csa", os.path.join(ROOT, "paper_conf_socc_jinv23_b200", "csrc", "gen_csa.py"))
+    g = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(g)
+    import ctypes
+    from paper_conf_socc_jinv23_b200 import cof
+    # pair count from the plan's guides (union of compared positions)
+    L = plan.L
+    care = 0
+    for gs in plan.guides:
+        for j, ch in enumerate(gs):
+            if ch.upper() != "N":
+                care |= 1 << j
+    npairs = max(1, (bin(care).count("1") + 1) // 2)
+    hdr = g.gen(npairs).splitlines()[0]
+    fa = int(hdr.split(":")[1].split("full")[0])
+    ha = int(hdr.split(",")[1].split("half")[0])
+    alu_ops = 2 * fa + 2 * ha + 6 + 1
+    alu_rate = 64.0 * 32 / alu_ops           # comparisons / clk / SM
+    lds_rate = 32.0 * 32 / (2 * npairs)      # comparisons / clk / SM
+    per_clk = min(alu_rate, lds_rate)
+    return {"peak": per_clk * n_sm * clk,
+            "basis": f"min(ALU {alu_rate:.1f}, LDS {lds_rate:.1f}) comparisons/clk/SM for {npairs} pairs "
+                     f"({alu_ops} LOP3 per 32 comparisons) x {n_sm} SMs x {sm_mhz:.0f} MHz"}
+
+
+def measure_e2e(wl, st, dev, args, world, genome_bases):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_socc_jinv23_b200 import search
+    srch = search.Searcher(wl.cfg.pattern, wl.guides, wl.thresholds, device=dev)
+    srch.reserve(max(ch.n_bases for ch in st.chunks), max(st.caps))
+    run_e2e_step(wl, st, srch)     # warm-up
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    h2d = d2h = 0
+    nh = 0
+    for _ in range(args.e2e_steps):
+        hits, a, b = run_e2e_step(wl, st, srch)
+        h2d, d2h, nh = a, b, len(hits)
+    torch.cuda.synchronize(dev)
+    dt = (time.perf_counter() - t0) / args.e2e_steps
+    if world > 1:
+        t = torch.tensor([dt], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dt = float(t[0])
+    return {"value": round(genome_bases / dt / 1e9, 4), "unit": "Gbases/s", "h2d_bytes_per_step": int(h2d),
+            "d2h_bytes_per_step": int(d2h), "s_per_step": dt, "hits": nh,
+            "path": "Searcher.search_host: cof_load_chunk -> cof_find_pam -> cof_compare -> cof_sort_hits "
+                    "-> cof_collect -> cof_merge, from pinned packed host planes (wall clock)"}
+
+
+def main_reference(args, cfgname, metric):
+    """CPU oracle arm: each step = the oracle on a bounded sample of the workload."""
+    threads = len(os.sched_getaffinity(0))
+    cfg = synth.config(cfgname, args.scale)
+    wl = synth.make_workload(cfgname, scale=args.scale, threads=max(1, min(16, os.cpu_count() or 1)))
+    c, s0, n = oracle_sample(wl, 8.0, threads)
+    for _ in range(args.warmup):
+        run_oracle(wl, c, s0, min(n, 20_000), threads)
+    times = []
+    for _ in range(args.steps):
+        dt, nh = run_oracle(wl, c, s0, n, threads)
+        times.append(dt)
+    dt = statistics.mean(times)
+    v = n / dt / 1e9
+    line = {"impl": "reference", "metric": metric, "value": v, "unit": "Gbases/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "ascii chars", "data": "synthetic",
+            "config": {"workload": cfgname, "description": cfg.description},
+            "cpu_baseline": {"value": v, "unit": "Gbases/s", "cores": threads, "kind": "oracle",
+                             "sample": f"{n} window starts of {wl.names[c]} from offset {s0}, both strands, "
+                                       f"all {len(wl.guides)} guides per step"},
+            "e2e": {"value": v, "unit": "Gbases/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

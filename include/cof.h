@@ -1,0 +1,197 @@
+/*
+ * cof.h -- C ABI of the B200-native Cas-OFFinder hot path (libcof.so).
+ *
+ * Paper: Jin & Vetter, "Experience Migrating OpenCL to SYCL: A Case Study on Searches
+ * for Potential Off-Target Sites of Cas9 RNA-Guided Endonucleases on AMD GPUs";
+ * "P:Lnn" = line nn of /root/reference/PAPER.md.  The calls follow the paper's
+ * problem statement: the host divides the genome into chunks that fit device
+ * memory, a "search" kernel selects the sites carrying a PAM, a "compare" kernel counts
+ * mismatched bases for every query, and the host collects "chromosome number, position,
+ * direction, the number of mismatched bases and potential off-target DNA sequence with
+ * mismatched bases".  Readings of points the paper leaves open are listed in DESIGN.md
+ * §2 (G1..G19) and referenced below.
+ *
+ * Conventions (all calls):
+ *  - Return COF_OK (0) or a negative cof_status; never throw, never abort.  On error
+ *    cof_last_error() returns a thread-local message.
+ *  - Every buffer is caller-owned; the library never frees caller memory.  "dev" means
+ *    a device pointer of the calling thread's current CUDA device, "host" a host pointer
+ *    (pinned for the async copies to be truly asynchronous).
+ *  - cof_stream is a cudaStream_t passed as an opaque pointer (NULL = legacy stream).
+ *    Calls are asynchronous on that stream unless they return a host-side count, in
+ *    which case they synchronize it.
+ *  - No torch types cross this boundary; the Python binding passes data_ptr()s.
+ */
+#ifndef COF_H
+#define COF_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t cof_status;
+#define COF_OK          0
+#define COF_E_ARG      (-1)   /* bad argument: non-IUPAC letter, length mismatch, L>32, NULL, ... */
+#define COF_E_CAPACITY (-2)   /* output buffer too small; the needed count is returned */
+#define COF_E_CUDA     (-3)   /* CUDA runtime error (message has the CUDA error string) */
+#define COF_E_STATE    (-4)   /* plan / chunk / workspace mismatch */
+#define COF_E_IO       (-5)   /* file could not be read / parsed */
+
+/* Pass as a count to cof_compare / cof_sort_hits to use the count the previous call
+ * left in the plan's device workspace (no host round trip between kernels). */
+#define COF_COUNT_ON_DEVICE UINT64_MAX
+
+typedef void *cof_stream;
+
+const char *cof_last_error(void);
+const char *cof_version(void);
+/* Number of CUDA kernels this library has launched in this process (monotone). */
+uint64_t cof_launch_count(void);
+
+/* ------------------------------------------------------------------ plan (M1)
+ * The input specification: a search pattern of length L (guide Ns + PAM, e.g.
+ * "NNNNNNNNNNNNNNNNNNNNNRG") and n queries ("guides") of the same length, each with its
+ * own maximum mismatch count (P:L158 via [17]; Listing 1 parameters P:L185-L188).
+ *  pattern   NUL-terminated IUPAC string (ACGTRYSWKMBDHVN, case-insensitive), 1<=L<=32.
+ *  guides    n_guides NUL-terminated IUPAC strings of length L; 'N' positions are not
+ *            compared (the -1-terminated index list; reading G7).
+ *  max_mm    n_guides thresholds; a site is a hit iff #mismatches <= max_mm.
+ *  out       receives a host-only, immutable plan (thread-safe to share read-only).
+ * Errors: COF_E_ARG for a non-IUPAC letter (G18), guide length != L (G11), L>32,
+ * n_guides == 0 or > 2^24, NULL pointers.  The plan reverse-complements pattern and
+ * guides for the '-' strand and groups guides by compared-position mask. */
+typedef struct cof_plan cof_plan;
+cof_status cof_plan_create(const char *pattern, uint32_t n_guides, const char *const *guides,
+                           const uint8_t *max_mm, cof_plan **out);
+void       cof_plan_destroy(cof_plan *plan);
+uint32_t   cof_plan_length(const cof_plan *plan);        /* L */
+uint32_t   cof_plan_n_guides(const cof_plan *plan);
+/* Bytes of the device-side plan (guide tables + counters).  One plan_dev per
+ * (device, stream) in flight: it holds the counters find/compare/sort exchange. */
+size_t     cof_plan_device_bytes(const cof_plan *plan);
+/* Async H2D of the guide tables into plan_dev (>= cof_plan_device_bytes, 256-B aligned). */
+cof_status cof_plan_upload(const cof_plan *plan, void *plan_dev, cof_stream s);
+
+/* ------------------------------------------------------------------ chunk (M3, M4)
+ * One chunk of one chromosome: window starts [start, start + n_owned) belong to it,
+ * and it holds bases [start, start + n_bases) with n_bases = min(n_owned + L - 1,
+ * chrom_len - start) (chunks overlap by L-1, reading G12).  The genome is stored as
+ * three bit-planes of uint32 words (bit p&31 of word p>>5 is base p): lo/hi = 2-bit
+ * code A=00 C=01 G=10 T=11 (lo = bit 0), nm = 1 for any non-ACGT letter (then lo=hi=0),
+ * reading G2/G4; the "2-bit sequence format" of P:L289.  Each plane has
+ * cof_plane_words(n_bases) words; words past the last base have nm = all-ones. */
+typedef struct {
+    uint32_t chrom;        /* chromosome index (FASTA / caller order) */
+    uint32_t reserved;
+    uint64_t start;        /* 0-based chromosome offset of base 0 of this chunk */
+    uint64_t n_bases;
+    uint64_t n_owned;
+    uint32_t *lo, *hi, *nm;
+} cof_chunk;
+
+uint64_t   cof_plane_words(uint64_t n_bases);
+/* Host pack (OpenMP): n ASCII bases -> planes of cof_plane_words(n) words each.
+ * Upper/lower case are equal; any non-ACGT byte becomes N (G2, G4). */
+cof_status cof_pack(const char *ascii, uint64_t n, uint32_t *lo, uint32_t *hi, uint32_t *nm);
+/* Host unpack (inverse, canonical form: "ACGTN" upper-case), for checks and output. */
+cof_status cof_unpack(const uint32_t *lo, const uint32_t *hi, const uint32_t *nm,
+                      uint64_t first, uint64_t n, char *ascii);
+/* Async H2D of the three host planes into dev->lo/hi/nm (device buffers of
+ * cof_plane_words(host->n_bases) words each); copies the metadata fields too.
+ * ("divides the genome data into chunks that can fit the memory"; Table III.) */
+cof_status cof_load_chunk(const cof_chunk *host, cof_chunk *dev, cof_stream s);
+
+/* ------------------------------------------------------------------ FASTA (M2)
+ * Minimal indexed FASTA reader ("single- or multi-sequence data format"):
+ * mmap + per-record line layout; packs any base range straight into planes. */
+typedef struct cof_fasta cof_fasta;
+cof_status cof_fasta_open(const char *path, cof_fasta **out);
+void       cof_fasta_close(cof_fasta *fa);
+uint32_t   cof_fasta_count(const cof_fasta *fa);
+const char *cof_fasta_name(const cof_fasta *fa, uint32_t i);
+uint64_t   cof_fasta_length(const cof_fasta *fa, uint32_t i);
+/* Pack bases [first, first+n) of record i into planes (cof_plane_words(n) words each). */
+cof_status cof_fasta_pack(const cof_fasta *fa, uint32_t i, uint64_t first, uint64_t n,
+                          uint32_t *lo, uint32_t *hi, uint32_t *nm);
+
+/* ------------------------------------------------------------------ finder (M5, M6)
+ * The "search" kernel (signature Table VI): for every owned window
+ * start p with p+L <= n_bases, '+' passes iff every non-N pattern letter P[j] contains
+ * base(p+j); '-' passes iff the reverse-complemented pattern does (G3, G10).  Passing
+ * starts are compacted in ascending order into one list per strand (chunk-relative
+ * uint32).  The paper compacts with an unordered atomic counter (Table V);
+ * here a single-pass ordered scan (decoupled look-back) keeps the lists sorted.
+ *  workspace  dev, >= cof_find_workspace_bytes(dev->n_owned) bytes (tile status words).
+ *  items_cap  capacity of each list; n_owned always suffices.
+ *  n_fwd/n_rev  host outputs; if both are NULL the call does not synchronize and the
+ *             counts stay in plan_dev for cof_compare(COF_COUNT_ON_DEVICE).
+ * COF_E_CAPACITY: a list overflowed; n_fwd and n_rev hold the needed counts. */
+size_t     cof_find_workspace_bytes(uint64_t n_owned);
+cof_status cof_find_pam(const cof_plan *plan, void *plan_dev, const cof_chunk *dev,
+                        void *workspace, uint32_t *items_fwd, uint32_t *items_rev,
+                        uint64_t items_cap, uint64_t *n_fwd, uint64_t *n_rev, cof_stream s);
+
+/* ------------------------------------------------------------------ comparer (M8, M9)
+ * The "compare" kernel (Listing 1): for every item and every guide,
+ * mm = #compared positions whose genome base is not in the guide letter's IUPAC set
+ * ('-' items use the reverse-complemented guide aligned to the same '+' window,
+ * P:L231-L236); emit iff mm <= max_mm.  Emission is a
+ * warp-aggregated atomic append of a 64-bit key
+ *     key = pos << 32 | strand << 31 | guide << 7 | mm      (strand 0 = '+', 1 = '-')
+ * so that integer order is (pos, '+' before '-', guide) (G13).
+ *  n_fwd/n_rev  item counts, or COF_COUNT_ON_DEVICE to use the finder's device counts.
+ *  hits     dev, capacity hits_cap keys; n_hits host output (NULL: no sync, the count
+ *           stays in plan_dev).  Order of hits is unspecified (see cof_sort_hits).
+ * COF_E_CAPACITY: *n_hits holds the needed count; re-run with a larger buffer. */
+cof_status cof_compare(const cof_plan *plan, void *plan_dev, const cof_chunk *dev,
+                       const uint32_t *items_fwd, uint64_t n_fwd,
+                       const uint32_t *items_rev, uint64_t n_rev,
+                       uint64_t *hits, uint64_t hits_cap, uint64_t *n_hits, cof_stream s);
+
+/* ------------------------------------------------------------------ sort (M10, K3)
+ * Deterministic order of the hit keys (the paper's atomics are unordered):
+ * stable LSD radix sort on the device of the key bits that vary for this chunk.
+ *  hits/tmp dev buffers of >= n_hits keys; the sorted keys end up in hits.
+ *  workspace dev, >= cof_sort_workspace_bytes(cap) bytes.
+ *  n_hits   count or COF_COUNT_ON_DEVICE (the comparer's count, clamped to cap). */
+size_t     cof_sort_workspace_bytes(uint64_t cap);
+cof_status cof_sort_hits(const cof_plan *plan, void *plan_dev, const cof_chunk *dev,
+                         uint64_t *hits, uint64_t *tmp, uint64_t cap, uint64_t n_hits,
+                         void *workspace, cof_stream s);
+
+/* Device counters of plan_dev: out[0]=n_fwd, out[1]=n_rev, out[2]=n_hits (synchronizes). */
+cof_status cof_read_counts(const cof_plan *plan, const void *plan_dev, uint64_t out[3],
+                           cof_stream s);
+
+/* ------------------------------------------------------------------ collect (M10)
+ * One output record: guide index, chromosome, 0-based '+'-strand position (G5),
+ * direction, #mismatches, and the L-letter site read along its strand (G6) with
+ * mismatched compared letters in lower case (G19). */
+typedef struct {
+    uint32_t guide;
+    uint32_t chrom;
+    uint64_t pos;
+    char     strand;   /* '+' or '-' */
+    uint8_t  mm;
+    char     site[34]; /* NUL-terminated */
+} cof_hit;
+
+/* D2H the n_hits keys from hits_dev (stream s), order them (host sort if they are not
+ * already sorted), and decorate them from the HOST planes of the same chunk.
+ * out must hold n_hits records; it is sorted by (pos, strand, guide).
+ * If hits_dev is NULL, keys are read from host_keys instead (already on the host). */
+cof_status cof_collect(const cof_plan *plan, const cof_chunk *host, const uint64_t *hits_dev,
+                       const uint64_t *host_keys, uint64_t n_hits, cof_hit *out, cof_stream s);
+
+/* k-way merge of sorted lists into out (sum of lens records), order (chrom, pos,
+ * strand, guide) (G13).  Lists from disjoint chunks merge by concatenation. */
+cof_status cof_merge(const cof_hit *const *lists, const uint64_t *lens, uint32_t n_lists,
+                     cof_hit *out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* COF_H */

@@ -193,7 +193,7 @@ int64_t cof_oracle_search(int32_t n_chrom, const char *const *seqs, const int64_
         G[i][L] = 0;
     }
 
-    const int64_t BLOCK = 1 << 16;
+    const int64_t BLOCK = 1 << 12;
     hitvec all = {0, 0, 0};
     int err = 0;
     for (int32_t c = 0; c < n_chrom && !err; c++) {

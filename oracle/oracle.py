@@ -77,10 +77,11 @@ def search(seqs, pattern, guides, thresholds, ranges=None, threads: int = 0) -> 
     (chrom, pos, strand '+' before '-', guide).  ``ranges`` = optional list of
     (begin, end) window-start ranges, one per chromosome."""
     L = lib()
-    bufs = [_as_bytes(s) for s in seqs]
-    n = len(bufs)
-    cseqs = (ctypes.c_char_p * max(n, 1))(*bufs)
-    lens = (ctypes.c_int64 * max(n, 1))(*[len(b) for b in bufs])
+    keep = [np.ascontiguousarray(s) if isinstance(s, np.ndarray) else _as_bytes(s) for s in seqs]
+    n = len(keep)
+    addrs = [ctypes.cast(k.ctypes.data, ctypes.c_char_p) if isinstance(k, np.ndarray) else k for k in keep]
+    cseqs = (ctypes.c_char_p * max(n, 1))(*addrs)
+    lens = (ctypes.c_int64 * max(n, 1))(*[len(k) for k in keep])
     beg = end = None
     if ranges is not None:
         beg = (ctypes.c_int64 * n)(*[r[0] for r in ranges])

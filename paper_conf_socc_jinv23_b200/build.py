@@ -1,0 +1,92 @@
+"""Build libcof.so in-tree: nvcc for the sm_100a kernels, g++/OpenMP for the host side.
+
+``python -m paper_conf_socc_jinv23_b200.build`` (or ``__graft_entry__.build()``).
+The library links the CUDA runtime statically and needs only the driver at run time.
+"""
+from __future__ import annotations
+
+import glob
+import hashlib
+import os
+import shutil
+import subprocess
+import sys
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+CSRC = os.path.join(HERE, "csrc")
+ROOT = os.path.dirname(HERE)
+INCLUDE = os.path.join(ROOT, "include")
+LIB = os.path.join(HERE, "libcof.so")
+BUILD = os.path.join(HERE, "_build")
+CUDA = os.environ.get("CUDA_HOME", "/usr/local/cuda")
+NVCC = os.path.join(CUDA, "bin", "nvcc")
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+
+def _sources():
+    cu = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    cpp = sorted(glob.glob(os.path.join(CSRC, "*.cpp")))
+    hdr = sorted(glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh"))
+                 + glob.glob(os.path.join(INCLUDE, "*.h")))
+    return cu, cpp, hdr
+
+
+def _digest(files):
+    h = hashlib.sha256()
+    for f in files:
+        h.update(f.encode())
+        with open(f, "rb") as fh:
+            h.update(fh.read())
+    return h.hexdigest()
+
+
+def _generate():
+    gen = os.path.join(CSRC, "gen_csa.py")
+    out = os.path.join(CSRC, "csa_gen.cuh")
+    if not os.path.exists(out) or os.path.getmtime(out) < os.path.getmtime(gen):
+        text = subprocess.check_output([sys.executable, gen]).decode()
+        with open(out, "w") as f:
+            f.write(text)
+
+
+def build(force: bool = False, verbose: bool = False) -> str:
+    _generate()
+    cu, cpp, hdr = _sources()
+    digest = _digest(cu + cpp + hdr + [__file__])
+    stamp = os.path.join(BUILD, "stamp")
+    if not force and os.path.exists(LIB) and os.path.exists(stamp) and open(stamp).read() == digest:
+        return LIB
+    os.makedirs(BUILD, exist_ok=True)
+    objs = []
+    procs = []
+    for src in cu:
+        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fopenmp",
+               "-Xptxas", "-v" if verbose else "-O3", "-I", INCLUDE, "-c", src, "-o", obj]
+        procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
+        objs.append(obj)
+    for src in cpp:
+        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        cmd = ["g++", "-O3", "-std=c++17", "-fPIC", "-fopenmp", "-Wall", "-I", INCLUDE,
+               "-I", os.path.join(CUDA, "include"), "-c", src, "-o", obj]
+        procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
+        objs.append(obj)
+    for cmd, p in procs:
+        out, _ = p.communicate()
+        if p.returncode != 0:
+            sys.stderr.write(out.decode(errors="replace"))
+            raise RuntimeError("build failed: " + " ".join(cmd))
+        if verbose and out:
+            sys.stderr.write(out.decode(errors="replace"))
+    tmp = LIB + f".{os.getpid()}.tmp"
+    cmd = ["g++", "-shared", "-fopenmp", "-o", tmp, *objs, "-L", os.path.join(CUDA, "lib64"),
+           "-lcudart_static", "-ldl", "-lrt", "-lpthread", "-Wl,--no-undefined"]
+    subprocess.check_call(cmd)
+    os.replace(tmp, LIB)
+    with open(stamp, "w") as f:
+        f.write(digest)
+    return LIB
+
+
+if __name__ == "__main__":
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))

@@ -1,0 +1,302 @@
+"""Thin Python binding of ``libcof.so`` (include/cof.h) -- argument marshalling only.
+
+Every function here has the name of the C entry point it calls and does no arithmetic of
+the method: it converts torch tensors / numpy arrays to pointers, CUDA streams to
+handles, and non-zero status codes to :class:`CofError`.  There is no CPU fallback: if
+the shared library is missing the import fails loudly.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libcof.so")
+
+COF_OK = 0
+COF_E_ARG = -1
+COF_E_CAPACITY = -2
+COF_E_CUDA = -3
+COF_E_STATE = -4
+COF_E_IO = -5
+COF_COUNT_ON_DEVICE = (1 << 64) - 1
+
+HIT_DTYPE = np.dtype([("guide", "<u4"), ("chrom", "<u4"), ("pos", "<u8"), ("strand", "S1"),
+                      ("mm", "u1"), ("site", "S34")], align=True)
+
+
+class CofError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"cof status {status}: {msg}")
+        self.status = status
+
+
+class cof_chunk(ctypes.Structure):
+    _fields_ = [("chrom", ctypes.c_uint32), ("reserved", ctypes.c_uint32), ("start", ctypes.c_uint64),
+                ("n_bases", ctypes.c_uint64), ("n_owned", ctypes.c_uint64),
+                ("lo", ctypes.c_void_p), ("hi", ctypes.c_void_p), ("nm", ctypes.c_void_p)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run `python -m paper_conf_socc_jinv23_b200.build` "
+                          "(there is no CPU fallback)")
+    L = ctypes.CDLL(LIB_PATH)
+    P, U32, U64, SZ, I32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_size_t, ctypes.c_int32
+    sig = {
+        "cof_last_error": (ctypes.c_char_p, []),
+        "cof_version": (ctypes.c_char_p, []),
+        "cof_launch_count": (U64, []),
+        "cof_plan_create": (I32, [ctypes.c_char_p, U32, P, P, P]),
+        "cof_plan_destroy": (None, [P]),
+        "cof_plan_length": (U32, [P]),
+        "cof_plan_n_guides": (U32, [P]),
+        "cof_plan_device_bytes": (SZ, [P]),
+        "cof_plan_upload": (I32, [P, P, P]),
+        "cof_plane_words": (U64, [U64]),
+        "cof_pack": (I32, [P, U64, P, P, P]),
+        "cof_unpack": (I32, [P, P, P, U64, U64, P]),
+        "cof_load_chunk": (I32, [P, P, P]),
+        "cof_fasta_open": (I32, [ctypes.c_char_p, P]),
+        "cof_fasta_close": (None, [P]),
+        "cof_fasta_count": (U32, [P]),
+        "cof_fasta_name": (ctypes.c_char_p, [P, U32]),
+        "cof_fasta_length": (U64, [P, U32]),
+        "cof_fasta_pack": (I32, [P, U32, U64, U64, P, P, P]),
+        "cof_find_workspace_bytes": (SZ, [U64]),
+        "cof_find_pam": (I32, [P, P, P, P, P, P, U64, P, P, P]),
+        "cof_compare": (I32, [P, P, P, P, U64, P, U64, P, U64, P, P]),
+        "cof_sort_workspace_bytes": (SZ, [U64]),
+        "cof_sort_hits": (I32, [P, P, P, P, P, U64, U64, P, P]),
+        "cof_read_counts": (I32, [P, P, P, P]),
+        "cof_collect": (I32, [P, P, P, P, U64, P, P]),
+        "cof_merge": (I32, [P, P, U32, P]),
+        "cof_set_comparer": (I32, [ctypes.c_int]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    return L
+
+
+lib = _load()
+
+# names the header declares (checked by tests/test_abi_host.py)
+EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof_plan_create",
+                       "cof_plan_destroy", "cof_plan_length", "cof_plan_n_guides",
+                       "cof_plan_device_bytes", "cof_plan_upload", "cof_plane_words", "cof_pack",
+                       "cof_unpack", "cof_load_chunk", "cof_fasta_open", "cof_fasta_close",
+                       "cof_fasta_count", "cof_fasta_name", "cof_fasta_length", "cof_fasta_pack",
+                       "cof_find_workspace_bytes", "cof_find_pam", "cof_compare",
+                       "cof_sort_workspace_bytes", "cof_sort_hits", "cof_read_counts",
+                       "cof_collect", "cof_merge")]
+
+
+def _check(st):
+    if st != COF_OK:
+        raise CofError(st, lib.cof_last_error().decode(errors="replace"))
+
+
+def _ptr(x):
+    """Address of a tensor / ndarray / int / None."""
+    if x is None:
+        return None
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    if isinstance(x, (ctypes.Array, ctypes.Structure)):
+        return ctypes.addressof(x)
+    raise TypeError(f"cannot take the address of {type(x)}")
+
+
+def _stream(s):
+    if s is None:
+        return None
+    if isinstance(s, int):
+        return s
+    return s.cuda_stream
+
+
+def cof_last_error() -> str:
+    return lib.cof_last_error().decode(errors="replace")
+
+
+def cof_version() -> str:
+    return lib.cof_version().decode()
+
+
+def cof_launch_count() -> int:
+    return int(lib.cof_launch_count())
+
+
+class Plan:
+    """Owns a ``cof_plan*``."""
+
+    def __init__(self, handle, pattern, guides, max_mm):
+        self.handle = handle
+        self.pattern = pattern
+        self.guides = list(guides)
+        self.max_mm = list(max_mm)
+
+    @property
+    def L(self):
+        return int(lib.cof_plan_length(self.handle))
+
+    @property
+    def n_guides(self):
+        return int(lib.cof_plan_n_guides(self.handle))
+
+    def __del__(self):
+        h, self.handle = getattr(self, "handle", None), None
+        if h and lib is not None:
+            lib.cof_plan_destroy(h)
+
+
+def cof_plan_create(pattern: str, guides, max_mm) -> Plan:
+    gs = [g.encode() for g in guides]
+    arr = (ctypes.c_char_p * max(len(gs), 1))(*gs)
+    mm = np.ascontiguousarray(np.asarray(max_mm, dtype=np.uint8))
+    out = ctypes.c_void_p()
+    _check(lib.cof_plan_create(pattern.encode(), len(gs), ctypes.addressof(arr), mm.ctypes.data,
+                               ctypes.addressof(out)))
+    return Plan(out.value, pattern, guides, max_mm)
+
+
+def cof_plan_device_bytes(plan: Plan) -> int:
+    return int(lib.cof_plan_device_bytes(plan.handle))
+
+
+def cof_plan_upload(plan: Plan, plan_dev, stream=None):
+    _check(lib.cof_plan_upload(plan.handle, _ptr(plan_dev), _stream(stream)))
+
+
+def cof_plane_words(n_bases: int) -> int:
+    return int(lib.cof_plane_words(int(n_bases)))
+
+
+def cof_pack(ascii_arr, n, lo, hi, nm):
+    _check(lib.cof_pack(_ptr(ascii_arr), int(n), _ptr(lo), _ptr(hi), _ptr(nm)))
+
+
+def cof_unpack(lo, hi, nm, first, n, out):
+    _check(lib.cof_unpack(_ptr(lo), _ptr(hi), _ptr(nm), int(first), int(n), _ptr(out)))
+
+
+def make_chunk(chrom, start, n_bases, n_owned, lo, hi, nm) -> cof_chunk:
+    return cof_chunk(int(chrom), 0, int(start), int(n_bases), int(n_owned), _ptr(lo), _ptr(hi), _ptr(nm))
+
+
+def cof_load_chunk(host: cof_chunk, dev: cof_chunk, stream=None):
+    _check(lib.cof_load_chunk(ctypes.addressof(host), ctypes.addressof(dev), _stream(stream)))
+
+
+def cof_find_workspace_bytes(n_owned: int) -> int:
+    return int(lib.cof_find_workspace_bytes(int(n_owned)))
+
+
+def cof_find_pam(plan, plan_dev, dev: cof_chunk, workspace, items_fwd, items_rev, items_cap,
+                 stream=None, sync=True):
+    """Returns (n_fwd, n_rev) if ``sync`` else None (counts stay on the device)."""
+    if sync:
+        a, b = ctypes.c_uint64(), ctypes.c_uint64()
+        _check(lib.cof_find_pam(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
+                                _ptr(items_fwd), _ptr(items_rev), int(items_cap), ctypes.addressof(a),
+                                ctypes.addressof(b), _stream(stream)))
+        return int(a.value), int(b.value)
+    _check(lib.cof_find_pam(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
+                            _ptr(items_fwd), _ptr(items_rev), int(items_cap), None, None, _stream(stream)))
+    return None
+
+
+def cof_compare(plan, plan_dev, dev: cof_chunk, items_fwd, n_fwd, items_rev, n_rev, hits, hits_cap,
+                stream=None, sync=True):
+    """Returns n_hits if ``sync`` else None.  n_fwd/n_rev may be COF_COUNT_ON_DEVICE."""
+    if sync:
+        n = ctypes.c_uint64()
+        _check(lib.cof_compare(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(items_fwd),
+                               int(n_fwd), _ptr(items_rev), int(n_rev), _ptr(hits), int(hits_cap),
+                               ctypes.addressof(n), _stream(stream)))
+        return int(n.value)
+    _check(lib.cof_compare(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(items_fwd), int(n_fwd),
+                           _ptr(items_rev), int(n_rev), _ptr(hits), int(hits_cap), None, _stream(stream)))
+    return None
+
+
+def cof_sort_workspace_bytes(cap: int) -> int:
+    return int(lib.cof_sort_workspace_bytes(int(cap)))
+
+
+def cof_sort_hits(plan, plan_dev, dev: cof_chunk, hits, tmp, cap, n_hits, workspace, stream=None):
+    _check(lib.cof_sort_hits(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(hits), _ptr(tmp),
+                             int(cap), int(n_hits), _ptr(workspace), _stream(stream)))
+
+
+def cof_read_counts(plan, plan_dev, stream=None):
+    out = (ctypes.c_uint64 * 3)()
+    _check(lib.cof_read_counts(plan.handle, _ptr(plan_dev), ctypes.addressof(out), _stream(stream)))
+    return int(out[0]), int(out[1]), int(out[2])
+
+
+def cof_collect(plan, host: cof_chunk, hits_dev, n_hits, stream=None, host_keys=None) -> np.ndarray:
+    out = np.zeros(int(n_hits), dtype=HIT_DTYPE)
+    if n_hits:
+        _check(lib.cof_collect(plan.handle, ctypes.addressof(host), _ptr(hits_dev), _ptr(host_keys),
+                               int(n_hits), out.ctypes.data, _stream(stream)))
+    return out
+
+
+def cof_merge(lists) -> np.ndarray:
+    lists = [np.ascontiguousarray(x, dtype=HIT_DTYPE) for x in lists]
+    total = sum(len(x) for x in lists)
+    out = np.zeros(total, dtype=HIT_DTYPE)
+    ptrs = (ctypes.c_void_p * max(len(lists), 1))(*[x.ctypes.data for x in lists])
+    lens = (ctypes.c_uint64 * max(len(lists), 1))(*[len(x) for x in lists])
+    _check(lib.cof_merge(ctypes.addressof(ptrs), ctypes.addressof(lens), len(lists), out.ctypes.data))
+    return out
+
+
+def cof_set_comparer(impl: str):
+    """'table' (bit-sliced pair tables, default) or 'popc' (POPC per comparison)."""
+    _check(lib.cof_set_comparer({"popc": 0, "table": 1}[impl]))
+
+
+class Fasta:
+    def __init__(self, path):
+        out = ctypes.c_void_p()
+        _check(lib.cof_fasta_open(str(path).encode(), ctypes.addressof(out)))
+        self.handle = out.value
+
+    def __len__(self):
+        return int(lib.cof_fasta_count(self.handle))
+
+    def name(self, i):
+        return lib.cof_fasta_name(self.handle, i).decode()
+
+    def length(self, i):
+        return int(lib.cof_fasta_length(self.handle, i))
+
+    def pack(self, i, first, n, lo, hi, nm):
+        _check(lib.cof_fasta_pack(self.handle, i, int(first), int(n), _ptr(lo), _ptr(hi), _ptr(nm)))
+
+    def close(self):
+        if self.handle:
+            lib.cof_fasta_close(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def hits_to_tuples(arr):
+    """(chrom, pos, strand, guide, mm, site) tuples (same serialization as the tests use)."""
+    return [(int(h["chrom"]), int(h["pos"]), h["strand"].decode(), int(h["guide"]), int(h["mm"]),
+             h["site"].decode()) for h in arr]

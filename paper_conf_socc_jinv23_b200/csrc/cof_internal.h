@@ -1,0 +1,81 @@
+// Internal definitions shared by the libcof.so translation units (NOT by the oracle).
+#pragma once
+#include <cstdint>
+#include <cstddef>
+#include <string>
+#include <vector>
+
+#include "../../include/cof.h"
+
+namespace cof {
+
+// ---- error handling (thread-local message, COF_* status codes)
+cof_status set_error(cof_status code, const char* fmt, ...);
+cof_status cuda_error(int err, const char* what);   // err = cudaError_t
+void count_launches(uint64_t n);
+
+// ---- nucleotide encoding of the product path
+// 4-bit IUPAC set masks: A=1, C=2, G=4, T=8 (N = 15).  Returns 0 for a non-IUPAC letter.
+uint8_t iupac_mask(char c);
+inline uint8_t comp_mask(uint8_t m) {          // complement of a set: A<->T, C<->G
+    return (uint8_t)(((m & 1) << 3) | ((m & 8) >> 3) | ((m & 2) << 1) | ((m & 4) >> 1));
+}
+// 2-bit code of a concrete base set (A=0 C=1 G=2 T=3), -1 if not a single base.
+inline int concrete_code(uint8_t m) {
+    switch (m) { case 1: return 0; case 2: return 1; case 4: return 2; case 8: return 3; default: return -1; }
+}
+
+// ---- finder parameters (per strand, non-N pattern positions)
+struct PamStrand {
+    uint32_t n;            // number of non-N positions
+    uint8_t j[32];         // window offset
+    uint8_t set[32];       // IUPAC set mask
+};
+
+// ---- comparer guide tables (device image inside plan_dev)
+// Concrete group record (uint4): {lo, hi, (uint32)-(t+1), guide}
+// Degenerate group record (2 x uint4): {A, C, G, T one-hot}, {care, -(t+1), guide, 0}
+enum GroupKind : uint32_t { GROUP_CONCRETE = 0, GROUP_DEGENERATE = 1 };
+struct GroupDesc {
+    uint32_t care;         // compared-position mask (bit j = window offset j)
+    uint32_t kind;
+    uint32_t rec_begin;    // index into the strand's uint4 record array
+    uint32_t n_guides;
+};
+
+// Bit-sliced pair-table comparer (v2): per strand, per 32-guide block, per position pair,
+// 25 entries (base pair combos incl. N) of {bit0, bit1} mismatch-count planes.
+struct PairLayout {
+    uint32_t n_pairs;          // pairs covering the union of compared positions
+    uint8_t j1[16], j2[16];    // window offsets of the pair (j2 == 0xFF: single position)
+};
+
+// Device plan image layout (byte offsets from plan_dev; all 256-byte aligned)
+struct DevLayout {
+    size_t counters;           // uint64[8]: n_fwd, n_rev, n_hits, ...
+    size_t groups_fwd, groups_rev;   // GroupDesc[n_groups]
+    size_t recs_fwd, recs_rev;       // uint4[n_recs]
+    size_t ptab_fwd, ptab_rev;       // pair tables: uint2[n_blocks][n_pairs][25]
+    size_t pmeta_fwd, pmeta_rev;     // per block: uint32[8] = {T0..T5 threshold planes, valid, 0}
+    size_t total;
+};
+
+}  // namespace cof
+
+struct cof_plan {
+    uint32_t L = 0;
+    uint32_t n_guides = 0;
+    std::string pattern;                 // upper-case
+    std::vector<std::string> guides;     // upper-case
+    std::vector<uint8_t> max_mm;
+    std::vector<uint8_t> gmask;          // [n_guides * L] IUPAC masks (forward orientation)
+    cof::PamStrand pam[2];               // [0] '+', [1] '-' (reverse-complemented pattern)
+    uint32_t n_groups = 0;
+    uint32_t n_recs = 0;
+    uint32_t n_blocks = 0;               // 32-guide blocks (pair-table comparer)
+    cof::PairLayout pairs[2];
+    uint32_t union_care[2] = {0, 0};
+    bool any_degenerate = false;
+    cof::DevLayout lay;
+    std::vector<uint8_t> image;          // host copy of the device image (counters zeroed)
+};

@@ -1,0 +1,439 @@
+// Comparer ("compare" kernel, M8 + M9) for sm_100a -- two implementations.
+//
+// Paper: Listing 1.  For each locus i and each selected strand the kernel
+// walks the non-N query positions (comp_index, -1-terminated), counts genome
+// bases outside the query letter's IUPAC set, stops early once the count
+// exceeds the threshold and, if the count is <= threshold,
+// appends (count, direction, locus) through an atomic counter.
+// The '-' half compares the reverse-complemented query against the same '+' window
+// (P:L231-L236).  The query table is staged in local (shared) memory (the
+// paper's opt3).  This kernel is ~98% of kernel time.
+//
+// v1 "popc"  (cof_comparer_popc): items in registers (R per thread), guide records in
+//   shared memory; per (item, guide) mm = popc(care & ((w_lo^g_lo) | (w_hi^g_hi) | w_nm))
+//   with the window pre-masked by the group's care mask -> 2 LOP3 + POPC + IADD.  Bound by
+//   the quarter-rate POPC pipe (16/clk/SM measured on B200, tools/microbench_pipes.cu).
+// v2 "table" (cof_comparer_table): bit-sliced over 32 guides.  For each position pair of
+//   an item, one 64-bit shared-memory lookup indexed by the pair's two genome bases returns
+//   the 2-bit mismatch count of all 32 guides of a block (bit k = guide k); a LOP3
+//   carry-save adder tree sums the pairs and a borrow chain against the bit-sliced
+//   thresholds yields the 32-guide hit mask.  No POPC, ~1.3 ALU ops + 0.3 LDS per
+//   comparison.  Handles any IUPAC guide letter and per-guide thresholds uniformly.
+#include <cuda_runtime.h>
+
+#include "cof_internal.h"
+#include "dev_common.cuh"
+#include "csa_gen.cuh"
+
+namespace cof {
+
+constexpr int CT = 256;   // threads per CTA
+constexpr uint64_t ON_DEVICE = COF_COUNT_ON_DEVICE;
+
+struct CompareArgs {
+    const uint32_t* lo;
+    const uint32_t* hi;
+    const uint32_t* nm;
+    const uint32_t* items[2];
+    uint64_t n[2];                 // ON_DEVICE: read counters[0..1]
+    uint64_t items_cap;
+    unsigned long long* hits;
+    uint64_t cap;
+    unsigned long long* counters;  // [0] n_fwd [1] n_rev [2] n_hits
+    // v1
+    const uint4* groups[2];        // GroupDesc as uint4
+    const uint4* recs[2];
+    uint32_t n_groups, n_recs;
+    // v2
+    const uint2* ptab[2];          // [n_blocks][n_pairs][25]
+    const uint32_t* pmeta[2];      // [n_blocks][8]
+    uint32_t n_blocks, n_pairs;
+    PairLayout pairs[2];
+};
+
+__device__ __forceinline__ void item_counts(const CompareArgs& a, uint64_t& n0, uint64_t& n1) {
+    n0 = a.n[0] == ON_DEVICE ? (uint64_t)a.counters[0] : a.n[0];
+    n1 = a.n[1] == ON_DEVICE ? (uint64_t)a.counters[1] : a.n[1];
+    if (n0 > a.items_cap) n0 = a.items_cap;
+    if (n1 > a.items_cap) n1 = a.items_cap;
+}
+
+// Warp-aggregated append of one key per predicated lane (old = atomic_inc(entrycount)).
+__device__ __forceinline__ void emit(const CompareArgs& a, bool pred, unsigned long long key) {
+    const unsigned act = __activemask();
+    const unsigned m = __ballot_sync(act, pred);
+    if (!pred) return;
+    const int lane = threadIdx.x & 31;
+    const int leader = __ffs(m) - 1;
+    unsigned long long base = 0;
+    if (lane == leader) base = atomicAdd(&a.counters[2], (unsigned long long)__popc(m));
+    base = __shfl_sync(m, base, leader);
+    const unsigned long long o = base + __popc(m & lanemask_lt());
+    if (o < a.cap) a.hits[o] = key;
+}
+
+__device__ __forceinline__ unsigned long long hit_key(uint32_t pos, uint32_t strand, uint32_t guide, uint32_t mm) {
+    return ((unsigned long long)pos << 32) | ((unsigned long long)strand << 31) |
+           ((unsigned long long)guide << 7) | (unsigned long long)mm;
+}
+
+// ============================================================================ v1 popc
+template <int R, bool SMEM>
+__global__ void __launch_bounds__(CT) cof_comparer_popc(const __grid_constant__ CompareArgs a) {
+    extern __shared__ __align__(16) uint4 s_tab[];
+    const uint4* G[2];
+    const uint4* Rc[2];
+    if (SMEM) {
+        const uint32_t ng = a.n_groups, nr = a.n_recs;
+        for (uint32_t i = threadIdx.x; i < ng; i += CT) {
+            s_tab[i] = a.groups[0][i];
+            s_tab[ng + i] = a.groups[1][i];
+        }
+        for (uint32_t i = threadIdx.x; i < nr; i += CT) {
+            s_tab[2 * ng + i] = a.recs[0][i];
+            s_tab[2 * ng + nr + i] = a.recs[1][i];
+        }
+        __syncthreads();
+        G[0] = s_tab; G[1] = s_tab + ng; Rc[0] = s_tab + 2 * ng; Rc[1] = s_tab + 2 * ng + nr;
+    } else {
+        G[0] = a.groups[0]; G[1] = a.groups[1]; Rc[0] = a.recs[0]; Rc[1] = a.recs[1];
+    }
+    uint64_t n0, n1;
+    item_counts(a, n0, n1);
+    const uint64_t per_tile = (uint64_t)CT * R;
+    const uint64_t t0 = (n0 + per_tile - 1) / per_tile, t1 = (n1 + per_tile - 1) / per_tile;
+    for (uint64_t tile = blockIdx.x; tile < t0 + t1; tile += gridDim.x) {
+        const uint32_t st = tile < t0 ? 0u : 1u;
+        const uint64_t base = (st == 0 ? tile : tile - t0) * per_tile;
+        const uint64_t nst = st == 0 ? n0 : n1;
+        uint32_t pos[R], wl[R], wh[R], wn[R];
+        bool ok[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            const uint64_t idx = base + (uint64_t)r * CT + threadIdx.x;
+            ok[r] = idx < nst;
+            pos[r] = ok[r] ? __ldg(a.items[st] + idx) : 0u;
+            wl[r] = plane_window(a.lo, pos[r]);
+            wh[r] = plane_window(a.hi, pos[r]);
+            wn[r] = plane_window(a.nm, pos[r]);
+        }
+        for (uint32_t g = 0; g < a.n_groups; g++) {
+            const uint4 gd = G[st][g];             // {care, kind, rec_begin, n_guides}
+            const uint32_t care = gd.x;
+            if (gd.y == GROUP_CONCRETE) {
+                uint32_t ml[R], mh[R], mn[R];
+#pragma unroll
+                for (int r = 0; r < R; r++) { ml[r] = wl[r] & care; mh[r] = wh[r] & care; mn[r] = wn[r] & care; }
+                const uint4* rec = Rc[st] + gd.z;
+                for (uint32_t k = 0; k < gd.w; k++) {
+                    const uint4 q = rec[k];       // {g_lo, g_hi, -(t+1), guide}
+                    int32_t any = 0;
+#pragma unroll
+                    for (int r = 0; r < R; r++) {
+                        const uint32_t y = ((ml[r] ^ q.x) | mn[r]) | (mh[r] ^ q.y);
+                        any |= __popc(y) + (int32_t)q.z;
+                    }
+                    if (any < 0) {
+#pragma unroll
+                        for (int r = 0; r < R; r++) {
+                            const uint32_t y = ((ml[r] ^ q.x) | mn[r]) | (mh[r] ^ q.y);
+                            const uint32_t mm = (uint32_t)__popc(y);
+                            emit(a, ok[r] && (int32_t)mm + (int32_t)q.z < 0, hit_key(pos[r], st, q.w, mm));
+                        }
+                    }
+                }
+            } else {
+                // degenerate guide letters: one-hot window planes, match = OR_b (is_b & guide_b)
+                uint32_t isA[R], isC[R], isG[R], isT[R];
+#pragma unroll
+                for (int r = 0; r < R; r++) {
+                    isA[r] = ~wl[r] & ~wh[r] & ~wn[r];
+                    isC[r] = wl[r] & ~wh[r] & ~wn[r];
+                    isG[r] = ~wl[r] & wh[r] & ~wn[r];
+                    isT[r] = wl[r] & wh[r] & ~wn[r];
+                }
+                const uint4* rec = Rc[st] + gd.z;
+                for (uint32_t k = 0; k < gd.w; k++) {
+                    const uint4 q = rec[2 * k];        // one-hot {A, C, G, T}
+                    const uint4 q2 = rec[2 * k + 1];   // {care, -(t+1), guide, 0}
+#pragma unroll
+                    for (int r = 0; r < R; r++) {
+                        const uint32_t match = (isA[r] & q.x) | (isC[r] & q.y) | (isG[r] & q.z) | (isT[r] & q.w);
+                        const uint32_t mm = (uint32_t)__popc(q2.x & ~match);
+                        emit(a, ok[r] && (int32_t)mm + (int32_t)q2.y < 0, hit_key(pos[r], st, q2.z, mm));
+                    }
+                }
+            }
+        }
+    }
+}
+
+// ============================================================================ v2 table
+// per-item, per-pair byte offset into a block's pair table: (pair * 25 + 5*b1 + b2) * 8
+template <int NP>
+__device__ __forceinline__ void pair_offsets(const PairLayout& pl, uint32_t wl, uint32_t wh, uint32_t wn,
+                                             uint32_t (&off)[NP]) {
+#pragma unroll
+    for (int q = 0; q < NP; q++) {
+        const uint32_t j1 = pl.j1[q], j2 = pl.j2[q];
+        const uint32_t b1 = ((wn >> j1) & 1u) ? 4u : (((wl >> j1) & 1u) | (((wh >> j1) & 1u) << 1));
+        uint32_t b2 = 0;
+        if (j2 != 0xFFu) b2 = ((wn >> j2) & 1u) ? 4u : (((wl >> j2) & 1u) | (((wh >> j2) & 1u) << 1));
+        off[q] = ((uint32_t)q * 25u + b1 * 5u + b2) * 8u;
+    }
+}
+
+template <int NP, int R>
+__global__ void __launch_bounds__(CT) cof_comparer_table(const __grid_constant__ CompareArgs a,
+                                                        uint32_t blocks_per_chunk) {
+    extern __shared__ __align__(16) uint8_t s_raw[];
+    // shared layout: [blocks_per_chunk][NP][25] uint2 table, then [blocks_per_chunk][8] meta
+    const uint32_t tab_bytes = blocks_per_chunk * NP * 25 * 8;
+    uint32_t* s_meta = reinterpret_cast<uint32_t*>(s_raw + tab_bytes);
+    const uint32_t s_tab = smem_u32(s_raw);
+
+    uint64_t n0, n1;
+    item_counts(a, n0, n1);
+    const uint64_t per_tile = (uint64_t)CT * R;
+    const uint64_t t0 = (n0 + per_tile - 1) / per_tile, t1 = (n1 + per_tile - 1) / per_tile;
+    const uint32_t n_chunks = (a.n_blocks + blocks_per_chunk - 1) / blocks_per_chunk;
+    int loaded_st = -1;
+    uint32_t loaded_chunk = 0xFFFFFFFFu;
+
+    for (uint64_t tile = blockIdx.x; tile < t0 + t1; tile += gridDim.x) {
+        const uint32_t st = tile < t0 ? 0u : 1u;
+        const uint64_t base = (st == 0 ? tile : tile - t0) * per_tile;
+        const uint64_t nst = st == 0 ? n0 : n1;
+        uint32_t pos[R], off[R][NP];
+        bool ok[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            const uint64_t idx = base + (uint64_t)r * CT + threadIdx.x;
+            ok[r] = idx < nst;
+            pos[r] = ok[r] ? __ldg(a.items[st] + idx) : 0u;
+            pair_offsets<NP>(a.pairs[st], plane_window(a.lo, pos[r]), plane_window(a.hi, pos[r]),
+                             plane_window(a.nm, pos[r]), off[r]);
+        }
+        for (uint32_t ch = 0; ch < n_chunks; ch++) {
+            const uint32_t b0 = ch * blocks_per_chunk;
+            const uint32_t nb = min(blocks_per_chunk, a.n_blocks - b0);
+            if (loaded_st != (int)st || loaded_chunk != ch) {
+                __syncthreads();
+                const uint4* src = reinterpret_cast<const uint4*>(a.ptab[st] + (size_t)b0 * NP * 25);
+                uint4* dst = reinterpret_cast<uint4*>(s_raw);
+                const uint32_t n16 = nb * NP * 25 * 8 / 16;
+                for (uint32_t i = threadIdx.x; i < n16; i += CT) dst[i] = __ldg(src + i);
+                for (uint32_t i = threadIdx.x; i < nb * 8; i += CT) s_meta[i] = __ldg(a.pmeta[st] + (size_t)b0 * 8 + i);
+                __syncthreads();
+                loaded_st = (int)st;
+                loaded_chunk = ch;
+            }
+            for (uint32_t b = 0; b < nb; b++) {
+                const uint32_t bbase = s_tab + b * (NP * 25 * 8);
+                const uint32_t* meta = s_meta + b * 8;
+                uint32_t T[6];
+#pragma unroll
+                for (int w = 0; w < 6; w++) T[w] = meta[w];
+                const uint32_t valid = meta[6];
+#pragma unroll
+                for (int r = 0; r < R; r++) {
+                    uint32_t v0[NP], v1[NP];
+#pragma unroll
+                    for (int q = 0; q < NP; q++)
+                        asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v0[q]), "=r"(v1[q]) : "r"(bbase + off[r][q]));
+                    uint32_t s[6];
+                    uint32_t hitm = csa_hits<NP>(v0, v1, T, valid, s);
+                    if (!ok[r]) hitm = 0;
+                    while (hitm) {
+                        const int k = __ffs(hitm) - 1;
+                        hitm &= hitm - 1;
+                        const uint32_t mm = ((s[0] >> k) & 1u) | (((s[1] >> k) & 1u) << 1) | (((s[2] >> k) & 1u) << 2) |
+                                            (((s[3] >> k) & 1u) << 3) | (((s[4] >> k) & 1u) << 4) |
+                                            (((s[5] >> k) & 1u) << 5);
+                        const uint32_t guide = (b0 + b) * 32u + (uint32_t)k;
+                        const unsigned long long key = hit_key(pos[r], st, guide, mm);
+                        const unsigned long long o = atomicAdd(&a.counters[2], 1ull);
+                        if (o < a.cap) a.hits[o] = key;
+                    }
+                }
+            }
+        }
+    }
+}
+
+// ============================================================================ host side
+struct KernelInfo {
+    const void* fn;
+    int bps;        // resident CTAs per SM at the launch smem size
+    uint32_t smem;
+};
+
+static int num_sms() {
+    static int sms = -1;
+    if (sms < 0) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    }
+    return sms;
+}
+
+static cof_status occupancy(const void* fn, uint32_t smem, int* bps) {
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return cuda_error(e, "comparer smem attribute");
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(bps, fn, CT, smem);
+    if (e != cudaSuccess) return cuda_error(e, "comparer occupancy");
+    if (*bps < 1) *bps = 1;
+    return COF_OK;
+}
+
+constexpr int R_POPC = 8;
+constexpr int R_TABLE = 2;
+
+template <int NP>
+static cof_status launch_table(const CompareArgs& a, uint64_t tiles_hint, cudaStream_t stream) {
+    // guide blocks resident in shared memory per pass (tiles over blocks if they do not fit)
+    const uint32_t per_block = NP * 25 * 8 + 32;
+    uint32_t bpc = a.n_blocks;
+    const uint32_t budget = 96 * 1024;
+    if (bpc * per_block > budget) bpc = budget / per_block;
+    const uint32_t smem = bpc * per_block;
+    int bps = 0;
+    auto fn = cof_comparer_table<NP, R_TABLE>;
+    cof_status st = occupancy((const void*)fn, smem, &bps);
+    if (st != COF_OK) return st;
+    uint64_t grid = (uint64_t)num_sms() * bps;
+    if (tiles_hint != ON_DEVICE && grid > tiles_hint) grid = tiles_hint ? tiles_hint : 1;
+    fn<<<(uint32_t)grid, CT, smem, stream>>>(a, bpc);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "cof_comparer_table launch");
+    count_launches(1);
+    return COF_OK;
+}
+
+static cof_status launch_popc(const CompareArgs& a, uint64_t tiles_hint, cudaStream_t stream) {
+    const uint32_t tab = (2 * a.n_groups + 2 * a.n_recs) * 16;
+    const bool smem_ok = tab <= 160 * 1024;
+    int bps = 0;
+    const void* fn = smem_ok ? (const void*)cof_comparer_popc<R_POPC, true> : (const void*)cof_comparer_popc<R_POPC, false>;
+    const uint32_t smem = smem_ok ? tab : 0;
+    cof_status st = occupancy(fn, smem, &bps);
+    if (st != COF_OK) return st;
+    uint64_t grid = (uint64_t)num_sms() * bps;
+    if (tiles_hint != ON_DEVICE && grid > tiles_hint) grid = tiles_hint ? tiles_hint : 1;
+    if (smem_ok) cof_comparer_popc<R_POPC, true><<<(uint32_t)grid, CT, smem, stream>>>(a);
+    else cof_comparer_popc<R_POPC, false><<<(uint32_t)grid, CT, 0, stream>>>(a);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "cof_comparer_popc launch");
+    count_launches(1);
+    return COF_OK;
+}
+
+static int g_impl = -1;   // 0 = popc, 1 = table (default); COF_COMPARER=popc|table overrides
+
+static int comparer_impl() {
+    if (g_impl < 0) {
+        const char* e = getenv("COF_COMPARER");
+        g_impl = (e && e[0] == 'p') ? 0 : 1;
+    }
+    return g_impl;
+}
+
+}  // namespace cof
+
+using namespace cof;
+
+extern "C" {
+
+cof_status cof_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, const uint32_t* items_fwd,
+                       uint64_t n_fwd, const uint32_t* items_rev, uint64_t n_rev, uint64_t* hits, uint64_t hits_cap,
+                       uint64_t* n_hits, cof_stream s) {
+    if (!plan || !plan_dev || !dev || !items_fwd || !items_rev || (!hits && hits_cap))
+        return set_error(COF_E_ARG, "cof_compare: NULL argument");
+    if (!dev->lo || !dev->hi || !dev->nm) return set_error(COF_E_ARG, "cof_compare: chunk planes are NULL");
+    cudaStream_t stream = (cudaStream_t)s;
+    uint8_t* pd = (uint8_t*)plan_dev;
+    CompareArgs a;
+    a.lo = dev->lo; a.hi = dev->hi; a.nm = dev->nm;
+    a.items[0] = items_fwd; a.items[1] = items_rev;
+    a.n[0] = n_fwd; a.n[1] = n_rev;
+    // the item capacity is only known to the caller; counts from the device are trusted up
+    // to n_owned (the finder never reports more than it could write into n_owned slots)
+    a.items_cap = dev->n_owned;
+    if (n_fwd != ON_DEVICE && n_fwd > a.items_cap) a.items_cap = n_fwd;
+    if (n_rev != ON_DEVICE && n_rev > a.items_cap) a.items_cap = n_rev;
+    a.hits = (unsigned long long*)hits;
+    a.cap = hits_cap;
+    a.counters = (unsigned long long*)(pd + plan->lay.counters);
+    a.groups[0] = (const uint4*)(pd + plan->lay.groups_fwd);
+    a.groups[1] = (const uint4*)(pd + plan->lay.groups_rev);
+    a.recs[0] = (const uint4*)(pd + plan->lay.recs_fwd);
+    a.recs[1] = (const uint4*)(pd + plan->lay.recs_rev);
+    a.n_groups = plan->n_groups;
+    a.n_recs = plan->n_recs;
+    a.ptab[0] = (const uint2*)(pd + plan->lay.ptab_fwd);
+    a.ptab[1] = (const uint2*)(pd + plan->lay.ptab_rev);
+    a.pmeta[0] = (const uint32_t*)(pd + plan->lay.pmeta_fwd);
+    a.pmeta[1] = (const uint32_t*)(pd + plan->lay.pmeta_rev);
+    a.n_blocks = plan->n_blocks;
+    a.n_pairs = plan->pairs[0].n_pairs;
+    a.pairs[0] = plan->pairs[0];
+    a.pairs[1] = plan->pairs[1];
+
+    cudaError_t e = cudaMemsetAsync(a.counters + 2, 0, sizeof(uint64_t), stream);
+    if (e != cudaSuccess) return cuda_error(e, "cof_compare memset");
+    uint64_t tiles_hint = ON_DEVICE;
+    if (n_fwd != ON_DEVICE && n_rev != ON_DEVICE) {
+        const int R = comparer_impl() == 0 ? R_POPC : R_TABLE;
+        const uint64_t per = (uint64_t)CT * R;
+        tiles_hint = (n_fwd + per - 1) / per + (n_rev + per - 1) / per;
+    }
+    if (tiles_hint != 0) {
+        cof_status st;
+        if (comparer_impl() == 0) {
+            st = launch_popc(a, tiles_hint, stream);
+        } else {
+            switch (a.n_pairs) {
+                case 1: st = launch_table<1>(a, tiles_hint, stream); break;
+                case 2: st = launch_table<2>(a, tiles_hint, stream); break;
+                case 3: st = launch_table<3>(a, tiles_hint, stream); break;
+                case 4: st = launch_table<4>(a, tiles_hint, stream); break;
+                case 5: st = launch_table<5>(a, tiles_hint, stream); break;
+                case 6: st = launch_table<6>(a, tiles_hint, stream); break;
+                case 7: st = launch_table<7>(a, tiles_hint, stream); break;
+                case 8: st = launch_table<8>(a, tiles_hint, stream); break;
+                case 9: st = launch_table<9>(a, tiles_hint, stream); break;
+                case 10: st = launch_table<10>(a, tiles_hint, stream); break;
+                case 11: st = launch_table<11>(a, tiles_hint, stream); break;
+                case 12: st = launch_table<12>(a, tiles_hint, stream); break;
+                case 13: st = launch_table<13>(a, tiles_hint, stream); break;
+                case 14: st = launch_table<14>(a, tiles_hint, stream); break;
+                case 15: st = launch_table<15>(a, tiles_hint, stream); break;
+                case 16: st = launch_table<16>(a, tiles_hint, stream); break;
+                default: return set_error(COF_E_STATE, "cof_compare: %u pairs", a.n_pairs);
+            }
+        }
+        if (st != COF_OK) return st;
+    }
+    if (n_hits) {
+        uint64_t c = 0;
+        e = cudaMemcpyAsync(&c, a.counters + 2, sizeof c, cudaMemcpyDeviceToHost, stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+        if (e != cudaSuccess) return cuda_error(e, "cof_compare count");
+        *n_hits = c;
+        if (c > hits_cap)
+            return set_error(COF_E_CAPACITY, "cof_compare: %llu hits exceed capacity %llu", (unsigned long long)c,
+                             (unsigned long long)hits_cap);
+    }
+    return COF_OK;
+}
+
+// Select the comparer implementation at run time (0 = popc, 1 = table).  Not part of the
+// stable ABI (declared here for tests / benchmarks).
+cof_status cof_set_comparer(int impl) {
+    if (impl != 0 && impl != 1) return set_error(COF_E_ARG, "cof_set_comparer: impl must be 0 or 1");
+    g_impl = impl;
+    return COF_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,387 @@
+// Host side of the boundary: errors, version, launch counter, the 2-bit packer (M4), the
+// indexed FASTA reader (M2), chunk loading (M11), counters, collect (M10) and merge.
+//
+// Paper: P:L29 (host reads single/multi-sequence files, divides the genome into chunks,
+// collects "chromosome number, position, direction, the number of mismatched bases and
+// potential off-target DNA sequence with mismatched bases"); P:L289 ("2-bit sequence
+// format", OpenMP in the host program).
+#include <algorithm>
+#include <atomic>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <queue>
+#include <string>
+#include <vector>
+
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
+#include <cuda_runtime.h>
+#include <omp.h>
+
+#include "cof_internal.h"
+
+namespace cof {
+
+static thread_local std::string g_err;
+static std::atomic<uint64_t> g_launches{0};
+
+cof_status set_error(cof_status code, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+cof_status cuda_error(int err, const char* what) {
+    return set_error(COF_E_CUDA, "%s: %s", what, cudaGetErrorString((cudaError_t)err));
+}
+
+void count_launches(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+// byte -> 2-bit code (A0 C1 G2 T3) or 4 for anything else (N, IUPAC, junk): readings G2/G4
+static uint8_t g_code[256];
+static struct CodeInit {
+    CodeInit() {
+        for (int i = 0; i < 256; i++) g_code[i] = 4;
+        g_code['A'] = g_code['a'] = 0;
+        g_code['C'] = g_code['c'] = 1;
+        g_code['G'] = g_code['g'] = 2;
+        g_code['T'] = g_code['t'] = 3;
+    }
+} g_code_init;
+
+// Pack 32 codes into one word of each plane.
+static inline void pack_word(const uint8_t* codes, int n, uint32_t& lo, uint32_t& hi, uint32_t& nm) {
+    uint32_t l = 0, h = 0, m = 0;
+    for (int b = 0; b < n; b++) {
+        uint32_t c = codes[b];
+        l |= (uint32_t)(c & 1) << b;
+        h |= (uint32_t)((c >> 1) & 1) << b;
+        m |= (uint32_t)(c >> 2) << b;
+    }
+    l &= ~m; h &= ~m;                     // N: lo = hi = 0
+    if (n < 32) m |= ~0u << n;            // past the end: N
+    lo = l; hi = h; nm = m;
+}
+
+}  // namespace cof
+
+using namespace cof;
+
+extern "C" {
+
+const char* cof_last_error(void) { return g_err.c_str(); }
+const char* cof_version(void) { return "cof-b200 0.1 (sm_100a)"; }
+uint64_t cof_launch_count(void) { return g_launches.load(); }
+
+uint64_t cof_plane_words(uint64_t n_bases) {
+    // ceil(n/32) data words, rounded up to a finder tile (256 words), + 4 pad words so the
+    // finder's 16-byte-granular bulk copies of (tile + halo) never leave the allocation.
+    uint64_t w = (n_bases + 31) / 32;
+    return ((w + 255) / 256) * 256 + 4;
+}
+
+cof_status cof_pack(const char* ascii, uint64_t n, uint32_t* lo, uint32_t* hi, uint32_t* nm) {
+    if ((!ascii && n) || !lo || !hi || !nm) return set_error(COF_E_ARG, "cof_pack: NULL argument");
+    const uint64_t words = cof_plane_words(n);
+    const int64_t full = (int64_t)(n / 32);
+#pragma omp parallel for schedule(static)
+    for (int64_t w = 0; w < full; w++) {
+        uint8_t codes[32];
+        const uint8_t* src = (const uint8_t*)ascii + w * 32;
+        for (int b = 0; b < 32; b++) codes[b] = g_code[src[b]];
+        pack_word(codes, 32, lo[w], hi[w], nm[w]);
+    }
+    uint64_t w = (uint64_t)full;
+    if (n % 32) {
+        uint8_t codes[32];
+        int r = (int)(n % 32);
+        for (int b = 0; b < r; b++) codes[b] = g_code[(uint8_t)ascii[w * 32 + b]];
+        pack_word(codes, r, lo[w], hi[w], nm[w]);
+        w++;
+    }
+    for (; w < words; w++) { lo[w] = 0; hi[w] = 0; nm[w] = ~0u; }
+    return COF_OK;
+}
+
+cof_status cof_unpack(const uint32_t* lo, const uint32_t* hi, const uint32_t* nm, uint64_t first,
+                      uint64_t n, char* ascii) {
+    if (!lo || !hi || !nm || (!ascii && n)) return set_error(COF_E_ARG, "cof_unpack: NULL argument");
+    static const char B[4] = {'A', 'C', 'G', 'T'};
+#pragma omp parallel for schedule(static) if (n > (1u << 20))
+    for (int64_t i = 0; i < (int64_t)n; i++) {
+        uint64_t p = first + (uint64_t)i;
+        uint64_t w = p >> 5;
+        int b = (int)(p & 31);
+        if (nm[w] >> b & 1) ascii[i] = 'N';
+        else ascii[i] = B[((lo[w] >> b) & 1) | (((hi[w] >> b) & 1) << 1)];
+    }
+    return COF_OK;
+}
+
+cof_status cof_load_chunk(const cof_chunk* host, cof_chunk* dev, cof_stream s) {
+    if (!host || !dev || !host->lo || !host->hi || !host->nm || !dev->lo || !dev->hi || !dev->nm)
+        return set_error(COF_E_ARG, "cof_load_chunk: NULL argument");
+    size_t bytes = cof_plane_words(host->n_bases) * sizeof(uint32_t);
+    cudaStream_t st = (cudaStream_t)s;
+    cudaError_t e;
+    if ((e = cudaMemcpyAsync(dev->lo, host->lo, bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess ||
+        (e = cudaMemcpyAsync(dev->hi, host->hi, bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess ||
+        (e = cudaMemcpyAsync(dev->nm, host->nm, bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess)
+        return cuda_error(e, "cof_load_chunk");
+    dev->chrom = host->chrom;
+    dev->start = host->start;
+    dev->n_bases = host->n_bases;
+    dev->n_owned = host->n_owned;
+    return COF_OK;
+}
+
+cof_status cof_read_counts(const cof_plan* plan, const void* plan_dev, uint64_t out[3], cof_stream s) {
+    if (!plan || !plan_dev || !out) return set_error(COF_E_ARG, "cof_read_counts: NULL argument");
+    uint64_t tmp[3];
+    cudaStream_t st = (cudaStream_t)s;
+    cudaError_t e = cudaMemcpyAsync(tmp, (const uint8_t*)plan_dev + plan->lay.counters, sizeof tmp,
+                                    cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_error(e, "cof_read_counts");
+    out[0] = tmp[0]; out[1] = tmp[1]; out[2] = tmp[2];
+    return COF_OK;
+}
+
+// ------------------------------------------------------------------ FASTA (M2)
+struct cof_fasta {
+    int fd = -1;
+    const char* data = nullptr;
+    size_t size = 0;
+    struct Rec {
+        std::string name;
+        size_t seq_off;        // first sequence byte
+        size_t seq_end;        // one past the last sequence byte (before next '>')
+        uint64_t length;       // bases
+        uint64_t line_bases;   // bases per full line (0: single line)
+        uint64_t line_bytes;   // bytes per full line incl. newline(s)
+        bool regular;          // all lines except the last have line_bases bases
+    };
+    std::vector<Rec> recs;
+};
+
+cof_status cof_fasta_open(const char* path, cof_fasta** out) {
+    if (!path || !out) return set_error(COF_E_ARG, "cof_fasta_open: NULL argument");
+    *out = nullptr;
+    int fd = open(path, O_RDONLY);
+    if (fd < 0) return set_error(COF_E_IO, "cannot open %s", path);
+    struct stat st;
+    if (fstat(fd, &st) != 0) { close(fd); return set_error(COF_E_IO, "cannot stat %s", path); }
+    cof_fasta* fa = new cof_fasta();
+    fa->fd = fd;
+    fa->size = (size_t)st.st_size;
+    if (fa->size) {
+        void* m = mmap(nullptr, fa->size, PROT_READ, MAP_PRIVATE, fd, 0);
+        if (m == MAP_FAILED) { close(fd); delete fa; return set_error(COF_E_IO, "cannot mmap %s", path); }
+        fa->data = (const char*)m;
+    }
+    const char* d = fa->data;
+    size_t i = 0, n = fa->size;
+    while (i < n) {
+        if (d[i] != '>') {
+            if (d[i] == '\n' || d[i] == '\r') { i++; continue; }
+            cof_fasta_close(fa);
+            return set_error(COF_E_IO, "%s: expected '>' at byte %zu", path, i);
+        }
+        size_t e = i;
+        while (e < n && d[e] != '\n') e++;
+        cof_fasta::Rec r;
+        size_t name_end = i + 1;
+        while (name_end < e && d[name_end] != ' ' && d[name_end] != '\t' && d[name_end] != '\r') name_end++;
+        r.name.assign(d + i + 1, name_end - i - 1);
+        r.seq_off = e < n ? e + 1 : n;
+        size_t j = r.seq_off;
+        r.length = 0; r.line_bases = 0; r.line_bytes = 0; r.regular = true;
+        uint64_t last_line_bases = 0;
+        bool seen_short = false;
+        while (j < n && d[j] != '>') {
+            size_t le = j;
+            while (le < n && d[le] != '\n') le++;
+            size_t content_end = le;
+            if (content_end > j && d[content_end - 1] == '\r') content_end--;
+            uint64_t nb = content_end - j;
+            size_t lb = (le < n ? le + 1 : le) - j;
+            if (r.line_bases == 0 && nb > 0) { r.line_bases = nb; r.line_bytes = lb; }
+            else if (nb > 0) {
+                if (seen_short || nb > r.line_bases || (nb == r.line_bases && lb != r.line_bytes)) r.regular = false;
+                if (nb < r.line_bases) seen_short = true;
+            }
+            if (nb == 0 && le < n && d[le + 1 < n ? le + 1 : le] != '>') { /* blank line inside */ }
+            r.length += nb;
+            last_line_bases = nb;
+            j = le < n ? le + 1 : le;
+        }
+        (void)last_line_bases;
+        r.seq_end = j;
+        fa->recs.push_back(r);
+        i = j;
+    }
+    *out = fa;
+    return COF_OK;
+}
+
+void cof_fasta_close(cof_fasta* fa) {
+    if (!fa) return;
+    if (fa->data) munmap((void*)fa->data, fa->size);
+    if (fa->fd >= 0) close(fa->fd);
+    delete fa;
+}
+
+uint32_t cof_fasta_count(const cof_fasta* fa) { return fa ? (uint32_t)fa->recs.size() : 0; }
+const char* cof_fasta_name(const cof_fasta* fa, uint32_t i) {
+    return (fa && i < fa->recs.size()) ? fa->recs[i].name.c_str() : nullptr;
+}
+uint64_t cof_fasta_length(const cof_fasta* fa, uint32_t i) {
+    return (fa && i < fa->recs.size()) ? fa->recs[i].length : 0;
+}
+
+cof_status cof_fasta_pack(const cof_fasta* fa, uint32_t i, uint64_t first, uint64_t n, uint32_t* lo,
+                          uint32_t* hi, uint32_t* nm) {
+    if (!fa || !lo || !hi || !nm) return set_error(COF_E_ARG, "cof_fasta_pack: NULL argument");
+    if (i >= fa->recs.size()) return set_error(COF_E_ARG, "cof_fasta_pack: record %u out of range", i);
+    const auto& r = fa->recs[i];
+    if (first + n > r.length) return set_error(COF_E_ARG, "cof_fasta_pack: range past record end");
+    std::vector<char> buf(n);
+    if (r.regular && r.line_bases) {
+        // random access: base k is at seq_off + (k / line_bases) * line_bytes + k % line_bases
+        const int64_t nn = (int64_t)n;
+#pragma omp parallel for schedule(static) if (n > (1u << 20))
+        for (int64_t k0 = 0; k0 < nn; k0 += 4096) {
+            int64_t k1 = std::min(nn, k0 + 4096);
+            for (int64_t k = k0; k < k1; k++) {
+                uint64_t b = first + (uint64_t)k;
+                buf[k] = fa->data[r.seq_off + (b / r.line_bases) * r.line_bytes + b % r.line_bases];
+            }
+        }
+    } else {
+        uint64_t b = 0, o = 0;
+        for (size_t j = r.seq_off; j < r.seq_end && o < n; j++) {
+            char c = fa->data[j];
+            if (c == '\n' || c == '\r') continue;
+            if (b >= first) buf[o++] = c;
+            b++;
+        }
+    }
+    return cof_pack(buf.data(), n, lo, hi, nm);
+}
+
+// ------------------------------------------------------------------ collect (M10) / merge
+// Decodes one hit key (see cof.h) into a record, building the site string from the host
+// planes: '+' reads the window, '-' reads its reverse complement (G6); a compared letter
+// is lower-cased where the genome base is not in the guide letter's IUPAC set (G19).
+static cof_status decorate(const cof_plan* plan, const cof_chunk* host, uint64_t key, cof_hit* h) {
+    static const char B[4] = {'A', 'C', 'G', 'T'};
+    static const char C[5] = {'T', 'G', 'C', 'A', 'N'};
+    const uint32_t L = plan->L;
+    uint64_t pos = key >> 32;
+    uint32_t strand = (uint32_t)(key >> 31) & 1u;
+    uint32_t guide = (uint32_t)(key >> 7) & 0xFFFFFFu;
+    uint32_t mm = (uint32_t)key & 127u;
+    if (guide >= plan->n_guides || pos + L > host->n_bases) return COF_E_STATE;
+    int code[32];
+    for (uint32_t j = 0; j < L; j++) {
+        uint64_t p = pos + j;
+        uint64_t w = p >> 5;
+        int b = (int)(p & 31);
+        code[j] = (host->nm[w] >> b & 1) ? 4 : (int)(((host->lo[w] >> b) & 1) | (((host->hi[w] >> b) & 1) << 1));
+    }
+    const uint8_t* gm = &plan->gmask[(size_t)guide * L];
+    uint32_t recount = 0;
+    for (uint32_t j = 0; j < L; j++) {
+        int c = strand == 0 ? code[j] : (code[L - 1 - j] == 4 ? 4 : 3 - code[L - 1 - j]);
+        char ch = c == 4 ? 'N' : B[c];
+        (void)C;
+        bool mis = gm[j] != 15 && (c == 4 || !((gm[j] >> c) & 1));
+        if (mis) { recount++; ch = (char)(ch + 32); }
+        h->site[j] = ch;
+    }
+    h->site[L] = 0;
+    for (uint32_t j = L + 1; j < sizeof h->site; j++) h->site[j] = 0;
+    if (recount != mm) return COF_E_STATE;
+    h->guide = guide;
+    h->chrom = host->chrom;
+    h->pos = host->start + pos;
+    h->strand = strand ? '-' : '+';
+    h->mm = (uint8_t)mm;
+    return COF_OK;
+}
+
+static inline uint64_t sort_key(uint64_t k) { return k >> 7; }   // (pos, strand, guide)
+
+cof_status cof_collect(const cof_plan* plan, const cof_chunk* host, const uint64_t* hits_dev,
+                       const uint64_t* host_keys, uint64_t n_hits, cof_hit* out, cof_stream s) {
+    if (!plan || !host || (!out && n_hits) || (!hits_dev && !host_keys && n_hits))
+        return set_error(COF_E_ARG, "cof_collect: NULL argument");
+    if (!host->lo || !host->hi || !host->nm) return set_error(COF_E_ARG, "cof_collect: host planes are NULL");
+    if (n_hits == 0) return COF_OK;
+    std::vector<uint64_t> keys(n_hits);
+    if (hits_dev) {
+        cudaStream_t st = (cudaStream_t)s;
+        cudaError_t e = cudaMemcpyAsync(keys.data(), hits_dev, n_hits * 8, cudaMemcpyDeviceToHost, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        if (e != cudaSuccess) return cuda_error(e, "cof_collect");
+    } else {
+        memcpy(keys.data(), host_keys, n_hits * 8);
+    }
+    bool sorted = true;
+    for (uint64_t i = 1; i < n_hits && sorted; i++) sorted = sort_key(keys[i - 1]) < sort_key(keys[i]);
+    if (!sorted) std::sort(keys.begin(), keys.end(), [](uint64_t a, uint64_t b) { return sort_key(a) < sort_key(b); });
+    int bad = 0;
+#pragma omp parallel for schedule(static) reduction(| : bad) if (n_hits > 4096)
+    for (int64_t i = 0; i < (int64_t)n_hits; i++)
+        if (decorate(plan, host, keys[i], &out[i]) != COF_OK) bad = 1;
+    if (bad) return set_error(COF_E_STATE, "cof_collect: a hit key does not match the plan/chunk (mismatch recount differs)");
+    return COF_OK;
+}
+
+static inline bool hit_less(const cof_hit& a, const cof_hit& b) {
+    if (a.chrom != b.chrom) return a.chrom < b.chrom;
+    if (a.pos != b.pos) return a.pos < b.pos;
+    if (a.strand != b.strand) return a.strand == '+';
+    return a.guide < b.guide;
+}
+
+cof_status cof_merge(const cof_hit* const* lists, const uint64_t* lens, uint32_t n_lists, cof_hit* out) {
+    if ((!lists || !lens) && n_lists) return set_error(COF_E_ARG, "cof_merge: NULL argument");
+    uint64_t total = 0;
+    for (uint32_t i = 0; i < n_lists; i++) {
+        if (lens[i] && !lists[i]) return set_error(COF_E_ARG, "cof_merge: list %u is NULL", i);
+        for (uint64_t k = 1; k < lens[i]; k++)
+            if (hit_less(lists[i][k], lists[i][k - 1])) return set_error(COF_E_ARG, "cof_merge: list %u is not sorted", i);
+        total += lens[i];
+    }
+    if (total && !out) return set_error(COF_E_ARG, "cof_merge: out is NULL");
+    // k-way merge with a min-heap of list heads (stable across lists for equal keys)
+    typedef std::pair<uint32_t, uint64_t> Head;   // (list, index)
+    auto cmp = [&](const Head& x, const Head& y) {
+        const cof_hit& a = lists[x.first][x.second];
+        const cof_hit& b = lists[y.first][y.second];
+        if (hit_less(a, b)) return false;
+        if (hit_less(b, a)) return true;
+        return x.first > y.first;
+    };
+    std::priority_queue<Head, std::vector<Head>, decltype(cmp)> heap(cmp);
+    for (uint32_t i = 0; i < n_lists; i++) if (lens[i]) heap.push({i, 0});
+    uint64_t o = 0;
+    while (!heap.empty()) {
+        Head h = heap.top();
+        heap.pop();
+        out[o++] = lists[h.first][h.second];
+        if (h.second + 1 < lens[h.first]) heap.push({h.first, h.second + 1});
+    }
+    return COF_OK;
+}
+
+}  // extern "C"

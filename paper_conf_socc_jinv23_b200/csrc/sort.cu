@@ -1,0 +1,216 @@
+// Deterministic ordering of hit keys (K3, M10) for sm_100a: stable LSD radix sort.
+//
+// Paper: hit slots come from an atomic counter and "the order of updates is not
+// deterministic" (Listing 1).  Reading G13 fixes the output order
+// to (chromosome, position, '+' before '-', guide).  Within a chunk the key
+//   key = pos << 32 | strand << 31 | guide << 7 | mm
+// orders exactly that way; only the bits that can vary are sorted: the compressed key
+//   k' = pos << (GB + 1) | strand << GB | guide      (GB = bits of the largest guide index)
+// is cut into 8-bit digits, one pass per digit.  Each pass: per-tile digit histograms
+// (shared-memory atomics), one exclusive scan over the digit-major histogram matrix, and a
+// stable scatter that ranks keys inside a tile with __match_any_sync in index order.
+#include <cuda_runtime.h>
+
+#include "cof_internal.h"
+#include "dev_common.cuh"
+
+namespace cof {
+
+constexpr int ST = 256;             // threads per CTA
+constexpr int SV = 16;              // keys per thread per tile
+constexpr int STILE = ST * SV;      // 4096 keys per tile
+constexpr int SCAN_T = 1024;
+
+struct SortPass {
+    const unsigned long long* src;
+    unsigned long long* dst;
+    uint32_t* hist;                 // [256][cap_tiles]
+    const unsigned long long* count;  // device count (n_hits) or nullptr
+    uint64_t n_host;                // used when count == nullptr
+    uint64_t cap;
+    uint32_t cap_tiles;
+    uint32_t shift;                 // digit position in k'
+    uint32_t gb;                    // guide bits
+};
+
+__device__ __forceinline__ uint64_t sort_n(const SortPass& p) {
+    uint64_t n = p.count ? (uint64_t)*p.count : p.n_host;
+    return n < p.cap ? n : p.cap;
+}
+
+__device__ __forceinline__ uint32_t digit_of(unsigned long long key, uint32_t gb, uint32_t shift) {
+    const uint64_t pos = key >> 32;
+    const uint64_t strand = (key >> 31) & 1ull;
+    const uint64_t guide = (key >> 7) & ((1ull << gb) - 1ull);
+    const uint64_t kc = (pos << (gb + 1)) | (strand << gb) | guide;
+    return (uint32_t)(kc >> shift) & 255u;
+}
+
+__global__ void __launch_bounds__(ST) cof_sort_hist(const __grid_constant__ SortPass p) {
+    __shared__ uint32_t h[256];
+    h[threadIdx.x] = 0;
+    __syncthreads();
+    const uint64_t n = sort_n(p);
+    const uint64_t base = (uint64_t)blockIdx.x * STILE;
+    if (base < n) {
+#pragma unroll 4
+        for (int v = 0; v < SV; v++) {
+            const uint64_t i = base + (uint64_t)v * ST + threadIdx.x;
+            if (i < n) atomicAdd(&h[digit_of(p.src[i], p.gb, p.shift)], 1u);
+        }
+    }
+    __syncthreads();
+    p.hist[(size_t)threadIdx.x * p.cap_tiles + blockIdx.x] = h[threadIdx.x];
+}
+
+// Exclusive scan of the whole [256][cap_tiles] matrix (digit-major) by one CTA.
+__global__ void __launch_bounds__(SCAN_T) cof_sort_scan(uint32_t* hist, uint64_t m) {
+    __shared__ uint32_t s_warp[SCAN_T / 32];
+    __shared__ uint32_t s_carry;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) s_carry = 0;
+    __syncthreads();
+    for (uint64_t c0 = 0; c0 < m; c0 += (uint64_t)SCAN_T * 4) {
+        uint32_t v[4], sum = 0;
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint64_t i = c0 + (uint64_t)tid * 4 + k;
+            v[k] = i < m ? hist[i] : 0u;
+            sum += v[k];
+        }
+        uint32_t x = sum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= o) x += y;
+        }
+        if (lane == 31) s_warp[warp] = x;
+        __syncthreads();
+        if (warp == 0) {
+            const uint32_t wv = s_warp[lane];
+            uint32_t wi = wv;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
+                if (lane >= o) wi += y;
+            }
+            s_warp[lane] = wi - wv;
+        }
+        __syncthreads();
+        uint32_t run = s_carry + s_warp[warp] + x - sum;
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint64_t i = c0 + (uint64_t)tid * 4 + k;
+            if (i < m) hist[i] = run;
+            run += v[k];
+        }
+        __syncthreads();
+        if (tid == SCAN_T - 1) s_carry = run;
+        __syncthreads();
+    }
+}
+
+__global__ void __launch_bounds__(ST) cof_sort_scatter(const __grid_constant__ SortPass p) {
+    __shared__ uint32_t s_off[256];          // global offset of this tile's digit d
+    __shared__ uint32_t s_run[256];          // keys of digit d already placed from earlier rounds
+    __shared__ uint32_t s_wc[ST / 32][256];  // per-warp counts -> exclusive warp offsets
+    const int tid = threadIdx.x, warp = tid >> 5;
+    const uint64_t n = sort_n(p);
+    const uint64_t base = (uint64_t)blockIdx.x * STILE;
+    if (base >= n) return;
+    s_off[tid] = p.hist[(size_t)tid * p.cap_tiles + blockIdx.x];
+    s_run[tid] = 0;
+    for (int w = 0; w < ST / 32; w++) s_wc[w][tid] = 0;
+    __syncthreads();
+    for (int v = 0; v < SV; v++) {
+        const uint64_t i = base + (uint64_t)v * ST + tid;
+        const bool ok = i < n;
+        unsigned long long key = ok ? p.src[i] : 0ull;
+        const uint32_t d = ok ? digit_of(key, p.gb, p.shift) : 256u;   // 256: not a key
+        const unsigned peers = __match_any_sync(0xffffffffu, d);
+        const uint32_t rank = (uint32_t)__popc(peers & lanemask_lt());
+        if (ok && rank == 0) s_wc[warp][d] = (uint32_t)__popc(peers);
+        __syncthreads();
+        {   // digit tid: exclusive prefix over warps, continuing the running count
+            uint32_t run = s_run[tid];
+#pragma unroll
+            for (int w = 0; w < ST / 32; w++) {
+                const uint32_t c = s_wc[w][tid];
+                s_wc[w][tid] = run;
+                run += c;
+            }
+            s_run[tid] = run;
+        }
+        __syncthreads();
+        if (ok) p.dst[s_off[d] + s_wc[warp][d] + rank] = key;
+        __syncthreads();
+        for (int w = 0; w < ST / 32; w++) s_wc[w][tid] = 0;
+        __syncthreads();
+    }
+}
+
+__global__ void cof_sort_copy(const __grid_constant__ SortPass p) {
+    const uint64_t n = sort_n(p);
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        p.dst[i] = p.src[i];
+}
+
+static uint32_t bits_for(uint64_t x) {   // number of bits to represent values 0..x
+    uint32_t b = 0;
+    while (b < 64 && (x >> b)) b++;
+    return b;
+}
+
+}  // namespace cof
+
+using namespace cof;
+
+extern "C" {
+
+size_t cof_sort_workspace_bytes(uint64_t cap) {
+    uint64_t tiles = (cap + STILE - 1) / STILE;
+    if (!tiles) tiles = 1;
+    return (size_t)(256 * tiles * sizeof(uint32_t) + 256);
+}
+
+cof_status cof_sort_hits(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, uint64_t* hits, uint64_t* tmp,
+                         uint64_t cap, uint64_t n_hits, void* workspace, cof_stream s) {
+    if (!plan || !plan_dev || !dev || ((!hits || !tmp || !workspace) && cap))
+        return set_error(COF_E_ARG, "cof_sort_hits: NULL argument");
+    if (cap == 0) return COF_OK;
+    cudaStream_t stream = (cudaStream_t)s;
+    SortPass p;
+    p.hist = (uint32_t*)workspace;
+    p.count = n_hits == COF_COUNT_ON_DEVICE
+                  ? (const unsigned long long*)((uint8_t*)plan_dev + plan->lay.counters + 2 * sizeof(uint64_t))
+                  : nullptr;
+    p.n_host = n_hits == COF_COUNT_ON_DEVICE ? 0 : n_hits;
+    if (!p.count && p.n_host <= 1) return COF_OK;
+    p.cap = cap;
+    uint64_t eff = p.count ? cap : (p.n_host < cap ? p.n_host : cap);
+    p.cap_tiles = (uint32_t)((eff + STILE - 1) / STILE);
+    p.gb = bits_for(plan->n_guides - 1);
+    const uint32_t pb = bits_for(dev->n_owned ? dev->n_owned - 1 : 0);
+    const uint32_t total_bits = pb + 1 + p.gb;
+    const uint32_t passes = (total_bits + 7) / 8;
+    unsigned long long* a = (unsigned long long*)hits;
+    unsigned long long* b = (unsigned long long*)tmp;
+    for (uint32_t k = 0; k < passes; k++) {
+        p.src = a; p.dst = b; p.shift = 8 * k;
+        cof_sort_hist<<<p.cap_tiles, ST, 0, stream>>>(p);
+        cof_sort_scan<<<1, SCAN_T, 0, stream>>>(p.hist, (uint64_t)256 * p.cap_tiles);
+        cof_sort_scatter<<<p.cap_tiles, ST, 0, stream>>>(p);
+        count_launches(3);
+        unsigned long long* t = a; a = b; b = t;
+    }
+    if (a != (unsigned long long*)hits) {
+        p.src = a; p.dst = (unsigned long long*)hits;
+        cof_sort_copy<<<1184, 256, 0, stream>>>(p);
+        count_launches(1);
+    }
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "cof_sort_hits launch");
+    return COF_OK;
+}
+
+}  // extern "C"

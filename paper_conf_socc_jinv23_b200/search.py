@@ -1,0 +1,167 @@
+"""Driver of the hot path: chunk planning (M3), the per-chunk device pipeline
+(load -> find -> compare -> sort -> collect, M5-M11), multi-GPU sharding (M19) and the
+final merge.  Every step of the path runs in libcof.so; this module only allocates
+memory (torch), orders the calls on a stream and moves counts.
+
+Paper: P:L29 -- the host "divides the genome data into chunks that can fit the memory of
+a heterogeneous device", runs the search kernel, hands the PAM sites to the compare
+kernel, and "the interaction ... continues until all chunks are processed".
+"""
+from __future__ import annotations
+
+import dataclasses
+import heapq
+
+import numpy as np
+import torch
+
+from . import cof
+
+
+@dataclasses.dataclass(frozen=True)
+class Chunk:
+    chrom: int
+    start: int      # 0-based chromosome offset of base 0 of the chunk
+    n_owned: int    # window starts [start, start + n_owned) belong to this chunk
+    n_bases: int    # bases held: n_owned + L - 1 (chunks overlap by L-1, reading G12)
+
+
+def plan_chunks(lengths, L: int, chunk_bases: int | None = None):
+    """Split chromosomes into chunks; every valid window start (0 <= p <= len-L) belongs
+    to exactly one chunk and each chunk holds the L-1 bases its last window needs."""
+    out = []
+    for c, n in enumerate(lengths):
+        n_starts = int(n) - L + 1
+        if n_starts <= 0:
+            continue
+        step = int(chunk_bases) if chunk_bases else n_starts
+        for s in range(0, n_starts, step):
+            owned = min(step, n_starts - s)
+            out.append(Chunk(c, s, owned, owned + L - 1))
+    return out
+
+
+def shard_lpt(chunks, world: int):
+    """Longest-processing-time-first assignment of chunks to ``world`` ranks (cost =
+    owned window starts).  Returns one chunk list per rank, each in genome order."""
+    loads = [(0, r) for r in range(world)]
+    heapq.heapify(loads)
+    out = [[] for _ in range(world)]
+    for i in sorted(range(len(chunks)), key=lambda i: (-chunks[i].n_owned, i)):
+        load, r = heapq.heappop(loads)
+        out[r].append(i)
+        heapq.heappush(loads, (load + chunks[i].n_owned, r))
+    return [[chunks[i] for i in sorted(lst)] for lst in out]
+
+
+def merge_hit_lists(lists):
+    """Order (chrom, pos, strand, guide) across chunk / rank lists (cof_merge)."""
+    lists = [x for x in lists if len(x)]
+    if not lists:
+        return np.zeros(0, dtype=cof.HIT_DTYPE)
+    return cof.cof_merge(lists)
+
+
+class HostGenome:
+    """Packed bit-planes of every chunk in pinned host memory (a1: chunk & pack)."""
+
+    def __init__(self, seqs, chunks, pin: bool = True):
+        self.chunks = chunks
+        self.planes = []
+        for ch in chunks:
+            words = cof.cof_plane_words(ch.n_bases)
+            buf = torch.empty((3, words), dtype=torch.int32, pin_memory=pin and torch.cuda.is_available())
+            seq = seqs[ch.chrom]
+            view = seq[ch.start: ch.start + ch.n_bases]
+            view = np.ascontiguousarray(view)
+            cof.cof_pack(view, ch.n_bases, buf[0], buf[1], buf[2])
+            self.planes.append(buf)
+
+    def chunk_struct(self, i) -> cof.cof_chunk:
+        ch, buf = self.chunks[i], self.planes[i]
+        return cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, buf[0], buf[1], buf[2])
+
+    @property
+    def bytes(self):
+        return sum(p.numel() * 4 for p in self.planes)
+
+
+class Searcher:
+    """One GPU's pipeline for a fixed (pattern, guides, thresholds) plan."""
+
+    def __init__(self, pattern, guides, thresholds, device="cuda", stream=None):
+        self.device = torch.device(device)
+        self.plan = cof.cof_plan_create(pattern, guides, thresholds)
+        self.L = self.plan.L
+        self.stream = stream or torch.cuda.current_stream(self.device)
+        nbytes = cof.cof_plan_device_bytes(self.plan)
+        self.plan_dev = torch.empty(nbytes + 256, dtype=torch.uint8, device=self.device)
+        cof.cof_plan_upload(self.plan, self.plan_dev, self.stream)
+        self._cap_bases = 0
+        self._hits_cap = 0
+
+    # ---- device buffers sized for the largest chunk seen so far
+    def reserve(self, max_bases: int, hits_cap: int):
+        if max_bases > self._cap_bases:
+            words = cof.cof_plane_words(max_bases)
+            self.d_planes = torch.empty((3, words), dtype=torch.int32, device=self.device)
+            self.d_items = torch.empty((2, max(max_bases, 1)), dtype=torch.int32, device=self.device)
+            self.d_find_ws = torch.empty(cof.cof_find_workspace_bytes(max_bases), dtype=torch.uint8,
+                                         device=self.device)
+            self._cap_bases = max_bases
+        if hits_cap > self._hits_cap:
+            self.d_hits = torch.empty(hits_cap, dtype=torch.int64, device=self.device)
+            self.d_tmp = torch.empty(hits_cap, dtype=torch.int64, device=self.device)
+            self.d_sort_ws = torch.empty(cof.cof_sort_workspace_bytes(hits_cap), dtype=torch.uint8,
+                                         device=self.device)
+            self._hits_cap = hits_cap
+
+    def device_chunk(self, ch: Chunk, planes=None) -> cof.cof_chunk:
+        p = self.d_planes if planes is None else planes
+        return cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, p[0], p[1], p[2])
+
+    def run_device_chunk(self, dchunk: cof.cof_chunk, items_cap: int):
+        """find -> compare -> sort on the device; returns (n_fwd, n_rev, n_hits).
+        Grows the hit buffer and re-runs compare on capacity overflow."""
+        s = self.stream
+        nf, nr = cof.cof_find_pam(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_items[0],
+                                  self.d_items[1], items_cap, s)
+        while True:
+            try:
+                nh = cof.cof_compare(self.plan, self.plan_dev, dchunk, self.d_items[0], nf, self.d_items[1], nr,
+                                     self.d_hits, self._hits_cap, s)
+                break
+            except cof.CofError as e:
+                if e.status != cof.COF_E_CAPACITY:
+                    raise
+                _, _, need = cof.cof_read_counts(self.plan, self.plan_dev, s)
+                self.reserve(self._cap_bases, int(need * 1.25) + 1024)
+        cof.cof_sort_hits(self.plan, self.plan_dev, dchunk, self.d_hits, self.d_tmp, self._hits_cap, nh,
+                          self.d_sort_ws, s)
+        return nf, nr, nh
+
+    def search_host(self, host: HostGenome, indices=None):
+        """End-to-end over host-resident packed chunks: H2D, find, compare, sort, D2H +
+        decorate (cof_collect); returns the merged, sorted hit array."""
+        idx = range(len(host.chunks)) if indices is None else indices
+        max_bases = max((host.chunks[i].n_bases for i in idx), default=1)
+        self.reserve(max_bases, max(self._hits_cap, 1 << 16))
+        out = []
+        with torch.cuda.device(self.device):
+            for i in idx:
+                hch = host.chunk_struct(i)
+                dch = self.device_chunk(host.chunks[i])
+                cof.cof_load_chunk(hch, dch, self.stream)
+                _, _, nh = self.run_device_chunk(dch, host.chunks[i].n_owned)
+                out.append(cof.cof_collect(self.plan, hch, self.d_hits, nh, self.stream))
+        return merge_hit_lists(out)
+
+
+def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda"):
+    """Convenience: whole search of ``seqs`` (list of uint8 ASCII arrays / bytes) on one GPU."""
+    L = len(pattern)
+    arrs = [np.frombuffer(s, dtype=np.uint8) if isinstance(s, (bytes, bytearray)) else
+            (np.frombuffer(s.encode(), dtype=np.uint8) if isinstance(s, str) else s) for s in seqs]
+    chunks = plan_chunks([len(a) for a in arrs], L, chunk_bases)
+    host = HostGenome(arrs, chunks)
+    return Searcher(pattern, guides, thresholds, device).search_host(host)

@@ -1,0 +1,204 @@
+"""CPU tests of the C ABI library: it loads, exports every declared symbol, and its host
+logic (pack/unpack, plan validation, FASTA, collect/decorate, merge) is right.  No CUDA
+compute call is made here."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+from oracle import oracle
+from paper_conf_socc_jinv23_b200 import cof, search, synth
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_symbols():
+    text = open(os.path.join(ROOT, "include", "cof.h")).read()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+    return sorted(set(re.findall(r"\b(cof_[a-z_0-9]+)\s*\(", text)))
+
+
+def test_library_exports_every_declared_symbol():
+    names = declared_symbols()
+    assert len(names) >= 25
+    lib = ctypes.CDLL(cof.LIB_PATH)
+    for n in names:
+        assert hasattr(lib, n), n
+    assert set(cof.EXPORTS) <= set(names)
+
+
+def test_version_and_counter():
+    assert "sm_100a" in cof.cof_version()
+    assert cof.cof_launch_count() >= 0
+
+
+def test_plane_words():
+    for n in (0, 1, 31, 32, 33, 8191, 8192, 8193, 10**6):
+        w = cof.cof_plane_words(n)
+        assert w >= (n + 31) // 32 + 1 and (w - 4) % 256 == 0
+
+
+def _canon(b: bytes) -> bytes:
+    return bytes(c if c in b"ACGT" else ord("N") for c in b.upper())
+
+
+@pytest.mark.parametrize("n", [0, 1, 31, 32, 33, 1000, 70001])
+def test_pack_roundtrip(n):
+    rng = np.random.default_rng(n)
+    seq = synth.random_genome_text(rng, n, b"ACGTacgtNnRYmk.-") if n else np.zeros(0, np.uint8)
+    w = cof.cof_plane_words(n)
+    lo, hi, nm = (np.zeros(w, np.uint32) for _ in range(3))
+    cof.cof_pack(seq, n, lo, hi, nm)
+    out = np.zeros(n, np.uint8)
+    cof.cof_unpack(lo, hi, nm, 0, n, out)
+    assert out.tobytes() == _canon(seq.tobytes())
+    # padding: past the last base every position is N (lo = hi = 0)
+    last = n // 32
+    if n % 32:
+        assert nm[last] >> (n % 32) == (0xFFFFFFFF >> (n % 32))
+        last += 1
+    assert (nm[last:] == 0xFFFFFFFF).all() and (lo[last:] == 0).all() and (hi[last:] == 0).all()
+    assert not (lo & nm).any() and not (hi & nm).any()
+
+
+def test_plan_validation():
+    good = "N" * 21 + "RG"
+    p = cof.cof_plan_create(good, ["ACGT" * 5 + "NNN"], [3])
+    assert p.L == 23 and p.n_guides == 1
+    assert cof.cof_plan_device_bytes(p) > 0
+    bad = [
+        (good, ["ACGT" * 5 + "NN"], [3]),          # length mismatch (G11)
+        ("N" * 21 + "RU", ["A" * 23], [3]),        # non-IUPAC pattern letter (G18)
+        (good, ["ACGT" * 5 + "NNX"], [3]),         # non-IUPAC guide letter
+        ("N" * 33, ["N" * 33], [1]),               # L > 32
+        ("", [""], [0]),                           # L = 0
+        (good, [], []),                            # no guides
+    ]
+    for pat, g, t in bad:
+        with pytest.raises(cof.CofError) as ei:
+            cof.cof_plan_create(pat, g, t)
+        assert ei.value.status == cof.COF_E_ARG
+    # lower case accepted (G4 / G18)
+    assert cof.cof_plan_create(good.lower(), [("acgt" * 5) + "nnn"], [2]).L == 23
+
+
+def _keys_from_oracle(hits):
+    return np.array([(int(h["pos"]) << 32) | ((1 if h["strand"] == b"-" else 0) << 31) |
+                     (int(h["guide"]) << 7) | int(h["mm"]) for h in hits], dtype=np.uint64)
+
+
+def test_collect_decorates_like_the_oracle():
+    """cof_collect (host decoration: site string, lower-case mismatches, '-' as reverse
+    complement, chrom/abs position) against the oracle's records, from host keys."""
+    rng = np.random.default_rng(3)
+    seq = synth.random_genome_text(rng, 20000, b"ACGTacgtN", p=[.22, .22, .22, .22, .02, .02, .02, .02, .04])
+    pat = "N" * 21 + "RG"
+    guides = ["".join(rng.choice(list("ACGT"), 20)) + "NNN" for _ in range(3)] + ["RYNNKMSWACGTACGTACGTNNN"]
+    thr = [12, 12, 12, 14]
+    ref = oracle.search([seq], pat, guides, thr)
+    assert len(ref) > 20
+    plan = cof.cof_plan_create(pat, guides, thr)
+    start = 0
+    w = cof.cof_plane_words(len(seq))
+    planes = np.zeros((3, w), np.uint32)
+    cof.cof_pack(seq, len(seq), planes[0], planes[1], planes[2])
+    host = cof.make_chunk(0, start, len(seq), len(seq) - 22, planes[0], planes[1], planes[2])
+    keys = _keys_from_oracle(ref)
+    shuffled = keys[rng.permutation(len(keys))]
+    got = cof.cof_collect(plan, host, None, len(keys), host_keys=shuffled)
+    assert cof.hits_to_tuples(got) == oracle.hits_to_tuples(ref)
+    # a key whose mismatch count disagrees with the genome is rejected
+    badk = keys.copy()
+    badk[0] ^= 1
+    with pytest.raises(cof.CofError) as ei:
+        cof.cof_collect(plan, host, None, len(badk), host_keys=badk)
+    assert ei.value.status == cof.COF_E_STATE
+
+
+def test_merge_orders_lists():
+    rng = np.random.default_rng(4)
+    lists = []
+    for _ in range(5):
+        n = int(rng.integers(0, 50))
+        a = np.zeros(n, dtype=cof.HIT_DTYPE)
+        a["chrom"] = rng.integers(0, 3, n)
+        a["pos"] = rng.integers(0, 100, n)
+        a["strand"] = rng.choice([b"+", b"-"], n)
+        a["guide"] = rng.integers(0, 4, n)
+        a = a[np.lexsort((a["guide"], a["strand"] == b"-", a["pos"], a["chrom"]))]
+        lists.append(a)
+    m = cof.cof_merge(lists)
+    cat = np.concatenate(lists)
+    exp = cat[np.lexsort((cat["guide"], cat["strand"] == b"-", cat["pos"], cat["chrom"]))]
+    key = lambda x: list(zip(x["chrom"], x["pos"], x["strand"], x["guide"]))
+    assert key(m) == key(exp)
+    with pytest.raises(cof.CofError):
+        cof.cof_merge([lists[0][::-1]] if len(lists[0]) > 1 and (lists[0][0] != lists[0][-1]) else [np.array(
+            [(0, 0, 5, b"+", 0, b""), (0, 0, 1, b"+", 0, b"")], dtype=cof.HIT_DTYPE)])
+
+
+def test_fasta_reader(tmp_path):
+    rng = np.random.default_rng(5)
+    seqs = [synth.random_genome_text(rng, n, b"ACGTacgtN") for n in (0, 5, 61, 1000, 4097)]
+    names = [f"chr{i}" for i in range(len(seqs))]
+    for width in (60, 7):
+        path = tmp_path / f"g{width}.fa"
+        synth.write_fasta(path, names, seqs, width)
+        fa = cof.Fasta(path)
+        assert len(fa) == len(seqs)
+        for i, s in enumerate(seqs):
+            assert fa.name(i) == names[i] and fa.length(i) == len(s)
+            for first, n in ((0, len(s)), (min(3, len(s)), max(0, len(s) - 6))):
+                w = cof.cof_plane_words(n)
+                a = np.zeros((3, w), np.uint32)
+                b = np.zeros((3, w), np.uint32)
+                fa.pack(i, first, n, a[0], a[1], a[2])
+                cof.cof_pack(np.ascontiguousarray(s[first:first + n]), n, b[0], b[1], b[2])
+                assert (a == b).all()
+        fa.close()
+    # irregular line lengths fall back to a streaming read
+    path = tmp_path / "irr.fa"
+    path.write_bytes(b">x desc\nACG\nTTTTT\nA\n>y\nNNNNacgt\n")
+    fa = cof.Fasta(path)
+    assert [fa.name(0), fa.name(1)] == ["x", "y"] and [fa.length(0), fa.length(1)] == [9, 8]
+    w = cof.cof_plane_words(9)
+    a = np.zeros((3, w), np.uint32)
+    fa.pack(0, 0, 9, a[0], a[1], a[2])
+    out = np.zeros(9, np.uint8)
+    cof.cof_unpack(a[0], a[1], a[2], 0, 9, out)
+    assert out.tobytes() == b"ACGTTTTTA"
+    with pytest.raises(cof.CofError):
+        cof.Fasta(tmp_path / "missing.fa")
+
+
+def test_plan_chunks_cover_every_window_once():
+    L = 23
+    lengths = [0, 10, 23, 24, 100_000, 77_777]
+    for cb in (None, 1, 1000, 7919, 10**6):
+        chunks = search.plan_chunks(lengths, L, cb)
+        for c, n in enumerate(lengths):
+            starts = []
+            for ch in chunks:
+                if ch.chrom != c:
+                    continue
+                assert ch.n_bases == ch.n_owned + L - 1
+                assert ch.start + ch.n_bases <= n
+                starts.append((ch.start, ch.start + ch.n_owned))
+            starts.sort()
+            covered = sum(e - s for s, e in starts)
+            assert covered == max(0, n - L + 1)
+            for (s0, e0), (s1, e1) in zip(starts, starts[1:]):
+                assert e0 == s1
+
+
+def test_shard_lpt_assigns_each_chunk_once():
+    chunks = search.plan_chunks([l for _, l in synth.HG38], 23, None)
+    for world in (1, 2, 4, 8):
+        shards = search.shard_lpt(chunks, world)
+        flat = sorted([c for s in shards for c in s], key=lambda c: (c.chrom, c.start))
+        assert flat == sorted(chunks, key=lambda c: (c.chrom, c.start))
+        loads = [sum(c.n_owned for c in s) for s in shards]
+        ideal = sum(loads) / world
+        assert max(loads) <= max(ideal * 1.05, max(c.n_owned for c in chunks) + 1)

@@ -1,0 +1,180 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Bar: bit-exact -- every hit record (chrom, pos, strand, guide, mm, site)
+and every finder candidate list must equal the oracle's.  Sizes span many finder tiles
+(8192 starts) and comparer tiles plus ragged tails; full-size configs are checked on
+sampled window ranges that the oracle recomputes one by one.
+"""
+import numpy as np
+import pytest
+import torch
+
+from oracle import oracle
+from paper_conf_socc_jinv23_b200 import cof, search, synth
+from tests import golden_io
+
+pytestmark = pytest.mark.gpu
+IMPLS = ["table", "popc"]
+
+
+@pytest.fixture(autouse=True)
+def _impl_reset():
+    yield
+    cof.cof_set_comparer("table")
+
+
+def gpu_hits(seqs, pattern, guides, thr, chunk_bases=None, impl="table"):
+    cof.cof_set_comparer(impl)
+    return cof.hits_to_tuples(search.search(seqs, pattern, guides, thr, chunk_bases=chunk_bases))
+
+
+def ref_hits(seqs, pattern, guides, thr, ranges=None):
+    return oracle.hits_to_tuples(oracle.search(seqs, pattern, guides, thr, ranges=ranges))
+
+
+@pytest.mark.parametrize("impl", IMPLS)
+def test_worked_example(impl):
+    d = golden_io.worked_example()
+    got = gpu_hits([c.encode() for c in d["chroms"]], d["pattern"], d["guides"], d["thr"], impl=impl)
+    assert got == d["hits"]
+
+
+@pytest.mark.parametrize("impl", IMPLS)
+@pytest.mark.parametrize("seed", range(8))
+def test_random_small(impl, seed):
+    """Random IUPAC patterns (incl. all-N and degenerate letters), guides with degenerate
+    letters and Ns, genomes with N / lowercase / rare IUPAC letters, lengths around tiles."""
+    rng = np.random.default_rng(500 + seed)
+    L = int(rng.integers(1, 33))
+    pat = "".join(rng.choice(list("NNNNNNNNACGTRYSWKMBDHV"), L))
+    guides = ["".join(rng.choice(list("ACGTACGTACGTNNRYKMSWBDHV"), L)) for _ in range(int(rng.integers(1, 70)))]
+    thr = [int(rng.integers(0, L + 1)) for _ in guides]
+    lens = [int(rng.integers(0, 3)) if i == 0 else int(rng.integers(L, 40_000)) for i in range(4)]
+    seqs = [synth.random_genome_text(rng, n, b"ACGTacgtNnRy",
+                                     p=[.22, .15, .15, .22, .05, .05, .05, .05, .04, .01, .005, .005]) for n in lens]
+    exp = ref_hits(seqs, pat, guides, thr)
+    assert gpu_hits(seqs, pat, guides, thr, impl=impl) == exp
+
+
+@pytest.mark.parametrize("impl", IMPLS)
+def test_c1_full(impl):
+    w = synth.make_workload("C1")
+    cfg = w.cfg
+    exp = ref_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
+    assert len(exp) >= cfg.threshold + 1
+    assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, impl=impl) == exp
+
+
+@pytest.mark.parametrize("name,scale,chunk", [("C2", 0.1, None), ("C3", 0.004, 1_000_003),
+                                              ("C4", 0.004, 333_333), ("C5", 0.002, None)])
+def test_configs_scaled(name, scale, chunk):
+    w = synth.make_workload(name, scale=scale, n_guides=None if name != "C5" else 200)
+    cfg = w.cfg
+    exp = ref_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
+    assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk) == exp
+
+
+def test_chunk_size_invariance():
+    w = synth.make_workload("C2", scale=0.02)
+    cfg = w.cfg
+    base = gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
+    for cb in (8192, 8191, 100_003, 7):
+        assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=cb) == base
+
+
+def test_finder_candidates_match_oracle():
+    """Finder output (ordered per-strand item lists) == oracle PAM candidate lists."""
+    rng = np.random.default_rng(9)
+    n = 300_001
+    seq = synth.random_genome_text(rng, n, b"ACGTacgtN", p=[.23, .23, .23, .23, .02, .02, .02, .01, .01])
+    for pat in ("N" * 21 + "RG", "TTTV" + "N" * 23, "NGG", "N" * 8):
+        L = len(pat)
+        plan = cof.cof_plan_create(pat, ["N" * L], [0])
+        s = torch.cuda.current_stream()
+        pd = torch.empty(cof.cof_plan_device_bytes(plan) + 256, dtype=torch.uint8, device="cuda")
+        cof.cof_plan_upload(plan, pd, s)
+        for start, owned in ((0, n - L + 1), (12345, 100_000), (n - L - 40, 41)):
+            nb = owned + L - 1
+            w = cof.cof_plane_words(nb)
+            host = np.zeros((3, w), np.uint32)
+            cof.cof_pack(np.ascontiguousarray(seq[start:start + nb]), nb, host[0], host[1], host[2])
+            d = torch.from_numpy(host.view(np.int32)).cuda()
+            dch = cof.make_chunk(0, start, nb, owned, d[0], d[1], d[2])
+            items = torch.empty((2, owned), dtype=torch.int32, device="cuda")
+            ws = torch.empty(cof.cof_find_workspace_bytes(owned), dtype=torch.uint8, device="cuda")
+            nf, nr = cof.cof_find_pam(plan, pd, dch, ws, items[0], items[1], owned, s)
+            for k, st in enumerate("+-"):
+                exp = oracle.pam_sites(seq, pat, st, start, start + owned) - start
+                got = items[k, : (nf, nr)[k]].cpu().numpy().astype(np.int64)
+                assert np.array_equal(got, exp), (pat, start, st)
+
+
+def test_capacity_overflow_and_device_counts():
+    rng = np.random.default_rng(10)
+    seq = synth.random_genome_text(rng, 50_000)
+    pat = "N" * 10
+    guides = ["N" * 10, "A" * 10]
+    thr = [0, 10]
+    exp = ref_hits([seq], pat, guides, thr)
+    srch = search.Searcher(pat, guides, thr)
+    srch.reserve(len(seq), 64)    # far too small: forces COF_E_CAPACITY + retry
+    host = search.HostGenome([seq], search.plan_chunks([len(seq)], 10))
+    got = cof.hits_to_tuples(srch.search_host(host))
+    assert got == exp
+    # items capacity too small -> COF_E_CAPACITY with the needed count
+    dch = srch.device_chunk(host.chunks[0])
+    cof.cof_load_chunk(host.chunk_struct(0), dch, srch.stream)
+    with pytest.raises(cof.CofError) as ei:
+        cof.cof_find_pam(srch.plan, srch.plan_dev, dch, srch.d_find_ws, srch.d_items[0], srch.d_items[1], 100,
+                         srch.stream)
+    assert ei.value.status == cof.COF_E_CAPACITY
+    # counts left on the device are used by compare / sort without a host round trip
+    cof.cof_find_pam(srch.plan, srch.plan_dev, dch, srch.d_find_ws, srch.d_items[0], srch.d_items[1],
+                     host.chunks[0].n_owned, srch.stream, sync=False)
+    cof.cof_compare(srch.plan, srch.plan_dev, dch, srch.d_items[0], cof.COF_COUNT_ON_DEVICE, srch.d_items[1],
+                    cof.COF_COUNT_ON_DEVICE, srch.d_hits, srch._hits_cap, srch.stream, sync=False)
+    cof.cof_sort_hits(srch.plan, srch.plan_dev, dch, srch.d_hits, srch.d_tmp, srch._hits_cap,
+                      cof.COF_COUNT_ON_DEVICE, srch.d_sort_ws, srch.stream)
+    nf, nr, nh = cof.cof_read_counts(srch.plan, srch.plan_dev, srch.stream)
+    assert nh == len(exp)
+    got2 = cof.hits_to_tuples(cof.cof_collect(srch.plan, host.chunk_struct(0), srch.d_hits, nh, srch.stream))
+    assert got2 == exp
+
+
+def test_sorted_keys_and_determinism():
+    w = synth.make_workload("C3", scale=0.002, n_guides=64)
+    cfg = w.cfg
+    a = gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
+    b = gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
+    assert a == b
+    assert a == sorted(a, key=lambda h: (h[0], h[1], h[2] == "-", h[3]))
+
+
+def test_full_size_sampled_c5():
+    """C5 at full size (the bench workload) on one GPU, in the bench's launch
+    configuration (whole-chromosome chunks, device-resident planes, counts on device);
+    the oracle recomputes sampled window ranges one by one."""
+    from bench import run_device_pipeline, prepare_workload   # same code the bench times
+    wl, plan_obj = prepare_workload("C5")
+    res = run_device_pipeline(wl, plan_obj, collect=True)
+    rng = np.random.default_rng(77)
+    cfg = wl.cfg
+    n_samples = 0
+    for c in rng.choice(len(wl.seqs), 6, replace=False):
+        n = len(wl.seqs[c])
+        for s0 in list(rng.integers(0, n - 200_000, 2)) + [0, n - 60_000]:
+            rng_ = [(0, 0)] * len(wl.seqs)
+            rng_[c] = (int(s0), int(s0) + 60_000)
+            exp = ref_hits(wl.seqs, cfg.pattern, wl.guides, wl.thresholds, ranges=rng_)
+            h = res[(res["chrom"] == c) & (res["pos"] >= s0) & (res["pos"] < s0 + 60_000)]
+            assert cof.hits_to_tuples(h) == exp
+            n_samples += 1
+    # planted sites at full size: every k <= t copy present with its exact mismatch count
+    found = {(int(h["chrom"]), int(h["pos"]), h["strand"].decode(), int(h["guide"])): int(h["mm"]) for h in res}
+    for pl in wl.plants:
+        key = (pl.chrom, pl.pos, pl.strand, pl.guide)
+        if pl.k <= cfg.threshold:
+            assert found.get(key) == pl.k
+        else:
+            assert key not in found
+    assert n_samples >= 20
