@@ -165,3 +165,23 @@ def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda"):
     chunks = plan_chunks([len(a) for a in arrs], L, chunk_bases)
     host = HostGenome(arrs, chunks)
     return Searcher(pattern, guides, thresholds, device).search_host(host)
+
+
+def shard_for_rank(chunks, rank: int, world: int):
+    """This rank's chunks (LPT over owned window starts; ranks are independent)."""
+    return shard_lpt(chunks, world)[rank]
+
+
+def gather_and_merge(local_hits: np.ndarray, group=None, dst: int = 0):
+    """Collect every rank's sorted hit list on ``dst`` (host objects over the process
+    group; the data path itself has no collective) and merge them there.  Returns the
+    merged array on ``dst`` and None elsewhere."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    buf = [None] * world if rank == dst else None
+    dist.gather_object(local_hits.tobytes(), buf, dst=dst, group=group)
+    if rank != dst:
+        return None
+    lists = [np.frombuffer(b, dtype=cof.HIT_DTYPE) for b in buf]
+    return merge_hit_lists(lists)

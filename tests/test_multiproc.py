@@ -1,0 +1,65 @@
+"""World-size-2 (gloo, CPU) test of the multi-GPU host logic: LPT sharding of chunks over
+ranks, per-rank independent search, gather + merge on rank 0 == single-process search.
+The per-rank search is the oracle here (no GPU on this box); the sharding, gather and
+merge code is the product's (search.shard_for_rank / gather_and_merge / cof_merge)."""
+import os
+import socket
+
+import numpy as np
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from oracle import oracle
+from paper_conf_socc_jinv23_b200 import cof, search, synth
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _oracle_chunk_hits(wl, ch):
+    cfg = wl.cfg
+    ranges = [(0, 0)] * len(wl.seqs)
+    ranges[ch.chrom] = (ch.start, ch.start + ch.n_owned)
+    h = oracle.search(wl.seqs, cfg.pattern, wl.guides, wl.thresholds, ranges=ranges)
+    out = np.zeros(len(h), dtype=cof.HIT_DTYPE)
+    for f in ("guide", "chrom", "pos", "strand", "mm", "site"):
+        out[f] = h[f]
+    return out
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    wl = synth.make_workload("C3", scale=0.0005, n_guides=8)
+    chunks = search.plan_chunks([len(s) for s in wl.seqs], wl.cfg.L, 40_000)
+    mine = search.shard_for_rank(chunks, rank, world)
+    lists = [_oracle_chunk_hits(wl, ch) for ch in mine]
+    local = search.merge_hit_lists(lists)
+    merged = search.gather_and_merge(local)
+    if rank == 0:
+        ref = oracle.search(wl.seqs, wl.cfg.pattern, wl.guides, wl.thresholds)
+        q.put((cof.hits_to_tuples(merged), oracle.hits_to_tuples(ref), len(mine), len(chunks)))
+    else:
+        q.put(("rank1", len(mine)))
+    dist.destroy_process_group()
+
+
+def test_two_rank_shard_gather_merge():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(2)]
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    r0 = [r for r in res if r[0] != "rank1"][0]
+    r1 = [r for r in res if r[0] == "rank1"][0]
+    got, exp, n0, n_all = r0
+    assert got == exp and len(exp) > 0
+    assert n0 + r1[1] == n_all and n0 > 0 and r1[1] > 0
