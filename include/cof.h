@@ -123,8 +123,10 @@ cof_status cof_fasta_pack(const cof_fasta *fa, uint32_t i, uint64_t first, uint6
  * base(p+j); '-' passes iff the reverse-complemented pattern does (G3, G10).  Passing
  * starts are compacted in ascending order into one list per strand (chunk-relative
  * uint32).  The paper compacts with an unordered atomic counter (Table V);
- * here a single-pass ordered scan (decoupled look-back) keeps the lists sorted.
- *  workspace  dev, >= cof_find_workspace_bytes(dev->n_owned) bytes (tile status words).
+ * here an ordered two-pass compaction (count, one grid-wide exchange, write) keeps the
+ * lists sorted.
+ *  workspace  dev, >= cof_find_workspace_bytes(dev->n_owned) bytes (per-CTA totals and a
+ *             grid barrier counter; reset by the call).
  *  items_cap  capacity of each list; n_owned always suffices.
  *  n_fwd/n_rev  host outputs; if both are NULL the call does not synchronize and the
  *             counts stay in plan_dev for cof_compare(COF_COUNT_ON_DEVICE).

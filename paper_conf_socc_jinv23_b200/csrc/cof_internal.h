@@ -43,6 +43,22 @@ struct GroupDesc {
     uint32_t n_guides;
 };
 
+#ifdef __CUDACC__
+#define COF_HD __host__ __device__ __forceinline__
+#else
+#define COF_HD inline
+#endif
+
+// Entry of a base pair (b1, b2 in 0..3 = A,C,G,T, 4 = N) of pair q in a 32-guide block of
+// the pair table (NP pairs, 25 entries each).  The 16 ACGT combos of a pair are 16
+// consecutive 8-byte entries (128 bytes = every shared-memory bank exactly once, so a
+// half-warp of lookups into one pair never conflicts); the 9 rare N combos of all pairs
+// follow in a separate region.
+COF_HD uint32_t pair_entry(uint32_t np, uint32_t q, uint32_t b1, uint32_t b2) {
+    if (b1 < 4 && b2 < 4) return q * 16u + b1 * 4u + b2;
+    return np * 16u + q * 9u + (b1 == 4 ? b2 : 5u + b1);
+}
+
 // Bit-sliced pair-table comparer (v2): per strand, per 32-guide block, per position pair,
 // 25 entries (base pair combos incl. N) of {bit0, bit1} mismatch-count planes.
 struct PairLayout {

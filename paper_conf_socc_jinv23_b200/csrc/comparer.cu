@@ -19,6 +19,8 @@
 //   carry-save adder tree sums the pairs and a borrow chain against the bit-sliced
 //   thresholds yields the 32-guide hit mask.  No POPC, ~1.3 ALU ops + 0.3 LDS per
 //   comparison.  Handles any IUPAC guide letter and per-guide thresholds uniformly.
+#include <algorithm>
+
 #include <cuda_runtime.h>
 
 #include "cof_internal.h"
@@ -29,6 +31,7 @@ namespace cof {
 
 constexpr int CT = 256;   // threads per CTA
 constexpr uint64_t ON_DEVICE = COF_COUNT_ON_DEVICE;
+constexpr uint32_t MAX_TABLE_BLOCKS = 128;   // 4096 guides per launch of the table comparer
 
 struct CompareArgs {
     const uint32_t* lo;
@@ -44,11 +47,6 @@ struct CompareArgs {
     const uint4* groups[2];        // GroupDesc as uint4
     const uint4* recs[2];
     uint32_t n_groups, n_recs;
-    // v2
-    const uint2* ptab[2];          // [n_blocks][n_pairs][25]
-    const uint32_t* pmeta[2];      // [n_blocks][8]
-    uint32_t n_blocks, n_pairs;
-    PairLayout pairs[2];
 };
 
 __device__ __forceinline__ void item_counts(const CompareArgs& a, uint64_t& n0, uint64_t& n1) {
@@ -179,86 +177,159 @@ __device__ __forceinline__ void pair_offsets(const PairLayout& pl, uint32_t wl, 
         const uint32_t b1 = ((wn >> j1) & 1u) ? 4u : (((wl >> j1) & 1u) | (((wh >> j1) & 1u) << 1));
         uint32_t b2 = 0;
         if (j2 != 0xFFu) b2 = ((wn >> j2) & 1u) ? 4u : (((wl >> j2) & 1u) | (((wh >> j2) & 1u) << 1));
-        off[q] = ((uint32_t)q * 25u + b1 * 5u + b2) * 8u;
+        off[q] = pair_entry(NP, (uint32_t)q, b1, b2) * 8u;
+    }
+}
+
+template <uint32_t OFF>
+__device__ __forceinline__ void lds64(uint32_t addr, uint32_t& x, uint32_t& y) {
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2+%3];" : "=r"(x), "=r"(y) : "r"(addr), "n"(OFF));
+}
+
+// Arguments of one table-comparer launch: ONE strand, up to MAX_TABLE_BLOCKS guide blocks.
+struct TableArgs {
+    const uint32_t* lo;
+    const uint32_t* hi;
+    const uint32_t* nm;
+    const uint32_t* items;
+    uint64_t n;                    // ON_DEVICE: read counters[strand]
+    uint64_t items_cap;
+    unsigned long long* hits;
+    uint64_t cap;
+    unsigned long long* counters;  // [0] n_fwd [1] n_rev [2] n_hits
+    const uint2* ptab;             // [n_blocks][NP][25] of this strand, first block = block_base
+    uint32_t strand;
+    uint32_t n_blocks;
+    uint32_t block_base;
+    uint32_t blocks_per_chunk;     // guide blocks resident in shared memory at a time
+    PairLayout pairs;
+    uint32_t meta[MAX_TABLE_BLOCKS][8];   // per block: T0..T5 threshold planes, valid mask
+};
+
+// Hit mask (bit k = guide k of the block) of one item against one 32-guide block whose
+// table starts OFF bytes past the item's base addresses.
+template <int NP, uint32_t OFF>
+__device__ __forceinline__ uint32_t table_hits(const uint32_t (&base)[NP], const uint32_t* __restrict__ T,
+                                               uint32_t (&s)[6]) {
+    uint32_t v0[NP], v1[NP];
+#pragma unroll
+    for (int q = 0; q < NP; q++) lds64<OFF>(base[q], v0[q], v1[q]);
+    const uint32_t Tl[6] = {T[0], T[1], T[2], T[3], T[4], T[5]};
+    return csa_hits<NP>(v0, v1, Tl, T[6], s);
+}
+
+__device__ __noinline__ void table_emit_v(const TableArgs& a, uint64_t item_idx, uint32_t hitm, uint32_t s0,
+                                          uint32_t s1, uint32_t s2, uint32_t s3, uint32_t s4, uint32_t s5,
+                                          uint32_t guide0) {
+    const uint32_t pos = __ldg(a.items + item_idx);
+    do {
+        const int k = __ffs(hitm) - 1;
+        hitm &= hitm - 1;
+        const uint32_t mm = ((s0 >> k) & 1u) | (((s1 >> k) & 1u) << 1) | (((s2 >> k) & 1u) << 2) |
+                            (((s3 >> k) & 1u) << 3) | (((s4 >> k) & 1u) << 4) | (((s5 >> k) & 1u) << 5);
+        const unsigned long long o = atomicAdd(&a.counters[2], 1ull);
+        if (o < a.cap) a.hits[o] = hit_key(pos, a.strand, guide0 + (uint32_t)k, mm);
+    } while (hitm);
+}
+
+__device__ __forceinline__ void table_emit(const TableArgs& a, uint64_t item_idx, uint32_t hitm, const uint32_t (&s)[6],
+                                           uint32_t guide0) {
+    table_emit_v(a, item_idx, hitm, s[0], s[1], s[2], s[3], s[4], s[5], guide0);
+}
+
+// All resident blocks [0, nb) for the R items of this thread.  base[r][q] = shared address of
+// item r's pair-q entry in block 0; groups of 4 blocks use immediate offsets.
+template <int NP, int R, bool TAIL>
+__device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base)[R][NP], uint32_t nb, uint32_t gb0,
+                                             uint64_t item0, const uint32_t (&okm)[R]) {
+    constexpr uint32_t BS = NP * 25 * 8;
+    uint32_t b = 0;
+    for (; b + 4 <= nb; b += 4) {
+        const uint32_t* m = a.meta[gb0 + b];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            uint32_t sx[6];
+            uint32_t h0 = table_hits<NP, 0 * BS>(base[r], m + 0, sx);
+            uint32_t h1 = table_hits<NP, 1 * BS>(base[r], m + 8, sx);
+            uint32_t h2 = table_hits<NP, 2 * BS>(base[r], m + 16, sx);
+            uint32_t h3 = table_hits<NP, 3 * BS>(base[r], m + 24, sx);
+            if (TAIL) { h0 &= okm[r]; h1 &= okm[r]; h2 &= okm[r]; h3 &= okm[r]; }
+            if (h0 | h1 | h2 | h3) {          // rare: ~1 hit per 2.5e4 comparisons at t = 6
+                // recompute the sums of the blocks that hit (keeps them out of the hot registers)
+                const uint64_t idx = item0 + (uint64_t)r * CT;
+                const uint32_t g0 = (a.block_base + gb0 + b) * 32u;
+                uint32_t sh[6];
+                if (h0) { table_hits<NP, 0 * BS>(base[r], m + 0, sh); table_emit(a, idx, h0, sh, g0); }
+                if (h1) { table_hits<NP, 1 * BS>(base[r], m + 8, sh); table_emit(a, idx, h1, sh, g0 + 32u); }
+                if (h2) { table_hits<NP, 2 * BS>(base[r], m + 16, sh); table_emit(a, idx, h2, sh, g0 + 64u); }
+                if (h3) { table_hits<NP, 3 * BS>(base[r], m + 24, sh); table_emit(a, idx, h3, sh, g0 + 96u); }
+            }
+#pragma unroll
+            for (int q = 0; q < NP; q++) base[r][q] += 4 * BS;
+        }
+    }
+    for (; b < nb; b++) {
+        const uint32_t* m = a.meta[gb0 + b];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            uint32_t s0[6];
+            uint32_t h0 = table_hits<NP, 0>(base[r], m, s0);
+            if (TAIL) h0 &= okm[r];
+            if (h0) table_emit(a, item0 + (uint64_t)r * CT, h0, s0, (a.block_base + gb0 + b) * 32u);
+#pragma unroll
+            for (int q = 0; q < NP; q++) base[r][q] += BS;
+        }
     }
 }
 
 template <int NP, int R>
-__global__ void __launch_bounds__(CT) cof_comparer_table(const __grid_constant__ CompareArgs a,
-                                                        uint32_t blocks_per_chunk) {
+__global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constant__ TableArgs a) {
     extern __shared__ __align__(16) uint8_t s_raw[];
-    // shared layout: [blocks_per_chunk][NP][25] uint2 table, then [blocks_per_chunk][8] meta
-    const uint32_t tab_bytes = blocks_per_chunk * NP * 25 * 8;
-    uint32_t* s_meta = reinterpret_cast<uint32_t*>(s_raw + tab_bytes);
+    // shared: [blocks_per_chunk][NP][25] uint2 pair table of the resident chunk of blocks
+    constexpr uint32_t BS = NP * 25 * 8;
     const uint32_t s_tab = smem_u32(s_raw);
-
-    uint64_t n0, n1;
-    item_counts(a, n0, n1);
+    uint64_t n = a.n == ON_DEVICE ? (uint64_t)a.counters[a.strand] : a.n;
+    if (n > a.items_cap) n = a.items_cap;
     const uint64_t per_tile = (uint64_t)CT * R;
-    const uint64_t t0 = (n0 + per_tile - 1) / per_tile, t1 = (n1 + per_tile - 1) / per_tile;
-    const uint32_t n_chunks = (a.n_blocks + blocks_per_chunk - 1) / blocks_per_chunk;
-    int loaded_st = -1;
-    uint32_t loaded_chunk = 0xFFFFFFFFu;
+    const uint64_t n_tiles = (n + per_tile - 1) / per_tile;
+    const uint32_t bpc = a.blocks_per_chunk;
+    const uint32_t n_chunks = (a.n_blocks + bpc - 1) / bpc;
+    uint32_t loaded = 0xFFFFFFFFu;
 
-    for (uint64_t tile = blockIdx.x; tile < t0 + t1; tile += gridDim.x) {
-        const uint32_t st = tile < t0 ? 0u : 1u;
-        const uint64_t base = (st == 0 ? tile : tile - t0) * per_tile;
-        const uint64_t nst = st == 0 ? n0 : n1;
-        uint32_t pos[R], off[R][NP];
-        bool ok[R];
+    for (uint64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        const uint64_t t0 = tile * per_tile;
+        const uint64_t item0 = t0 + threadIdx.x;
+        const bool tail = t0 + per_tile > n;
+        uint32_t off[R][NP], okm[R];
 #pragma unroll
         for (int r = 0; r < R; r++) {
-            const uint64_t idx = base + (uint64_t)r * CT + threadIdx.x;
-            ok[r] = idx < nst;
-            pos[r] = ok[r] ? __ldg(a.items[st] + idx) : 0u;
-            pair_offsets<NP>(a.pairs[st], plane_window(a.lo, pos[r]), plane_window(a.hi, pos[r]),
-                             plane_window(a.nm, pos[r]), off[r]);
+            const uint64_t idx = item0 + (uint64_t)r * CT;
+            okm[r] = idx < n ? ~0u : 0u;
+            const uint32_t pos = idx < n ? __ldg(a.items + idx) : 0u;
+            pair_offsets<NP>(a.pairs, plane_window(a.lo, pos), plane_window(a.hi, pos), plane_window(a.nm, pos), off[r]);
         }
         for (uint32_t ch = 0; ch < n_chunks; ch++) {
-            const uint32_t b0 = ch * blocks_per_chunk;
-            const uint32_t nb = min(blocks_per_chunk, a.n_blocks - b0);
-            if (loaded_st != (int)st || loaded_chunk != ch) {
+            const uint32_t b0 = ch * bpc;
+            const uint32_t nb = min(bpc, a.n_blocks - b0);
+            if (loaded != ch) {
                 __syncthreads();
-                const uint4* src = reinterpret_cast<const uint4*>(a.ptab[st] + (size_t)b0 * NP * 25);
-                uint4* dst = reinterpret_cast<uint4*>(s_raw);
-                const uint32_t n16 = nb * NP * 25 * 8 / 16;
-                for (uint32_t i = threadIdx.x; i < n16; i += CT) dst[i] = __ldg(src + i);
-                for (uint32_t i = threadIdx.x; i < nb * 8; i += CT) s_meta[i] = __ldg(a.pmeta[st] + (size_t)b0 * 8 + i);
+                const uint2* src = a.ptab + (size_t)b0 * NP * 25;
+                uint2* dst = reinterpret_cast<uint2*>(s_raw);
+                const uint32_t n8 = nb * NP * 25;
+                for (uint32_t i = threadIdx.x; i < n8; i += CT) dst[i] = __ldg(src + i);
                 __syncthreads();
-                loaded_st = (int)st;
-                loaded_chunk = ch;
+                loaded = ch;
             }
-            for (uint32_t b = 0; b < nb; b++) {
-                const uint32_t bbase = s_tab + b * (NP * 25 * 8);
-                const uint32_t* meta = s_meta + b * 8;
-                uint32_t T[6];
+            uint32_t base[R][NP];
 #pragma unroll
-                for (int w = 0; w < 6; w++) T[w] = meta[w];
-                const uint32_t valid = meta[6];
+            for (int r = 0; r < R; r++)
 #pragma unroll
-                for (int r = 0; r < R; r++) {
-                    uint32_t v0[NP], v1[NP];
-#pragma unroll
-                    for (int q = 0; q < NP; q++)
-                        asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v0[q]), "=r"(v1[q]) : "r"(bbase + off[r][q]));
-                    uint32_t s[6];
-                    uint32_t hitm = csa_hits<NP>(v0, v1, T, valid, s);
-                    if (!ok[r]) hitm = 0;
-                    while (hitm) {
-                        const int k = __ffs(hitm) - 1;
-                        hitm &= hitm - 1;
-                        const uint32_t mm = ((s[0] >> k) & 1u) | (((s[1] >> k) & 1u) << 1) | (((s[2] >> k) & 1u) << 2) |
-                                            (((s[3] >> k) & 1u) << 3) | (((s[4] >> k) & 1u) << 4) |
-                                            (((s[5] >> k) & 1u) << 5);
-                        const uint32_t guide = (b0 + b) * 32u + (uint32_t)k;
-                        const unsigned long long key = hit_key(pos[r], st, guide, mm);
-                        const unsigned long long o = atomicAdd(&a.counters[2], 1ull);
-                        if (o < a.cap) a.hits[o] = key;
-                    }
-                }
-            }
+                for (int q = 0; q < NP; q++) base[r][q] = s_tab + off[r][q];
+            if (tail) table_blocks<NP, R, true>(a, base, nb, b0, item0, okm);
+            else table_blocks<NP, R, false>(a, base, nb, b0, item0, okm);
         }
     }
+    (void)BS;
 }
 
 // ============================================================================ host side
@@ -288,26 +359,92 @@ static cof_status occupancy(const void* fn, uint32_t smem, int* bps) {
 }
 
 constexpr int R_POPC = 8;
-constexpr int R_TABLE = 2;
+constexpr int R_TABLE = 2;   // items per thread (COF_TABLE_R=4 selects 4)
 
-template <int NP>
-static cof_status launch_table(const CompareArgs& a, uint64_t tiles_hint, cudaStream_t stream) {
+static int table_r() {
+    static int r = -1;
+    if (r < 0) {
+        const char* e = getenv("COF_TABLE_R");
+        r = (e && e[0] == '4') ? 4 : R_TABLE;
+    }
+    return r;
+}
+
+template <int NP, int R>
+static cof_status launch_table_r(TableArgs& t, uint64_t n_hint, cudaStream_t stream) {
     // guide blocks resident in shared memory per pass (tiles over blocks if they do not fit)
-    const uint32_t per_block = NP * 25 * 8 + 32;
-    uint32_t bpc = a.n_blocks;
-    const uint32_t budget = 96 * 1024;
+    const uint32_t per_block = NP * 25 * 8;
+    uint32_t bpc = t.n_blocks;
+    const uint32_t budget = 72 * 1024;
     if (bpc * per_block > budget) bpc = budget / per_block;
+    t.blocks_per_chunk = bpc;
     const uint32_t smem = bpc * per_block;
     int bps = 0;
-    auto fn = cof_comparer_table<NP, R_TABLE>;
+    auto fn = cof_comparer_table<NP, R>;
     cof_status st = occupancy((const void*)fn, smem, &bps);
     if (st != COF_OK) return st;
     uint64_t grid = (uint64_t)num_sms() * bps;
-    if (tiles_hint != ON_DEVICE && grid > tiles_hint) grid = tiles_hint ? tiles_hint : 1;
-    fn<<<(uint32_t)grid, CT, smem, stream>>>(a, bpc);
+    if (n_hint != ON_DEVICE) {
+        const uint64_t tiles = (n_hint + (uint64_t)CT * R - 1) / ((uint64_t)CT * R);
+        if (tiles == 0) return COF_OK;
+        if (grid > tiles) grid = tiles;
+    }
+    fn<<<(uint32_t)grid, CT, smem, stream>>>(t);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "cof_comparer_table launch");
     count_launches(1);
+    return COF_OK;
+}
+
+template <int NP>
+static cof_status launch_table(TableArgs& t, uint64_t n_hint, cudaStream_t stream) {
+    if (table_r() == 4) return launch_table_r<NP, 4>(t, n_hint, stream);
+    return launch_table_r<NP, R_TABLE>(t, n_hint, stream);
+}
+
+// One launch per (strand, range of <= MAX_TABLE_BLOCKS guide blocks); thresholds travel in
+// the parameter space; hit counts accumulate on the device.
+static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs& a, cudaStream_t stream) {
+    static thread_local TableArgs T;   // ~4.5 KB parameter block, one per calling thread
+    const uint32_t np = plan->pairs[0].n_pairs;
+    for (uint32_t sd = 0; sd < 2; sd++) {
+        T.lo = a.lo; T.hi = a.hi; T.nm = a.nm;
+        T.items = a.items[sd];
+        T.n = a.n[sd];
+        T.items_cap = a.items_cap;
+        T.hits = a.hits; T.cap = a.cap; T.counters = a.counters;
+        T.strand = sd;
+        T.pairs = plan->pairs[sd];
+        const uint32_t* pm = (const uint32_t*)(plan->image.data() + (sd == 0 ? plan->lay.pmeta_fwd : plan->lay.pmeta_rev));
+        for (uint32_t bb = 0; bb < plan->n_blocks; bb += MAX_TABLE_BLOCKS) {
+            T.block_base = bb;
+            T.n_blocks = std::min<uint32_t>(MAX_TABLE_BLOCKS, plan->n_blocks - bb);
+            T.ptab = (const uint2*)(pd + (sd == 0 ? plan->lay.ptab_fwd : plan->lay.ptab_rev)) + (size_t)bb * np * 25;
+            for (uint32_t k = 0; k < T.n_blocks; k++)
+                for (int w = 0; w < 8; w++) T.meta[k][w] = pm[(size_t)(bb + k) * 8 + w];
+            cof_status st;
+            switch (np) {
+                case 1: st = launch_table<1>(T, T.n, stream); break;
+                case 2: st = launch_table<2>(T, T.n, stream); break;
+                case 3: st = launch_table<3>(T, T.n, stream); break;
+                case 4: st = launch_table<4>(T, T.n, stream); break;
+                case 5: st = launch_table<5>(T, T.n, stream); break;
+                case 6: st = launch_table<6>(T, T.n, stream); break;
+                case 7: st = launch_table<7>(T, T.n, stream); break;
+                case 8: st = launch_table<8>(T, T.n, stream); break;
+                case 9: st = launch_table<9>(T, T.n, stream); break;
+                case 10: st = launch_table<10>(T, T.n, stream); break;
+                case 11: st = launch_table<11>(T, T.n, stream); break;
+                case 12: st = launch_table<12>(T, T.n, stream); break;
+                case 13: st = launch_table<13>(T, T.n, stream); break;
+                case 14: st = launch_table<14>(T, T.n, stream); break;
+                case 15: st = launch_table<15>(T, T.n, stream); break;
+                case 16: st = launch_table<16>(T, T.n, stream); break;
+                default: return set_error(COF_E_STATE, "cof_compare: %u pairs", np);
+            }
+            if (st != COF_OK) return st;
+        }
+    }
     return COF_OK;
 }
 
@@ -371,20 +508,12 @@ cof_status cof_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* de
     a.recs[1] = (const uint4*)(pd + plan->lay.recs_rev);
     a.n_groups = plan->n_groups;
     a.n_recs = plan->n_recs;
-    a.ptab[0] = (const uint2*)(pd + plan->lay.ptab_fwd);
-    a.ptab[1] = (const uint2*)(pd + plan->lay.ptab_rev);
-    a.pmeta[0] = (const uint32_t*)(pd + plan->lay.pmeta_fwd);
-    a.pmeta[1] = (const uint32_t*)(pd + plan->lay.pmeta_rev);
-    a.n_blocks = plan->n_blocks;
-    a.n_pairs = plan->pairs[0].n_pairs;
-    a.pairs[0] = plan->pairs[0];
-    a.pairs[1] = plan->pairs[1];
 
     cudaError_t e = cudaMemsetAsync(a.counters + 2, 0, sizeof(uint64_t), stream);
     if (e != cudaSuccess) return cuda_error(e, "cof_compare memset");
     uint64_t tiles_hint = ON_DEVICE;
     if (n_fwd != ON_DEVICE && n_rev != ON_DEVICE) {
-        const int R = comparer_impl() == 0 ? R_POPC : R_TABLE;
+        const int R = comparer_impl() == 0 ? R_POPC : table_r();
         const uint64_t per = (uint64_t)CT * R;
         tiles_hint = (n_fwd + per - 1) / per + (n_rev + per - 1) / per;
     }
@@ -393,25 +522,7 @@ cof_status cof_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* de
         if (comparer_impl() == 0) {
             st = launch_popc(a, tiles_hint, stream);
         } else {
-            switch (a.n_pairs) {
-                case 1: st = launch_table<1>(a, tiles_hint, stream); break;
-                case 2: st = launch_table<2>(a, tiles_hint, stream); break;
-                case 3: st = launch_table<3>(a, tiles_hint, stream); break;
-                case 4: st = launch_table<4>(a, tiles_hint, stream); break;
-                case 5: st = launch_table<5>(a, tiles_hint, stream); break;
-                case 6: st = launch_table<6>(a, tiles_hint, stream); break;
-                case 7: st = launch_table<7>(a, tiles_hint, stream); break;
-                case 8: st = launch_table<8>(a, tiles_hint, stream); break;
-                case 9: st = launch_table<9>(a, tiles_hint, stream); break;
-                case 10: st = launch_table<10>(a, tiles_hint, stream); break;
-                case 11: st = launch_table<11>(a, tiles_hint, stream); break;
-                case 12: st = launch_table<12>(a, tiles_hint, stream); break;
-                case 13: st = launch_table<13>(a, tiles_hint, stream); break;
-                case 14: st = launch_table<14>(a, tiles_hint, stream); break;
-                case 15: st = launch_table<15>(a, tiles_hint, stream); break;
-                case 16: st = launch_table<16>(a, tiles_hint, stream); break;
-                default: return set_error(COF_E_STATE, "cof_compare: %u pairs", a.n_pairs);
-            }
+            st = run_table(plan, pd, a, stream);
         }
         if (st != COF_OK) return st;
     }

@@ -65,6 +65,12 @@ __device__ __forceinline__ uint64_t ld_relaxed_gpu(const uint64_t* p) {
     return v;
 }
 
+__device__ __forceinline__ uint32_t ld_acquire_gpu_u32(const unsigned int* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
 __device__ __forceinline__ uint32_t lanemask_lt() {
     uint32_t m;
     asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));

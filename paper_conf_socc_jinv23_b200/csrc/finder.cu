@@ -11,10 +11,11 @@
 // (cp.async.bulk + mbarrier).  One thread owns one plane word = 32 window starts and
 // tests the pattern and its reverse complement bit-parallel: per non-N pattern letter, a
 // funnel shift of each plane and a 3-LOP3 multiplexer select membership in the letter's
-// IUPAC set, AND-ed over letters.  Passing starts are compacted in order: CTA scan of the
-// per-thread popcounts, single-pass decoupled look-back across tiles for the global
-// offset, staging in shared memory and coalesced stores.  Bytes per base: 3/8 read +
-// 4 x items written.
+// IUPAC set, AND-ed over letters.  Passing starts are compacted in order: each CTA owns
+// a contiguous tile range, counts it (pass 1), exchanges its total with all CTAs once
+// (grid barrier), then re-streams the range (pass 2: CTA scan of the per-thread popcounts,
+// staging in shared memory, coalesced stores).  Algorithmic bytes per base: 3/8 read +
+// 4 x items written (pass 2 re-reads the planes, largely from L2).
 #include <cuda_runtime.h>
 
 #include "cof_internal.h"
@@ -26,6 +27,8 @@ constexpr int FT = 256;          // threads per CTA; one plane word per thread p
 constexpr int FW = 256;          // words per tile (8192 window starts)
 constexpr int FSTAGES = 4;       // TMA ring depth
 constexpr int FLOAD = FW + 4;    // words per plane per stage: tile + halo, 16-byte multiple
+constexpr uint32_t FMAX_CTAS = 4096;                      // grid cap (co-residency)
+constexpr size_t FWS_BARRIER = 2 * FMAX_CTAS * sizeof(uint64_t);
 constexpr uint32_t FSMEM = FSTAGES * 3 * FLOAD * 4 + FSTAGES * 8 + FW * 32 * 4;
 
 struct FinderArgs {
@@ -35,25 +38,51 @@ struct FinderArgs {
     uint64_t limit;              // valid window starts are [0, limit)
     uint32_t* out[2];            // '+' / '-' item lists
     uint64_t cap;
-    uint64_t* status;            // workspace: one look-back word per tile (zeroed)
+    uint64_t* status;            // workspace: per CTA (fwd, rev) totals
+    unsigned int* barrier;       // workspace: grid barrier counter (zeroed)
     unsigned long long* counters;  // plan_dev counters: [0] n_fwd, [1] n_rev
     uint32_t n_tiles;
-    PamStrand pam[2];
+    uint32_t ne;                 // non-N pattern letters per strand (same for both)
+    uint32_t pj[2][32];          // window offset of entry e
+    uint4 psel[2][32];           // entry e's IUPAC set as splat words {A, C, G, T} (0 / ~0)
 };
 
 // Membership of each of 32 bases (bit-parallel) in the IUPAC set `set` (A=1 C=2 G=4 T=8):
 // a multiplexer on the 2-bit code selects the set bit; N (nm=1) is in no set (G2).
-__device__ __forceinline__ uint32_t member(uint32_t lo, uint32_t hi, uint32_t nm, uint32_t set) {
-    const uint32_t sA = 0u - (set & 1u), sC = 0u - ((set >> 1) & 1u);
-    const uint32_t sG = 0u - ((set >> 2) & 1u), sT = 0u - ((set >> 3) & 1u);
-    const uint32_t t0 = (hi & sG) | (~hi & sA);      // lo = 0: A or G
-    const uint32_t t1 = (hi & sT) | (~hi & sC);      // lo = 1: C or T
+__device__ __forceinline__ uint32_t member(uint32_t lo, uint32_t hi, uint32_t nm, uint4 sel) {
+    const uint32_t t0 = (hi & sel.z) | (~hi & sel.x);      // lo = 0: A or G
+    const uint32_t t1 = (hi & sel.w) | (~hi & sel.y);      // lo = 1: C or T
     const uint32_t r = (lo & t1) | (~lo & t0);
     return r & ~nm;
 }
 
-constexpr uint64_t LB_AGG = 1ull << 62, LB_INC = 2ull << 62, LB_VAL = (1ull << 62) - 1;
+// PAM masks of the 32 window starts of one plane word, both strands.  NE > 0: entry count
+// known at compile time (fully unrolled); NE < 0: generic loop.
+template <int NE>
+__device__ __forceinline__ void pam_masks(const FinderArgs& a, uint32_t valid, uint32_t lo0, uint32_t lo1,
+                                          uint32_t hi0, uint32_t hi1, uint32_t nm0, uint32_t nm1, uint32_t (&m)[2]) {
+#pragma unroll
+    for (int st = 0; st < 2; st++) {
+        uint32_t acc = valid;
+        const uint32_t n = NE >= 0 ? (uint32_t)NE : a.ne;
+#pragma unroll
+        for (uint32_t e = 0; e < (NE >= 0 ? (uint32_t)NE : n); e++) {
+            const uint32_t j = a.pj[st][e];
+            acc &= member(__funnelshift_r(lo0, lo1, j), __funnelshift_r(hi0, hi1, j), __funnelshift_r(nm0, nm1, j),
+                          a.psel[st][e]);
+        }
+        m[st] = acc;
+    }
+}
 
+// Two passes over a contiguous tile range per CTA with one grid-wide exchange in between:
+//  pass 1 counts the passing starts of the CTA's range (no writes), publishes the CTA
+//  total and waits at a grid barrier (all CTAs are co-resident: the grid is sized from the
+//  occupancy calculator); every CTA then sums the totals of the CTAs before it (its global
+//  offset) and pass 2 re-streams its range (mostly from L2) and writes the items in order.
+// One exchange per CTA replaces a decoupled look-back per tile, whose depth (all
+// concurrently running tiles) made it latency-bound.
+template <int NE>
 __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ FinderArgs a) {
     extern __shared__ __align__(128) uint8_t smem[];
     uint32_t* stage = reinterpret_cast<uint32_t*>(smem);
@@ -61,9 +90,15 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
     uint32_t* items = reinterpret_cast<uint32_t*>(bars + FSTAGES);
     __shared__ uint32_t s_warp[FT / 32];
     __shared__ uint32_t s_tile_tot;
-    __shared__ uint64_t s_prefix;
+    __shared__ unsigned long long s_red[FT / 32][2];
+    __shared__ unsigned long long s_base[2];
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t per = (a.n_tiles + gridDim.x - 1) / gridDim.x;
+    const uint32_t t_begin = min(a.n_tiles, blockIdx.x * per);
+    const uint32_t t_end = min(a.n_tiles, t_begin + per);
+    const uint32_t n_mine = t_end - t_begin;
+
     if (tid == 0) {
         for (int s = 0; s < FSTAGES; s++) mbar_init(&bars[s], 1);
         fence_mbar_init();
@@ -77,135 +112,132 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
         bulk_g2s(stage + (s * 3 + 1) * FLOAD, a.hi + w0, FLOAD * 4, &bars[s]);
         bulk_g2s(stage + (s * 3 + 2) * FLOAD, a.nm + w0, FLOAD * 4, &bars[s]);
     };
-    if (tid == 0) {
-        for (int s = 0; s < FSTAGES; s++) {
-            uint32_t t = blockIdx.x + (uint32_t)s * gridDim.x;
-            if (t < a.n_tiles) issue(t, s);
-        }
-    }
 
-    uint32_t it = 0;
-    for (uint32_t tile = blockIdx.x; tile < a.n_tiles; tile += gridDim.x, it++) {
-        const int s = (int)(it % FSTAGES);
-        mbar_wait_parity(&bars[s], (it / FSTAGES) & 1u);
-        const uint32_t* Slo = stage + (s * 3 + 0) * FLOAD;
-        const uint32_t* Shi = stage + (s * 3 + 1) * FLOAD;
-        const uint32_t* Snm = stage + (s * 3 + 2) * FLOAD;
-        const uint32_t lo0 = Slo[tid], lo1 = Slo[tid + 1];
-        const uint32_t hi0 = Shi[tid], hi1 = Shi[tid + 1];
-        const uint32_t nm0 = Snm[tid], nm1 = Snm[tid + 1];
+    uint32_t it = 0;                       // ring position across both passes
+    unsigned long long cnt_f = 0, cnt_r = 0;   // pass 1: this thread's counts
+    unsigned long long run_f = 0, run_r = 0;   // pass 2: items of this CTA written so far
 
-        const uint64_t p0 = ((uint64_t)tile * FW + tid) * 32;
-        uint32_t valid;
-        if (p0 >= a.limit) valid = 0;
-        else if (a.limit - p0 >= 32) valid = ~0u;
-        else valid = (1u << (uint32_t)(a.limit - p0)) - 1u;
-
-        uint32_t m[2];
+    for (int pass = 0; pass < 2; pass++) {
+        if (pass == 1) {
+            // ---- CTA totals -> grid exchange -> this CTA's global offsets
 #pragma unroll
-        for (int st = 0; st < 2; st++) {
-            uint32_t acc = valid;
-            const uint32_t n = a.pam[st].n;
-            for (uint32_t e = 0; e < n; e++) {
-                const uint32_t j = a.pam[st].j[e];
-                const uint32_t l = __funnelshift_r(lo0, lo1, j);
-                const uint32_t h = __funnelshift_r(hi0, hi1, j);
-                const uint32_t x = __funnelshift_r(nm0, nm1, j);
-                acc &= member(l, h, x, a.pam[st].set[e]);
+            for (int o = 16; o > 0; o >>= 1) {
+                cnt_f += __shfl_xor_sync(0xffffffffu, cnt_f, o);
+                cnt_r += __shfl_xor_sync(0xffffffffu, cnt_r, o);
             }
-            m[st] = acc;
+            if (lane == 0) { s_red[warp][0] = cnt_f; s_red[warp][1] = cnt_r; }
+            __syncthreads();
+            if (tid == 0) {
+                unsigned long long f = 0, r = 0;
+                for (int w = 0; w < FT / 32; w++) { f += s_red[w][0]; r += s_red[w][1]; }
+                st_relaxed_gpu(&a.status[2 * blockIdx.x], f);
+                st_relaxed_gpu(&a.status[2 * blockIdx.x + 1], r);
+                __threadfence();
+                atomicAdd(a.barrier, 1u);
+                while (ld_acquire_gpu_u32(a.barrier) < gridDim.x) __nanosleep(64);
+            }
+            __syncthreads();
+            unsigned long long f = 0, r = 0;
+            for (uint32_t c = tid; c < blockIdx.x; c += FT) {
+                f += ld_relaxed_gpu(&a.status[2 * c]);
+                r += ld_relaxed_gpu(&a.status[2 * c + 1]);
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                f += __shfl_xor_sync(0xffffffffu, f, o);
+                r += __shfl_xor_sync(0xffffffffu, r, o);
+            }
+            __syncthreads();
+            if (lane == 0) { s_red[warp][0] = f; s_red[warp][1] = r; }
+            __syncthreads();
+            if (tid == 0) {
+                unsigned long long bf = 0, br = 0;
+                for (int w = 0; w < FT / 32; w++) { bf += s_red[w][0]; br += s_red[w][1]; }
+                s_base[0] = bf;
+                s_base[1] = br;
+                if (blockIdx.x == gridDim.x - 1) {     // last CTA knows the chunk totals
+                    a.counters[0] = bf + ld_relaxed_gpu(&a.status[2 * blockIdx.x]);
+                    a.counters[1] = br + ld_relaxed_gpu(&a.status[2 * blockIdx.x + 1]);
+                }
+            }
+            __syncthreads();
         }
-        __syncthreads();   // every thread has read stage s: refill it
         if (tid == 0) {
-            const uint32_t nt = tile + FSTAGES * gridDim.x;
-            if (nt < a.n_tiles) {
+            for (int s = 0; s < FSTAGES && (uint32_t)s < n_mine; s++) issue(t_begin + s, (int)((it + s) % FSTAGES));
+        }
+        for (uint32_t k = 0; k < n_mine; k++, it++) {
+            const uint32_t tile = t_begin + k;
+            const int s = (int)(it % FSTAGES);
+            mbar_wait_parity(&bars[s], (it / FSTAGES) & 1u);
+            const uint32_t* Slo = stage + (s * 3 + 0) * FLOAD;
+            const uint32_t* Shi = stage + (s * 3 + 1) * FLOAD;
+            const uint32_t* Snm = stage + (s * 3 + 2) * FLOAD;
+            const uint32_t lo0 = Slo[tid], lo1 = Slo[tid + 1];
+            const uint32_t hi0 = Shi[tid], hi1 = Shi[tid + 1];
+            const uint32_t nm0 = Snm[tid], nm1 = Snm[tid + 1];
+
+            const uint64_t p0 = ((uint64_t)tile * FW + tid) * 32;
+            uint32_t valid = ~0u;
+            if (p0 + 32 > a.limit) valid = p0 >= a.limit ? 0u : (1u << (uint32_t)(a.limit - p0)) - 1u;
+            uint32_t m[2];
+            pam_masks<NE>(a, valid, lo0, lo1, hi0, hi1, nm0, nm1, m);
+            __syncthreads();   // every thread has read stage s: refill it
+            if (tid == 0 && k + FSTAGES < n_mine) {
                 fence_proxy_async_smem();
-                issue(nt, s);
+                issue(tile + FSTAGES, s);
             }
-        }
+            if (pass == 0) {
+                cnt_f += (unsigned)__popc(m[0]);
+                cnt_r += (unsigned)__popc(m[1]);
+                continue;
+            }
 
-        // ---- CTA exclusive scan of packed counts (fwd in bits 0..15, rev in 16..31)
-        const uint32_t cnt = (uint32_t)__popc(m[0]) | ((uint32_t)__popc(m[1]) << 16);
-        uint32_t x = cnt;
+            // ---- pass 2: CTA exclusive scan of packed counts (fwd bits 0..15, rev 16..31)
+            const uint32_t cnt = (uint32_t)__popc(m[0]) | ((uint32_t)__popc(m[1]) << 16);
+            uint32_t x = cnt;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= o) x += y;
-        }
-        if (lane == 31) s_warp[warp] = x;
-        __syncthreads();
-        if (warp == 0) {
-            uint32_t wv = lane < FT / 32 ? s_warp[lane] : 0u;
-            uint32_t wi = wv;
-#pragma unroll
-            for (int o = 1; o < FT / 32; o <<= 1) {
-                uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
-                if (lane >= o) wi += y;
+            for (int o = 1; o < 32; o <<= 1) {
+                uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= o) x += y;
             }
-            if (lane < FT / 32) s_warp[lane] = wi - wv;          // exclusive warp offsets
-            const uint32_t tot = __shfl_sync(0xffffffffu, wi, FT / 32 - 1);
-            // ---- decoupled look-back over tiles (values: fwd bits 0..30, rev bits 31..61)
-            const uint64_t agg = (uint64_t)(tot & 0xFFFFu) | ((uint64_t)(tot >> 16) << 31);
-            uint64_t excl = 0;
-            if (tile == 0) {
-                if (lane == 0) st_relaxed_gpu(&a.status[0], LB_INC | agg);
-            } else {
-                if (lane == 0) st_relaxed_gpu(&a.status[tile], LB_AGG | agg);
-                int64_t pred = (int64_t)tile - 1;
-                while (true) {
-                    const int64_t idx = pred - lane;
-                    const uint64_t v = idx >= 0 ? ld_relaxed_gpu(&a.status[idx]) : LB_INC;
-                    const uint32_t flag = (uint32_t)(v >> 62);
-                    if (__any_sync(0xffffffffu, flag == 0)) continue;
-                    const uint32_t inc = __ballot_sync(0xffffffffu, flag == 2);
-                    uint64_t val = v & LB_VAL;
-                    if (inc) {
-                        const int first = __ffs(inc) - 1;
-                        if (lane > first) val = 0;
-                    }
+            if (lane == 31) s_warp[warp] = x;
+            __syncthreads();
+            if (warp == 0) {
+                uint32_t wv = lane < FT / 32 ? s_warp[lane] : 0u;
+                uint32_t wi = wv;
 #pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) val += __shfl_xor_sync(0xffffffffu, val, o);
-                    excl += val;
-                    if (inc) break;
-                    pred -= 32;
+                for (int o = 1; o < FT / 32; o <<= 1) {
+                    uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
+                    if (lane >= o) wi += y;
                 }
-                if (lane == 0) st_relaxed_gpu(&a.status[tile], LB_INC | (excl + agg));
-            }
-            if (lane == 0) {
-                s_prefix = excl;
-                s_tile_tot = tot;
-                if (tile == a.n_tiles - 1) {
-                    const uint64_t inc_all = excl + agg;
-                    a.counters[0] = inc_all & 0x7FFFFFFFull;
-                    a.counters[1] = (inc_all >> 31) & 0x7FFFFFFFull;
-                }
-            }
-        }
-        __syncthreads();
-        const uint32_t local = s_warp[warp] + x - cnt;    // exclusive, packed
-        const uint64_t pre = s_prefix;
-        const uint32_t tot = s_tile_tot;
-
-        // ---- ordered, coalesced output per strand through the shared staging buffer
-#pragma unroll
-        for (int st = 0; st < 2; st++) {
-            uint32_t off = st == 0 ? (local & 0xFFFFu) : (local >> 16);
-            uint32_t mm = m[st];
-            const uint32_t pbase = (uint32_t)p0;
-            while (mm) {
-                const int b = __ffs(mm) - 1;
-                items[off++] = pbase + (uint32_t)b;
-                mm &= mm - 1;
+                if (lane < FT / 32) s_warp[lane] = wi - wv;
+                if (lane == FT / 32 - 1) s_tile_tot = wi;
             }
             __syncthreads();
-            const uint32_t total = st == 0 ? (tot & 0xFFFFu) : (tot >> 16);
-            const uint64_t base = st == 0 ? (pre & 0x7FFFFFFFull) : ((pre >> 31) & 0x7FFFFFFFull);
-            uint32_t* out = a.out[st];
-            for (uint32_t i = tid; i < total; i += FT) {
-                const uint64_t o = base + i;
-                if (o < a.cap) out[o] = items[i];
+            const uint32_t local = s_warp[warp] + x - cnt;
+            const uint32_t tot = s_tile_tot;
+#pragma unroll
+            for (int st = 0; st < 2; st++) {
+                uint32_t off = st == 0 ? (local & 0xFFFFu) : (local >> 16);
+                uint32_t mm = m[st];
+                const uint32_t pbase = (uint32_t)p0;
+                while (mm) {
+                    const int b = __ffs(mm) - 1;
+                    items[off++] = pbase + (uint32_t)b;
+                    mm &= mm - 1;
+                }
+                __syncthreads();
+                const uint32_t total = st == 0 ? (tot & 0xFFFFu) : (tot >> 16);
+                const unsigned long long base = s_base[st] + (st == 0 ? run_f : run_r);
+                uint32_t* out = a.out[st];
+                for (uint32_t i = tid; i < total; i += FT) {
+                    const unsigned long long o = base + i;
+                    if (o < a.cap) out[o] = items[i];
+                }
+                __syncthreads();
             }
-            __syncthreads();
+            run_f += tot & 0xFFFFu;
+            run_r += tot >> 16;
         }
     }
 }
@@ -213,17 +245,37 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
 static int g_finder_blocks_per_sm = -1;
 static int g_num_sms = -1;
 
+typedef void (*FinderFn)(FinderArgs);
+static FinderFn finder_fn(uint32_t ne) {
+    switch (ne) {
+        case 0: return cof_finder_kernel<0>;
+        case 1: return cof_finder_kernel<1>;
+        case 2: return cof_finder_kernel<2>;
+        case 3: return cof_finder_kernel<3>;
+        case 4: return cof_finder_kernel<4>;
+        case 5: return cof_finder_kernel<5>;
+        case 6: return cof_finder_kernel<6>;
+        default: return cof_finder_kernel<-1>;
+    }
+}
+
 static cof_status finder_setup() {
     if (g_finder_blocks_per_sm > 0) return COF_OK;
-    cudaError_t e = cudaFuncSetAttribute(cof_finder_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM);
-    if (e != cudaSuccess) return cuda_error(e, "finder setup");
-    int dev = 0, sms = 0, bps = 0;
+    int bps_min = 1 << 30;
+    for (uint32_t ne = 0; ne <= 7; ne++) {
+        FinderFn fn = finder_fn(ne);
+        cudaError_t e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM);
+        if (e != cudaSuccess) return cuda_error(e, "finder setup");
+        int bps = 0;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, (const void*)fn, FT, FSMEM);
+        if (e != cudaSuccess) return cuda_error(e, "finder occupancy");
+        if (bps < bps_min) bps_min = bps;
+    }
+    int dev = 0, sms = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, cof_finder_kernel, FT, FSMEM);
-    if (e != cudaSuccess) return cuda_error(e, "finder occupancy");
     g_num_sms = sms;
-    g_finder_blocks_per_sm = bps > 0 ? bps : 1;
+    g_finder_blocks_per_sm = bps_min > 0 ? bps_min : 1;
     return COF_OK;
 }
 
@@ -234,8 +286,8 @@ using namespace cof;
 extern "C" {
 
 size_t cof_find_workspace_bytes(uint64_t n_owned) {
-    uint64_t tiles = (n_owned + (uint64_t)FW * 32 - 1) / ((uint64_t)FW * 32);
-    return (size_t)(tiles ? tiles : 1) * sizeof(uint64_t);
+    (void)n_owned;   // per-CTA totals (at most FMAX_CTAS CTAs) + the grid barrier counter
+    return FWS_BARRIER + 64;
 }
 
 cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
@@ -257,7 +309,7 @@ cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* d
     unsigned long long* counters = (unsigned long long*)((uint8_t*)plan_dev + plan->lay.counters);
     cudaError_t e = cudaMemsetAsync(counters, 0, 2 * sizeof(uint64_t), stream);
     if (e == cudaSuccess && n_tiles)
-        e = cudaMemsetAsync(workspace, 0, (size_t)n_tiles * sizeof(uint64_t), stream);
+        e = cudaMemsetAsync((uint8_t*)workspace + FWS_BARRIER, 0, 64, stream);
     if (e != cudaSuccess) return cuda_error(e, "cof_find_pam memset");
     if (n_tiles) {
         FinderArgs a;
@@ -266,13 +318,21 @@ cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* d
         a.out[0] = items_fwd; a.out[1] = items_rev;
         a.cap = items_cap;
         a.status = (uint64_t*)workspace;
+        a.barrier = (unsigned int*)((uint8_t*)workspace + FWS_BARRIER);
         a.counters = counters;
         a.n_tiles = n_tiles;
-        a.pam[0] = plan->pam[0];
-        a.pam[1] = plan->pam[1];
+        a.ne = plan->pam[0].n;
+        for (int st = 0; st < 2; st++)
+            for (uint32_t k = 0; k < plan->pam[st].n; k++) {
+                const uint32_t set = plan->pam[st].set[k];
+                a.pj[st][k] = plan->pam[st].j[k];
+                a.psel[st][k] = make_uint4(0u - (set & 1u), 0u - ((set >> 1) & 1u), 0u - ((set >> 2) & 1u),
+                                           0u - ((set >> 3) & 1u));
+            }
         uint32_t grid = (uint32_t)g_num_sms * (uint32_t)g_finder_blocks_per_sm;
+        if (grid > FMAX_CTAS) grid = FMAX_CTAS;
         if (grid > n_tiles) grid = n_tiles;
-        cof_finder_kernel<<<grid, FT, FSMEM, stream>>>(a);
+        finder_fn(a.ne)<<<grid, FT, FSMEM, stream>>>(a);
         e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "cof_finder_kernel launch");
         count_launches(1);

@@ -213,7 +213,7 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
                         w0 |= (cnt & 1u) << k;
                         w1 |= (cnt >> 1) << k;
                     }
-                    size_t e = ((size_t)b * NPAIR + q) * 25 + c;
+                    size_t e = (size_t)b * NPAIR * 25 + pair_entry(NPAIR, q, b1, b2);
                     tab[e * 2 + 0] = w0;
                     tab[e * 2 + 1] = w1;
                 }

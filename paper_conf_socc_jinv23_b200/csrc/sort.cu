@@ -7,7 +7,7 @@
 // orders exactly that way; only the bits that can vary are sorted: the compressed key
 //   k' = pos << (GB + 1) | strand << GB | guide      (GB = bits of the largest guide index)
 // is cut into 8-bit digits, one pass per digit.  Each pass: per-tile digit histograms
-// (shared-memory atomics), one exclusive scan over the digit-major histogram matrix, and a
+// (shared-memory atomics) + digit totals, a per-digit scan over tiles (one CTA per digit), and a
 // stable scatter that ranks keys inside a tile with __match_any_sync in index order.
 #include <cuda_runtime.h>
 
@@ -19,12 +19,12 @@ namespace cof {
 constexpr int ST = 256;             // threads per CTA
 constexpr int SV = 16;              // keys per thread per tile
 constexpr int STILE = ST * SV;      // 4096 keys per tile
-constexpr int SCAN_T = 1024;
 
 struct SortPass {
     const unsigned long long* src;
     unsigned long long* dst;
     uint32_t* hist;                 // [256][cap_tiles]
+    uint32_t* totals;               // [256] keys per digit (zeroed before the pass)
     const unsigned long long* count;  // device count (n_hits) or nullptr
     uint64_t n_host;                // used when count == nullptr
     uint64_t cap;
@@ -61,21 +61,35 @@ __global__ void __launch_bounds__(ST) cof_sort_hist(const __grid_constant__ Sort
     }
     __syncthreads();
     p.hist[(size_t)threadIdx.x * p.cap_tiles + blockIdx.x] = h[threadIdx.x];
+    if (h[threadIdx.x]) atomicAdd(&p.totals[threadIdx.x], h[threadIdx.x]);
 }
 
-// Exclusive scan of the whole [256][cap_tiles] matrix (digit-major) by one CTA.
-__global__ void __launch_bounds__(SCAN_T) cof_sort_scan(uint32_t* hist, uint64_t m) {
-    __shared__ uint32_t s_warp[SCAN_T / 32];
+// Offsets: CTA d turns row d of the [256][cap_tiles] histogram into global offsets
+// (exclusive scan over tiles + the number of keys with a smaller digit).
+__global__ void __launch_bounds__(ST) cof_sort_scan(const __grid_constant__ SortPass p) {
+    __shared__ uint32_t s_warp[ST / 32];
     __shared__ uint32_t s_carry;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid == 0) s_carry = 0;
+    const uint32_t d = blockIdx.x;
+    uint32_t below = tid < (int)d ? p.totals[tid] : 0u;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) below += __shfl_xor_sync(0xffffffffu, below, o);
+    if (lane == 0) s_warp[warp] = below;
     __syncthreads();
-    for (uint64_t c0 = 0; c0 < m; c0 += (uint64_t)SCAN_T * 4) {
+    if (tid == 0) {
+        uint32_t b = 0;
+        for (int w = 0; w < ST / 32; w++) b += s_warp[w];
+        s_carry = b;
+    }
+    __syncthreads();
+    uint32_t* row = p.hist + (size_t)d * p.cap_tiles;
+    const uint32_t m = p.cap_tiles;
+    for (uint32_t c0 = 0; c0 < m; c0 += ST * 4) {
         uint32_t v[4], sum = 0;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
-            const uint64_t i = c0 + (uint64_t)tid * 4 + k;
-            v[k] = i < m ? hist[i] : 0u;
+            const uint32_t i = c0 + (uint32_t)tid * 4 + k;
+            v[k] = i < m ? row[i] : 0u;
             sum += v[k];
         }
         uint32_t x = sum;
@@ -84,28 +98,29 @@ __global__ void __launch_bounds__(SCAN_T) cof_sort_scan(uint32_t* hist, uint64_t
             const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
             if (lane >= o) x += y;
         }
+        __syncthreads();
         if (lane == 31) s_warp[warp] = x;
         __syncthreads();
         if (warp == 0) {
-            const uint32_t wv = s_warp[lane];
+            const uint32_t wv = lane < ST / 32 ? s_warp[lane] : 0u;
             uint32_t wi = wv;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
+            for (int o = 1; o < ST / 32; o <<= 1) {
                 const uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
                 if (lane >= o) wi += y;
             }
-            s_warp[lane] = wi - wv;
+            if (lane < ST / 32) s_warp[lane] = wi - wv;
         }
         __syncthreads();
         uint32_t run = s_carry + s_warp[warp] + x - sum;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
-            const uint64_t i = c0 + (uint64_t)tid * 4 + k;
-            if (i < m) hist[i] = run;
+            const uint32_t i = c0 + (uint32_t)tid * 4 + k;
+            if (i < m) row[i] = run;
             run += v[k];
         }
         __syncthreads();
-        if (tid == SCAN_T - 1) s_carry = run;
+        if (tid == ST - 1) s_carry = run;
         __syncthreads();
     }
 }
@@ -170,7 +185,7 @@ extern "C" {
 size_t cof_sort_workspace_bytes(uint64_t cap) {
     uint64_t tiles = (cap + STILE - 1) / STILE;
     if (!tiles) tiles = 1;
-    return (size_t)(256 * tiles * sizeof(uint32_t) + 256);
+    return (size_t)(256 * tiles * sizeof(uint32_t) + 256 * sizeof(uint32_t));
 }
 
 cof_status cof_sort_hits(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, uint64_t* hits, uint64_t* tmp,
@@ -195,10 +210,12 @@ cof_status cof_sort_hits(const cof_plan* plan, void* plan_dev, const cof_chunk* 
     const uint32_t passes = (total_bits + 7) / 8;
     unsigned long long* a = (unsigned long long*)hits;
     unsigned long long* b = (unsigned long long*)tmp;
+    p.totals = p.hist + (size_t)256 * p.cap_tiles;
     for (uint32_t k = 0; k < passes; k++) {
         p.src = a; p.dst = b; p.shift = 8 * k;
+        cudaMemsetAsync(p.totals, 0, 256 * sizeof(uint32_t), stream);
         cof_sort_hist<<<p.cap_tiles, ST, 0, stream>>>(p);
-        cof_sort_scan<<<1, SCAN_T, 0, stream>>>(p.hist, (uint64_t)256 * p.cap_tiles);
+        cof_sort_scan<<<256, ST, 0, stream>>>(p);
         cof_sort_scatter<<<p.cap_tiles, ST, 0, stream>>>(p);
         count_launches(3);
         unsigned long long* t = a; a = b; b = t;
