@@ -244,17 +244,27 @@ def cof_read_counts(plan, plan_dev, stream=None):
 
 
 def cof_collect(plan, host: cof_chunk, hits_dev, n_hits, stream=None, host_keys=None) -> np.ndarray:
-    out = np.zeros(int(n_hits), dtype=HIT_DTYPE)
+    out = np.empty(int(n_hits), dtype=HIT_DTYPE)
     if n_hits:
         _check(lib.cof_collect(plan.handle, ctypes.addressof(host), _ptr(hits_dev), _ptr(host_keys),
                                int(n_hits), out.ctypes.data, _stream(stream)))
     return out
 
 
+def cof_collect_into(plan, host: cof_chunk, host_keys, n_hits, out: np.ndarray):
+    """cof_collect from host keys into a caller-provided (contiguous) record array."""
+    if not out.flags["C_CONTIGUOUS"] or out.dtype != HIT_DTYPE or len(out) < n_hits:
+        raise ValueError("out must be a contiguous HIT_DTYPE array of >= n_hits records")
+    if n_hits:
+        _check(lib.cof_collect(plan.handle, ctypes.addressof(host), None, _ptr(host_keys), int(n_hits),
+                               out.ctypes.data, None))
+    return out
+
+
 def cof_merge(lists) -> np.ndarray:
     lists = [np.ascontiguousarray(x, dtype=HIT_DTYPE) for x in lists]
     total = sum(len(x) for x in lists)
-    out = np.zeros(total, dtype=HIT_DTYPE)
+    out = np.empty(total, dtype=HIT_DTYPE)
     ptrs = (ctypes.c_void_p * max(len(lists), 1))(*[x.ctypes.data for x in lists])
     lens = (ctypes.c_uint64 * max(len(lists), 1))(*[len(x) for x in lists])
     _check(lib.cof_merge(ctypes.addressof(ptrs), ctypes.addressof(lens), len(lists), out.ctypes.data))

@@ -85,6 +85,7 @@ struct cof_plan {
     std::vector<std::string> guides;     // upper-case
     std::vector<uint8_t> max_mm;
     std::vector<uint8_t> gmask;          // [n_guides * L] IUPAC masks (forward orientation)
+    std::vector<uint32_t> onehot;        // [2][n_guides][5]: A, C, G, T membership + care, window offsets
     cof::PamStrand pam[2];               // [0] '+', [1] '-' (reverse-complemented pattern)
     uint32_t n_groups = 0;
     uint32_t n_recs = 0;

@@ -208,14 +208,22 @@ struct TableArgs {
 
 // Hit mask (bit k = guide k of the block) of one item against one 32-guide block whose
 // table starts OFF bytes past the item's base addresses.
-template <int NP, uint32_t OFF>
+// TC >= 0: every guide of the launch has threshold TC (compile-time constant: the borrow
+// chain folds to a couple of LOP3); TC < 0: per-guide thresholds from the bit planes.
+template <int NP, uint32_t OFF, int TC>
 __device__ __forceinline__ uint32_t table_hits(const uint32_t (&base)[NP], const uint32_t* __restrict__ T,
                                                uint32_t (&s)[6]) {
     uint32_t v0[NP], v1[NP];
 #pragma unroll
     for (int q = 0; q < NP; q++) lds64<OFF>(base[q], v0[q], v1[q]);
-    const uint32_t Tl[6] = {T[0], T[1], T[2], T[3], T[4], T[5]};
-    return csa_hits<NP>(v0, v1, Tl, T[6], s);
+    if constexpr (TC >= 0) {
+        const uint32_t Tl[6] = {0u - (TC & 1u), 0u - ((TC >> 1) & 1u), 0u - ((TC >> 2) & 1u),
+                                0u - ((TC >> 3) & 1u), 0u - ((TC >> 4) & 1u), 0u - ((TC >> 5) & 1u)};
+        return csa_hits<NP>(v0, v1, Tl, T[6], s);
+    } else {
+        const uint32_t Tl[6] = {T[0], T[1], T[2], T[3], T[4], T[5]};
+        return csa_hits<NP>(v0, v1, Tl, T[6], s);
+    }
 }
 
 __device__ __noinline__ void table_emit_v(const TableArgs& a, uint64_t item_idx, uint32_t hitm, uint32_t s0,
@@ -239,7 +247,7 @@ __device__ __forceinline__ void table_emit(const TableArgs& a, uint64_t item_idx
 
 // All resident blocks [0, nb) for the R items of this thread.  base[r][q] = shared address of
 // item r's pair-q entry in block 0; groups of 4 blocks use immediate offsets.
-template <int NP, int R, bool TAIL>
+template <int NP, int R, bool TAIL, int TC>
 __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base)[R][NP], uint32_t nb, uint32_t gb0,
                                              uint64_t item0, const uint32_t (&okm)[R]) {
     constexpr uint32_t BS = NP * 25 * 8;
@@ -249,20 +257,20 @@ __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base
 #pragma unroll
         for (int r = 0; r < R; r++) {
             uint32_t sx[6];
-            uint32_t h0 = table_hits<NP, 0 * BS>(base[r], m + 0, sx);
-            uint32_t h1 = table_hits<NP, 1 * BS>(base[r], m + 8, sx);
-            uint32_t h2 = table_hits<NP, 2 * BS>(base[r], m + 16, sx);
-            uint32_t h3 = table_hits<NP, 3 * BS>(base[r], m + 24, sx);
+            uint32_t h0 = table_hits<NP, 0 * BS, TC>(base[r], m + 0, sx);
+            uint32_t h1 = table_hits<NP, 1 * BS, TC>(base[r], m + 8, sx);
+            uint32_t h2 = table_hits<NP, 2 * BS, TC>(base[r], m + 16, sx);
+            uint32_t h3 = table_hits<NP, 3 * BS, TC>(base[r], m + 24, sx);
             if (TAIL) { h0 &= okm[r]; h1 &= okm[r]; h2 &= okm[r]; h3 &= okm[r]; }
             if (h0 | h1 | h2 | h3) {          // rare: ~1 hit per 2.5e4 comparisons at t = 6
                 // recompute the sums of the blocks that hit (keeps them out of the hot registers)
                 const uint64_t idx = item0 + (uint64_t)r * CT;
                 const uint32_t g0 = (a.block_base + gb0 + b) * 32u;
                 uint32_t sh[6];
-                if (h0) { table_hits<NP, 0 * BS>(base[r], m + 0, sh); table_emit(a, idx, h0, sh, g0); }
-                if (h1) { table_hits<NP, 1 * BS>(base[r], m + 8, sh); table_emit(a, idx, h1, sh, g0 + 32u); }
-                if (h2) { table_hits<NP, 2 * BS>(base[r], m + 16, sh); table_emit(a, idx, h2, sh, g0 + 64u); }
-                if (h3) { table_hits<NP, 3 * BS>(base[r], m + 24, sh); table_emit(a, idx, h3, sh, g0 + 96u); }
+                if (h0) { table_hits<NP, 0 * BS, TC>(base[r], m + 0, sh); table_emit(a, idx, h0, sh, g0); }
+                if (h1) { table_hits<NP, 1 * BS, TC>(base[r], m + 8, sh); table_emit(a, idx, h1, sh, g0 + 32u); }
+                if (h2) { table_hits<NP, 2 * BS, TC>(base[r], m + 16, sh); table_emit(a, idx, h2, sh, g0 + 64u); }
+                if (h3) { table_hits<NP, 3 * BS, TC>(base[r], m + 24, sh); table_emit(a, idx, h3, sh, g0 + 96u); }
             }
 #pragma unroll
             for (int q = 0; q < NP; q++) base[r][q] += 4 * BS;
@@ -273,7 +281,7 @@ __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base
 #pragma unroll
         for (int r = 0; r < R; r++) {
             uint32_t s0[6];
-            uint32_t h0 = table_hits<NP, 0>(base[r], m, s0);
+            uint32_t h0 = table_hits<NP, 0, TC>(base[r], m, s0);
             if (TAIL) h0 &= okm[r];
             if (h0) table_emit(a, item0 + (uint64_t)r * CT, h0, s0, (a.block_base + gb0 + b) * 32u);
 #pragma unroll
@@ -282,7 +290,7 @@ __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base
     }
 }
 
-template <int NP, int R>
+template <int NP, int R, int TC>
 __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constant__ TableArgs a) {
     extern __shared__ __align__(16) uint8_t s_raw[];
     // shared: [blocks_per_chunk][NP][25] uint2 pair table of the resident chunk of blocks
@@ -325,8 +333,8 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constan
             for (int r = 0; r < R; r++)
 #pragma unroll
                 for (int q = 0; q < NP; q++) base[r][q] = s_tab + off[r][q];
-            if (tail) table_blocks<NP, R, true>(a, base, nb, b0, item0, okm);
-            else table_blocks<NP, R, false>(a, base, nb, b0, item0, okm);
+            if (tail) table_blocks<NP, R, true, TC>(a, base, nb, b0, item0, okm);
+            else table_blocks<NP, R, false, TC>(a, base, nb, b0, item0, okm);
         }
     }
     (void)BS;
@@ -359,28 +367,33 @@ static cof_status occupancy(const void* fn, uint32_t smem, int* bps) {
 }
 
 constexpr int R_POPC = 8;
-constexpr int R_TABLE = 2;   // items per thread (COF_TABLE_R=4 selects 4)
+constexpr int R_TABLE = 2;   // items per thread
 
-static int table_r() {
-    static int r = -1;
-    if (r < 0) {
-        const char* e = getenv("COF_TABLE_R");
-        r = (e && e[0] == '4') ? 4 : R_TABLE;
+// Tuning knobs (defaults chosen from B200 measurements):
+//  COF_TABLE_SMEM_KB     shared-memory budget per CTA for resident guide blocks
+static bool g_uniform_t_enabled = getenv("COF_TABLE_GENERIC") == nullptr;
+static uint32_t table_smem_budget() {
+    static uint32_t v = 0;
+    if (!v) {
+        const char* e = getenv("COF_TABLE_SMEM_KB");
+        v = (e ? (uint32_t)atoi(e) : 72u) * 1024u;
+        if (v < 4096) v = 4096;
     }
-    return r;
+    return v;
 }
+static int table_r() { return R_TABLE; }
 
-template <int NP, int R>
+template <int NP, int R, int TC>
 static cof_status launch_table_r(TableArgs& t, uint64_t n_hint, cudaStream_t stream) {
     // guide blocks resident in shared memory per pass (tiles over blocks if they do not fit)
     const uint32_t per_block = NP * 25 * 8;
     uint32_t bpc = t.n_blocks;
-    const uint32_t budget = 72 * 1024;
-    if (bpc * per_block > budget) bpc = budget / per_block;
+    const uint32_t budget = table_smem_budget();
+    if (bpc * per_block > budget) bpc = std::max<uint32_t>(1, budget / per_block);
     t.blocks_per_chunk = bpc;
     const uint32_t smem = bpc * per_block;
     int bps = 0;
-    auto fn = cof_comparer_table<NP, R>;
+    auto fn = cof_comparer_table<NP, R, TC>;
     cof_status st = occupancy((const void*)fn, smem, &bps);
     if (st != COF_OK) return st;
     uint64_t grid = (uint64_t)num_sms() * bps;
@@ -396,10 +409,25 @@ static cof_status launch_table_r(TableArgs& t, uint64_t n_hint, cudaStream_t str
     return COF_OK;
 }
 
+// Uniform-threshold specializations for the common guide shapes (20-nt SpCas9 guides:
+// 10 pairs; 23-nt Cas12a guides: 12 pairs) and t <= 7; everything else runs the generic
+// per-guide-threshold kernel.
 template <int NP>
-static cof_status launch_table(TableArgs& t, uint64_t n_hint, cudaStream_t stream) {
-    if (table_r() == 4) return launch_table_r<NP, 4>(t, n_hint, stream);
-    return launch_table_r<NP, R_TABLE>(t, n_hint, stream);
+static cof_status launch_table(TableArgs& t, int uniform_t, uint64_t n_hint, cudaStream_t stream) {
+    if constexpr (NP == 10 || NP == 12) {
+        switch (uniform_t) {
+            case 0: return launch_table_r<NP, R_TABLE, 0>(t, n_hint, stream);
+            case 1: return launch_table_r<NP, R_TABLE, 1>(t, n_hint, stream);
+            case 2: return launch_table_r<NP, R_TABLE, 2>(t, n_hint, stream);
+            case 3: return launch_table_r<NP, R_TABLE, 3>(t, n_hint, stream);
+            case 4: return launch_table_r<NP, R_TABLE, 4>(t, n_hint, stream);
+            case 5: return launch_table_r<NP, R_TABLE, 5>(t, n_hint, stream);
+            case 6: return launch_table_r<NP, R_TABLE, 6>(t, n_hint, stream);
+            case 7: return launch_table_r<NP, R_TABLE, 7>(t, n_hint, stream);
+            default: break;
+        }
+    }
+    return launch_table_r<NP, R_TABLE, -1>(t, n_hint, stream);
 }
 
 // One launch per (strand, range of <= MAX_TABLE_BLOCKS guide blocks); thresholds travel in
@@ -407,6 +435,9 @@ static cof_status launch_table(TableArgs& t, uint64_t n_hint, cudaStream_t strea
 static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs& a, cudaStream_t stream) {
     static thread_local TableArgs T;   // ~4.5 KB parameter block, one per calling thread
     const uint32_t np = plan->pairs[0].n_pairs;
+    int ut = g_uniform_t_enabled ? (int)plan->max_mm[0] : -1;   // same threshold for every guide?
+    for (uint32_t i = 1; i < plan->n_guides && ut >= 0; i++)
+        if (plan->max_mm[i] != plan->max_mm[0]) ut = -1;
     for (uint32_t sd = 0; sd < 2; sd++) {
         T.lo = a.lo; T.hi = a.hi; T.nm = a.nm;
         T.items = a.items[sd];
@@ -424,22 +455,22 @@ static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs
                 for (int w = 0; w < 8; w++) T.meta[k][w] = pm[(size_t)(bb + k) * 8 + w];
             cof_status st;
             switch (np) {
-                case 1: st = launch_table<1>(T, T.n, stream); break;
-                case 2: st = launch_table<2>(T, T.n, stream); break;
-                case 3: st = launch_table<3>(T, T.n, stream); break;
-                case 4: st = launch_table<4>(T, T.n, stream); break;
-                case 5: st = launch_table<5>(T, T.n, stream); break;
-                case 6: st = launch_table<6>(T, T.n, stream); break;
-                case 7: st = launch_table<7>(T, T.n, stream); break;
-                case 8: st = launch_table<8>(T, T.n, stream); break;
-                case 9: st = launch_table<9>(T, T.n, stream); break;
-                case 10: st = launch_table<10>(T, T.n, stream); break;
-                case 11: st = launch_table<11>(T, T.n, stream); break;
-                case 12: st = launch_table<12>(T, T.n, stream); break;
-                case 13: st = launch_table<13>(T, T.n, stream); break;
-                case 14: st = launch_table<14>(T, T.n, stream); break;
-                case 15: st = launch_table<15>(T, T.n, stream); break;
-                case 16: st = launch_table<16>(T, T.n, stream); break;
+                case 1: st = launch_table<1>(T, ut, T.n, stream); break;
+                case 2: st = launch_table<2>(T, ut, T.n, stream); break;
+                case 3: st = launch_table<3>(T, ut, T.n, stream); break;
+                case 4: st = launch_table<4>(T, ut, T.n, stream); break;
+                case 5: st = launch_table<5>(T, ut, T.n, stream); break;
+                case 6: st = launch_table<6>(T, ut, T.n, stream); break;
+                case 7: st = launch_table<7>(T, ut, T.n, stream); break;
+                case 8: st = launch_table<8>(T, ut, T.n, stream); break;
+                case 9: st = launch_table<9>(T, ut, T.n, stream); break;
+                case 10: st = launch_table<10>(T, ut, T.n, stream); break;
+                case 11: st = launch_table<11>(T, ut, T.n, stream); break;
+                case 12: st = launch_table<12>(T, ut, T.n, stream); break;
+                case 13: st = launch_table<13>(T, ut, T.n, stream); break;
+                case 14: st = launch_table<14>(T, ut, T.n, stream); break;
+                case 15: st = launch_table<15>(T, ut, T.n, stream); break;
+                case 16: st = launch_table<16>(T, ut, T.n, stream); break;
                 default: return set_error(COF_E_STATE, "cof_compare: %u pairs", np);
             }
             if (st != COF_OK) return st;

@@ -23,13 +23,15 @@
 
 namespace cof {
 
-constexpr int FT = 256;          // threads per CTA; one plane word per thread per tile
-constexpr int FW = 256;          // words per tile (8192 window starts)
+constexpr int FT = 256;          // threads per CTA
+constexpr int FWPT = 2;          // consecutive plane words (x 32 window starts) per thread
+constexpr int FW = FT * FWPT;    // words per tile (16384 window starts)
+constexpr int FSTAGE_ITEMS = 8192;   // shared staging capacity per output round
 constexpr int FSTAGES = 4;       // TMA ring depth
 constexpr int FLOAD = FW + 4;    // words per plane per stage: tile + halo, 16-byte multiple
 constexpr uint32_t FMAX_CTAS = 4096;                      // grid cap (co-residency)
 constexpr size_t FWS_BARRIER = 2 * FMAX_CTAS * sizeof(uint64_t);
-constexpr uint32_t FSMEM = FSTAGES * 3 * FLOAD * 4 + FSTAGES * 8 + FW * 32 * 4;
+constexpr uint32_t FSMEM = FSTAGES * 3 * FLOAD * 4 + FSTAGES * 8 + FSTAGE_ITEMS * 4;
 
 struct FinderArgs {
     const uint32_t* lo;
@@ -169,31 +171,41 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
             const uint32_t tile = t_begin + k;
             const int s = (int)(it % FSTAGES);
             mbar_wait_parity(&bars[s], (it / FSTAGES) & 1u);
-            const uint32_t* Slo = stage + (s * 3 + 0) * FLOAD;
-            const uint32_t* Shi = stage + (s * 3 + 1) * FLOAD;
-            const uint32_t* Snm = stage + (s * 3 + 2) * FLOAD;
-            const uint32_t lo0 = Slo[tid], lo1 = Slo[tid + 1];
-            const uint32_t hi0 = Shi[tid], hi1 = Shi[tid + 1];
-            const uint32_t nm0 = Snm[tid], nm1 = Snm[tid + 1];
+            const uint32_t* Slo = stage + (s * 3 + 0) * FLOAD + FWPT * tid;
+            const uint32_t* Shi = stage + (s * 3 + 1) * FLOAD + FWPT * tid;
+            const uint32_t* Snm = stage + (s * 3 + 2) * FLOAD + FWPT * tid;
+            uint32_t lo[FWPT + 1], hi[FWPT + 1], nm[FWPT + 1];
+#pragma unroll
+            for (int w = 0; w <= FWPT; w++) { lo[w] = Slo[w]; hi[w] = Shi[w]; nm[w] = Snm[w]; }
 
-            const uint64_t p0 = ((uint64_t)tile * FW + tid) * 32;
-            uint32_t valid = ~0u;
-            if (p0 + 32 > a.limit) valid = p0 >= a.limit ? 0u : (1u << (uint32_t)(a.limit - p0)) - 1u;
-            uint32_t m[2];
-            pam_masks<NE>(a, valid, lo0, lo1, hi0, hi1, nm0, nm1, m);
+            const uint64_t p0 = ((uint64_t)tile * FW + FWPT * tid) * 32;   // first start of this thread
+            uint32_t m[2][FWPT];
+#pragma unroll
+            for (int w = 0; w < FWPT; w++) {
+                const uint64_t pw = p0 + 32u * w;
+                uint32_t valid = ~0u;
+                if (pw + 32 > a.limit) valid = pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
+                uint32_t mw[2];
+                pam_masks<NE>(a, valid, lo[w], lo[w + 1], hi[w], hi[w + 1], nm[w], nm[w + 1], mw);
+                m[0][w] = mw[0];
+                m[1][w] = mw[1];
+            }
             __syncthreads();   // every thread has read stage s: refill it
             if (tid == 0 && k + FSTAGES < n_mine) {
                 fence_proxy_async_smem();
                 issue(tile + FSTAGES, s);
             }
+            uint32_t cf = 0, cr = 0;
+#pragma unroll
+            for (int w = 0; w < FWPT; w++) { cf += (uint32_t)__popc(m[0][w]); cr += (uint32_t)__popc(m[1][w]); }
             if (pass == 0) {
-                cnt_f += (unsigned)__popc(m[0]);
-                cnt_r += (unsigned)__popc(m[1]);
+                cnt_f += cf;
+                cnt_r += cr;
                 continue;
             }
 
             // ---- pass 2: CTA exclusive scan of packed counts (fwd bits 0..15, rev 16..31)
-            const uint32_t cnt = (uint32_t)__popc(m[0]) | ((uint32_t)__popc(m[1]) << 16);
+            const uint32_t cnt = cf | (cr << 16);
             uint32_t x = cnt;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -216,25 +228,48 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
             __syncthreads();
             const uint32_t local = s_warp[warp] + x - cnt;
             const uint32_t tot = s_tile_tot;
+            const uint32_t pbase = (uint32_t)p0;
 #pragma unroll
             for (int st = 0; st < 2; st++) {
-                uint32_t off = st == 0 ? (local & 0xFFFFu) : (local >> 16);
-                uint32_t mm = m[st];
-                const uint32_t pbase = (uint32_t)p0;
-                while (mm) {
-                    const int b = __ffs(mm) - 1;
-                    items[off++] = pbase + (uint32_t)b;
-                    mm &= mm - 1;
-                }
-                __syncthreads();
                 const uint32_t total = st == 0 ? (tot & 0xFFFFu) : (tot >> 16);
+                const uint32_t first = st == 0 ? (local & 0xFFFFu) : (local >> 16);
                 const unsigned long long base = s_base[st] + (st == 0 ? run_f : run_r);
                 uint32_t* out = a.out[st];
-                for (uint32_t i = tid; i < total; i += FT) {
-                    const unsigned long long o = base + i;
-                    if (o < a.cap) out[o] = items[i];
+                // staged in rounds of FSTAGE_ITEMS (one round unless the pattern is very permissive)
+                for (uint32_t r0 = 0; r0 < total; r0 += FSTAGE_ITEMS) {
+                    if (total <= FSTAGE_ITEMS) {
+                        uint32_t off = first;
+#pragma unroll
+                        for (int w = 0; w < FWPT; w++) {
+                            uint32_t mm = m[st][w];
+                            while (mm) {
+                                const int b = __ffs(mm) - 1;
+                                items[off++] = pbase + 32u * w + (uint32_t)b;
+                                mm &= mm - 1;
+                            }
+                        }
+                    } else {
+                        uint32_t rank = first;
+#pragma unroll
+                        for (int w = 0; w < FWPT; w++) {
+                            uint32_t mm = m[st][w];
+                            while (mm) {
+                                const int b = __ffs(mm) - 1;
+                                if (rank >= r0 && rank < r0 + FSTAGE_ITEMS) items[rank - r0] = pbase + 32u * w + (uint32_t)b;
+                                rank++;
+                                mm &= mm - 1;
+                            }
+                        }
+                    }
+                    __syncthreads();
+                    uint32_t n_round = min(total - r0, (uint32_t)FSTAGE_ITEMS);
+                    const unsigned long long o0 = base + r0;
+                    if (o0 >= a.cap) n_round = 0;
+                    else if (a.cap - o0 < n_round) n_round = (uint32_t)(a.cap - o0);
+                    uint32_t* __restrict__ dst = out + o0;
+                    for (uint32_t i = tid; i < n_round; i += FT) dst[i] = items[i];
+                    __syncthreads();
                 }
-                __syncthreads();
             }
             run_f += tot & 0xFFFFu;
             run_r += tot >> 16;

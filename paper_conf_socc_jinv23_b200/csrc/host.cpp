@@ -82,10 +82,10 @@ const char* cof_version(void) { return "cof-b200 0.1 (sm_100a)"; }
 uint64_t cof_launch_count(void) { return g_launches.load(); }
 
 uint64_t cof_plane_words(uint64_t n_bases) {
-    // ceil(n/32) data words, rounded up to a finder tile (256 words), + 4 pad words so the
+    // ceil(n/32) data words, rounded up to a finder tile (512 words), + 4 pad words so the
     // finder's 16-byte-granular bulk copies of (tile + halo) never leave the allocation.
     uint64_t w = (n_bases + 31) / 32;
-    return ((w + 255) / 256) * 256 + 4;
+    return ((w + 511) / 512) * 512 + 4;
 }
 
 cof_status cof_pack(const char* ascii, uint64_t n, uint32_t* lo, uint32_t* hi, uint32_t* nm) {
@@ -282,34 +282,41 @@ cof_status cof_fasta_pack(const cof_fasta* fa, uint32_t i, uint64_t first, uint6
 // planes: '+' reads the window, '-' reads its reverse complement (G6); a compared letter
 // is lower-cased where the genome base is not in the guide letter's IUPAC set (G19).
 static cof_status decorate(const cof_plan* plan, const cof_chunk* host, uint64_t key, cof_hit* h) {
-    static const char B[4] = {'A', 'C', 'G', 'T'};
-    static const char C[5] = {'T', 'G', 'C', 'A', 'N'};
+    // char of a (code | N << 2 | mismatch << 3) index: ACGT/N, lower-cased when mismatched
+    static const char CH[16] = {'A', 'C', 'G', 'T', 'N', 'N', 'N', 'N', 'a', 'c', 'g', 't', 'n', 'n', 'n', 'n'};
     const uint32_t L = plan->L;
-    uint64_t pos = key >> 32;
-    uint32_t strand = (uint32_t)(key >> 31) & 1u;
-    uint32_t guide = (uint32_t)(key >> 7) & 0xFFFFFFu;
-    uint32_t mm = (uint32_t)key & 127u;
+    const uint64_t pos = key >> 32;
+    const uint32_t strand = (uint32_t)(key >> 31) & 1u;
+    const uint32_t guide = (uint32_t)(key >> 7) & 0xFFFFFFu;
+    const uint32_t mm = (uint32_t)key & 127u;
     if (guide >= plan->n_guides || pos + L > host->n_bases) return COF_E_STATE;
-    int code[32];
-    for (uint32_t j = 0; j < L; j++) {
-        uint64_t p = pos + j;
-        uint64_t w = p >> 5;
-        int b = (int)(p & 31);
-        code[j] = (host->nm[w] >> b & 1) ? 4 : (int)(((host->lo[w] >> b) & 1) | (((host->hi[w] >> b) & 1) << 1));
+    // the L-base window as 32-bit slices of the three planes (bit j = base pos + j)
+    const uint64_t w = pos >> 5;
+    const uint32_t sh = (uint32_t)(pos & 31);
+    auto win = [&](const uint32_t* pl) -> uint32_t {
+        const uint64_t v = ((uint64_t)pl[w + 1] << 32) | pl[w];
+        return (uint32_t)(v >> sh);
+    };
+    const uint32_t lo = win(host->lo), hi = win(host->hi), nm = win(host->nm);
+    // mismatched window offsets against the guide in this strand's orientation (bit-parallel)
+    const uint32_t* oh = &plan->onehot[((size_t)strand * plan->n_guides + guide) * 5];
+    const uint32_t match = (~lo & ~hi & ~nm & oh[0]) | (lo & ~hi & ~nm & oh[1]) | (~lo & hi & ~nm & oh[2]) |
+                           (lo & hi & ~nm & oh[3]);
+    const uint32_t mis = oh[4] & ~match;
+    if ((uint32_t)__builtin_popcount(mis) != mm) return COF_E_STATE;
+    // site read along the strand (G6): '+' = window offset j, '-' = complement of offset L-1-j
+    if (strand == 0) {
+        for (uint32_t j = 0; j < L; j++)
+            h->site[j] = CH[((lo >> j) & 1u) | (((hi >> j) & 1u) << 1) | (((nm >> j) & 1u) << 2) | (((mis >> j) & 1u) << 3)];
+    } else {
+        for (uint32_t j = 0; j < L; j++) {
+            const uint32_t k = L - 1 - j;
+            // complement of code c is 3 - c (= c ^ 3); N stays N
+            h->site[j] = CH[((((lo >> k) & 1u) | (((hi >> k) & 1u) << 1)) ^ 3u) | (((nm >> k) & 1u) << 2) |
+                            (((mis >> k) & 1u) << 3)];
+        }
     }
-    const uint8_t* gm = &plan->gmask[(size_t)guide * L];
-    uint32_t recount = 0;
-    for (uint32_t j = 0; j < L; j++) {
-        int c = strand == 0 ? code[j] : (code[L - 1 - j] == 4 ? 4 : 3 - code[L - 1 - j]);
-        char ch = c == 4 ? 'N' : B[c];
-        (void)C;
-        bool mis = gm[j] != 15 && (c == 4 || !((gm[j] >> c) & 1));
-        if (mis) { recount++; ch = (char)(ch + 32); }
-        h->site[j] = ch;
-    }
-    h->site[L] = 0;
-    for (uint32_t j = L + 1; j < sizeof h->site; j++) h->site[j] = 0;
-    if (recount != mm) return COF_E_STATE;
+    memset(h->site + L, 0, sizeof h->site - L);
     h->guide = guide;
     h->chrom = host->chrom;
     h->pos = host->start + pos;
@@ -363,6 +370,32 @@ cof_status cof_merge(const cof_hit* const* lists, const uint64_t* lens, uint32_t
         total += lens[i];
     }
     if (total && !out) return set_error(COF_E_ARG, "cof_merge: out is NULL");
+    // fast path: non-empty lists already in global order (disjoint chunks in genome order)
+    {
+        bool ordered = true;
+        const cof_hit* prev = nullptr;
+        for (uint32_t i = 0; i < n_lists && ordered; i++) {
+            if (!lens[i]) continue;
+            if (prev && !hit_less(*prev, lists[i][0])) ordered = false;
+            prev = &lists[i][lens[i] - 1];
+        }
+        if (ordered) {
+            std::vector<uint64_t> at(n_lists + 1, 0);
+            for (uint32_t i = 0; i < n_lists; i++) at[i + 1] = at[i] + lens[i];
+            const int64_t CH = 1 << 16;   // records per copy task
+            std::vector<std::pair<uint32_t, uint64_t>> tasks;
+            for (uint32_t i = 0; i < n_lists; i++)
+                for (uint64_t k = 0; k < lens[i]; k += CH) tasks.push_back({i, k});
+#pragma omp parallel for schedule(dynamic, 4)
+            for (int64_t t = 0; t < (int64_t)tasks.size(); t++) {
+                const uint32_t i = tasks[t].first;
+                const uint64_t k = tasks[t].second;
+                const uint64_t n = std::min<uint64_t>(CH, lens[i] - k);
+                memcpy(out + at[i] + k, lists[i] + k, n * sizeof(cof_hit));
+            }
+            return COF_OK;
+        }
+    }
     // k-way merge with a min-heap of list heads (stable across lists for equal keys)
     typedef std::pair<uint32_t, uint64_t> Head;   // (list, index)
     auto cmp = [&](const Head& x, const Head& y) {

@@ -86,6 +86,18 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
         return s == 0 ? p->gmask[(size_t)i * L + j] : comp_mask(p->gmask[(size_t)i * L + (L - 1 - j)]);
     };
 
+    // ---- host decoration: one-hot membership masks per guide and strand (window offsets)
+    p->onehot.assign((size_t)2 * n_guides * 5, 0u);
+    for (int s = 0; s < 2; s++)
+        for (uint32_t i = 0; i < n_guides; i++) {
+            uint32_t* oh = &p->onehot[((size_t)s * n_guides + i) * 5];
+            for (uint32_t j = 0; j < L; j++) {
+                const uint8_t m = gm(s, i, j);
+                for (int b = 0; b < 4; b++) oh[b] |= (uint32_t)((m >> b) & 1u) << j;
+                if (m != 15) oh[4] |= 1u << j;
+            }
+        }
+
     // ---- v1 comparer: group guides by (care mask, kind); records per strand
     std::map<std::pair<uint32_t, uint32_t>, std::vector<uint32_t>> groups;  // (care_fwd, kind) -> guides
     for (uint32_t i = 0; i < n_guides; i++) {

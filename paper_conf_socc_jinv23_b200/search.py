@@ -140,22 +140,103 @@ class Searcher:
                           self.d_sort_ws, s)
         return nf, nr, nh
 
-    def search_host(self, host: HostGenome, indices=None):
-        """End-to-end over host-resident packed chunks: H2D, find, compare, sort, D2H +
-        decorate (cof_collect); returns the merged, sorted hit array."""
-        idx = range(len(host.chunks)) if indices is None else indices
+    def search_host(self, host: HostGenome, indices=None, out=None):
+        """End-to-end over host-resident packed chunks.  Per chunk: H2D on a copy stream
+        (double-buffered device planes, overlapping the previous chunk's kernels), find,
+        compare, device sort and an async D2H of the sorted keys; a host thread decorates
+        chunk i (cof_collect, OpenMP) while the GPU works on chunk i+1.
+
+        Returns the sorted hit array.  If ``out`` (a ``cof.HIT_DTYPE`` array) is large
+        enough, each chunk is decorated straight into its slice of ``out`` (chunks are
+        disjoint and in genome order, so no merge copy is needed) and a view of ``out`` is
+        returned; otherwise per-chunk arrays are merged with cof_merge."""
+        import queue
+        import threading
+
+        idx = list(range(len(host.chunks)) if indices is None else indices)
         max_bases = max((host.chunks[i].n_bases for i in idx), default=1)
         self.reserve(max_bases, max(self._hits_cap, 1 << 16))
-        out = []
-        with torch.cuda.device(self.device):
-            for i in idx:
-                hch = host.chunk_struct(i)
-                dch = self.device_chunk(host.chunks[i])
-                cof.cof_load_chunk(hch, dch, self.stream)
-                _, _, nh = self.run_device_chunk(dch, host.chunks[i].n_owned)
-                out.append(cof.cof_collect(self.plan, hch, self.d_hits, nh, self.stream))
-        return merge_hit_lists(out)
+        if not hasattr(self, "d_planes2") or self.d_planes2.shape != self.d_planes.shape:
+            self.d_planes2 = torch.empty_like(self.d_planes)
+            self.copy_stream = torch.cuda.Stream(self.device)
+        planes = [self.d_planes, self.d_planes2]
+        results = {}
+        errors = []
+        work = queue.Queue()
+        ordered = all(a < b for a, b in zip(idx, idx[1:]))
+        use_out = out is not None and ordered
 
+        def collector():
+            while True:
+                job = work.get()
+                if job is None:
+                    return
+                i, ev, keys, nh, dst = job
+                try:
+                    ev.synchronize()
+                    if dst is not None:
+                        if nh:
+                            cof.cof_collect_into(self.plan, host.chunk_struct(i), keys, nh, dst)
+                        results[i] = dst
+                    else:
+                        results[i] = cof.cof_collect(self.plan, host.chunk_struct(i), None, nh, host_keys=keys)
+                except Exception as e:      # surfaced after the join
+                    errors.append(e)
+
+        th = threading.Thread(target=collector, daemon=True)
+        th.start()
+        total = 0
+        overflow = False
+        try:
+            with torch.cuda.device(self.device):
+                loaded = [None, None]          # events: planes buffer k loaded
+                freed = [None, None]           # events: compute done with planes buffer k
+
+                def load(j, k):
+                    with torch.cuda.stream(self.copy_stream):
+                        if freed[k] is not None:
+                            self.copy_stream.wait_event(freed[k])
+                        dch = self.device_chunk(host.chunks[idx[j]], planes[k])
+                        cof.cof_load_chunk(host.chunk_struct(idx[j]), dch, self.copy_stream)
+                        ev = torch.cuda.Event()
+                        ev.record(self.copy_stream)
+                        loaded[k] = ev
+                        return dch
+
+                dchs = [None, None]
+                if idx:
+                    dchs[0] = load(0, 0)
+                for j, i in enumerate(idx):
+                    k = j & 1
+                    self.stream.wait_event(loaded[k])
+                    if j + 1 < len(idx):
+                        dchs[(j + 1) & 1] = load(j + 1, (j + 1) & 1)
+                    _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned)
+                    fr = torch.cuda.Event()
+                    fr.record(self.stream)
+                    freed[k] = fr
+                    keys = torch.empty(max(nh, 1), dtype=torch.int64, pin_memory=True)
+                    with torch.cuda.stream(self.stream):
+                        if nh:
+                            keys[:nh].copy_(self.d_hits[:nh], non_blocking=True)
+                        ev = torch.cuda.Event()
+                        ev.record(self.stream)
+                    dst = None
+                    if use_out and not overflow:
+                        if total + nh <= len(out):
+                            dst = out[total:total + nh]
+                        else:
+                            overflow = True
+                    total += nh
+                    work.put((i, ev, keys.numpy().view(np.uint64), nh, dst))
+        finally:
+            work.put(None)
+            th.join()
+        if errors:
+            raise errors[0]
+        if use_out and not overflow:
+            return out[:total]
+        return merge_hit_lists([results[i] for i in idx])
 
 def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda"):
     """Convenience: whole search of ``seqs`` (list of uint8 ASCII arrays / bytes) on one GPU."""

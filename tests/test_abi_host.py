@@ -37,7 +37,7 @@ def test_version_and_counter():
 def test_plane_words():
     for n in (0, 1, 31, 32, 33, 8191, 8192, 8193, 10**6):
         w = cof.cof_plane_words(n)
-        assert w >= (n + 31) // 32 + 1 and (w - 4) % 256 == 0
+        assert w >= (n + 31) // 32 + 1 and (w - 4) % 512 == 0
 
 
 def _canon(b: bytes) -> bytes:

@@ -178,3 +178,20 @@ def test_full_size_sampled_c5():
         else:
             assert key not in found
     assert n_samples >= 20
+
+
+def test_search_host_into_caller_buffer_and_chunk_pipeline():
+    """The pipelined public path (double-buffered H2D, overlapped host decoration) writing
+    straight into a caller buffer equals the oracle; a too-small buffer falls back to merge."""
+    w = synth.make_workload("C3", scale=0.003, n_guides=40)
+    cfg = w.cfg
+    exp = ref_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
+    chunks = search.plan_chunks([len(s) for s in w.seqs], cfg.L, 200_003)
+    host = search.HostGenome(w.seqs, chunks)
+    srch = search.Searcher(cfg.pattern, w.guides, w.thresholds)
+    out = np.empty(len(exp) + 10, dtype=cof.HIT_DTYPE)
+    got = srch.search_host(host, out=out)
+    assert got.base is out or np.shares_memory(got, out)
+    assert cof.hits_to_tuples(got) == exp
+    small = np.empty(max(1, len(exp) // 3), dtype=cof.HIT_DTYPE)
+    assert cof.hits_to_tuples(srch.search_host(host, out=small)) == exp
