@@ -33,6 +33,9 @@ sys.path.insert(0, ROOT)
 from paper_conf_socc_jinv23_b200 import synth  # noqa: E402
 
 
+E2E_CHUNK_BASES = 250_000_000   # e2e: chromosomes packed into chunks of <= this many bases
+
+
 def _peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -105,8 +108,8 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
 
     wl = synth.make_workload(name, scale=scale, threads=max(1, min(16, os.cpu_count() or 1)))
     L = wl.cfg.L
-    all_chunks = search.plan_chunks([len(s) for s in wl.seqs], L, None)
-    chunks = all_chunks if chunks is None else chunks
+    if chunks is None:   # the whole genome as one multi-segment chunk (the bench's default)
+        chunks = [search.pack_shard(search.plan_chunks([len(s) for s in wl.seqs], L, None))]
     st = type("State", (), {})()
     st.device = device or torch.device("cuda", torch.cuda.current_device())
     st.stream = torch.cuda.current_stream(st.device)
@@ -118,7 +121,10 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
     for i, ch in enumerate(chunks):
         d = st.host.planes[i].to(st.device, non_blocking=True)
         st.d_planes.append(d)
-        st.d_chunks.append(cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, d[0], d[1], d[2]))
+        if ch.multi:
+            st.d_chunks.append(cof.make_chunk(0, 0, ch.n_bases, ch.n_owned, d[0], d[1], d[2], d[3], st.host.segs[i]))
+        else:
+            st.d_chunks.append(cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, d[0], d[1], d[2]))
         pd = torch.empty(nbytes + 256, dtype=torch.uint8, device=st.device)
         cof.cof_plan_upload(st.plan, pd, st.stream)
         st.plan_devs.append(pd)
@@ -197,9 +203,9 @@ def step_counts(st):
 def run_e2e_step(wl, st, searcher, out=None):
     """Public-API end-to-end step from pinned host planes; returns (hits, h2d, d2h bytes).
     ``out``: the caller's result buffer (reused between steps, as an application would)."""
-    hits = searcher.search_host(st.host, out=out)
-    h2d = st.host.bytes
-    d2h = len(hits) * 8 + 24 * len(st.chunks)      # sorted keys + per-chunk counts
+    hits = searcher.search_host(st.e2e_host, out=out)
+    h2d = st.e2e_host.bytes
+    d2h = len(hits) * 8 + 24 * len(st.e2e_host.chunks)      # sorted keys + per-chunk counts
     return hits, h2d, d2h
 
 
@@ -271,7 +277,7 @@ def main():
     L = cfg.L
     all_chunks = search.plan_chunks([l for _, l in cfg.genome.chroms], L, None)
     shards = search.shard_lpt(all_chunks, world)
-    mine = shards[rank]
+    mine = [search.pack_shard(shards[rank])]          # this rank's chromosomes as ONE chunk
     wl, st = prepare_workload(cfgname, args.scale, chunks=mine, device=dev)
     genome_bases = wl.total_bases
     my_items = sum(c[0] + c[1] for c in st.counts)
@@ -353,7 +359,9 @@ def main():
             "comparisons_per_s": comps_s, "hits_per_step": int(hits_all), "items_per_step": int(items_all),
             "config": {"workload": cfgname, "description": cfg.description, "genome_bases": genome_bases,
                        "chromosomes": len(wl.seqs), "guides": len(wl.guides), "threshold": cfg.threshold,
-                       "pattern": cfg.pattern, "chunking": "whole chromosome per chunk",
+                       "pattern": cfg.pattern,
+                       "chunking": "device: this rank's chromosomes as one multi-segment chunk; "
+                                   "e2e: packed chunks of <= 250 Mbp, pipelined",
                        "parallelism": f"chromosome LPT shards over {world} GPU(s)",
                        "comparer": args.comparer,
                        "l2": "inputs larger than L2 (1.16 GB planes + item lists), no flush"},
@@ -416,8 +424,10 @@ def measure_e2e(wl, st, dev, args, world, genome_bases):
     import torch
     import torch.distributed as dist
     from paper_conf_socc_jinv23_b200 import search
+    chunks = search.pack_pieces([p for ch in st.chunks for p in ch.pieces], E2E_CHUNK_BASES)
+    st.e2e_host = search.HostGenome(wl.seqs, chunks)
     srch = search.Searcher(wl.cfg.pattern, wl.guides, wl.thresholds, device=dev)
-    srch.reserve(max(ch.n_bases for ch in st.chunks), max(st.caps))
+    srch.reserve(max(ch.n_bases for ch in chunks), max(st.caps))
     from paper_conf_socc_jinv23_b200 import cof
     hits0, _, _ = run_e2e_step(wl, st, srch)     # warm-up; sizes the caller's result buffer
     out = np.empty(int(len(hits0) * 1.05) + 1024, dtype=cof.HIT_DTYPE)

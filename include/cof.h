@@ -76,20 +76,39 @@ size_t     cof_plan_device_bytes(const cof_plan *plan);
 cof_status cof_plan_upload(const cof_plan *plan, void *plan_dev, cof_stream s);
 
 /* ------------------------------------------------------------------ chunk (M3, M4)
- * One chunk of one chromosome: window starts [start, start + n_owned) belong to it,
- * and it holds bases [start, start + n_bases) with n_bases = min(n_owned + L - 1,
- * chrom_len - start) (chunks overlap by L-1, reading G12).  The genome is stored as
- * three bit-planes of uint32 words (bit p&31 of word p>>5 is base p): lo/hi = 2-bit
- * code A=00 C=01 G=10 T=11 (lo = bit 0), nm = 1 for any non-ACGT letter (then lo=hi=0),
- * reading G2/G4; the "2-bit sequence format" of P:L289.  Each plane has
- * cof_plane_words(n_bases) words; words past the last base have nm = all-ones. */
+ * A chunk is the unit the device works on ("divides the genome data into chunks that
+ * can fit the memory of a heterogeneous device").  It holds n_bases bases stored as three
+ * bit-planes of uint32 words (bit p&31 of word p>>5 is base p): lo/hi = 2-bit code A=00
+ * C=01 G=10 T=11 (lo = bit 0), nm = 1 for any non-ACGT letter (then lo=hi=0), readings
+ * G2/G4; the "2-bit sequence format" of P:L289.  Each plane has cof_plane_words(n_bases)
+ * words; words past the last base have nm = all-ones.  Positions inside a chunk are
+ * chunk coordinates (< 2^32).
+ *
+ * Single-segment chunk (n_segs == 0): bases [start, start + n_bases) of chromosome `chrom`;
+ * window starts [0, n_owned) belong to it, n_bases = min(n_owned + L - 1, chrom_len - start)
+ * (chunks of one chromosome overlap by L-1, reading G12).
+ * Multi-segment chunk (n_segs > 0): several chromosome pieces laid back to back (e.g. a
+ * whole genome or one GPU's shard); segs[k] (HOST array, ascending chunk_off) says which
+ * chromosome piece starts at chunk offset chunk_off and which window starts it owns; vs is
+ * the valid-start plane (bit p = 1 iff start p is owned, see cof_valid_starts), so no window
+ * spanning two pieces is ever reported. */
 typedef struct {
-    uint32_t chrom;        /* chromosome index (FASTA / caller order) */
+    uint32_t chrom;        /* chromosome index */
     uint32_t reserved;
-    uint64_t start;        /* 0-based chromosome offset of base 0 of this chunk */
+    uint64_t chunk_off;    /* chunk offset of the piece's first base */
+    uint64_t chrom_off;    /* chromosome offset of that base */
+    uint64_t n_owned;      /* window starts [chunk_off, chunk_off + n_owned) belong to the chunk */
+} cof_segment;
+
+typedef struct {
+    uint32_t chrom;        /* single-segment: chromosome index (FASTA / caller order) */
+    uint32_t n_segs;       /* 0 = single segment; else number of entries in segs */
+    uint64_t start;        /* single-segment: 0-based chromosome offset of base 0 */
     uint64_t n_bases;
-    uint64_t n_owned;
+    uint64_t n_owned;      /* owned window starts (single: [0, n_owned); multi: total) */
     uint32_t *lo, *hi, *nm;
+    uint32_t *vs;          /* multi-segment: valid-start plane (same word count); else NULL */
+    const cof_segment *segs;   /* multi-segment: HOST segment table (collect, valid starts) */
 } cof_chunk;
 
 uint64_t   cof_plane_words(uint64_t n_bases);
@@ -99,9 +118,13 @@ cof_status cof_pack(const char *ascii, uint64_t n, uint32_t *lo, uint32_t *hi, u
 /* Host unpack (inverse, canonical form: "ACGTN" upper-case), for checks and output. */
 cof_status cof_unpack(const uint32_t *lo, const uint32_t *hi, const uint32_t *nm,
                       uint64_t first, uint64_t n, char *ascii);
-/* Async H2D of the three host planes into dev->lo/hi/nm (device buffers of
- * cof_plane_words(host->n_bases) words each); copies the metadata fields too.
- * ("divides the genome data into chunks that can fit the memory"; Table III.) */
+/* Valid-start plane of a multi-segment chunk: bit p = 1 iff p lies in
+ * [segs[k].chunk_off, segs[k].chunk_off + segs[k].n_owned) for some k (host, OpenMP).
+ * vs has cof_plane_words(n_bases) words.  COF_E_ARG if a segment leaves the chunk. */
+cof_status cof_valid_starts(const cof_segment *segs, uint32_t n_segs, uint64_t n_bases, uint32_t *vs);
+/* Async H2D of the host planes (and vs, if both chunks have one) into the device buffers
+ * of dev (cof_plane_words(host->n_bases) words each); copies the metadata fields and the
+ * segs pointer too.  (Table III.) */
 cof_status cof_load_chunk(const cof_chunk *host, cof_chunk *dev, cof_stream s);
 
 /* ------------------------------------------------------------------ FASTA (M2)
@@ -119,7 +142,8 @@ cof_status cof_fasta_pack(const cof_fasta *fa, uint32_t i, uint64_t first, uint6
 
 /* ------------------------------------------------------------------ finder (M5, M6)
  * The "search" kernel (signature Table VI): for every owned window
- * start p with p+L <= n_bases, '+' passes iff every non-N pattern letter P[j] contains
+ * start p (single segment: p < n_owned; multi: vs bit set) with p+L <= n_bases, '+'
+ * passes iff every non-N pattern letter P[j] contains
  * base(p+j); '-' passes iff the reverse-complemented pattern does (G3, G10).  Passing
  * starts are compacted in ascending order into one list per strand (chunk-relative
  * uint32).  The paper compacts with an unordered atomic counter (Table V);
@@ -169,7 +193,8 @@ cof_status cof_read_counts(const cof_plan *plan, const void *plan_dev, uint64_t 
                            cof_stream s);
 
 /* ------------------------------------------------------------------ collect (M10)
- * One output record: guide index, chromosome, 0-based '+'-strand position (G5),
+ * One output record: guide index, chromosome, 0-based '+'-strand chromosome
+ * position (G5; chunk coordinates are mapped back through the segment table),
  * direction, #mismatches, and the L-letter site read along its strand (G6) with
  * mismatched compared letters in lower case (G19). */
 typedef struct {

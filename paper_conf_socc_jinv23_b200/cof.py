@@ -33,10 +33,16 @@ class CofError(RuntimeError):
         self.status = status
 
 
+class cof_segment(ctypes.Structure):
+    _fields_ = [("chrom", ctypes.c_uint32), ("reserved", ctypes.c_uint32), ("chunk_off", ctypes.c_uint64),
+                ("chrom_off", ctypes.c_uint64), ("n_owned", ctypes.c_uint64)]
+
+
 class cof_chunk(ctypes.Structure):
-    _fields_ = [("chrom", ctypes.c_uint32), ("reserved", ctypes.c_uint32), ("start", ctypes.c_uint64),
+    _fields_ = [("chrom", ctypes.c_uint32), ("n_segs", ctypes.c_uint32), ("start", ctypes.c_uint64),
                 ("n_bases", ctypes.c_uint64), ("n_owned", ctypes.c_uint64),
-                ("lo", ctypes.c_void_p), ("hi", ctypes.c_void_p), ("nm", ctypes.c_void_p)]
+                ("lo", ctypes.c_void_p), ("hi", ctypes.c_void_p), ("nm", ctypes.c_void_p),
+                ("vs", ctypes.c_void_p), ("segs", ctypes.c_void_p)]
 
 
 def _load():
@@ -59,6 +65,7 @@ def _load():
         "cof_pack": (I32, [P, U64, P, P, P]),
         "cof_unpack": (I32, [P, P, P, U64, U64, P]),
         "cof_load_chunk": (I32, [P, P, P]),
+        "cof_valid_starts": (I32, [P, U32, U64, P]),
         "cof_fasta_open": (I32, [ctypes.c_char_p, P]),
         "cof_fasta_close": (None, [P]),
         "cof_fasta_count": (U32, [P]),
@@ -88,7 +95,7 @@ lib = _load()
 EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof_plan_create",
                        "cof_plan_destroy", "cof_plan_length", "cof_plan_n_guides",
                        "cof_plan_device_bytes", "cof_plan_upload", "cof_plane_words", "cof_pack",
-                       "cof_unpack", "cof_load_chunk", "cof_fasta_open", "cof_fasta_close",
+                       "cof_unpack", "cof_valid_starts", "cof_load_chunk", "cof_fasta_open", "cof_fasta_close",
                        "cof_fasta_count", "cof_fasta_name", "cof_fasta_length", "cof_fasta_pack",
                        "cof_find_workspace_bytes", "cof_find_pam", "cof_compare",
                        "cof_sort_workspace_bytes", "cof_sort_hits", "cof_read_counts",
@@ -188,8 +195,24 @@ def cof_unpack(lo, hi, nm, first, n, out):
     _check(lib.cof_unpack(_ptr(lo), _ptr(hi), _ptr(nm), int(first), int(n), _ptr(out)))
 
 
-def make_chunk(chrom, start, n_bases, n_owned, lo, hi, nm) -> cof_chunk:
-    return cof_chunk(int(chrom), 0, int(start), int(n_bases), int(n_owned), _ptr(lo), _ptr(hi), _ptr(nm))
+def make_chunk(chrom, start, n_bases, n_owned, lo, hi, nm, vs=None, segs=None) -> cof_chunk:
+    """Single-segment chunk (segs None) or multi-segment chunk (segs = cof_segment array, vs plane)."""
+    c = cof_chunk(int(chrom), 0 if segs is None else len(segs), int(start), int(n_bases), int(n_owned),
+                  _ptr(lo), _ptr(hi), _ptr(nm), _ptr(vs), None if segs is None else ctypes.addressof(segs))
+    c._keep = segs          # the host segment table must outlive the struct
+    return c
+
+
+def make_segments(rows):
+    """rows = [(chrom, chunk_off, chrom_off, n_owned), ...] -> cof_segment array."""
+    arr = (cof_segment * max(len(rows), 1))()
+    for k, (c, co, so, no) in enumerate(rows):
+        arr[k] = cof_segment(int(c), 0, int(co), int(so), int(no))
+    return arr
+
+
+def cof_valid_starts(segs, n_segs, n_bases, vs):
+    _check(lib.cof_valid_starts(ctypes.addressof(segs), int(n_segs), int(n_bases), _ptr(vs)))
 
 
 def cof_load_chunk(host: cof_chunk, dev: cof_chunk, stream=None):

@@ -53,9 +53,11 @@ struct GroupDesc {
 // the pair table (NP pairs, 25 entries each).  The 16 ACGT combos of a pair are 16
 // consecutive 8-byte entries (128 bytes = every shared-memory bank exactly once, so a
 // half-warp of lookups into one pair never conflicts); the 9 rare N combos of all pairs
-// follow in a separate region.
+// follow in a separate region.  Inside the 16 the index is lo(b1) | lo(b2)<<1 | hi(b1)<<2 |
+// hi(b2)<<3 (lo/hi = the two bits of the 2-bit code): for two adjacent window positions
+// that is one nibble of (lo-plane bits | hi-plane bits << 2), see the comparer's fast path.
 COF_HD uint32_t pair_entry(uint32_t np, uint32_t q, uint32_t b1, uint32_t b2) {
-    if (b1 < 4 && b2 < 4) return q * 16u + b1 * 4u + b2;
+    if (b1 < 4 && b2 < 4) return q * 16u + ((b1 & 1u) | ((b2 & 1u) << 1) | ((b1 >> 1) << 2) | ((b2 >> 1) << 3));
     return np * 16u + q * 9u + (b1 == 4 ? b2 : 5u + b1);
 }
 
@@ -64,6 +66,8 @@ COF_HD uint32_t pair_entry(uint32_t np, uint32_t q, uint32_t b1, uint32_t b2) {
 struct PairLayout {
     uint32_t n_pairs;          // pairs covering the union of compared positions
     uint8_t j1[16], j2[16];    // window offsets of the pair (j2 == 0xFF: single position)
+    uint32_t contig;           // 1: compared positions are the contiguous range [p0, p0 + n_cmp)
+    uint32_t p0, n_cmp;        //    so pair q = window offsets (p0 + 2q, p0 + 2q + 1)
 };
 
 // Device plan image layout (byte offsets from plan_dev; all 256-byte aligned)

@@ -314,7 +314,30 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constan
             const uint64_t idx = item0 + (uint64_t)r * CT;
             okm[r] = idx < n ? ~0u : 0u;
             const uint32_t pos = idx < n ? __ldg(a.items + idx) : 0u;
-            pair_offsets<NP>(a.pairs, plane_window(a.lo, pos), plane_window(a.hi, pos), plane_window(a.nm, pos), off[r]);
+            bool done = false;
+            if (a.pairs.contig) {
+                // fast path: window starting at the first compared offset; with no N among the
+                // compared positions every pair index is one nibble of Y (even pairs) or Z (odd)
+                const uint32_t p = pos + a.pairs.p0;
+                const uint32_t wn = plane_window(a.nm, p);
+                const uint32_t cm = a.pairs.n_cmp >= 32 ? ~0u : ((1u << a.pairs.n_cmp) - 1u);
+                if ((wn & cm) == 0) {
+                    const uint32_t wl = plane_window(a.lo, p), wh = plane_window(a.hi, p);
+                    const uint32_t Y = (wl & 0x33333333u) | ((wh & 0x33333333u) << 2);
+                    const uint32_t Z = ((wl >> 2) & 0x33333333u) | (wh & 0xCCCCCCCCu);
+#pragma unroll
+                    for (int q = 0; q < NP; q++) {
+                        const uint32_t src = (q & 1) ? Z : Y;
+                        const int k = q >> 1;
+                        const uint32_t nib8 = k == 0 ? (src << 3) & 0x78u : (src >> (4 * k - 3)) & 0x78u;
+                        off[r][q] = (uint32_t)q * 128u + nib8;
+                    }
+                    done = true;
+                }
+            }
+            if (!done)
+                pair_offsets<NP>(a.pairs, plane_window(a.lo, pos), plane_window(a.hi, pos), plane_window(a.nm, pos),
+                                 off[r]);
         }
         for (uint32_t ch = 0; ch < n_chunks; ch++) {
             const uint32_t b0 = ch * bpc;

@@ -31,13 +31,15 @@ constexpr int FSTAGES = 4;       // TMA ring depth
 constexpr int FLOAD = FW + 4;    // words per plane per stage: tile + halo, 16-byte multiple
 constexpr uint32_t FMAX_CTAS = 4096;                      // grid cap (co-residency)
 constexpr size_t FWS_BARRIER = 2 * FMAX_CTAS * sizeof(uint64_t);
-constexpr uint32_t FSMEM = FSTAGES * 3 * FLOAD * 4 + FSTAGES * 8 + FSTAGE_ITEMS * 4;
+constexpr int FPL = 4;           // planes per stage: lo, hi, nm, vs (valid starts; multi-segment chunks)
+constexpr uint32_t FSMEM = FSTAGES * FPL * FLOAD * 4 + FSTAGES * 8 + FSTAGE_ITEMS * 4;
 
 struct FinderArgs {
     const uint32_t* lo;
     const uint32_t* hi;
     const uint32_t* nm;
-    uint64_t limit;              // valid window starts are [0, limit)
+    const uint32_t* vs;          // valid-start plane or nullptr (then starts [0, limit) are valid)
+    uint64_t limit;              // no start >= limit is valid
     uint32_t* out[2];            // '+' / '-' item lists
     uint64_t cap;
     uint64_t* status;            // workspace: per CTA (fwd, rev) totals
@@ -84,11 +86,11 @@ __device__ __forceinline__ void pam_masks(const FinderArgs& a, uint32_t valid, u
 //  offset) and pass 2 re-streams its range (mostly from L2) and writes the items in order.
 // One exchange per CTA replaces a decoupled look-back per tile, whose depth (all
 // concurrently running tiles) made it latency-bound.
-template <int NE>
+template <int NE, bool VS>
 __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ FinderArgs a) {
     extern __shared__ __align__(128) uint8_t smem[];
     uint32_t* stage = reinterpret_cast<uint32_t*>(smem);
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + FSTAGES * 3 * FLOAD * 4);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + FSTAGES * FPL * FLOAD * 4);
     uint32_t* items = reinterpret_cast<uint32_t*>(bars + FSTAGES);
     __shared__ uint32_t s_warp[FT / 32];
     __shared__ uint32_t s_tile_tot;
@@ -109,10 +111,11 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
 
     auto issue = [&](uint32_t tile, int s) {
         const size_t w0 = (size_t)tile * FW;
-        mbar_arrive_expect_tx(&bars[s], 3 * FLOAD * 4);
-        bulk_g2s(stage + (s * 3 + 0) * FLOAD, a.lo + w0, FLOAD * 4, &bars[s]);
-        bulk_g2s(stage + (s * 3 + 1) * FLOAD, a.hi + w0, FLOAD * 4, &bars[s]);
-        bulk_g2s(stage + (s * 3 + 2) * FLOAD, a.nm + w0, FLOAD * 4, &bars[s]);
+        mbar_arrive_expect_tx(&bars[s], (VS ? 4 : 3) * FLOAD * 4);
+        bulk_g2s(stage + (s * FPL + 0) * FLOAD, a.lo + w0, FLOAD * 4, &bars[s]);
+        bulk_g2s(stage + (s * FPL + 1) * FLOAD, a.hi + w0, FLOAD * 4, &bars[s]);
+        bulk_g2s(stage + (s * FPL + 2) * FLOAD, a.nm + w0, FLOAD * 4, &bars[s]);
+        if (VS) bulk_g2s(stage + (s * FPL + 3) * FLOAD, a.vs + w0, FLOAD * 4, &bars[s]);
     };
 
     uint32_t it = 0;                       // ring position across both passes
@@ -171,9 +174,10 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
             const uint32_t tile = t_begin + k;
             const int s = (int)(it % FSTAGES);
             mbar_wait_parity(&bars[s], (it / FSTAGES) & 1u);
-            const uint32_t* Slo = stage + (s * 3 + 0) * FLOAD + FWPT * tid;
-            const uint32_t* Shi = stage + (s * 3 + 1) * FLOAD + FWPT * tid;
-            const uint32_t* Snm = stage + (s * 3 + 2) * FLOAD + FWPT * tid;
+            const uint32_t* Slo = stage + (s * FPL + 0) * FLOAD + FWPT * tid;
+            const uint32_t* Shi = stage + (s * FPL + 1) * FLOAD + FWPT * tid;
+            const uint32_t* Snm = stage + (s * FPL + 2) * FLOAD + FWPT * tid;
+            const uint32_t* Svs = stage + (s * FPL + 3) * FLOAD + FWPT * tid;
             uint32_t lo[FWPT + 1], hi[FWPT + 1], nm[FWPT + 1];
 #pragma unroll
             for (int w = 0; w <= FWPT; w++) { lo[w] = Slo[w]; hi[w] = Shi[w]; nm[w] = Snm[w]; }
@@ -183,8 +187,8 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
 #pragma unroll
             for (int w = 0; w < FWPT; w++) {
                 const uint64_t pw = p0 + 32u * w;
-                uint32_t valid = ~0u;
-                if (pw + 32 > a.limit) valid = pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
+                uint32_t valid = VS ? Svs[w] : ~0u;
+                if (pw + 32 > a.limit) valid &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
                 uint32_t mw[2];
                 pam_masks<NE>(a, valid, lo[w], lo[w + 1], hi[w], hi[w + 1], nm[w], nm[w + 1], mw);
                 m[0][w] = mw[0];
@@ -281,24 +285,26 @@ static int g_finder_blocks_per_sm = -1;
 static int g_num_sms = -1;
 
 typedef void (*FinderFn)(FinderArgs);
-static FinderFn finder_fn(uint32_t ne) {
+template <bool VS>
+static FinderFn finder_fn_vs(uint32_t ne) {
     switch (ne) {
-        case 0: return cof_finder_kernel<0>;
-        case 1: return cof_finder_kernel<1>;
-        case 2: return cof_finder_kernel<2>;
-        case 3: return cof_finder_kernel<3>;
-        case 4: return cof_finder_kernel<4>;
-        case 5: return cof_finder_kernel<5>;
-        case 6: return cof_finder_kernel<6>;
-        default: return cof_finder_kernel<-1>;
+        case 0: return cof_finder_kernel<0, VS>;
+        case 1: return cof_finder_kernel<1, VS>;
+        case 2: return cof_finder_kernel<2, VS>;
+        case 3: return cof_finder_kernel<3, VS>;
+        case 4: return cof_finder_kernel<4, VS>;
+        case 5: return cof_finder_kernel<5, VS>;
+        case 6: return cof_finder_kernel<6, VS>;
+        default: return cof_finder_kernel<-1, VS>;
     }
 }
+static FinderFn finder_fn(uint32_t ne, bool vs) { return vs ? finder_fn_vs<true>(ne) : finder_fn_vs<false>(ne); }
 
 static cof_status finder_setup() {
     if (g_finder_blocks_per_sm > 0) return COF_OK;
     int bps_min = 1 << 30;
-    for (uint32_t ne = 0; ne <= 7; ne++) {
-        FinderFn fn = finder_fn(ne);
+    for (uint32_t k = 0; k < 16; k++) {
+        FinderFn fn = finder_fn(k & 7, k >= 8);
         cudaError_t e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM);
         if (e != cudaSuccess) return cuda_error(e, "finder setup");
         int bps = 0;
@@ -331,15 +337,16 @@ cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* d
     if (!plan || !plan_dev || !dev || !workspace || !items_fwd || !items_rev)
         return set_error(COF_E_ARG, "cof_find_pam: NULL argument");
     if (!dev->lo || !dev->hi || !dev->nm) return set_error(COF_E_ARG, "cof_find_pam: chunk planes are NULL");
-    if (dev->n_owned >= (1ull << 31)) return set_error(COF_E_ARG, "cof_find_pam: n_owned must be < 2^31");
-    if (((uintptr_t)dev->lo | (uintptr_t)dev->hi | (uintptr_t)dev->nm) & 15)
+    if (((uintptr_t)dev->lo | (uintptr_t)dev->hi | (uintptr_t)dev->nm | (uintptr_t)dev->vs) & 15)
         return set_error(COF_E_ARG, "cof_find_pam: planes must be 16-byte aligned");
     cof_status st = finder_setup();
     if (st != COF_OK) return st;
     cudaStream_t stream = (cudaStream_t)s;
     const uint64_t L = plan->L;
+    if (dev->n_segs && !dev->vs) return set_error(COF_E_ARG, "cof_find_pam: multi-segment chunk without vs plane");
+    if (dev->n_bases >= (1ull << 32)) return set_error(COF_E_ARG, "cof_find_pam: n_bases must be < 2^32");
     uint64_t limit = dev->n_bases >= L ? dev->n_bases - L + 1 : 0;
-    if (limit > dev->n_owned) limit = dev->n_owned;
+    if (!dev->n_segs && limit > dev->n_owned) limit = dev->n_owned;
     const uint32_t n_tiles = (uint32_t)((limit + (uint64_t)FW * 32 - 1) / ((uint64_t)FW * 32));
     unsigned long long* counters = (unsigned long long*)((uint8_t*)plan_dev + plan->lay.counters);
     cudaError_t e = cudaMemsetAsync(counters, 0, 2 * sizeof(uint64_t), stream);
@@ -349,6 +356,7 @@ cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* d
     if (n_tiles) {
         FinderArgs a;
         a.lo = dev->lo; a.hi = dev->hi; a.nm = dev->nm;
+        a.vs = dev->n_segs ? dev->vs : nullptr;
         a.limit = limit;
         a.out[0] = items_fwd; a.out[1] = items_rev;
         a.cap = items_cap;
@@ -367,7 +375,7 @@ cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* d
         uint32_t grid = (uint32_t)g_num_sms * (uint32_t)g_finder_blocks_per_sm;
         if (grid > FMAX_CTAS) grid = FMAX_CTAS;
         if (grid > n_tiles) grid = n_tiles;
-        finder_fn(a.ne)<<<grid, FT, FSMEM, stream>>>(a);
+        finder_fn(a.ne, a.vs != nullptr)<<<grid, FT, FSMEM, stream>>>(a);
         e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "cof_finder_kernel launch");
         count_launches(1);

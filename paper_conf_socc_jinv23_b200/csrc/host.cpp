@@ -126,9 +126,33 @@ cof_status cof_unpack(const uint32_t* lo, const uint32_t* hi, const uint32_t* nm
     return COF_OK;
 }
 
+cof_status cof_valid_starts(const cof_segment* segs, uint32_t n_segs, uint64_t n_bases, uint32_t* vs) {
+    if (!vs || (!segs && n_segs)) return set_error(COF_E_ARG, "cof_valid_starts: NULL argument");
+    const uint64_t words = cof_plane_words(n_bases);
+    memset(vs, 0, words * sizeof(uint32_t));
+    for (uint32_t k = 0; k < n_segs; k++) {
+        const uint64_t a = segs[k].chunk_off, b = a + segs[k].n_owned;
+        if (b > n_bases) return set_error(COF_E_ARG, "cof_valid_starts: segment %u ends past the chunk", k);
+        if (a == b) continue;
+        const uint64_t wa = a >> 5, wb = (b - 1) >> 5;
+        if (wa == wb) {
+            vs[wa] |= (uint32_t)(((1ull << (b - a)) - 1ull) << (a & 31));
+            continue;
+        }
+        vs[wa] |= ~0u << (a & 31);
+#pragma omp parallel for schedule(static) if (wb - wa > (1u << 16))
+        for (int64_t w = (int64_t)wa + 1; w < (int64_t)wb; w++) vs[w] = ~0u;
+        const uint32_t tail = (uint32_t)(b - (wb << 5));          // 1..32 bits in the last word
+        vs[wb] |= tail >= 32 ? ~0u : ((1u << tail) - 1u);
+    }
+    return COF_OK;
+}
+
 cof_status cof_load_chunk(const cof_chunk* host, cof_chunk* dev, cof_stream s) {
     if (!host || !dev || !host->lo || !host->hi || !host->nm || !dev->lo || !dev->hi || !dev->nm)
         return set_error(COF_E_ARG, "cof_load_chunk: NULL argument");
+    if (host->n_segs && (!host->vs || !dev->vs))
+        return set_error(COF_E_ARG, "cof_load_chunk: multi-segment chunk needs vs planes on both sides");
     size_t bytes = cof_plane_words(host->n_bases) * sizeof(uint32_t);
     cudaStream_t st = (cudaStream_t)s;
     cudaError_t e;
@@ -136,10 +160,15 @@ cof_status cof_load_chunk(const cof_chunk* host, cof_chunk* dev, cof_stream s) {
         (e = cudaMemcpyAsync(dev->hi, host->hi, bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess ||
         (e = cudaMemcpyAsync(dev->nm, host->nm, bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess)
         return cuda_error(e, "cof_load_chunk");
+    if (host->n_segs && (e = cudaMemcpyAsync(dev->vs, host->vs, bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess)
+        return cuda_error(e, "cof_load_chunk");
     dev->chrom = host->chrom;
+    dev->n_segs = host->n_segs;
     dev->start = host->start;
     dev->n_bases = host->n_bases;
     dev->n_owned = host->n_owned;
+    dev->segs = host->segs;
+    if (!host->n_segs) dev->vs = nullptr;
     return COF_OK;
 }
 
@@ -318,8 +347,21 @@ static cof_status decorate(const cof_plan* plan, const cof_chunk* host, uint64_t
     }
     memset(h->site + L, 0, sizeof h->site - L);
     h->guide = guide;
-    h->chrom = host->chrom;
-    h->pos = host->start + pos;
+    if (host->n_segs == 0) {
+        h->chrom = host->chrom;
+        h->pos = host->start + pos;
+    } else {   // chunk coordinate -> (chromosome, chromosome position) through the segment table
+        uint32_t lo_k = 0, hi_k = host->n_segs;
+        while (hi_k - lo_k > 1) {
+            const uint32_t mid = (lo_k + hi_k) / 2;
+            if (host->segs[mid].chunk_off <= pos) lo_k = mid;
+            else hi_k = mid;
+        }
+        const cof_segment& sg = host->segs[lo_k];
+        if (pos < sg.chunk_off || pos >= sg.chunk_off + sg.n_owned) return COF_E_STATE;
+        h->chrom = sg.chrom;
+        h->pos = sg.chrom_off + (pos - sg.chunk_off);
+    }
     h->strand = strand ? '-' : '+';
     h->mm = (uint8_t)mm;
     return COF_OK;

@@ -165,6 +165,10 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
         if (pl.n_pairs == 0) {   // all guides all-N: one dummy pair that never counts
             pl.j1[0] = 0; pl.j2[0] = 0xFF; pl.n_pairs = 1;
         }
+        pl.n_cmp = (uint32_t)__builtin_popcount(uc);
+        pl.p0 = uc ? (uint32_t)__builtin_ctz(uc) : 0u;
+        pl.contig = uc != 0 && (uc >> pl.p0) == (pl.n_cmp >= 32 ? 0xFFFFFFFFu : ((1u << pl.n_cmp) - 1u)) &&
+                    pl.p0 + 2 * pl.n_pairs <= 32;
     }
     // (both strands have the same number of compared positions, hence of pairs)
     const uint32_t NPAIR = p->pairs[0].n_pairs;

@@ -205,7 +205,7 @@ cof_status cof_sort_hits(const cof_plan* plan, void* plan_dev, const cof_chunk* 
     uint64_t eff = p.count ? cap : (p.n_host < cap ? p.n_host : cap);
     p.cap_tiles = (uint32_t)((eff + STILE - 1) / STILE);
     p.gb = bits_for(plan->n_guides - 1);
-    const uint32_t pb = bits_for(dev->n_owned ? dev->n_owned - 1 : 0);
+    const uint32_t pb = bits_for(dev->n_bases ? dev->n_bases - 1 : 0);   // positions are < n_bases
     const uint32_t total_bits = pb + 1 + p.gb;
     const uint32_t passes = (total_bits + 7) / 8;
     unsigned long long* a = (unsigned long long*)hits;

@@ -19,17 +19,57 @@ from . import cof
 
 
 @dataclasses.dataclass(frozen=True)
-class Chunk:
+class Piece:
+    """Window starts [chrom_off, chrom_off + n_owned) of chromosome ``chrom`` plus the
+    L-1 bases their last window needs (length = n_owned + L - 1, reading G12)."""
     chrom: int
-    start: int      # 0-based chromosome offset of base 0 of the chunk
-    n_owned: int    # window starts [start, start + n_owned) belong to this chunk
-    n_bases: int    # bases held: n_owned + L - 1 (chunks overlap by L-1, reading G12)
+    chrom_off: int
+    n_owned: int
+    length: int
 
 
-def plan_chunks(lengths, L: int, chunk_bases: int | None = None):
-    """Split chromosomes into chunks; every valid window start (0 <= p <= len-L) belongs
-    to exactly one chunk and each chunk holds the L-1 bases its last window needs."""
-    out = []
+@dataclasses.dataclass(frozen=True)
+class Chunk:
+    """One device work unit: one or more pieces laid back to back (chunk coordinates)."""
+    pieces: tuple
+
+    @property
+    def n_bases(self):
+        return sum(p.length for p in self.pieces)
+
+    @property
+    def n_owned(self):
+        return sum(p.n_owned for p in self.pieces)
+
+    @property
+    def multi(self):
+        return len(self.pieces) > 1
+
+    # single-segment conveniences
+    @property
+    def chrom(self):
+        return self.pieces[0].chrom
+
+    @property
+    def start(self):
+        return self.pieces[0].chrom_off
+
+    def segments(self):
+        """(chrom, chunk_off, chrom_off, n_owned) per piece."""
+        rows, off = [], 0
+        for p in self.pieces:
+            rows.append((p.chrom, off, p.chrom_off, p.n_owned))
+            off += p.length
+        return rows
+
+
+def plan_chunks(lengths, L: int, chunk_bases: int | None = None, pack_bases: int | None = None):
+    """Split chromosomes into pieces of at most ``chunk_bases`` owned window starts (whole
+    chromosomes if None): every valid start 0 <= p <= len-L belongs to exactly one piece.
+    Without ``pack_bases`` each piece is its own chunk; with it, consecutive pieces are
+    packed into multi-segment chunks of at most ``pack_bases`` bases (a piece longer than
+    that gets a chunk of its own); ``pack_bases=0`` packs everything into one chunk."""
+    pieces = []
     for c, n in enumerate(lengths):
         n_starts = int(n) - L + 1
         if n_starts <= 0:
@@ -37,7 +77,23 @@ def plan_chunks(lengths, L: int, chunk_bases: int | None = None):
         step = int(chunk_bases) if chunk_bases else n_starts
         for s in range(0, n_starts, step):
             owned = min(step, n_starts - s)
-            out.append(Chunk(c, s, owned, owned + L - 1))
+            pieces.append(Piece(c, s, owned, owned + L - 1))
+    if pack_bases is None:
+        return [Chunk((p,)) for p in pieces]
+    return pack_pieces(pieces, pack_bases)
+
+
+def pack_pieces(pieces, pack_bases: int):
+    """Consecutive pieces -> multi-segment chunks of at most ``pack_bases`` bases (0: one)."""
+    out, cur, cur_bases = [], [], 0
+    for p in pieces:
+        if cur and pack_bases and cur_bases + p.length > pack_bases:
+            out.append(Chunk(tuple(cur)))
+            cur, cur_bases = [], 0
+        cur.append(p)
+        cur_bases += p.length
+    if cur:
+        out.append(Chunk(tuple(cur)))
     return out
 
 
@@ -54,6 +110,11 @@ def shard_lpt(chunks, world: int):
     return [[chunks[i] for i in sorted(lst)] for lst in out]
 
 
+def pack_shard(chunks):
+    """All pieces of a list of chunks as ONE multi-segment chunk (a rank's whole shard)."""
+    return Chunk(tuple(p for ch in chunks for p in ch.pieces))
+
+
 def merge_hit_lists(lists):
     """Order (chrom, pos, strand, guide) across chunk / rank lists (cof_merge)."""
     lists = [x for x in lists if len(x)]
@@ -63,22 +124,34 @@ def merge_hit_lists(lists):
 
 
 class HostGenome:
-    """Packed bit-planes of every chunk in pinned host memory (a1: chunk & pack)."""
+    """Packed bit-planes of every chunk in pinned host memory (a1: chunk & pack); multi-
+    segment chunks also get their valid-start plane and segment table."""
 
     def __init__(self, seqs, chunks, pin: bool = True):
         self.chunks = chunks
         self.planes = []
+        self.segs = []
+        pin = pin and torch.cuda.is_available()
         for ch in chunks:
             words = cof.cof_plane_words(ch.n_bases)
-            buf = torch.empty((3, words), dtype=torch.int32, pin_memory=pin and torch.cuda.is_available())
-            seq = seqs[ch.chrom]
-            view = seq[ch.start: ch.start + ch.n_bases]
-            view = np.ascontiguousarray(view)
-            cof.cof_pack(view, ch.n_bases, buf[0], buf[1], buf[2])
+            buf = torch.empty((4 if ch.multi else 3, words), dtype=torch.int32, pin_memory=pin)
+            if ch.multi:
+                text = np.concatenate([np.asarray(seqs[p.chrom][p.chrom_off: p.chrom_off + p.length])
+                                       for p in ch.pieces])
+                segs = cof.make_segments(ch.segments())
+                cof.cof_valid_starts(segs, len(ch.pieces), ch.n_bases, buf[3])
+            else:
+                p = ch.pieces[0]
+                text = np.ascontiguousarray(seqs[p.chrom][p.chrom_off: p.chrom_off + p.length])
+                segs = None
+            cof.cof_pack(text, ch.n_bases, buf[0], buf[1], buf[2])
             self.planes.append(buf)
+            self.segs.append(segs)
 
     def chunk_struct(self, i) -> cof.cof_chunk:
-        ch, buf = self.chunks[i], self.planes[i]
+        ch, buf, segs = self.chunks[i], self.planes[i], self.segs[i]
+        if ch.multi:
+            return cof.make_chunk(0, 0, ch.n_bases, ch.n_owned, buf[0], buf[1], buf[2], buf[3], segs)
         return cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, buf[0], buf[1], buf[2])
 
     @property
@@ -104,7 +177,7 @@ class Searcher:
     def reserve(self, max_bases: int, hits_cap: int):
         if max_bases > self._cap_bases:
             words = cof.cof_plane_words(max_bases)
-            self.d_planes = torch.empty((3, words), dtype=torch.int32, device=self.device)
+            self.d_planes = torch.empty((4, words), dtype=torch.int32, device=self.device)
             self.d_items = torch.empty((2, max(max_bases, 1)), dtype=torch.int32, device=self.device)
             self.d_find_ws = torch.empty(cof.cof_find_workspace_bytes(max_bases), dtype=torch.uint8,
                                          device=self.device)
@@ -116,8 +189,11 @@ class Searcher:
                                          device=self.device)
             self._hits_cap = hits_cap
 
-    def device_chunk(self, ch: Chunk, planes=None) -> cof.cof_chunk:
+    def device_chunk(self, ch: Chunk, planes=None, segs=None) -> cof.cof_chunk:
         p = self.d_planes if planes is None else planes
+        if ch.multi:
+            return cof.make_chunk(0, 0, ch.n_bases, ch.n_owned, p[0], p[1], p[2], p[3],
+                                  segs if segs is not None else cof.make_segments(ch.segments()))
         return cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, p[0], p[1], p[2])
 
     def run_device_chunk(self, dchunk: cof.cof_chunk, items_cap: int):
@@ -196,7 +272,7 @@ class Searcher:
                     with torch.cuda.stream(self.copy_stream):
                         if freed[k] is not None:
                             self.copy_stream.wait_event(freed[k])
-                        dch = self.device_chunk(host.chunks[idx[j]], planes[k])
+                        dch = self.device_chunk(host.chunks[idx[j]], planes[k], host.segs[idx[j]])
                         cof.cof_load_chunk(host.chunk_struct(idx[j]), dch, self.copy_stream)
                         ev = torch.cuda.Event()
                         ev.record(self.copy_stream)
@@ -238,12 +314,13 @@ class Searcher:
             return out[:total]
         return merge_hit_lists([results[i] for i in idx])
 
-def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda"):
-    """Convenience: whole search of ``seqs`` (list of uint8 ASCII arrays / bytes) on one GPU."""
+def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda", pack_bases=None):
+    """Convenience: whole search of ``seqs`` (list of uint8 ASCII arrays / bytes) on one GPU.
+    ``pack_bases`` packs chromosome pieces into multi-segment chunks (0 = one chunk)."""
     L = len(pattern)
     arrs = [np.frombuffer(s, dtype=np.uint8) if isinstance(s, (bytes, bytearray)) else
             (np.frombuffer(s.encode(), dtype=np.uint8) if isinstance(s, str) else s) for s in seqs]
-    chunks = plan_chunks([len(a) for a in arrs], L, chunk_bases)
+    chunks = plan_chunks([len(a) for a in arrs], L, chunk_bases, pack_bases)
     host = HostGenome(arrs, chunks)
     return Searcher(pattern, guides, thresholds, device).search_host(host)
 

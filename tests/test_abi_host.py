@@ -202,3 +202,65 @@ def test_shard_lpt_assigns_each_chunk_once():
         loads = [sum(c.n_owned for c in s) for s in shards]
         ideal = sum(loads) / world
         assert max(loads) <= max(ideal * 1.05, max(c.n_owned for c in chunks) + 1)
+
+
+def test_valid_starts_plane():
+    segs_rows = [(0, 0, 0, 5), (1, 10, 0, 40), (2, 60, 7, 33), (3, 100, 0, 0), (4, 200, 3, 64)]
+    n = 300
+    segs = cof.make_segments(segs_rows)
+    vs = np.zeros(cof.cof_plane_words(n), np.uint32)
+    cof.cof_valid_starts(segs, len(segs_rows), n, vs)
+    bits = np.unpackbits(vs.view(np.uint8), bitorder="little")
+    exp = np.zeros(len(bits), np.uint8)
+    for _, off, _, owned in segs_rows:
+        exp[off:off + owned] = 1
+    assert np.array_equal(bits, exp)
+    with pytest.raises(cof.CofError):
+        cof.cof_valid_starts(cof.make_segments([(0, 290, 0, 20)]), 1, n, vs)
+
+
+def test_collect_maps_multi_segment_chunks():
+    """Chunk coordinates of a multi-segment chunk map back to (chromosome, position)."""
+    rng = np.random.default_rng(8)
+    seqs = [synth.random_genome_text(rng, n, b"ACGTacgtN", p=[.22, .22, .22, .22, .02, .02, .02, .02, .04])
+            for n in (5000, 30, 7000, 4000)]
+    pat = "N" * 21 + "RG"
+    guides = ["".join(rng.choice(list("ACGT"), 20)) + "NNN" for _ in range(3)]
+    thr = [12, 12, 12]
+    ref = oracle.search(seqs, pat, guides, thr)
+    chunks = search.plan_chunks([len(s) for s in seqs], 23, 2500, pack_bases=0)
+    assert len(chunks) == 1 and chunks[0].multi
+    ch = chunks[0]
+    host = search.HostGenome(seqs, chunks, pin=False)
+    segs = ch.segments()
+    keys = []
+    for h in ref:   # oracle record -> chunk coordinate of its window start
+        c, p = int(h["chrom"]), int(h["pos"])
+        off = [co + (p - so) for (cc, co, so, no) in segs if cc == c and so <= p < so + no]
+        assert len(off) == 1
+        keys.append((off[0] << 32) | ((1 if h["strand"] == b"-" else 0) << 31) | (int(h["guide"]) << 7) | int(h["mm"]))
+    keys = np.array(keys, dtype=np.uint64)
+    plan = cof.cof_plan_create(pat, guides, thr)
+    got = cof.cof_collect(plan, host.chunk_struct(0), None, len(keys), host_keys=np.sort(keys))
+    assert cof.hits_to_tuples(got) == oracle.hits_to_tuples(ref)
+
+
+def test_plan_chunks_packed():
+    L = 23
+    lengths = [100_000, 10, 77_777, 5000]
+    for cb, pb in ((None, 0), (7919, 0), (7919, 50_000), (None, 1)):
+        chunks = search.plan_chunks(lengths, L, cb, pack_bases=pb)
+        cover = {}
+        for ch in chunks:
+            off = 0
+            for p in ch.pieces:
+                cover.setdefault(p.chrom, []).append((p.chrom_off, p.chrom_off + p.n_owned))
+                assert p.length == p.n_owned + L - 1 and p.chrom_off + p.length <= lengths[p.chrom]
+                off += p.length
+            assert ch.n_bases == off
+            if pb:
+                assert ch.n_bases <= pb or len(ch.pieces) == 1
+        for c, n in enumerate(lengths):
+            iv = sorted(cover.get(c, []))
+            assert sum(e - s for s, e in iv) == max(0, n - L + 1)
+            assert all(a[1] == b[0] for a, b in zip(iv, iv[1:]))

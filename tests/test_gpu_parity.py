@@ -23,9 +23,10 @@ def _impl_reset():
     cof.cof_set_comparer("table")
 
 
-def gpu_hits(seqs, pattern, guides, thr, chunk_bases=None, impl="table"):
+def gpu_hits(seqs, pattern, guides, thr, chunk_bases=None, impl="table", pack_bases=None):
     cof.cof_set_comparer(impl)
-    return cof.hits_to_tuples(search.search(seqs, pattern, guides, thr, chunk_bases=chunk_bases))
+    return cof.hits_to_tuples(search.search(seqs, pattern, guides, thr, chunk_bases=chunk_bases,
+                                            pack_bases=pack_bases))
 
 
 def ref_hits(seqs, pattern, guides, thr, ranges=None):
@@ -54,6 +55,9 @@ def test_random_small(impl, seed):
                                      p=[.22, .15, .15, .22, .05, .05, .05, .05, .04, .01, .005, .005]) for n in lens]
     exp = ref_hits(seqs, pat, guides, thr)
     assert gpu_hits(seqs, pat, guides, thr, impl=impl) == exp
+    # the same genome as one multi-segment chunk and as packed pieces
+    assert gpu_hits(seqs, pat, guides, thr, impl=impl, pack_bases=0) == exp
+    assert gpu_hits(seqs, pat, guides, thr, impl=impl, chunk_bases=9973, pack_bases=30_000) == exp
 
 
 @pytest.mark.parametrize("impl", IMPLS)
@@ -65,13 +69,14 @@ def test_c1_full(impl):
     assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, impl=impl) == exp
 
 
-@pytest.mark.parametrize("name,scale,chunk", [("C2", 0.1, None), ("C3", 0.004, 1_000_003),
-                                              ("C4", 0.004, 333_333), ("C5", 0.002, None)])
-def test_configs_scaled(name, scale, chunk):
+@pytest.mark.parametrize("name,scale,chunk,pack", [("C2", 0.1, None, None), ("C3", 0.004, 1_000_003, None),
+                                                   ("C4", 0.004, 333_333, 0), ("C5", 0.002, None, 0),
+                                                   ("C3", 0.003, None, 2_000_000)])
+def test_configs_scaled(name, scale, chunk, pack):
     w = synth.make_workload(name, scale=scale, n_guides=None if name != "C5" else 200)
     cfg = w.cfg
     exp = ref_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
-    assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk) == exp
+    assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk, pack_bases=pack) == exp
 
 
 def test_chunk_size_invariance():
