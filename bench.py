@@ -130,7 +130,7 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
         st.plan_devs.append(pd)
     max_owned = max(ch.n_owned for ch in chunks)
     st.items = torch.empty((2, max_owned), dtype=torch.int32, device=st.device)
-    st.find_ws = torch.empty(cof.cof_find_workspace_bytes(max_owned), dtype=torch.uint8, device=st.device)
+    st.find_ws = torch.empty(cof.cof_find_workspace_bytes(max(ch.n_bases for ch in chunks)), dtype=torch.uint8, device=st.device)
     # first pass with host counts: exact item / hit counts per chunk
     st.counts = []
     tmp_cap = 1 << 20

@@ -149,13 +149,13 @@ cof_status cof_fasta_pack(const cof_fasta *fa, uint32_t i, uint64_t first, uint6
  * uint32).  The paper compacts with an unordered atomic counter (Table V);
  * here an ordered two-pass compaction (count, one grid-wide exchange, write) keeps the
  * lists sorted.
- *  workspace  dev, >= cof_find_workspace_bytes(dev->n_owned) bytes (per-CTA totals and a
- *             grid barrier counter; reset by the call).
+ *  workspace  dev, >= cof_find_workspace_bytes(dev->n_bases) bytes (per-CTA totals, a
+ *             grid barrier counter and the pass-1 PAM masks, 8 bytes per plane word).
  *  items_cap  capacity of each list; n_owned always suffices.
  *  n_fwd/n_rev  host outputs; if both are NULL the call does not synchronize and the
  *             counts stay in plan_dev for cof_compare(COF_COUNT_ON_DEVICE).
  * COF_E_CAPACITY: a list overflowed; n_fwd and n_rev hold the needed counts. */
-size_t     cof_find_workspace_bytes(uint64_t n_owned);
+size_t     cof_find_workspace_bytes(uint64_t n_bases);
 cof_status cof_find_pam(const cof_plan *plan, void *plan_dev, const cof_chunk *dev,
                         void *workspace, uint32_t *items_fwd, uint32_t *items_rev,
                         uint64_t items_cap, uint64_t *n_fwd, uint64_t *n_rev, cof_stream s);

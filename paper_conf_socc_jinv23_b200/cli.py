@@ -1,0 +1,116 @@
+"""Cas-OFFinder-style command line (I/O compatibility).
+
+    python -m paper_conf_socc_jinv23_b200 INPUT [G] OUTPUT [--chunk-bases N] [--device cuda:0]
+
+INPUT follows the tool's input file ("the desired pattern, query sequences, and maximum
+mismatch number", P:L158 via [17]):
+
+    /path/to/genome.fa            (a FASTA file, or a directory of .fa/.fasta/.fna files)
+    NNNNNNNNNNNNNNNNNNNNNRG       (pattern; N = any base, PAM letters in IUPAC)
+    GGCCGACCTGTCGCTGACGCNNN 5     (query and its maximum mismatch count, one per line)
+    ...
+
+OUTPUT is tab-separated, one hit per line ("chromosome number, position, direction,
+the number of mismatched bases and potential off-target DNA sequence with mismatched
+bases"): query, chromosome name, 0-based position, site (mismatches lower-case),
+strand, mismatches — in (chromosome, position, strand, query) order (reading G13).
+The second positional argument (the original tool's C/G/A device letter) is accepted and
+ignored: the search always runs on the GPU.
+"""
+from __future__ import annotations
+
+import argparse
+import dataclasses
+import os
+import sys
+
+import numpy as np
+
+
+@dataclasses.dataclass
+class InputSpec:
+    genome: str
+    pattern: str
+    queries: list
+    thresholds: list
+
+
+def parse_input(text: str, base_dir: str = ".") -> InputSpec:
+    lines = [ln.strip() for ln in text.splitlines()]
+    lines = [ln for ln in lines if ln and not ln.startswith("#")]
+    if len(lines) < 3:
+        raise ValueError("input needs a genome path, a pattern and at least one query line")
+    genome = lines[0]
+    if not os.path.isabs(genome):
+        genome = os.path.join(base_dir, genome)
+    pattern = lines[1].split()[0]
+    queries, thr = [], []
+    for ln in lines[2:]:
+        parts = ln.split()
+        if len(parts) < 2:
+            raise ValueError(f"query line needs a sequence and a mismatch count: {ln!r}")
+        q, t = parts[0], int(parts[1])
+        if len(q) != len(pattern):
+            raise ValueError(f"query {q} has length {len(q)}, pattern has {len(pattern)}")
+        if t < 0:
+            raise ValueError(f"negative mismatch count in {ln!r}")
+        queries.append(q)
+        thr.append(t)
+    return InputSpec(genome, pattern, queries, thr)
+
+
+def genome_files(path: str):
+    if os.path.isdir(path):
+        ext = (".fa", ".fasta", ".fna", ".fa.txt")
+        return sorted(os.path.join(path, f) for f in os.listdir(path) if f.lower().endswith(ext))
+    return [path]
+
+
+def format_hits(hits, queries, names) -> str:
+    """TSV lines for a cof.HIT_DTYPE array."""
+    out = []
+    for h in hits:
+        out.append(f"{queries[int(h['guide'])]}\t{names[int(h['chrom'])]}\t{int(h['pos'])}\t"
+                   f"{h['site'].decode()}\t{h['strand'].decode()}\t{int(h['mm'])}")
+    return "\n".join(out) + ("\n" if out else "")
+
+
+def run(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = None):
+    """Search the genome of ``spec`` on one GPU; returns (hits, chromosome names)."""
+    import torch
+    from . import cof, search
+
+    fastas = [cof.Fasta(f) for f in genome_files(spec.genome)]
+    names, recs = [], []
+    for fi, fa in enumerate(fastas):
+        for i in range(len(fa)):
+            names.append(fa.name(i))
+            recs.append((fi, i, fa.length(i)))
+    L = len(spec.pattern)
+    chunks = search.plan_chunks([r[2] for r in recs], L, chunk_bases)
+    host = search.HostGenome.from_packer(chunks, lambda c, first, n, lo, hi, nm:
+                                         fastas[recs[c][0]].pack(recs[c][1], first, n, lo, hi, nm))
+    srch = search.Searcher(spec.pattern, spec.queries, spec.thresholds, device=device)
+    hits = srch.search_host(host)
+    torch.cuda.synchronize()
+    return hits, names
+
+
+def main(argv=None) -> int:
+    ap = argparse.ArgumentParser(prog="python -m paper_conf_socc_jinv23_b200", description=__doc__.split("\n")[0])
+    ap.add_argument("input")
+    ap.add_argument("args", nargs="+", help="[C|G|A] OUTPUT")
+    ap.add_argument("--chunk-bases", type=int, default=None)
+    ap.add_argument("--device", default="cuda")
+    a = ap.parse_args(argv)
+    output = a.args[-1]
+    with open(a.input) as f:
+        spec = parse_input(f.read(), os.path.dirname(os.path.abspath(a.input)))
+    hits, names = run(spec, a.device, a.chunk_bases)
+    text = format_hits(hits, spec.queries, names)
+    if output == "-":
+        sys.stdout.write(text)
+    else:
+        with open(output, "w") as f:
+            f.write(text)
+    return 0

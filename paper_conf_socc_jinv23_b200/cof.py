@@ -219,8 +219,8 @@ def cof_load_chunk(host: cof_chunk, dev: cof_chunk, stream=None):
     _check(lib.cof_load_chunk(ctypes.addressof(host), ctypes.addressof(dev), _stream(stream)))
 
 
-def cof_find_workspace_bytes(n_owned: int) -> int:
-    return int(lib.cof_find_workspace_bytes(int(n_owned)))
+def cof_find_workspace_bytes(n_bases: int) -> int:
+    return int(lib.cof_find_workspace_bytes(int(n_bases)))
 
 
 def cof_find_pam(plan, plan_dev, dev: cof_chunk, workspace, items_fwd, items_rev, items_cap,

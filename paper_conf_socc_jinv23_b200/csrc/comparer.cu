@@ -304,16 +304,31 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constan
     const uint32_t n_chunks = (a.n_blocks + bpc - 1) / bpc;
     uint32_t loaded = 0xFFFFFFFFu;
 
+    // item positions are prefetched one tile ahead (their load latency overlaps the
+    // previous tile's table work; only the dependent window loads remain exposed)
+    uint32_t pos_next[R];
+#pragma unroll
+    for (int r = 0; r < R; r++) {
+        const uint64_t idx = (uint64_t)blockIdx.x * per_tile + threadIdx.x + (uint64_t)r * CT;
+        pos_next[r] = (blockIdx.x < n_tiles && idx < n) ? __ldg(a.items + idx) : 0u;
+    }
     for (uint64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
         const uint64_t t0 = tile * per_tile;
         const uint64_t item0 = t0 + threadIdx.x;
         const bool tail = t0 + per_tile > n;
+        uint32_t cur[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            cur[r] = pos_next[r];
+            const uint64_t nidx = item0 + (uint64_t)gridDim.x * per_tile + (uint64_t)r * CT;
+            pos_next[r] = nidx < n ? __ldg(a.items + nidx) : 0u;
+        }
         uint32_t off[R][NP], okm[R];
 #pragma unroll
         for (int r = 0; r < R; r++) {
             const uint64_t idx = item0 + (uint64_t)r * CT;
             okm[r] = idx < n ? ~0u : 0u;
-            const uint32_t pos = idx < n ? __ldg(a.items + idx) : 0u;
+            const uint32_t pos = cur[r];
             bool done = false;
             if (a.pairs.contig) {
                 // fast path: window starting at the first compared offset; with no N among the

@@ -31,6 +31,7 @@ constexpr int FSTAGES = 4;       // TMA ring depth
 constexpr int FLOAD = FW + 4;    // words per plane per stage: tile + halo, 16-byte multiple
 constexpr uint32_t FMAX_CTAS = 4096;                      // grid cap (co-residency)
 constexpr size_t FWS_BARRIER = 2 * FMAX_CTAS * sizeof(uint64_t);
+constexpr size_t FWS_MASKS = FWS_BARRIER + 256;
 constexpr int FPL = 4;           // planes per stage: lo, hi, nm, vs (valid starts; multi-segment chunks)
 constexpr uint32_t FSMEM = FSTAGES * FPL * FLOAD * 4 + FSTAGES * 8 + FSTAGE_ITEMS * 4;
 
@@ -43,6 +44,7 @@ struct FinderArgs {
     uint32_t* out[2];            // '+' / '-' item lists
     uint64_t cap;
     uint64_t* status;            // workspace: per CTA (fwd, rev) totals
+    uint32_t* masks;             // workspace: per plane word {fwd, rev} PAM masks (pass 1 -> pass 2)
     unsigned int* barrier;       // workspace: grid barrier counter (zeroed)
     unsigned long long* counters;  // plan_dev counters: [0] n_fwd, [1] n_rev
     uint32_t n_tiles;
@@ -118,166 +120,173 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
         if (VS) bulk_g2s(stage + (s * FPL + 3) * FLOAD, a.vs + w0, FLOAD * 4, &bars[s]);
     };
 
-    uint32_t it = 0;                       // ring position across both passes
-    unsigned long long cnt_f = 0, cnt_r = 0;   // pass 1: this thread's counts
-    unsigned long long run_f = 0, run_r = 0;   // pass 2: items of this CTA written so far
-
-    for (int pass = 0; pass < 2; pass++) {
-        if (pass == 1) {
-            // ---- CTA totals -> grid exchange -> this CTA's global offsets
+    // ---------------- pass 1: stream the planes (TMA ring), PAM masks -> workspace, counts
+    unsigned long long cnt_f = 0, cnt_r = 0;
+    if (tid == 0)
+        for (int s = 0; s < FSTAGES && (uint32_t)s < n_mine; s++) issue(t_begin + s, s);
+    for (uint32_t k = 0; k < n_mine; k++) {
+        const uint32_t tile = t_begin + k;
+        const int s = (int)(k % FSTAGES);
+        mbar_wait_parity(&bars[s], (k / FSTAGES) & 1u);
+        const uint32_t* Slo = stage + (s * FPL + 0) * FLOAD + FWPT * tid;
+        const uint32_t* Shi = stage + (s * FPL + 1) * FLOAD + FWPT * tid;
+        const uint32_t* Snm = stage + (s * FPL + 2) * FLOAD + FWPT * tid;
+        const uint32_t* Svs = stage + (s * FPL + 3) * FLOAD + FWPT * tid;
+        uint32_t lo[FWPT + 1], hi[FWPT + 1], nm[FWPT + 1], vsw[FWPT];
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) {
-                cnt_f += __shfl_xor_sync(0xffffffffu, cnt_f, o);
-                cnt_r += __shfl_xor_sync(0xffffffffu, cnt_r, o);
-            }
-            if (lane == 0) { s_red[warp][0] = cnt_f; s_red[warp][1] = cnt_r; }
-            __syncthreads();
-            if (tid == 0) {
-                unsigned long long f = 0, r = 0;
-                for (int w = 0; w < FT / 32; w++) { f += s_red[w][0]; r += s_red[w][1]; }
-                st_relaxed_gpu(&a.status[2 * blockIdx.x], f);
-                st_relaxed_gpu(&a.status[2 * blockIdx.x + 1], r);
-                __threadfence();
-                atomicAdd(a.barrier, 1u);
-                while (ld_acquire_gpu_u32(a.barrier) < gridDim.x) __nanosleep(64);
-            }
-            __syncthreads();
-            unsigned long long f = 0, r = 0;
-            for (uint32_t c = tid; c < blockIdx.x; c += FT) {
-                f += ld_relaxed_gpu(&a.status[2 * c]);
-                r += ld_relaxed_gpu(&a.status[2 * c + 1]);
-            }
+        for (int w = 0; w <= FWPT; w++) { lo[w] = Slo[w]; hi[w] = Shi[w]; nm[w] = Snm[w]; }
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) {
-                f += __shfl_xor_sync(0xffffffffu, f, o);
-                r += __shfl_xor_sync(0xffffffffu, r, o);
-            }
-            __syncthreads();
-            if (lane == 0) { s_red[warp][0] = f; s_red[warp][1] = r; }
-            __syncthreads();
-            if (tid == 0) {
-                unsigned long long bf = 0, br = 0;
-                for (int w = 0; w < FT / 32; w++) { bf += s_red[w][0]; br += s_red[w][1]; }
-                s_base[0] = bf;
-                s_base[1] = br;
-                if (blockIdx.x == gridDim.x - 1) {     // last CTA knows the chunk totals
-                    a.counters[0] = bf + ld_relaxed_gpu(&a.status[2 * blockIdx.x]);
-                    a.counters[1] = br + ld_relaxed_gpu(&a.status[2 * blockIdx.x + 1]);
-                }
-            }
-            __syncthreads();
+        for (int w = 0; w < FWPT; w++) vsw[w] = VS ? Svs[w] : ~0u;
+        __syncthreads();   // every thread has read stage s: refill it
+        if (tid == 0 && k + FSTAGES < n_mine) {
+            fence_proxy_async_smem();
+            issue(tile + FSTAGES, s);
         }
+        const uint64_t p0 = ((uint64_t)tile * FW + FWPT * tid) * 32;
+        uint32_t mk[2 * FWPT];
+#pragma unroll
+        for (int w = 0; w < FWPT; w++) {
+            const uint64_t pw = p0 + 32u * w;
+            uint32_t valid = vsw[w];
+            if (pw + 32 > a.limit) valid &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
+            uint32_t mw[2];
+            pam_masks<NE>(a, valid, lo[w], lo[w + 1], hi[w], hi[w + 1], nm[w], nm[w + 1], mw);
+            mk[2 * w] = mw[0];
+            mk[2 * w + 1] = mw[1];
+            cnt_f += (unsigned)__popc(mw[0]);
+            cnt_r += (unsigned)__popc(mw[1]);
+        }
+        // masks of this thread's FWPT words: {fwd0, rev0, fwd1, rev1} (one 16-byte store)
+        reinterpret_cast<uint4*>(a.masks)[(size_t)tile * FT + tid] = make_uint4(mk[0], mk[1], mk[2], mk[3]);
+    }
+
+    // ---------------- grid exchange: CTA totals -> this CTA's global offsets
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        cnt_f += __shfl_xor_sync(0xffffffffu, cnt_f, o);
+        cnt_r += __shfl_xor_sync(0xffffffffu, cnt_r, o);
+    }
+    if (lane == 0) { s_red[warp][0] = cnt_f; s_red[warp][1] = cnt_r; }
+    __syncthreads();
+    if (tid == 0) {
+        unsigned long long f = 0, r = 0;
+        for (int w = 0; w < FT / 32; w++) { f += s_red[w][0]; r += s_red[w][1]; }
+        st_relaxed_gpu(&a.status[2 * blockIdx.x], f);
+        st_relaxed_gpu(&a.status[2 * blockIdx.x + 1], r);
+        __threadfence();
+        atomicAdd(a.barrier, 1u);
+        while (ld_acquire_gpu_u32(a.barrier) < gridDim.x) __nanosleep(64);
+    }
+    __syncthreads();
+    {
+        unsigned long long f = 0, r = 0;
+        for (uint32_t c = tid; c < blockIdx.x; c += FT) {
+            f += ld_relaxed_gpu(&a.status[2 * c]);
+            r += ld_relaxed_gpu(&a.status[2 * c + 1]);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            f += __shfl_xor_sync(0xffffffffu, f, o);
+            r += __shfl_xor_sync(0xffffffffu, r, o);
+        }
+        __syncthreads();
+        if (lane == 0) { s_red[warp][0] = f; s_red[warp][1] = r; }
+        __syncthreads();
         if (tid == 0) {
-            for (int s = 0; s < FSTAGES && (uint32_t)s < n_mine; s++) issue(t_begin + s, (int)((it + s) % FSTAGES));
+            unsigned long long bf = 0, br = 0;
+            for (int w = 0; w < FT / 32; w++) { bf += s_red[w][0]; br += s_red[w][1]; }
+            s_base[0] = bf;
+            s_base[1] = br;
+            if (blockIdx.x == gridDim.x - 1) {     // last CTA knows the chunk totals
+                a.counters[0] = bf + ld_relaxed_gpu(&a.status[2 * blockIdx.x]);
+                a.counters[1] = br + ld_relaxed_gpu(&a.status[2 * blockIdx.x + 1]);
+            }
         }
-        for (uint32_t k = 0; k < n_mine; k++, it++) {
-            const uint32_t tile = t_begin + k;
-            const int s = (int)(it % FSTAGES);
-            mbar_wait_parity(&bars[s], (it / FSTAGES) & 1u);
-            const uint32_t* Slo = stage + (s * FPL + 0) * FLOAD + FWPT * tid;
-            const uint32_t* Shi = stage + (s * FPL + 1) * FLOAD + FWPT * tid;
-            const uint32_t* Snm = stage + (s * FPL + 2) * FLOAD + FWPT * tid;
-            const uint32_t* Svs = stage + (s * FPL + 3) * FLOAD + FWPT * tid;
-            uint32_t lo[FWPT + 1], hi[FWPT + 1], nm[FWPT + 1];
-#pragma unroll
-            for (int w = 0; w <= FWPT; w++) { lo[w] = Slo[w]; hi[w] = Shi[w]; nm[w] = Snm[w]; }
+        __syncthreads();
+    }
 
-            const uint64_t p0 = ((uint64_t)tile * FW + FWPT * tid) * 32;   // first start of this thread
-            uint32_t m[2][FWPT];
-#pragma unroll
-            for (int w = 0; w < FWPT; w++) {
-                const uint64_t pw = p0 + 32u * w;
-                uint32_t valid = VS ? Svs[w] : ~0u;
-                if (pw + 32 > a.limit) valid &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
-                uint32_t mw[2];
-                pam_masks<NE>(a, valid, lo[w], lo[w + 1], hi[w], hi[w + 1], nm[w], nm[w + 1], mw);
-                m[0][w] = mw[0];
-                m[1][w] = mw[1];
-            }
-            __syncthreads();   // every thread has read stage s: refill it
-            if (tid == 0 && k + FSTAGES < n_mine) {
-                fence_proxy_async_smem();
-                issue(tile + FSTAGES, s);
-            }
-            uint32_t cf = 0, cr = 0;
-#pragma unroll
-            for (int w = 0; w < FWPT; w++) { cf += (uint32_t)__popc(m[0][w]); cr += (uint32_t)__popc(m[1][w]); }
-            if (pass == 0) {
-                cnt_f += cf;
-                cnt_r += cr;
-                continue;
-            }
+    // ---------------- pass 2: masks (workspace, mostly L2) -> ordered item lists
+    unsigned long long run_f = 0, run_r = 0;
+    const uint4* mptr = reinterpret_cast<const uint4*>(a.masks);
+    uint4 mnext = n_mine ? __ldcg(mptr + (size_t)t_begin * FT + tid) : make_uint4(0, 0, 0, 0);
+    for (uint32_t k = 0; k < n_mine; k++) {
+        const uint32_t tile = t_begin + k;
+        const uint4 mv = mnext;
+        if (k + 1 < n_mine) mnext = __ldcg(mptr + (size_t)(tile + 1) * FT + tid);
+        const uint32_t m[2][FWPT] = {{mv.x, mv.z}, {mv.y, mv.w}};
+        const uint32_t cf = (uint32_t)(__popc(mv.x) + __popc(mv.z));
+        const uint32_t cr = (uint32_t)(__popc(mv.y) + __popc(mv.w));
+        const uint64_t p0 = ((uint64_t)tile * FW + FWPT * tid) * 32;
 
-            // ---- pass 2: CTA exclusive scan of packed counts (fwd bits 0..15, rev 16..31)
-            const uint32_t cnt = cf | (cr << 16);
-            uint32_t x = cnt;
+        // CTA exclusive scan of packed counts (fwd bits 0..15, rev 16..31)
+        const uint32_t cnt = cf | (cr << 16);
+        uint32_t x = cnt;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-                if (lane >= o) x += y;
+        for (int o = 1; o < 32; o <<= 1) {
+            uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= o) x += y;
+        }
+        if (lane == 31) s_warp[warp] = x;
+        __syncthreads();
+        if (warp == 0) {
+            uint32_t wv = lane < FT / 32 ? s_warp[lane] : 0u;
+            uint32_t wi = wv;
+#pragma unroll
+            for (int o = 1; o < FT / 32; o <<= 1) {
+                uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
+                if (lane >= o) wi += y;
             }
-            if (lane == 31) s_warp[warp] = x;
-            __syncthreads();
-            if (warp == 0) {
-                uint32_t wv = lane < FT / 32 ? s_warp[lane] : 0u;
-                uint32_t wi = wv;
+            if (lane < FT / 32) s_warp[lane] = wi - wv;
+            if (lane == FT / 32 - 1) s_tile_tot = wi;
+        }
+        __syncthreads();
+        const uint32_t local = s_warp[warp] + x - cnt;
+        const uint32_t tot = s_tile_tot;
+        const uint32_t pbase = (uint32_t)p0;
 #pragma unroll
-                for (int o = 1; o < FT / 32; o <<= 1) {
-                    uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
-                    if (lane >= o) wi += y;
-                }
-                if (lane < FT / 32) s_warp[lane] = wi - wv;
-                if (lane == FT / 32 - 1) s_tile_tot = wi;
-            }
-            __syncthreads();
-            const uint32_t local = s_warp[warp] + x - cnt;
-            const uint32_t tot = s_tile_tot;
-            const uint32_t pbase = (uint32_t)p0;
+        for (int st = 0; st < 2; st++) {
+            const uint32_t total = st == 0 ? (tot & 0xFFFFu) : (tot >> 16);
+            const uint32_t first = st == 0 ? (local & 0xFFFFu) : (local >> 16);
+            const unsigned long long base = s_base[st] + (st == 0 ? run_f : run_r);
+            uint32_t* out = a.out[st];
+            // staged in rounds of FSTAGE_ITEMS (one round unless the pattern is very permissive)
+            for (uint32_t r0 = 0; r0 < total; r0 += FSTAGE_ITEMS) {
+                if (total <= FSTAGE_ITEMS) {
+                    uint32_t off = first;
 #pragma unroll
-            for (int st = 0; st < 2; st++) {
-                const uint32_t total = st == 0 ? (tot & 0xFFFFu) : (tot >> 16);
-                const uint32_t first = st == 0 ? (local & 0xFFFFu) : (local >> 16);
-                const unsigned long long base = s_base[st] + (st == 0 ? run_f : run_r);
-                uint32_t* out = a.out[st];
-                // staged in rounds of FSTAGE_ITEMS (one round unless the pattern is very permissive)
-                for (uint32_t r0 = 0; r0 < total; r0 += FSTAGE_ITEMS) {
-                    if (total <= FSTAGE_ITEMS) {
-                        uint32_t off = first;
-#pragma unroll
-                        for (int w = 0; w < FWPT; w++) {
-                            uint32_t mm = m[st][w];
-                            while (mm) {
-                                const int b = __ffs(mm) - 1;
-                                items[off++] = pbase + 32u * w + (uint32_t)b;
-                                mm &= mm - 1;
-                            }
-                        }
-                    } else {
-                        uint32_t rank = first;
-#pragma unroll
-                        for (int w = 0; w < FWPT; w++) {
-                            uint32_t mm = m[st][w];
-                            while (mm) {
-                                const int b = __ffs(mm) - 1;
-                                if (rank >= r0 && rank < r0 + FSTAGE_ITEMS) items[rank - r0] = pbase + 32u * w + (uint32_t)b;
-                                rank++;
-                                mm &= mm - 1;
-                            }
+                    for (int w = 0; w < FWPT; w++) {
+                        uint32_t mm = m[st][w];
+                        while (mm) {
+                            const int b = __ffs(mm) - 1;
+                            items[off++] = pbase + 32u * w + (uint32_t)b;
+                            mm &= mm - 1;
                         }
                     }
-                    __syncthreads();
-                    uint32_t n_round = min(total - r0, (uint32_t)FSTAGE_ITEMS);
-                    const unsigned long long o0 = base + r0;
-                    if (o0 >= a.cap) n_round = 0;
-                    else if (a.cap - o0 < n_round) n_round = (uint32_t)(a.cap - o0);
-                    uint32_t* __restrict__ dst = out + o0;
-                    for (uint32_t i = tid; i < n_round; i += FT) dst[i] = items[i];
-                    __syncthreads();
+                } else {
+                    uint32_t rank = first;
+#pragma unroll
+                    for (int w = 0; w < FWPT; w++) {
+                        uint32_t mm = m[st][w];
+                        while (mm) {
+                            const int b = __ffs(mm) - 1;
+                            if (rank >= r0 && rank < r0 + FSTAGE_ITEMS) items[rank - r0] = pbase + 32u * w + (uint32_t)b;
+                            rank++;
+                            mm &= mm - 1;
+                        }
+                    }
                 }
+                __syncthreads();
+                uint32_t n_round = min(total - r0, (uint32_t)FSTAGE_ITEMS);
+                const unsigned long long o0 = base + r0;
+                if (o0 >= a.cap) n_round = 0;
+                else if (a.cap - o0 < n_round) n_round = (uint32_t)(a.cap - o0);
+                uint32_t* __restrict__ dst = out + o0;
+                for (uint32_t i = tid; i < n_round; i += FT) dst[i] = items[i];
+                __syncthreads();
             }
-            run_f += tot & 0xFFFFu;
-            run_r += tot >> 16;
         }
+        run_f += tot & 0xFFFFu;
+        run_r += tot >> 16;
     }
 }
 
@@ -326,9 +335,10 @@ using namespace cof;
 
 extern "C" {
 
-size_t cof_find_workspace_bytes(uint64_t n_owned) {
-    (void)n_owned;   // per-CTA totals (at most FMAX_CTAS CTAs) + the grid barrier counter
-    return FWS_BARRIER + 64;
+size_t cof_find_workspace_bytes(uint64_t n_bases) {
+    // per-CTA totals (at most FMAX_CTAS CTAs) + the grid barrier counter + 8 bytes of PAM
+    // masks per plane word (the tiles cover cof_plane_words(n_bases) words)
+    return FWS_MASKS + (size_t)cof_plane_words(n_bases) * 8;
 }
 
 cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
@@ -362,6 +372,7 @@ cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* d
         a.cap = items_cap;
         a.status = (uint64_t*)workspace;
         a.barrier = (unsigned int*)((uint8_t*)workspace + FWS_BARRIER);
+        a.masks = (uint32_t*)((uint8_t*)workspace + FWS_MASKS);
         a.counters = counters;
         a.n_tiles = n_tiles;
         a.ne = plan->pam[0].n;

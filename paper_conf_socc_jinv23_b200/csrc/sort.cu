@@ -53,10 +53,16 @@ __global__ void __launch_bounds__(ST) cof_sort_hist(const __grid_constant__ Sort
     const uint64_t n = sort_n(p);
     const uint64_t base = (uint64_t)blockIdx.x * STILE;
     if (base < n) {
-#pragma unroll 4
+        unsigned long long kk[SV];
+#pragma unroll
         for (int v = 0; v < SV; v++) {
             const uint64_t i = base + (uint64_t)v * ST + threadIdx.x;
-            if (i < n) atomicAdd(&h[digit_of(p.src[i], p.gb, p.shift)], 1u);
+            kk[v] = i < n ? __ldcg(p.src + i) : 0ull;
+        }
+#pragma unroll
+        for (int v = 0; v < SV; v++) {
+            const uint64_t i = base + (uint64_t)v * ST + threadIdx.x;
+            if (i < n) atomicAdd(&h[digit_of(kk[v], p.gb, p.shift)], 1u);
         }
     }
     __syncthreads();
@@ -125,42 +131,86 @@ __global__ void __launch_bounds__(ST) cof_sort_scan(const __grid_constant__ Sort
     }
 }
 
+// Stable scatter of one 4096-key tile.  Warp w owns keys [w*512, w*512+512) of the tile,
+// lane l holds slots k = 0..15 (index w*512 + 32k + l, coalesced): going slot by slot with
+// __match_any_sync and a warp-private digit counter gives every key its rank among the
+// equal-digit keys of its warp in index order (no block barrier per slot).  One block-wide
+// prefix then turns (warp, digit) counts into tile-local digit starts; keys are staged in
+// shared memory in digit order and written out with consecutive threads writing
+// consecutive keys of a digit run (coalesced).
 __global__ void __launch_bounds__(ST) cof_sort_scatter(const __grid_constant__ SortPass p) {
-    __shared__ uint32_t s_off[256];          // global offset of this tile's digit d
-    __shared__ uint32_t s_run[256];          // keys of digit d already placed from earlier rounds
-    __shared__ uint32_t s_wc[ST / 32][256];  // per-warp counts -> exclusive warp offsets
-    const int tid = threadIdx.x, warp = tid >> 5;
+    constexpr int NW = ST / 32;
+    __shared__ uint32_t s_cnt[NW][256];          // per-warp digit counts -> exclusive prefixes
+    __shared__ uint32_t s_goff[256];             // global offset of this tile's digit d
+    __shared__ uint32_t s_dstart[256];           // tile-local start of digit d
+    __shared__ uint32_t s_warp[NW];
+    __shared__ unsigned long long s_keys[STILE];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const uint64_t n = sort_n(p);
     const uint64_t base = (uint64_t)blockIdx.x * STILE;
     if (base >= n) return;
-    s_off[tid] = p.hist[(size_t)tid * p.cap_tiles + blockIdx.x];
-    s_run[tid] = 0;
-    for (int w = 0; w < ST / 32; w++) s_wc[w][tid] = 0;
-    __syncthreads();
-    for (int v = 0; v < SV; v++) {
-        const uint64_t i = base + (uint64_t)v * ST + tid;
-        const bool ok = i < n;
-        unsigned long long key = ok ? p.src[i] : 0ull;
-        const uint32_t d = ok ? digit_of(key, p.gb, p.shift) : 256u;   // 256: not a key
-        const unsigned peers = __match_any_sync(0xffffffffu, d);
-        const uint32_t rank = (uint32_t)__popc(peers & lanemask_lt());
-        if (ok && rank == 0) s_wc[warp][d] = (uint32_t)__popc(peers);
-        __syncthreads();
-        {   // digit tid: exclusive prefix over warps, continuing the running count
-            uint32_t run = s_run[tid];
+    const uint32_t n_tile = (uint32_t)min((uint64_t)STILE, n - base);
 #pragma unroll
-            for (int w = 0; w < ST / 32; w++) {
-                const uint32_t c = s_wc[w][tid];
-                s_wc[w][tid] = run;
-                run += c;
-            }
-            s_run[tid] = run;
+    for (int w = 0; w < NW; w++) s_cnt[w][tid] = 0;
+    s_goff[tid] = p.hist[(size_t)tid * p.cap_tiles + blockIdx.x];
+    __syncthreads();
+
+    unsigned long long key[SV];
+    uint32_t rank[SV];
+#pragma unroll
+    for (int k = 0; k < SV; k++) {   // all loads first: 16 independent requests in flight
+        const uint32_t li = (uint32_t)warp * (STILE / NW) + (uint32_t)k * 32 + lane;
+        key[k] = li < n_tile ? __ldcs(p.src + base + li) : 0ull;
+    }
+#pragma unroll
+    for (int k = 0; k < SV; k++) {
+        const uint32_t li = (uint32_t)warp * (STILE / NW) + (uint32_t)k * 32 + lane;
+        const bool ok = li < n_tile;
+        const uint32_t d = ok ? digit_of(key[k], p.gb, p.shift) : 256u;
+        const unsigned peers = __match_any_sync(0xffffffffu, d);
+        const int leader = __ffs(peers) - 1;
+        uint32_t old = 0;
+        if (lane == leader && ok) old = s_cnt[warp][d];
+        old = __shfl_sync(0xffffffffu, old, leader);
+        if (lane == leader && ok) s_cnt[warp][d] = old + (uint32_t)__popc(peers);
+        __syncwarp();
+        rank[k] = old + (uint32_t)__popc(peers & lanemask_lt());
+    }
+    __syncthreads();
+    // digit tid: exclusive prefix over warps, then exclusive scan of the digit totals
+    uint32_t run = 0;
+#pragma unroll
+    for (int w = 0; w < NW; w++) {
+        const uint32_t c = s_cnt[w][tid];
+        s_cnt[w][tid] = run;
+        run += c;
+    }
+    uint32_t x = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+    }
+    if (lane == 31) s_warp[warp] = x;
+    __syncthreads();
+    uint32_t wbase = 0;
+#pragma unroll
+    for (int w = 0; w < NW; w++) wbase += w < warp ? s_warp[w] : 0u;
+    s_dstart[tid] = wbase + x - run;
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < SV; k++) {
+        const uint32_t li = (uint32_t)warp * (STILE / NW) + (uint32_t)k * 32 + lane;
+        if (li < n_tile) {
+            const uint32_t d = digit_of(key[k], p.gb, p.shift);
+            s_keys[s_dstart[d] + s_cnt[warp][d] + rank[k]] = key[k];
         }
-        __syncthreads();
-        if (ok) p.dst[s_off[d] + s_wc[warp][d] + rank] = key;
-        __syncthreads();
-        for (int w = 0; w < ST / 32; w++) s_wc[w][tid] = 0;
-        __syncthreads();
+    }
+    __syncthreads();
+    for (uint32_t j = tid; j < n_tile; j += ST) {
+        const unsigned long long kk = s_keys[j];
+        const uint32_t d = digit_of(kk, p.gb, p.shift);
+        p.dst[s_goff[d] + (j - s_dstart[d])] = kk;
     }
 }
 

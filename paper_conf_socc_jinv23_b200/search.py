@@ -148,6 +148,23 @@ class HostGenome:
             self.planes.append(buf)
             self.segs.append(segs)
 
+    @classmethod
+    def from_packer(cls, chunks, pack, pin: bool = True):
+        """Single-segment chunks packed by ``pack(chrom, first, n, lo, hi, nm)`` (e.g. straight
+        from an indexed FASTA file, cof_fasta_pack) without materialising the ASCII."""
+        self = cls.__new__(cls)
+        self.chunks, self.planes, self.segs = chunks, [], []
+        pin = pin and torch.cuda.is_available()
+        for ch in chunks:
+            if ch.multi:
+                raise ValueError("from_packer builds single-segment chunks")
+            words = cof.cof_plane_words(ch.n_bases)
+            buf = torch.empty((3, words), dtype=torch.int32, pin_memory=pin)
+            pack(ch.chrom, ch.start, ch.n_bases, buf[0], buf[1], buf[2])
+            self.planes.append(buf)
+            self.segs.append(None)
+        return self
+
     def chunk_struct(self, i) -> cof.cof_chunk:
         ch, buf, segs = self.chunks[i], self.planes[i], self.segs[i]
         if ch.multi:

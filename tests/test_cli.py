@@ -1,0 +1,47 @@
+"""Cas-OFFinder-style input file / TSV output."""
+import os
+
+import numpy as np
+import pytest
+
+from oracle import oracle
+from paper_conf_socc_jinv23_b200 import cli, cof, synth
+
+
+def test_parse_input(tmp_path):
+    spec = cli.parse_input("genome.fa\nNNNNNRG\nACGTANN 1\n# comment\nTTTTTNN 0\n", str(tmp_path))
+    assert spec.genome == os.path.join(str(tmp_path), "genome.fa")
+    assert spec.pattern == "NNNNNRG" and spec.queries == ["ACGTANN", "TTTTTNN"] and spec.thresholds == [1, 0]
+    for bad in ("g\nNNRG\n", "g\nNNRG\nACG 1\n", "g\nNNRG\nACGT\n", "g\nNNRG\nACGT -1\n"):
+        with pytest.raises(ValueError):
+            cli.parse_input(bad)
+
+
+def test_format_hits():
+    h = np.zeros(2, dtype=cof.HIT_DTYPE)
+    h[0] = (1, 0, 12, b"+", 2, b"ACgTaGG")
+    h[1] = (0, 1, 7, b"-", 0, b"ACGTAGG")
+    txt = cli.format_hits(h, ["Q0NNNNN", "Q1NNNNN"], ["chrA", "chrB"])
+    assert txt == "Q1NNNNN\tchrA\t12\tACgTaGG\t+\t2\nQ0NNNNN\tchrB\t7\tACGTAGG\t-\t0\n"
+
+
+@pytest.mark.gpu
+def test_cli_end_to_end(tmp_path):
+    rng = np.random.default_rng(31)
+    seqs = [synth.random_genome_text(rng, n, b"ACGTacgtN", p=[.23, .2, .2, .23, .03, .03, .03, .03, .02])
+            for n in (40_000, 25_001, 500)]
+    names = ["chr1", "chr2", "chrM"]
+    gdir = tmp_path / "genome"
+    gdir.mkdir()
+    synth.write_fasta(gdir / "a.fa", names[:2], seqs[:2])
+    synth.write_fasta(gdir / "b.fa", names[2:], seqs[2:], width=70)
+    guides = ["".join(rng.choice(list("ACGT"), 20)) + "NNN" for _ in range(5)]
+    inp = tmp_path / "input.txt"
+    inp.write_text("genome\n" + "N" * 21 + "RG\n" + "".join(f"{g} 9\n" for g in guides))
+    out = tmp_path / "out.txt"
+    assert cli.main([str(inp), "G", str(out), "--chunk-bases", "9999"]) == 0
+    ref = oracle.search(seqs, "N" * 21 + "RG", guides, [9] * 5)
+    exp = "".join(f"{guides[int(h['guide'])]}\t{names[int(h['chrom'])]}\t{int(h['pos'])}\t{h['site'].decode()}\t"
+                  f"{h['strand'].decode()}\t{int(h['mm'])}\n" for h in ref)
+    assert len(ref) > 10
+    assert out.read_text() == exp

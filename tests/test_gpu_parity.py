@@ -106,7 +106,7 @@ def test_finder_candidates_match_oracle():
             d = torch.from_numpy(host.view(np.int32)).cuda()
             dch = cof.make_chunk(0, start, nb, owned, d[0], d[1], d[2])
             items = torch.empty((2, owned), dtype=torch.int32, device="cuda")
-            ws = torch.empty(cof.cof_find_workspace_bytes(owned), dtype=torch.uint8, device="cuda")
+            ws = torch.empty(cof.cof_find_workspace_bytes(nb), dtype=torch.uint8, device="cuda")
             nf, nr = cof.cof_find_pam(plan, pd, dch, ws, items[0], items[1], owned, s)
             for k, st in enumerate("+-"):
                 exp = oracle.pam_sites(seq, pat, st, start, start + owned) - start
@@ -200,3 +200,18 @@ def test_search_host_into_caller_buffer_and_chunk_pipeline():
     assert cof.hits_to_tuples(got) == exp
     small = np.empty(max(1, len(exp) // 3), dtype=cof.HIT_DTYPE)
     assert cof.hits_to_tuples(srch.search_host(host, out=small)) == exp
+
+
+def test_many_guides_multiple_table_launches():
+    """> 4096 guides: the table comparer splits the guides into launches of 128 blocks
+    (thresholds in the parameter space) and tiles them through shared memory."""
+    rng = np.random.default_rng(21)
+    seq = synth.random_genome_text(rng, 30_000)
+    n_g = 4096 + 300
+    guides = ["".join(rng.choice(list("ACGT"), 20)) + "NNN" for _ in range(n_g)]
+    thr = [int(t) for t in rng.integers(4, 8, n_g)]
+    exp = ref_hits([seq], "N" * 21 + "RG", guides, thr)
+    assert len(exp) > 0
+    assert gpu_hits([seq], "N" * 21 + "RG", guides, thr) == exp
+    thr_u = [7] * n_g
+    assert gpu_hits([seq], "N" * 21 + "RG", guides, thr_u) == ref_hits([seq], "N" * 21 + "RG", guides, thr_u)
