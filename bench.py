@@ -129,22 +129,31 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
         cof.cof_plan_upload(st.plan, pd, st.stream)
         st.plan_devs.append(pd)
     max_owned = max(ch.n_owned for ch in chunks)
-    st.items = torch.empty((2, max_owned), dtype=torch.int32, device=st.device)
-    st.find_ws = torch.empty(cof.cof_find_workspace_bytes(max(ch.n_bases for ch in chunks)), dtype=torch.uint8, device=st.device)
+    # fused find+compare (finder masks -> comparer, no item lists) unless the guide table is
+    # too large for it or COF_FUSED=0; the two-call path writes / reads ordered item lists
+    st.fused = search.use_fused(st.plan, len(wl.guides))
+    st.items = torch.empty((2, 1 if st.fused else max_owned), dtype=torch.int32, device=st.device)
+    st.find_ws = torch.empty(cof.cof_find_compare_workspace_bytes(max(ch.n_bases for ch in chunks)),
+                             dtype=torch.uint8, device=st.device)
     # first pass with host counts: exact item / hit counts per chunk
     st.counts = []
     tmp_cap = 1 << 20
     tmp_hits = torch.empty(tmp_cap, dtype=torch.int64, device=st.device)
     for i, ch in enumerate(chunks):
-        nf, nr = cof.cof_find_pam(st.plan, st.plan_devs[i], st.d_chunks[i], st.find_ws, st.items[0], st.items[1],
-                                  max_owned, st.stream)
         try:
-            nh = cof.cof_compare(st.plan, st.plan_devs[i], st.d_chunks[i], st.items[0], nf, st.items[1], nr,
-                                 tmp_hits, tmp_cap, st.stream)
+            if st.fused:
+                cof.cof_find_masks(st.plan, st.plan_devs[i], st.d_chunks[i], st.find_ws, st.stream)
+                nh = cof.cof_compare_masks(st.plan, st.plan_devs[i], st.d_chunks[i], st.find_ws, tmp_hits, tmp_cap,
+                                           st.stream)
+            else:
+                nf, nr = cof.cof_find_pam(st.plan, st.plan_devs[i], st.d_chunks[i], st.find_ws, st.items[0],
+                                          st.items[1], max_owned, st.stream)
+                nh = cof.cof_compare(st.plan, st.plan_devs[i], st.d_chunks[i], st.items[0], nf, st.items[1], nr,
+                                     tmp_hits, tmp_cap, st.stream)
         except cof.CofError as e:
             if e.status != cof.COF_E_CAPACITY:
                 raise
-            nh = cof.cof_read_counts(st.plan, st.plan_devs[i], st.stream)[2]
+        nf, nr, nh = cof.cof_read_counts(st.plan, st.plan_devs[i], st.stream)
         st.counts.append((nf, nr, nh))
     del tmp_hits
     st.caps = [max(1024, int(c[2] * 1.1) + 1024) for c in st.counts]
@@ -156,26 +165,38 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
     return wl, st
 
 
-def run_device_pipeline(wl, st, collect=False, events=None):
+def run_device_pipeline(wl, st, collect=False, events=None, fevents=None):
     """One step on the device: per chunk find -> compare -> sort, counts kept on the
-    device (no host round trip between kernels).  ``events``: list to append
-    (start, end) CUDA event pairs bracketing each comparer launch.  With ``collect``
+    device (no host round trip between kernels).  ``events`` / ``fevents``: lists to append
+    (start, end) CUDA event pairs bracketing each comparer / finder call.  With ``collect``
     returns the merged, decorated hit array (cof_collect + cof_merge)."""
     import torch
     from paper_conf_socc_jinv23_b200 import cof, search
 
     ON = cof.COF_COUNT_ON_DEVICE
     s = st.stream
+
+    def ev():
+        e = torch.cuda.Event(enable_timing=True)
+        e.record(s)
+        return e
+
     for i in range(len(st.chunks)):
         dch, pd = st.d_chunks[i], st.plan_devs[i]
-        cof.cof_find_pam(st.plan, pd, dch, st.find_ws, st.items[0], st.items[1], st.max_owned, s, sync=False)
+        f0 = ev() if fevents is not None else None
+        if st.fused:
+            cof.cof_find_masks(st.plan, pd, dch, st.find_ws, s)
+        else:
+            cof.cof_find_pam(st.plan, pd, dch, st.find_ws, st.items[0], st.items[1], st.max_owned, s, sync=False)
+        if fevents is not None:
+            fevents.append((f0, ev()))
+        e0 = ev() if events is not None else None
+        if st.fused:
+            cof.cof_compare_masks(st.plan, pd, dch, st.find_ws, st.hits[i], st.caps[i], s, sync=False)
+        else:
+            cof.cof_compare(st.plan, pd, dch, st.items[0], ON, st.items[1], ON, st.hits[i], st.caps[i], s, sync=False)
         if events is not None:
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(s)
-        cof.cof_compare(st.plan, pd, dch, st.items[0], ON, st.items[1], ON, st.hits[i], st.caps[i], s, sync=False)
-        if events is not None:
-            e1.record(s)
-            events.append((e0, e1))
+            events.append((e0, ev()))
         cof.cof_sort_hits(st.plan, pd, dch, st.hits[i], st.tmp, st.caps[i], ON, st.sort_ws, s)
     if not collect:
         return None
@@ -205,7 +226,7 @@ def run_e2e_step(wl, st, searcher, out=None):
     ``out``: the caller's result buffer (reused between steps, as an application would)."""
     hits = searcher.search_host(st.e2e_host, out=out)
     h2d = st.e2e_host.bytes
-    d2h = len(hits) * 8 + 24 * len(st.e2e_host.chunks)      # sorted keys + per-chunk counts
+    d2h = len(hits) * 56 + 24 * len(st.e2e_host.chunks)     # decorated records + per-chunk counts
     return hits, h2d, d2h
 
 
@@ -295,12 +316,12 @@ def main():
 
     clocks = ClockSampler(local)
     clocks.start()
-    events = []
+    events, fevents = [], []
     launches0 = cof.cof_launch_count()
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     t_start.record(st.stream)
     for _ in range(args.steps):
-        run_device_pipeline(wl, st, events=events)
+        run_device_pipeline(wl, st, events=events, fevents=fevents)
     t_end.record(st.stream)
     torch.cuda.synchronize(dev)
     launches = cof.cof_launch_count() - launches0
@@ -308,6 +329,7 @@ def main():
     barrier()
     ms_total = t_start.elapsed_time(t_end)
     cmp_ms = sum(a.elapsed_time(b) for a, b in events)
+    find_ms = sum(a.elapsed_time(b) for a, b in fevents)
     totals = step_counts(st)   # verifies capacities
 
     # max over ranks
@@ -334,6 +356,22 @@ def main():
     roof = comparer_roof(st.plan, n_sm, sm_max, args.comparer)
     cmp_rate = comps_mine * args.steps / (cmp_ms * 1e-3) if cmp_ms > 0 else 0.0
     n_cmp_launch = len(events)
+
+    # finder roofline (HBM): algorithmic bytes of the search kernel per step
+    plane_bytes = sum(cof.cof_plane_words(ch.n_bases) * 4 * (4 if ch.multi else 3) for ch in st.chunks)
+    words = sum(cof.cof_plane_words(ch.n_bases) for ch in st.chunks)
+    if st.fused:      # planes (+ valid-start plane) read, {fwd, rev} masks written
+        find_bytes = plane_bytes + words * 8
+        find_basis = "planes read + 8 B of PAM masks per plane word written (fused path)"
+    else:             # planes read, 4 B per item written
+        find_bytes = plane_bytes + 4 * my_items
+        find_basis = "planes read + 4 B per item written (two-call path)"
+    find_gbs = find_bytes * args.steps / (find_ms * 1e-3) / 1e9 if find_ms > 0 else 0.0
+    hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
+    finder_roof = {"bound": "hbm", "kernel": "cof_finder_kernel", "achieved": round(find_gbs, 1),
+                   "peak": hbm_peak, "unit": "GB/s", "frac": find_gbs / hbm_peak,
+                   "bytes_per_step": int(find_bytes), "basis": find_basis,
+                   "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_finder_kernel", st)}
 
     e2e = None
     if not args.no_e2e:
@@ -365,11 +403,13 @@ def main():
                        "parallelism": f"chromosome LPT shards over {world} GPU(s)",
                        "comparer": args.comparer,
                        "l2": "inputs larger than L2 (1.16 GB planes + item lists), no flush"},
-            "roofline": {"bound": "alu", "kernel": f"cof_comparer_{args.comparer}",
+            "roofline": {"bound": "alu", "kernel": f"cof_comparer_{'fused' if st.fused else args.comparer}",
                          "achieved": cmp_rate, "peak": roof["peak"], "unit": "comparisons/s",
-                         "frac": cmp_rate / roof["peak"] if roof["peak"] else None, "traffic": None,
+                         "frac": cmp_rate / roof["peak"] if roof["peak"] else None,
+                         "traffic": traffic_for("cof_comparer", st),
                          "peak_basis": roof["basis"], "launches": n_cmp_launch,
                          "share_of_step": cmp_ms_max / ms_total if ms_total else None},
+            "finder_roofline": finder_roof,
             "gpu_launches": int(launches // args.steps) if args.steps else 0,
             "gpu_launches_timed_region": int(launches),
             "clocks": clk,
@@ -381,6 +421,18 @@ def main():
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def traffic_for(kernel, st):
+    """DRAM bytes per launch of ``kernel`` from the committed ncu --set full capture
+    (profiles/roofline_traffic.json), or None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "roofline_traffic.json")) as f:
+            d = json.load(f)
+        key = f"{kernel}_{'fused' if st.fused else 'twocall'}"
+        return d.get(key, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
 
 
 def comparer_roof(plan, n_sm, sm_mhz, impl):
@@ -430,8 +482,10 @@ def measure_e2e(wl, st, dev, args, world, genome_bases):
     srch.reserve(max(ch.n_bases for ch in chunks), max(st.caps))
     from paper_conf_socc_jinv23_b200 import cof
     hits0, _, _ = run_e2e_step(wl, st, srch)     # warm-up; sizes the caller's result buffer
-    out = np.empty(int(len(hits0) * 1.05) + 1024, dtype=cof.HIT_DTYPE)
-    out[:] = np.zeros(1, dtype=cof.HIT_DTYPE)    # touch the pages once, outside the timed steps
+    n_out = int(len(hits0) * 1.05) + 1024
+    # the caller's result buffer: pinned host memory, so the device-decorated records DMA
+    # straight into it (allocated and touched once, outside the timed steps)
+    out = torch.zeros(n_out * cof.HIT_DTYPE.itemsize, dtype=torch.uint8, pin_memory=True).numpy().view(cof.HIT_DTYPE)
     del hits0
     torch.cuda.synchronize(dev)
     if world > 1:
@@ -450,9 +504,9 @@ def measure_e2e(wl, st, dev, args, world, genome_bases):
         dt = float(t[0])
     return {"value": round(genome_bases / dt / 1e9, 4), "unit": "Gbases/s", "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "s_per_step": dt, "hits": nh,
-            "path": "Searcher.search_host: cof_load_chunk -> cof_find_pam -> cof_compare -> cof_sort_hits "
-                    "-> D2H keys -> cof_collect (host thread, overlapped with the next chunk) -> cof_merge, "
-                    "from pinned packed host planes (wall clock)"}
+            "path": "Searcher.search_host: cof_load_chunk (copy stream, double-buffered) -> cof_find_pam -> "
+                    "cof_compare -> cof_sort_hits -> cof_decorate (device) -> D2H of the records into the "
+                    "caller's pinned buffer, from pinned packed host planes (wall clock)"}
 
 
 def main_reference(args, cfgname, metric):

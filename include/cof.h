@@ -177,6 +177,28 @@ cof_status cof_compare(const cof_plan *plan, void *plan_dev, const cof_chunk *de
                        const uint32_t *items_rev, uint64_t n_rev,
                        uint64_t *hits, uint64_t hits_cap, uint64_t *n_hits, cof_stream s);
 
+/* ------------------------------------------------------------------ fused find + compare
+ * the search and compare kernels of P:L29 without the host hand-off and
+ * without the item lists: the finder (pass 1 only) writes per-word PAM masks into the
+ * workspace and the comparer expands them itself (shared-memory queue) before the table
+ * comparison.  Same hits as cof_find_pam + cof_compare (same key format, unordered); the
+ * item counts land in plan_dev (cof_read_counts).  Requires the whole guide table to fit
+ * in shared memory (cof_find_compare_supported); otherwise COF_E_ARG.
+ *  workspace  dev, >= cof_find_compare_workspace_bytes(dev->n_bases) bytes. */
+int        cof_find_compare_supported(const cof_plan *plan);
+size_t     cof_find_compare_workspace_bytes(uint64_t n_bases);
+/* = cof_find_masks + cof_compare_masks */
+cof_status cof_find_compare(const cof_plan *plan, void *plan_dev, const cof_chunk *dev, void *workspace,
+                            uint64_t *hits, uint64_t hits_cap, uint64_t *n_hits, cof_stream s);
+/* The search kernel's pass 1 alone: PAM masks of every plane word, both strands, into the
+ * workspace ({fwd, rev} 32-bit masks per plane word, bit b = window start 32w + b);
+ * item counts into plan_dev.  Asynchronous. */
+cof_status cof_find_masks(const cof_plan *plan, void *plan_dev, const cof_chunk *dev, void *workspace,
+                          cof_stream s);
+/* The comparer over those masks (n_hits: host count, NULL = no sync). */
+cof_status cof_compare_masks(const cof_plan *plan, void *plan_dev, const cof_chunk *dev, void *workspace,
+                             uint64_t *hits, uint64_t hits_cap, uint64_t *n_hits, cof_stream s);
+
 /* ------------------------------------------------------------------ sort (M10, K3)
  * Deterministic order of the hit keys (the paper's atomics are unordered):
  * stable LSD radix sort on the device of the key bits that vary for this chunk.
@@ -212,6 +234,18 @@ typedef struct {
  * If hits_dev is NULL, keys are read from host_keys instead (already on the host). */
 cof_status cof_collect(const cof_plan *plan, const cof_chunk *host, const uint64_t *hits_dev,
                        const uint64_t *host_keys, uint64_t n_hits, cof_hit *out, cof_stream s);
+
+/* The same decoration on the device: n_hits (sorted) keys of hits_dev -> n_hits records in
+ * the DEVICE buffer out_dev (same order), one thread per hit, from the device planes of
+ * the chunk and the guide masks in plan_dev; dev->segs (host) is copied into workspace
+ * (>= cof_decorate_workspace_bytes(dev->n_segs) device bytes).  Asynchronous; a key that
+ * does not match the chunk/plan sets a flag that cof_decorate_check reports (COF_E_STATE,
+ * synchronizes).  The caller copies the records to the host (pinned memory: no staging). */
+size_t     cof_decorate_workspace_bytes(uint32_t n_segs);
+cof_status cof_decorate(const cof_plan *plan, const void *plan_dev, const cof_chunk *dev,
+                        const uint64_t *hits_dev, uint64_t n_hits, cof_hit *out_dev,
+                        void *workspace, cof_stream s);
+cof_status cof_decorate_check(const void *workspace, cof_stream s);
 
 /* k-way merge of sorted lists into out (sum of lens records), order (chrom, pos,
  * strand, guide) (G13).  Lists from disjoint chunks merge by concatenation. */

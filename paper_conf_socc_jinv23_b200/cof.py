@@ -80,6 +80,14 @@ def _load():
         "cof_read_counts": (I32, [P, P, P, P]),
         "cof_collect": (I32, [P, P, P, P, U64, P, P]),
         "cof_merge": (I32, [P, P, U32, P]),
+        "cof_decorate_workspace_bytes": (SZ, [U32]),
+        "cof_decorate": (I32, [P, P, P, P, U64, P, P, P]),
+        "cof_decorate_check": (I32, [P, P]),
+        "cof_find_compare_supported": (ctypes.c_int, [P]),
+        "cof_find_compare_workspace_bytes": (SZ, [U64]),
+        "cof_find_compare": (I32, [P, P, P, P, P, U64, P, P]),
+        "cof_find_masks": (I32, [P, P, P, P, P]),
+        "cof_compare_masks": (I32, [P, P, P, P, P, U64, P, P]),
         "cof_set_comparer": (I32, [ctypes.c_int]),
     }
     for name, (res, args) in sig.items():
@@ -99,7 +107,10 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_fasta_count", "cof_fasta_name", "cof_fasta_length", "cof_fasta_pack",
                        "cof_find_workspace_bytes", "cof_find_pam", "cof_compare",
                        "cof_sort_workspace_bytes", "cof_sort_hits", "cof_read_counts",
-                       "cof_collect", "cof_merge")]
+                       "cof_collect", "cof_merge", "cof_decorate_workspace_bytes", "cof_decorate",
+                       "cof_decorate_check", "cof_find_compare_supported",
+                       "cof_find_compare_workspace_bytes", "cof_find_compare", "cof_find_masks",
+                       "cof_compare_masks")]
 
 
 def _check(st):
@@ -251,6 +262,41 @@ def cof_compare(plan, plan_dev, dev: cof_chunk, items_fwd, n_fwd, items_rev, n_r
     return None
 
 
+def cof_find_compare_supported(plan) -> bool:
+    return bool(lib.cof_find_compare_supported(plan.handle))
+
+
+def cof_find_compare_workspace_bytes(n_bases: int) -> int:
+    return int(lib.cof_find_compare_workspace_bytes(int(n_bases)))
+
+
+def cof_find_compare(plan, plan_dev, dev: cof_chunk, workspace, hits, hits_cap, stream=None, sync=True):
+    """Fused finder + comparer; returns n_hits if ``sync`` else None (count stays on the device)."""
+    if sync:
+        n = ctypes.c_uint64()
+        _check(lib.cof_find_compare(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
+                                    _ptr(hits), int(hits_cap), ctypes.addressof(n), _stream(stream)))
+        return int(n.value)
+    _check(lib.cof_find_compare(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
+                                _ptr(hits), int(hits_cap), None, _stream(stream)))
+    return None
+
+
+def cof_find_masks(plan, plan_dev, dev: cof_chunk, workspace, stream=None):
+    _check(lib.cof_find_masks(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace), _stream(stream)))
+
+
+def cof_compare_masks(plan, plan_dev, dev: cof_chunk, workspace, hits, hits_cap, stream=None, sync=True):
+    if sync:
+        n = ctypes.c_uint64()
+        _check(lib.cof_compare_masks(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
+                                     _ptr(hits), int(hits_cap), ctypes.addressof(n), _stream(stream)))
+        return int(n.value)
+    _check(lib.cof_compare_masks(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
+                                 _ptr(hits), int(hits_cap), None, _stream(stream)))
+    return None
+
+
 def cof_sort_workspace_bytes(cap: int) -> int:
     return int(lib.cof_sort_workspace_bytes(int(cap)))
 
@@ -282,6 +328,20 @@ def cof_collect_into(plan, host: cof_chunk, host_keys, n_hits, out: np.ndarray):
         _check(lib.cof_collect(plan.handle, ctypes.addressof(host), None, _ptr(host_keys), int(n_hits),
                                out.ctypes.data, None))
     return out
+
+
+def cof_decorate_workspace_bytes(n_segs: int) -> int:
+    return int(lib.cof_decorate_workspace_bytes(int(n_segs)))
+
+
+def cof_decorate(plan, plan_dev, dev: cof_chunk, hits_dev, n_hits, out_dev, workspace, stream=None):
+    """Device decoration: n_hits keys -> n_hits cof_hit records in the device buffer out_dev."""
+    _check(lib.cof_decorate(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(hits_dev), int(n_hits),
+                            _ptr(out_dev), _ptr(workspace), _stream(stream)))
+
+
+def cof_decorate_check(workspace, stream=None):
+    _check(lib.cof_decorate_check(_ptr(workspace), _stream(stream)))
 
 
 def cof_merge(lists) -> np.ndarray:

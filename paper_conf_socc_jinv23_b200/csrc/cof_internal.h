@@ -77,6 +77,7 @@ struct DevLayout {
     size_t recs_fwd, recs_rev;       // uint4[n_recs]
     size_t ptab_fwd, ptab_rev;       // pair tables: uint2[n_blocks][n_pairs][25]
     size_t pmeta_fwd, pmeta_rev;     // per block: uint32[8] = {T0..T5 threshold planes, valid, 0}
+    size_t onehot;                   // uint32[2][n_guides][5] decoration masks (see cof_plan::onehot)
     size_t total;
 };
 

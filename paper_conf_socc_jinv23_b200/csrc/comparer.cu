@@ -204,6 +204,10 @@ struct TableArgs {
     uint32_t blocks_per_chunk;     // guide blocks resident in shared memory at a time
     PairLayout pairs;
     uint32_t meta[MAX_TABLE_BLOCKS][8];   // per block: T0..T5 threshold planes, valid mask
+    // fused find+compare: the finder's PAM masks replace the item list
+    const uint4* masks;            // one {fwd0, rev0, fwd1, rev1} per word pair
+    uint64_t n_wp;
+    unsigned int* ticket;          // dynamic grab counter (zeroed per launch)
 };
 
 // Hit mask (bit k = guide k of the block) of one item against one 32-guide block whose
@@ -226,10 +230,10 @@ __device__ __forceinline__ uint32_t table_hits(const uint32_t (&base)[NP], const
     }
 }
 
-__device__ __noinline__ void table_emit_v(const TableArgs& a, uint64_t item_idx, uint32_t hitm, uint32_t s0,
+__device__ __noinline__ void table_emit_v(const TableArgs& a, const uint32_t* pos_ptr, uint32_t hitm, uint32_t s0,
                                           uint32_t s1, uint32_t s2, uint32_t s3, uint32_t s4, uint32_t s5,
                                           uint32_t guide0) {
-    const uint32_t pos = __ldg(a.items + item_idx);
+    const uint32_t pos = *pos_ptr;   // item list (global) or the fused kernel's queue (shared)
     do {
         const int k = __ffs(hitm) - 1;
         hitm &= hitm - 1;
@@ -240,16 +244,16 @@ __device__ __noinline__ void table_emit_v(const TableArgs& a, uint64_t item_idx,
     } while (hitm);
 }
 
-__device__ __forceinline__ void table_emit(const TableArgs& a, uint64_t item_idx, uint32_t hitm, const uint32_t (&s)[6],
-                                           uint32_t guide0) {
-    table_emit_v(a, item_idx, hitm, s[0], s[1], s[2], s[3], s[4], s[5], guide0);
+__device__ __forceinline__ void table_emit(const TableArgs& a, const uint32_t* pos_ptr, uint32_t hitm,
+                                           const uint32_t (&s)[6], uint32_t guide0) {
+    table_emit_v(a, pos_ptr, hitm, s[0], s[1], s[2], s[3], s[4], s[5], guide0);
 }
 
 // All resident blocks [0, nb) for the R items of this thread.  base[r][q] = shared address of
 // item r's pair-q entry in block 0; groups of 4 blocks use immediate offsets.
-template <int NP, int R, bool TAIL, int TC>
+template <int NP, int R, bool TAIL, int TC, int STRIDE = CT>
 __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base)[R][NP], uint32_t nb, uint32_t gb0,
-                                             uint64_t item0, const uint32_t (&okm)[R]) {
+                                             const uint32_t* pos0, const uint32_t (&okm)[R]) {
     constexpr uint32_t BS = NP * 25 * 8;
     uint32_t b = 0;
     for (; b + 4 <= nb; b += 4) {
@@ -264,7 +268,7 @@ __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base
             if (TAIL) { h0 &= okm[r]; h1 &= okm[r]; h2 &= okm[r]; h3 &= okm[r]; }
             if (h0 | h1 | h2 | h3) {          // rare: ~1 hit per 2.5e4 comparisons at t = 6
                 // recompute the sums of the blocks that hit (keeps them out of the hot registers)
-                const uint64_t idx = item0 + (uint64_t)r * CT;
+                const uint32_t* idx = pos0 + r * STRIDE;
                 const uint32_t g0 = (a.block_base + gb0 + b) * 32u;
                 uint32_t sh[6];
                 if (h0) { table_hits<NP, 0 * BS, TC>(base[r], m + 0, sh); table_emit(a, idx, h0, sh, g0); }
@@ -283,11 +287,37 @@ __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base
             uint32_t s0[6];
             uint32_t h0 = table_hits<NP, 0, TC>(base[r], m, s0);
             if (TAIL) h0 &= okm[r];
-            if (h0) table_emit(a, item0 + (uint64_t)r * CT, h0, s0, (a.block_base + gb0 + b) * 32u);
+            if (h0) table_emit(a, pos0 + r * STRIDE, h0, s0, (a.block_base + gb0 + b) * 32u);
 #pragma unroll
             for (int q = 0; q < NP; q++) base[r][q] += BS;
         }
     }
+}
+
+// Byte offsets (within a guide block's table) of the NP pair entries of the window at pos.
+template <int NP>
+__device__ __forceinline__ void item_offsets(const TableArgs& a, uint32_t pos, uint32_t (&off)[NP]) {
+    if (a.pairs.contig) {
+        // fast path: window starting at the first compared offset; with no N among the
+        // compared positions every pair index is one nibble of Y (even pairs) or Z (odd)
+        const uint32_t p = pos + a.pairs.p0;
+        const uint32_t wn = plane_window(a.nm, p);
+        const uint32_t cm = a.pairs.n_cmp >= 32 ? ~0u : ((1u << a.pairs.n_cmp) - 1u);
+        if ((wn & cm) == 0) {
+            const uint32_t wl = plane_window(a.lo, p), wh = plane_window(a.hi, p);
+            const uint32_t Y = (wl & 0x33333333u) | ((wh & 0x33333333u) << 2);
+            const uint32_t Z = ((wl >> 2) & 0x33333333u) | (wh & 0xCCCCCCCCu);
+#pragma unroll
+            for (int q = 0; q < NP; q++) {
+                const uint32_t src = (q & 1) ? Z : Y;
+                const int k = q >> 1;
+                const uint32_t nib8 = k == 0 ? (src << 3) & 0x78u : (src >> (4 * k - 3)) & 0x78u;
+                off[q] = (uint32_t)q * 128u + nib8;
+            }
+            return;
+        }
+    }
+    pair_offsets<NP>(a.pairs, plane_window(a.lo, pos), plane_window(a.hi, pos), plane_window(a.nm, pos), off);
 }
 
 template <int NP, int R, int TC>
@@ -328,31 +358,7 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constan
         for (int r = 0; r < R; r++) {
             const uint64_t idx = item0 + (uint64_t)r * CT;
             okm[r] = idx < n ? ~0u : 0u;
-            const uint32_t pos = cur[r];
-            bool done = false;
-            if (a.pairs.contig) {
-                // fast path: window starting at the first compared offset; with no N among the
-                // compared positions every pair index is one nibble of Y (even pairs) or Z (odd)
-                const uint32_t p = pos + a.pairs.p0;
-                const uint32_t wn = plane_window(a.nm, p);
-                const uint32_t cm = a.pairs.n_cmp >= 32 ? ~0u : ((1u << a.pairs.n_cmp) - 1u);
-                if ((wn & cm) == 0) {
-                    const uint32_t wl = plane_window(a.lo, p), wh = plane_window(a.hi, p);
-                    const uint32_t Y = (wl & 0x33333333u) | ((wh & 0x33333333u) << 2);
-                    const uint32_t Z = ((wl >> 2) & 0x33333333u) | (wh & 0xCCCCCCCCu);
-#pragma unroll
-                    for (int q = 0; q < NP; q++) {
-                        const uint32_t src = (q & 1) ? Z : Y;
-                        const int k = q >> 1;
-                        const uint32_t nib8 = k == 0 ? (src << 3) & 0x78u : (src >> (4 * k - 3)) & 0x78u;
-                        off[r][q] = (uint32_t)q * 128u + nib8;
-                    }
-                    done = true;
-                }
-            }
-            if (!done)
-                pair_offsets<NP>(a.pairs, plane_window(a.lo, pos), plane_window(a.hi, pos), plane_window(a.nm, pos),
-                                 off[r]);
+            item_offsets<NP>(a, cur[r], off[r]);
         }
         for (uint32_t ch = 0; ch < n_chunks; ch++) {
             const uint32_t b0 = ch * bpc;
@@ -371,11 +377,111 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constan
             for (int r = 0; r < R; r++)
 #pragma unroll
                 for (int q = 0; q < NP; q++) base[r][q] = s_tab + off[r][q];
-            if (tail) table_blocks<NP, R, true, TC>(a, base, nb, b0, item0, okm);
-            else table_blocks<NP, R, false, TC>(a, base, nb, b0, item0, okm);
+            if (tail) table_blocks<NP, R, true, TC>(a, base, nb, b0, a.items + item0, okm);
+            else table_blocks<NP, R, false, TC>(a, base, nb, b0, a.items + item0, okm);
         }
     }
     (void)BS;
+}
+
+
+// ============================================================================ fused find+compare
+// the comparer consumes the finder's per-word PAM masks directly.  Each
+// CTA grabs ranges of FGRAB word pairs (dynamic), expands the set bits of its strand into
+// a shared-memory queue of positions (block scan -> ordered), and runs the table
+// comparison on full batches of CT*R queued items; leftovers carry over to the next grab.
+// No item list is written or read (4 B/item x 2), and the finder shrinks to its pass 1.
+constexpr uint32_t FGRAB = 32;            // word pairs per grab (one per lane of a warp)
+constexpr uint32_t FWQ = 256;             // per-warp ring of queued positions (multiple of 32 * R)
+
+// Per-warp queues: each warp grabs its own word-pair ranges (dynamic ticket), expands its
+// strand's set bits into its ring (warp scan, ordered), and compares full batches of 32*R
+// positions; no CTA-wide barrier after the table load, so warps hide each other's latency.
+template <int NP, int R, int TC>
+__global__ void __launch_bounds__(CT, 3) cof_comparer_fused(const __grid_constant__ TableArgs a) {
+    extern __shared__ __align__(16) uint8_t s_raw[];
+    constexpr uint32_t BS = NP * 25 * 8;
+    constexpr uint32_t BATCH = 32 * R;
+    static_assert(FWQ % BATCH == 0 && FWQ >= 2 * BATCH, "ring");
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const uint32_t tab_bytes = (a.n_blocks * BS + 15u) & ~15u;
+    uint32_t* queue = reinterpret_cast<uint32_t*>(s_raw + tab_bytes) + warp * FWQ;
+    const uint32_t s_tab = smem_u32(s_raw);
+    {
+        const uint2* src = a.ptab;
+        uint2* dst = reinterpret_cast<uint2*>(s_raw);
+        const uint32_t n8 = a.n_blocks * NP * 25;
+        for (uint32_t i = tid; i < n8; i += CT) dst[i] = __ldg(src + i);
+    }
+    __syncthreads();
+
+    // batches start at multiples of BATCH in the ring, so a batch never wraps
+    uint32_t head = 0, q_n = 0;          // warp-uniform
+    auto process = [&](uint32_t n_items) {   // ring[head, head + n_items), n_items <= BATCH
+        const uint32_t* q = queue + head;
+        uint32_t off[R][NP], okm[R];
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            const uint32_t i = (uint32_t)r * 32 + lane;
+            okm[r] = i < n_items ? ~0u : 0u;
+            item_offsets<NP>(a, i < n_items ? q[i] : 0u, off[r]);
+        }
+        uint32_t base[R][NP];
+#pragma unroll
+        for (int r = 0; r < R; r++)
+#pragma unroll
+            for (int qq = 0; qq < NP; qq++) base[r][qq] = s_tab + off[r][qq];
+        if (n_items < BATCH) table_blocks<NP, R, true, TC, 32>(a, base, a.n_blocks, 0, q + lane, okm);
+        else table_blocks<NP, R, false, TC, 32>(a, base, a.n_blocks, 0, q + lane, okm);
+        __syncwarp();                     // the slots may be refilled after this
+        head = (head + BATCH) & (FWQ - 1);
+        q_n -= n_items;
+    };
+
+    for (;;) {
+        uint32_t grab = 0;
+        if (lane == 0) grab = atomicAdd(a.ticket, 1u);
+        grab = __shfl_sync(0xffffffffu, grab, 0);
+        const uint64_t wp0 = (uint64_t)grab * FGRAB;
+        if (wp0 >= a.n_wp) break;
+        const uint64_t wp = wp0 + lane;
+        uint32_t m0 = 0, m1 = 0;
+        if (wp < a.n_wp) {
+            const uint4 v = __ldcs(a.masks + wp);
+            m0 = a.strand ? v.y : v.x;
+            m1 = a.strand ? v.w : v.z;
+        }
+        const uint32_t c = (uint32_t)(__popc(m0) + __popc(m1));
+        uint32_t x = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= o) x += y;
+        }
+        const uint32_t total = __shfl_sync(0xffffffffu, x, 31);
+        const uint32_t first = x - c;
+        const uint32_t pbase = (uint32_t)(wp * 64);
+        for (uint32_t done = 0; done < total;) {
+            const uint32_t take = min(FWQ - q_n, total - done);
+            const uint32_t tail = head + q_n;
+            uint32_t rank = first;
+#pragma unroll
+            for (int w = 0; w < 2; w++) {
+                uint32_t mm = w ? m1 : m0;
+                while (mm) {
+                    const int b = __ffs(mm) - 1;
+                    if (rank - done < take) queue[(tail + rank - done) & (FWQ - 1)] = pbase + 32u * w + (uint32_t)b;
+                    rank++;
+                    mm &= mm - 1;
+                }
+            }
+            __syncwarp();
+            q_n += take;
+            done += take;
+            while (q_n >= BATCH) process(BATCH);
+        }
+    }
+    while (q_n > 0) process(min(q_n, BATCH));
 }
 
 // ============================================================================ host side
@@ -450,27 +556,52 @@ static cof_status launch_table_r(TableArgs& t, uint64_t n_hint, cudaStream_t str
 // Uniform-threshold specializations for the common guide shapes (20-nt SpCas9 guides:
 // 10 pairs; 23-nt Cas12a guides: 12 pairs) and t <= 7; everything else runs the generic
 // per-guide-threshold kernel.
+template <int NP, int R, int TC>
+static cof_status launch_fused_r(TableArgs& t, cudaStream_t stream) {
+    const uint32_t smem = ((t.n_blocks * NP * 25 * 8 + 15u) & ~15u) + (CT / 32) * FWQ * 4;   // table + rings
+    int bps = 0;
+    auto fn = cof_comparer_fused<NP, R, TC>;
+    cof_status st = occupancy((const void*)fn, smem, &bps);
+    if (st != COF_OK) return st;
+    const uint64_t grabs = (t.n_wp + FGRAB - 1) / FGRAB;
+    uint64_t grid = (uint64_t)num_sms() * bps;
+    const uint64_t ctas_needed = (grabs + CT / 32 - 1) / (CT / 32);
+    if (grid > ctas_needed) grid = ctas_needed ? ctas_needed : 1;
+    fn<<<(uint32_t)grid, CT, smem, stream>>>(t);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "cof_comparer_fused launch");
+    count_launches(1);
+    return COF_OK;
+}
+
+template <int NP, int R, int TC>
+static cof_status launch_any_r(TableArgs& t, bool fused, uint64_t n_hint, cudaStream_t stream) {
+    return fused ? launch_fused_r<NP, R, TC>(t, stream) : launch_table_r<NP, R, TC>(t, n_hint, stream);
+}
+
 template <int NP>
-static cof_status launch_table(TableArgs& t, int uniform_t, uint64_t n_hint, cudaStream_t stream) {
+static cof_status launch_table(TableArgs& t, int uniform_t, uint64_t n_hint, cudaStream_t stream, bool fused = false) {
     if constexpr (NP == 10 || NP == 12) {
         switch (uniform_t) {
-            case 0: return launch_table_r<NP, R_TABLE, 0>(t, n_hint, stream);
-            case 1: return launch_table_r<NP, R_TABLE, 1>(t, n_hint, stream);
-            case 2: return launch_table_r<NP, R_TABLE, 2>(t, n_hint, stream);
-            case 3: return launch_table_r<NP, R_TABLE, 3>(t, n_hint, stream);
-            case 4: return launch_table_r<NP, R_TABLE, 4>(t, n_hint, stream);
-            case 5: return launch_table_r<NP, R_TABLE, 5>(t, n_hint, stream);
-            case 6: return launch_table_r<NP, R_TABLE, 6>(t, n_hint, stream);
-            case 7: return launch_table_r<NP, R_TABLE, 7>(t, n_hint, stream);
+            case 0: return launch_any_r<NP, R_TABLE, 0>(t, fused, n_hint, stream);
+            case 1: return launch_any_r<NP, R_TABLE, 1>(t, fused, n_hint, stream);
+            case 2: return launch_any_r<NP, R_TABLE, 2>(t, fused, n_hint, stream);
+            case 3: return launch_any_r<NP, R_TABLE, 3>(t, fused, n_hint, stream);
+            case 4: return launch_any_r<NP, R_TABLE, 4>(t, fused, n_hint, stream);
+            case 5: return launch_any_r<NP, R_TABLE, 5>(t, fused, n_hint, stream);
+            case 6: return launch_any_r<NP, R_TABLE, 6>(t, fused, n_hint, stream);
+            case 7: return launch_any_r<NP, R_TABLE, 7>(t, fused, n_hint, stream);
             default: break;
         }
     }
-    return launch_table_r<NP, R_TABLE, -1>(t, n_hint, stream);
+    return launch_any_r<NP, R_TABLE, -1>(t, fused, n_hint, stream);
 }
 
 // One launch per (strand, range of <= MAX_TABLE_BLOCKS guide blocks); thresholds travel in
 // the parameter space; hit counts accumulate on the device.
-static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs& a, cudaStream_t stream) {
+static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs& a, cudaStream_t stream,
+                            const uint4* masks = nullptr, uint64_t n_wp = 0, unsigned int* tickets = nullptr) {
+    const bool fused = masks != nullptr;
     static thread_local TableArgs T;   // ~4.5 KB parameter block, one per calling thread
     const uint32_t np = plan->pairs[0].n_pairs;
     int ut = g_uniform_t_enabled ? (int)plan->max_mm[0] : -1;   // same threshold for every guide?
@@ -484,6 +615,9 @@ static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs
         T.hits = a.hits; T.cap = a.cap; T.counters = a.counters;
         T.strand = sd;
         T.pairs = plan->pairs[sd];
+        T.masks = masks;
+        T.n_wp = n_wp;
+        T.ticket = tickets ? tickets + sd : nullptr;
         const uint32_t* pm = (const uint32_t*)(plan->image.data() + (sd == 0 ? plan->lay.pmeta_fwd : plan->lay.pmeta_rev));
         for (uint32_t bb = 0; bb < plan->n_blocks; bb += MAX_TABLE_BLOCKS) {
             T.block_base = bb;
@@ -493,22 +627,22 @@ static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs
                 for (int w = 0; w < 8; w++) T.meta[k][w] = pm[(size_t)(bb + k) * 8 + w];
             cof_status st;
             switch (np) {
-                case 1: st = launch_table<1>(T, ut, T.n, stream); break;
-                case 2: st = launch_table<2>(T, ut, T.n, stream); break;
-                case 3: st = launch_table<3>(T, ut, T.n, stream); break;
-                case 4: st = launch_table<4>(T, ut, T.n, stream); break;
-                case 5: st = launch_table<5>(T, ut, T.n, stream); break;
-                case 6: st = launch_table<6>(T, ut, T.n, stream); break;
-                case 7: st = launch_table<7>(T, ut, T.n, stream); break;
-                case 8: st = launch_table<8>(T, ut, T.n, stream); break;
-                case 9: st = launch_table<9>(T, ut, T.n, stream); break;
-                case 10: st = launch_table<10>(T, ut, T.n, stream); break;
-                case 11: st = launch_table<11>(T, ut, T.n, stream); break;
-                case 12: st = launch_table<12>(T, ut, T.n, stream); break;
-                case 13: st = launch_table<13>(T, ut, T.n, stream); break;
-                case 14: st = launch_table<14>(T, ut, T.n, stream); break;
-                case 15: st = launch_table<15>(T, ut, T.n, stream); break;
-                case 16: st = launch_table<16>(T, ut, T.n, stream); break;
+                case 1: st = launch_table<1>(T, ut, T.n, stream, fused); break;
+                case 2: st = launch_table<2>(T, ut, T.n, stream, fused); break;
+                case 3: st = launch_table<3>(T, ut, T.n, stream, fused); break;
+                case 4: st = launch_table<4>(T, ut, T.n, stream, fused); break;
+                case 5: st = launch_table<5>(T, ut, T.n, stream, fused); break;
+                case 6: st = launch_table<6>(T, ut, T.n, stream, fused); break;
+                case 7: st = launch_table<7>(T, ut, T.n, stream, fused); break;
+                case 8: st = launch_table<8>(T, ut, T.n, stream, fused); break;
+                case 9: st = launch_table<9>(T, ut, T.n, stream, fused); break;
+                case 10: st = launch_table<10>(T, ut, T.n, stream, fused); break;
+                case 11: st = launch_table<11>(T, ut, T.n, stream, fused); break;
+                case 12: st = launch_table<12>(T, ut, T.n, stream, fused); break;
+                case 13: st = launch_table<13>(T, ut, T.n, stream, fused); break;
+                case 14: st = launch_table<14>(T, ut, T.n, stream, fused); break;
+                case 15: st = launch_table<15>(T, ut, T.n, stream, fused); break;
+                case 16: st = launch_table<16>(T, ut, T.n, stream, fused); break;
                 default: return set_error(COF_E_STATE, "cof_compare: %u pairs", np);
             }
             if (st != COF_OK) return st;
@@ -545,11 +679,90 @@ static int comparer_impl() {
     return g_impl;
 }
 
+cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
+                       uint32_t* items_fwd, uint32_t* items_rev, uint64_t items_cap, bool masks_only,
+                       cudaStream_t stream);
+const uint4* finder_masks(const void* workspace);
+uint64_t finder_word_pairs(const cof_plan* plan, const cof_chunk* dev);
+
+static bool fusable(const cof_plan* plan) {
+    const uint32_t np = plan->pairs[0].n_pairs;
+    return plan->n_blocks <= MAX_TABLE_BLOCKS &&
+           (size_t)plan->n_blocks * np * 25 * 8 + (CT / 32) * FWQ * 4 + 1024 <= table_smem_budget() + 16 * 1024;
+}
+
 }  // namespace cof
 
 using namespace cof;
 
 extern "C" {
+
+int cof_find_compare_supported(const cof_plan* plan) {
+    return plan && comparer_impl() == 1 && fusable(plan) ? 1 : 0;
+}
+
+size_t cof_find_compare_workspace_bytes(uint64_t n_bases) { return cof_find_workspace_bytes(n_bases) + 256; }
+
+cof_status cof_find_masks(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace, cof_stream s) {
+    if (!plan || !plan_dev || !dev || !workspace) return set_error(COF_E_ARG, "cof_find_masks: NULL argument");
+    if (!dev->lo || !dev->hi || !dev->nm) return set_error(COF_E_ARG, "cof_find_masks: chunk planes are NULL");
+    cudaStream_t stream = (cudaStream_t)s;
+    unsigned long long* counters = (unsigned long long*)((uint8_t*)plan_dev + plan->lay.counters);
+    cudaError_t e = cudaMemsetAsync(counters, 0, 2 * sizeof(uint64_t), stream);
+    if (e != cudaSuccess) return cuda_error(e, "cof_find_masks memset");
+    return find_launch(plan, plan_dev, dev, workspace, nullptr, nullptr, 0, true, stream);
+}
+
+cof_status cof_compare_masks(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
+                             uint64_t* hits, uint64_t hits_cap, uint64_t* n_hits, cof_stream s) {
+    if (!plan || !plan_dev || !dev || !workspace || (!hits && hits_cap))
+        return set_error(COF_E_ARG, "cof_compare_masks: NULL argument");
+    if (!dev->lo || !dev->hi || !dev->nm) return set_error(COF_E_ARG, "cof_compare_masks: chunk planes are NULL");
+    if (comparer_impl() != 1 || !fusable(plan))
+        return set_error(COF_E_ARG, "cof_compare_masks: guide table too large for the fused kernel "
+                                    "(use cof_find_pam + cof_compare)");
+    cudaStream_t stream = (cudaStream_t)s;
+    uint8_t* pd = (uint8_t*)plan_dev;
+    unsigned long long* counters = (unsigned long long*)(pd + plan->lay.counters);
+    unsigned int* tickets = (unsigned int*)((uint8_t*)workspace + cof_find_workspace_bytes(dev->n_bases));
+    cudaError_t e = cudaMemsetAsync(counters + 2, 0, sizeof(uint64_t), stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(tickets, 0, 2 * sizeof(unsigned int), stream);
+    if (e != cudaSuccess) return cuda_error(e, "cof_compare_masks memset");
+    CompareArgs a;
+    a.lo = dev->lo; a.hi = dev->hi; a.nm = dev->nm;
+    a.items[0] = a.items[1] = nullptr;
+    a.n[0] = a.n[1] = 0;
+    a.items_cap = 0;
+    a.hits = (unsigned long long*)hits;
+    a.cap = hits_cap;
+    a.counters = counters;
+    const uint64_t n_wp = finder_word_pairs(plan, dev);
+    if (n_wp) {
+        cof_status st = run_table(plan, pd, a, stream, finder_masks(workspace), n_wp, tickets);
+        if (st != COF_OK) return st;
+    }
+    if (n_hits) {
+        uint64_t c = 0;
+        e = cudaMemcpyAsync(&c, counters + 2, sizeof c, cudaMemcpyDeviceToHost, stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+        if (e != cudaSuccess) return cuda_error(e, "cof_compare_masks count");
+        *n_hits = c;
+        if (c > hits_cap)
+            return set_error(COF_E_CAPACITY, "cof_compare_masks: %llu hits exceed capacity %llu",
+                             (unsigned long long)c, (unsigned long long)hits_cap);
+    }
+    return COF_OK;
+}
+
+cof_status cof_find_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
+                            uint64_t* hits, uint64_t hits_cap, uint64_t* n_hits, cof_stream s) {
+    if (plan && !fusable(plan))
+        return set_error(COF_E_ARG, "cof_find_compare: guide table too large for the fused kernel "
+                                    "(use cof_find_pam + cof_compare)");
+    cof_status st = cof_find_masks(plan, plan_dev, dev, workspace, s);
+    if (st != COF_OK) return st;
+    return cof_compare_masks(plan, plan_dev, dev, workspace, hits, hits_cap, n_hits, s);
+}
 
 cof_status cof_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, const uint32_t* items_fwd,
                        uint64_t n_fwd, const uint32_t* items_rev, uint64_t n_rev, uint64_t* hits, uint64_t hits_cap,

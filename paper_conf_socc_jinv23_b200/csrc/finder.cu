@@ -88,7 +88,7 @@ __device__ __forceinline__ void pam_masks(const FinderArgs& a, uint32_t valid, u
 //  offset) and pass 2 re-streams its range (mostly from L2) and writes the items in order.
 // One exchange per CTA replaces a decoupled look-back per tile, whose depth (all
 // concurrently running tiles) made it latency-bound.
-template <int NE, bool VS>
+template <int NE, bool VS, bool MASKS_ONLY>
 __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ FinderArgs a) {
     extern __shared__ __align__(128) uint8_t smem[];
     uint32_t* stage = reinterpret_cast<uint32_t*>(smem);
@@ -168,6 +168,15 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
     }
     if (lane == 0) { s_red[warp][0] = cnt_f; s_red[warp][1] = cnt_r; }
     __syncthreads();
+    if (MASKS_ONLY) {   // fused find+compare: the masks are the output; counts for reporting only
+        if (tid == 0) {
+            unsigned long long f = 0, r = 0;
+            for (int w = 0; w < FT / 32; w++) { f += s_red[w][0]; r += s_red[w][1]; }
+            atomicAdd(&a.counters[0], f);
+            atomicAdd(&a.counters[1], r);
+        }
+        return;
+    }
     if (tid == 0) {
         unsigned long long f = 0, r = 0;
         for (int w = 0; w < FT / 32; w++) { f += s_red[w][0]; r += s_red[w][1]; }
@@ -294,26 +303,29 @@ static int g_finder_blocks_per_sm = -1;
 static int g_num_sms = -1;
 
 typedef void (*FinderFn)(FinderArgs);
-template <bool VS>
+template <bool VS, bool MO>
 static FinderFn finder_fn_vs(uint32_t ne) {
     switch (ne) {
-        case 0: return cof_finder_kernel<0, VS>;
-        case 1: return cof_finder_kernel<1, VS>;
-        case 2: return cof_finder_kernel<2, VS>;
-        case 3: return cof_finder_kernel<3, VS>;
-        case 4: return cof_finder_kernel<4, VS>;
-        case 5: return cof_finder_kernel<5, VS>;
-        case 6: return cof_finder_kernel<6, VS>;
-        default: return cof_finder_kernel<-1, VS>;
+        case 0: return cof_finder_kernel<0, VS, MO>;
+        case 1: return cof_finder_kernel<1, VS, MO>;
+        case 2: return cof_finder_kernel<2, VS, MO>;
+        case 3: return cof_finder_kernel<3, VS, MO>;
+        case 4: return cof_finder_kernel<4, VS, MO>;
+        case 5: return cof_finder_kernel<5, VS, MO>;
+        case 6: return cof_finder_kernel<6, VS, MO>;
+        default: return cof_finder_kernel<-1, VS, MO>;
     }
 }
-static FinderFn finder_fn(uint32_t ne, bool vs) { return vs ? finder_fn_vs<true>(ne) : finder_fn_vs<false>(ne); }
+static FinderFn finder_fn(uint32_t ne, bool vs, bool masks_only = false) {
+    if (masks_only) return vs ? finder_fn_vs<true, true>(ne) : finder_fn_vs<false, true>(ne);
+    return vs ? finder_fn_vs<true, false>(ne) : finder_fn_vs<false, false>(ne);
+}
 
 static cof_status finder_setup() {
     if (g_finder_blocks_per_sm > 0) return COF_OK;
     int bps_min = 1 << 30;
-    for (uint32_t k = 0; k < 16; k++) {
-        FinderFn fn = finder_fn(k & 7, k >= 8);
+    for (uint32_t k = 0; k < 32; k++) {
+        FinderFn fn = finder_fn(k & 7, (k >> 3) & 1, k >= 16);
         cudaError_t e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM);
         if (e != cudaSuccess) return cuda_error(e, "finder setup");
         int bps = 0;
@@ -341,17 +353,63 @@ size_t cof_find_workspace_bytes(uint64_t n_bases) {
     return FWS_MASKS + (size_t)cof_plane_words(n_bases) * 8;
 }
 
+}  // extern "C"
+
+namespace cof {
+// Shared by cof_find_pam (ordered item lists) and cof_find_compare (masks only).
+cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
+                       uint32_t* items_fwd, uint32_t* items_rev, uint64_t items_cap, bool masks_only,
+                       cudaStream_t stream);
+}
+
+extern "C" {
+
 cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
                         uint32_t* items_fwd, uint32_t* items_rev, uint64_t items_cap, uint64_t* n_fwd,
                         uint64_t* n_rev, cof_stream s) {
     if (!plan || !plan_dev || !dev || !workspace || !items_fwd || !items_rev)
         return set_error(COF_E_ARG, "cof_find_pam: NULL argument");
+    cudaStream_t stream = (cudaStream_t)s;
+    cof_status st = find_launch(plan, plan_dev, dev, workspace, items_fwd, items_rev, items_cap, false, stream);
+    if (st != COF_OK) return st;
+    unsigned long long* counters = (unsigned long long*)((uint8_t*)plan_dev + plan->lay.counters);
+    if (n_fwd || n_rev) {
+        uint64_t c[2];
+        cudaError_t e = cudaMemcpyAsync(c, counters, sizeof c, cudaMemcpyDeviceToHost, stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+        if (e != cudaSuccess) return cuda_error(e, "cof_find_pam counts");
+        if (n_fwd) *n_fwd = c[0];
+        if (n_rev) *n_rev = c[1];
+        if (c[0] > items_cap || c[1] > items_cap)
+            return set_error(COF_E_CAPACITY, "cof_find_pam: %llu/%llu items exceed capacity %llu",
+                             (unsigned long long)c[0], (unsigned long long)c[1], (unsigned long long)items_cap);
+    }
+    return COF_OK;
+}
+
+}  // extern "C"
+
+namespace cof {
+const uint4* finder_masks(const void* workspace) {
+    return reinterpret_cast<const uint4*>((const uint8_t*)workspace + FWS_MASKS);
+}
+uint64_t finder_word_pairs(const cof_plan* plan, const cof_chunk* dev) {
+    const uint64_t L = plan->L;
+    uint64_t limit = dev->n_bases >= L ? dev->n_bases - L + 1 : 0;
+    if (!dev->n_segs && limit > dev->n_owned) limit = dev->n_owned;
+    const uint64_t n_tiles = (limit + (uint64_t)FW * 32 - 1) / ((uint64_t)FW * 32);
+    return n_tiles * FT;   // one uint4 {fwd0, rev0, fwd1, rev1} per thread-slot of every tile
+}
+
+cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
+                       uint32_t* items_fwd, uint32_t* items_rev, uint64_t items_cap, bool masks_only,
+                       cudaStream_t stream) {
+    if (!plan || !plan_dev || !dev || !workspace) return set_error(COF_E_ARG, "find: NULL argument");
     if (!dev->lo || !dev->hi || !dev->nm) return set_error(COF_E_ARG, "cof_find_pam: chunk planes are NULL");
     if (((uintptr_t)dev->lo | (uintptr_t)dev->hi | (uintptr_t)dev->nm | (uintptr_t)dev->vs) & 15)
         return set_error(COF_E_ARG, "cof_find_pam: planes must be 16-byte aligned");
     cof_status st = finder_setup();
     if (st != COF_OK) return st;
-    cudaStream_t stream = (cudaStream_t)s;
     const uint64_t L = plan->L;
     if (dev->n_segs && !dev->vs) return set_error(COF_E_ARG, "cof_find_pam: multi-segment chunk without vs plane");
     if (dev->n_bases >= (1ull << 32)) return set_error(COF_E_ARG, "cof_find_pam: n_bases must be < 2^32");
@@ -386,23 +444,11 @@ cof_status cof_find_pam(const cof_plan* plan, void* plan_dev, const cof_chunk* d
         uint32_t grid = (uint32_t)g_num_sms * (uint32_t)g_finder_blocks_per_sm;
         if (grid > FMAX_CTAS) grid = FMAX_CTAS;
         if (grid > n_tiles) grid = n_tiles;
-        finder_fn(a.ne, a.vs != nullptr)<<<grid, FT, FSMEM, stream>>>(a);
+        finder_fn(a.ne, a.vs != nullptr, masks_only)<<<grid, FT, FSMEM, stream>>>(a);
         e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "cof_finder_kernel launch");
         count_launches(1);
     }
-    if (n_fwd || n_rev) {
-        uint64_t c[2];
-        e = cudaMemcpyAsync(c, counters, sizeof c, cudaMemcpyDeviceToHost, stream);
-        if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
-        if (e != cudaSuccess) return cuda_error(e, "cof_find_pam counts");
-        if (n_fwd) *n_fwd = c[0];
-        if (n_rev) *n_rev = c[1];
-        if (c[0] > items_cap || c[1] > items_cap)
-            return set_error(COF_E_CAPACITY, "cof_find_pam: %llu/%llu items exceed capacity %llu",
-                             (unsigned long long)c[0], (unsigned long long)c[1], (unsigned long long)items_cap);
-    }
     return COF_OK;
 }
-
-}  // extern "C"
+}  // namespace cof

@@ -188,9 +188,11 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     size_t pmeta_bytes = (size_t)p->n_blocks * 8 * 4;
     lay.pmeta_fwd = off; off = align256(off + pmeta_bytes);
     lay.pmeta_rev = off; off = align256(off + pmeta_bytes);
+    lay.onehot = off; off = align256(off + p->onehot.size() * 4);
     lay.total = off;
     p->image.assign(lay.total, 0);
     uint8_t* img = p->image.data();
+    memcpy(img + lay.onehot, p->onehot.data(), p->onehot.size() * 4);
     memcpy(img + lay.groups_fwd, gd[0].data(), gd[0].size() * sizeof(GroupDesc));
     memcpy(img + lay.groups_rev, gd[1].data(), gd[1].size() * sizeof(GroupDesc));
     memcpy(img + lay.recs_fwd, recs[0].data(), recs[0].size() * 4);

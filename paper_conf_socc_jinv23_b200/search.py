@@ -11,6 +11,7 @@ from __future__ import annotations
 
 import dataclasses
 import heapq
+import os
 
 import numpy as np
 import torch
@@ -61,6 +62,19 @@ class Chunk:
             rows.append((p.chrom, off, p.chrom_off, p.n_owned))
             off += p.length
         return rows
+
+
+FUSED_MIN_GUIDES = 256   # measured crossover on B200: 100 guides two-call 12.4 ms vs fused 13.6 ms
+                         # (C3); 1000 guides fused 56.3 ms vs two-call 57.5 ms (C5)
+
+
+def use_fused(plan, n_guides: int) -> bool:
+    env = os.environ.get("COF_FUSED")
+    if not cof.cof_find_compare_supported(plan):
+        return False
+    if env is not None:
+        return env != "0"
+    return n_guides >= FUSED_MIN_GUIDES
 
 
 def plan_chunks(lengths, L: int, chunk_bases: int | None = None, pack_bases: int | None = None):
@@ -189,14 +203,21 @@ class Searcher:
         cof.cof_plan_upload(self.plan, self.plan_dev, self.stream)
         self._cap_bases = 0
         self._hits_cap = 0
+        self._rec_cap = 0
+        self.d_records = None
+        # fused find+compare (no item lists) when the guide table fits the fused kernel and there
+        # are enough guides to amortise the in-kernel expansion (COF_FUSED=0/1 overrides)
+        self.fused = use_fused(self.plan, len(guides))
 
     # ---- device buffers sized for the largest chunk seen so far
     def reserve(self, max_bases: int, hits_cap: int):
         if max_bases > self._cap_bases:
             words = cof.cof_plane_words(max_bases)
             self.d_planes = torch.empty((4, words), dtype=torch.int32, device=self.device)
-            self.d_items = torch.empty((2, max(max_bases, 1)), dtype=torch.int32, device=self.device)
-            self.d_find_ws = torch.empty(cof.cof_find_workspace_bytes(max_bases), dtype=torch.uint8,
+            # item lists only for the two-call path (the fused path never materialises them)
+            self.d_items = torch.empty((2, 1 if self.fused else max(max_bases, 1)), dtype=torch.int32,
+                                       device=self.device)
+            self.d_find_ws = torch.empty(cof.cof_find_compare_workspace_bytes(max_bases), dtype=torch.uint8,
                                          device=self.device)
             self._cap_bases = max_bases
         if hits_cap > self._hits_cap:
@@ -217,12 +238,21 @@ class Searcher:
         """find -> compare -> sort on the device; returns (n_fwd, n_rev, n_hits).
         Grows the hit buffer and re-runs compare on capacity overflow."""
         s = self.stream
-        nf, nr = cof.cof_find_pam(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_items[0],
-                                  self.d_items[1], items_cap, s)
+        if not self.fused and self.d_items.shape[1] < items_cap:   # path switched after reserve()
+            self.d_items = torch.empty((2, items_cap), dtype=torch.int32, device=self.device)
+        if self.fused:
+            cof.cof_find_masks(self.plan, self.plan_dev, dchunk, self.d_find_ws, s)
+        else:
+            nf, nr = cof.cof_find_pam(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_items[0],
+                                      self.d_items[1], items_cap, s)
         while True:
             try:
-                nh = cof.cof_compare(self.plan, self.plan_dev, dchunk, self.d_items[0], nf, self.d_items[1], nr,
-                                     self.d_hits, self._hits_cap, s)
+                if self.fused:
+                    nh = cof.cof_compare_masks(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_hits,
+                                               self._hits_cap, s)
+                else:
+                    nh = cof.cof_compare(self.plan, self.plan_dev, dchunk, self.d_items[0], nf, self.d_items[1],
+                                         nr, self.d_hits, self._hits_cap, s)
                 break
             except cof.CofError as e:
                 if e.status != cof.COF_E_CAPACITY:
@@ -231,21 +261,23 @@ class Searcher:
                 self.reserve(self._cap_bases, int(need * 1.25) + 1024)
         cof.cof_sort_hits(self.plan, self.plan_dev, dchunk, self.d_hits, self.d_tmp, self._hits_cap, nh,
                           self.d_sort_ws, s)
+        if self.fused:
+            nf, nr, _ = cof.cof_read_counts(self.plan, self.plan_dev, s)
         return nf, nr, nh
 
-    def search_host(self, host: HostGenome, indices=None, out=None):
+    def search_host(self, host: HostGenome, indices=None, out=None, decorate="device"):
         """End-to-end over host-resident packed chunks.  Per chunk: H2D on a copy stream
         (double-buffered device planes, overlapping the previous chunk's kernels), find,
-        compare, device sort and an async D2H of the sorted keys; a host thread decorates
-        chunk i (cof_collect, OpenMP) while the GPU works on chunk i+1.
+        compare, device sort, device decoration (cof_decorate) and an async D2H of the
+        finished records; nothing waits on the host except the item/hit counts.
 
-        Returns the sorted hit array.  If ``out`` (a ``cof.HIT_DTYPE`` array) is large
-        enough, each chunk is decorated straight into its slice of ``out`` (chunks are
-        disjoint and in genome order, so no merge copy is needed) and a view of ``out`` is
-        returned; otherwise per-chunk arrays are merged with cof_merge."""
-        import queue
-        import threading
-
+        Returns the sorted hit array.  If ``out`` (a ``cof.HIT_DTYPE`` array, ideally in
+        pinned memory) is large enough, each chunk's records land straight in its slice of
+        ``out`` (chunks are disjoint and in genome order, so no merge copy is needed) and a
+        view of ``out`` is returned; otherwise per-chunk arrays are merged with cof_merge.
+        ``decorate="host"`` decorates on CPU threads instead (cof_collect)."""
+        if decorate == "host":
+            return self._search_host_cpu_decorate(host, indices, out)
         idx = list(range(len(host.chunks)) if indices is None else indices)
         max_bases = max((host.chunks[i].n_bases for i in idx), default=1)
         self.reserve(max_bases, max(self._hits_cap, 1 << 16))
@@ -253,6 +285,80 @@ class Searcher:
             self.d_planes2 = torch.empty_like(self.d_planes)
             self.copy_stream = torch.cuda.Stream(self.device)
         planes = [self.d_planes, self.d_planes2]
+        ordered = all(a < b for a, b in zip(idx, idx[1:]))
+        use_out = out is not None and ordered
+        max_segs = max((len(host.chunks[i].pieces) for i in idx), default=1)
+        ws = torch.empty((len(idx), cof.cof_decorate_workspace_bytes(max_segs)), dtype=torch.uint8,
+                         device=self.device)
+        results = []
+        total = 0
+        overflow = False
+        with torch.cuda.device(self.device):
+            loaded = [None, None]
+            freed = [None, None]
+
+            def load(j, k):
+                with torch.cuda.stream(self.copy_stream):
+                    if freed[k] is not None:
+                        self.copy_stream.wait_event(freed[k])
+                    dch = self.device_chunk(host.chunks[idx[j]], planes[k], host.segs[idx[j]])
+                    cof.cof_load_chunk(host.chunk_struct(idx[j]), dch, self.copy_stream)
+                    ev = torch.cuda.Event()
+                    ev.record(self.copy_stream)
+                    loaded[k] = ev
+                    return dch
+
+            dchs = [None, None]
+            if idx:
+                dchs[0] = load(0, 0)
+            for j, i in enumerate(idx):
+                k = j & 1
+                self.stream.wait_event(loaded[k])
+                if j + 1 < len(idx):
+                    dchs[(j + 1) & 1] = load(j + 1, (j + 1) & 1)
+                _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned)
+                if nh > self._rec_cap:
+                    self._reserve_records(nh)
+                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, self.d_records, ws[j],
+                                 self.stream)
+                fr = torch.cuda.Event()
+                fr.record(self.stream)
+                freed[k] = fr
+                dst = None
+                if use_out and not overflow:
+                    if total + nh <= len(out):
+                        dst = out[total:total + nh]
+                    else:
+                        overflow = True
+                if dst is None:
+                    dst = torch.empty(max(nh, 1) * cof.HIT_DTYPE.itemsize, dtype=torch.uint8,
+                                      pin_memory=True).numpy().view(cof.HIT_DTYPE)[:nh]
+                if nh:
+                    with torch.cuda.stream(self.stream):
+                        torch.from_numpy(dst.view(np.uint8)).copy_(self.d_records[: nh * cof.HIT_DTYPE.itemsize],
+                                                                   non_blocking=True)
+                results.append(dst)
+                total += nh
+            self.stream.synchronize()
+            for j in range(len(idx)):
+                cof.cof_decorate_check(ws[j], self.stream)
+        if use_out and not overflow:
+            return out[:total]
+        return merge_hit_lists(results)
+
+    def _reserve_records(self, n):
+        self.d_records = torch.empty(int(n * 1.25 + 1024) * cof.HIT_DTYPE.itemsize, dtype=torch.uint8,
+                                     device=self.device)
+        self._rec_cap = int(n * 1.25 + 1024)
+
+    def _search_host_cpu_decorate(self, host: HostGenome, indices=None, out=None):
+        """As search_host, decorating on CPU threads (cof_collect) overlapped with the GPU."""
+        import queue
+        import threading
+
+        idx = list(range(len(host.chunks)) if indices is None else indices)
+        max_bases = max((host.chunks[i].n_bases for i in idx), default=1)
+        self.reserve(max_bases, max(self._hits_cap, 1 << 16))
         results = {}
         errors = []
         work = queue.Queue()
@@ -282,32 +388,10 @@ class Searcher:
         overflow = False
         try:
             with torch.cuda.device(self.device):
-                loaded = [None, None]          # events: planes buffer k loaded
-                freed = [None, None]           # events: compute done with planes buffer k
-
-                def load(j, k):
-                    with torch.cuda.stream(self.copy_stream):
-                        if freed[k] is not None:
-                            self.copy_stream.wait_event(freed[k])
-                        dch = self.device_chunk(host.chunks[idx[j]], planes[k], host.segs[idx[j]])
-                        cof.cof_load_chunk(host.chunk_struct(idx[j]), dch, self.copy_stream)
-                        ev = torch.cuda.Event()
-                        ev.record(self.copy_stream)
-                        loaded[k] = ev
-                        return dch
-
-                dchs = [None, None]
-                if idx:
-                    dchs[0] = load(0, 0)
-                for j, i in enumerate(idx):
-                    k = j & 1
-                    self.stream.wait_event(loaded[k])
-                    if j + 1 < len(idx):
-                        dchs[(j + 1) & 1] = load(j + 1, (j + 1) & 1)
-                    _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned)
-                    fr = torch.cuda.Event()
-                    fr.record(self.stream)
-                    freed[k] = fr
+                for i in idx:
+                    dch = self.device_chunk(host.chunks[i], None, host.segs[i])
+                    cof.cof_load_chunk(host.chunk_struct(i), dch, self.stream)
+                    _, _, nh = self.run_device_chunk(dch, host.chunks[i].n_owned)
                     keys = torch.empty(max(nh, 1), dtype=torch.int64, pin_memory=True)
                     with torch.cuda.stream(self.stream):
                         if nh:
@@ -322,6 +406,7 @@ class Searcher:
                             overflow = True
                     total += nh
                     work.put((i, ev, keys.numpy().view(np.uint64), nh, dst))
+                    self.stream.synchronize()    # the single plane buffer is reused next chunk
         finally:
             work.put(None)
             th.join()
@@ -331,15 +416,19 @@ class Searcher:
             return out[:total]
         return merge_hit_lists([results[i] for i in idx])
 
-def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda", pack_bases=None):
+def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda", pack_bases=None, fused=None):
     """Convenience: whole search of ``seqs`` (list of uint8 ASCII arrays / bytes) on one GPU.
-    ``pack_bases`` packs chromosome pieces into multi-segment chunks (0 = one chunk)."""
+    ``pack_bases`` packs chromosome pieces into multi-segment chunks (0 = one chunk);
+    ``fused`` False forces the two-call path (item lists) even when the fused one fits."""
     L = len(pattern)
     arrs = [np.frombuffer(s, dtype=np.uint8) if isinstance(s, (bytes, bytearray)) else
             (np.frombuffer(s.encode(), dtype=np.uint8) if isinstance(s, str) else s) for s in seqs]
     chunks = plan_chunks([len(a) for a in arrs], L, chunk_bases, pack_bases)
     host = HostGenome(arrs, chunks)
-    return Searcher(pattern, guides, thresholds, device).search_host(host)
+    srch = Searcher(pattern, guides, thresholds, device)
+    if fused is not None:
+        srch.fused = bool(fused) and cof.cof_find_compare_supported(srch.plan)
+    return srch.search_host(host)
 
 
 def shard_for_rank(chunks, rank: int, world: int):

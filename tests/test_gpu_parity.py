@@ -23,10 +23,10 @@ def _impl_reset():
     cof.cof_set_comparer("table")
 
 
-def gpu_hits(seqs, pattern, guides, thr, chunk_bases=None, impl="table", pack_bases=None):
+def gpu_hits(seqs, pattern, guides, thr, chunk_bases=None, impl="table", pack_bases=None, fused=None):
     cof.cof_set_comparer(impl)
     return cof.hits_to_tuples(search.search(seqs, pattern, guides, thr, chunk_bases=chunk_bases,
-                                            pack_bases=pack_bases))
+                                            pack_bases=pack_bases, fused=fused))
 
 
 def ref_hits(seqs, pattern, guides, thr, ranges=None):
@@ -58,6 +58,11 @@ def test_random_small(impl, seed):
     # the same genome as one multi-segment chunk and as packed pieces
     assert gpu_hits(seqs, pat, guides, thr, impl=impl, pack_bases=0) == exp
     assert gpu_hits(seqs, pat, guides, thr, impl=impl, chunk_bases=9973, pack_bases=30_000) == exp
+    if impl == "table":   # both table paths: fused (masks) and two-call (item lists)
+        assert gpu_hits(seqs, pat, guides, thr, impl=impl, fused=False) == exp
+        assert gpu_hits(seqs, pat, guides, thr, impl=impl, fused=False, pack_bases=0) == exp
+        assert gpu_hits(seqs, pat, guides, thr, impl=impl, fused=True) == exp
+        assert gpu_hits(seqs, pat, guides, thr, impl=impl, fused=True, chunk_bases=9973, pack_bases=30_000) == exp
 
 
 @pytest.mark.parametrize("impl", IMPLS)
@@ -77,6 +82,10 @@ def test_configs_scaled(name, scale, chunk, pack):
     cfg = w.cfg
     exp = ref_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
     assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk, pack_bases=pack) == exp
+    assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk, pack_bases=pack,
+                    fused=False) == exp
+    assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk, pack_bases=pack,
+                    fused=True) == exp
 
 
 def test_chunk_size_invariance():
@@ -122,6 +131,7 @@ def test_capacity_overflow_and_device_counts():
     thr = [0, 10]
     exp = ref_hits([seq], pat, guides, thr)
     srch = search.Searcher(pat, guides, thr)
+    srch.fused = False            # this test drives the two-call API (item lists) directly
     srch.reserve(len(seq), 64)    # far too small: forces COF_E_CAPACITY + retry
     host = search.HostGenome([seq], search.plan_chunks([len(seq)], 10))
     got = cof.hits_to_tuples(srch.search_host(host))
@@ -185,8 +195,9 @@ def test_full_size_sampled_c5():
     assert n_samples >= 20
 
 
-def test_search_host_into_caller_buffer_and_chunk_pipeline():
-    """The pipelined public path (double-buffered H2D, overlapped host decoration) writing
+@pytest.mark.parametrize("decorate", ["device", "host"])
+def test_search_host_into_caller_buffer_and_chunk_pipeline(decorate):
+    """The pipelined public path (double-buffered H2D, device or host decoration) writing
     straight into a caller buffer equals the oracle; a too-small buffer falls back to merge."""
     w = synth.make_workload("C3", scale=0.003, n_guides=40)
     cfg = w.cfg
@@ -195,11 +206,16 @@ def test_search_host_into_caller_buffer_and_chunk_pipeline():
     host = search.HostGenome(w.seqs, chunks)
     srch = search.Searcher(cfg.pattern, w.guides, w.thresholds)
     out = np.empty(len(exp) + 10, dtype=cof.HIT_DTYPE)
-    got = srch.search_host(host, out=out)
+    got = srch.search_host(host, out=out, decorate=decorate)
     assert got.base is out or np.shares_memory(got, out)
     assert cof.hits_to_tuples(got) == exp
     small = np.empty(max(1, len(exp) // 3), dtype=cof.HIT_DTYPE)
-    assert cof.hits_to_tuples(srch.search_host(host, out=small)) == exp
+    assert cof.hits_to_tuples(srch.search_host(host, out=small, decorate=decorate)) == exp
+    # multi-segment chunks through the same path
+    packed = search.HostGenome(w.seqs, search.plan_chunks([len(s) for s in w.seqs], cfg.L, 150_001,
+                                                          pack_bases=1_000_000))
+    assert any(c.multi for c in packed.chunks)
+    assert cof.hits_to_tuples(srch.search_host(packed, decorate=decorate)) == exp
 
 
 def test_many_guides_multiple_table_launches():
