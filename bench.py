@@ -46,7 +46,7 @@ def _peaks():
 
 # ----------------------------------------------------------------------------- clocks
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """nvidia-smi clocks + throttle reasons sampled every 100 ms during the timed region."""
 
     FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
@@ -61,7 +61,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.thread = threading.Thread(target=self._read, daemon=True)
             self.thread.start()
         except Exception:
@@ -238,7 +238,7 @@ def oracle_sample(wl, target_s: float, threads: int):
     cfg = wl.cfg
     c = int(np.argmax([len(s) for s in wl.seqs]))
     s0 = 1_000_000 if len(wl.seqs[c]) > 3_000_000 else 0
-    probe = 20_000
+    probe = 100_000
     t = time.perf_counter()
     orc.search([wl.seqs[c]], cfg.pattern, wl.guides, wl.thresholds, ranges=[(s0, s0 + probe)], threads=threads)
     dt = max(time.perf_counter() - t, 1e-3)
@@ -263,7 +263,7 @@ def items_per_base_estimate(st, wl):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C5")
     ap.add_argument("--scale", type=float, default=1.0)
@@ -289,10 +289,17 @@ def main():
     import torch.distributed as dist
     from paper_conf_socc_jinv23_b200 import cof, search
 
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # one process per GPU; COF_DIST_BACKEND=gloo lets several ranks share a device (tests)
+    local_dev = local % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
+    backend = os.environ.get("COF_DIST_BACKEND", "nccl")
+    coll_dev = dev if backend == "nccl" else torch.device("cpu")
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     cof.cof_set_comparer(args.comparer)
     cfg = synth.config(cfgname, args.scale)
     L = cfg.L
@@ -334,7 +341,7 @@ def main():
 
     # max over ranks
     t = torch.tensor([ms_total, cmp_ms, float(comps_mine), float(totals[2]), float(my_items)],
-                     dtype=torch.float64, device=dev)
+                     dtype=torch.float64, device=coll_dev)
     if world > 1:
         tmax = t.clone()
         dist.all_reduce(tmax[:2], op=dist.ReduceOp.MAX)
@@ -375,12 +382,12 @@ def main():
 
     e2e = None
     if not args.no_e2e:
-        e2e = measure_e2e(wl, st, dev, args, world, genome_bases)
+        e2e = measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         threads = len(os.sched_getaffinity(0))
-        c, s0, n = oracle_sample(wl, 12.0, threads)
+        c, s0, n = oracle_sample(wl, 15.0, threads)
         dt, nh = run_oracle(wl, c, s0, n, threads)
         ipb = items_per_base_estimate(st, wl)
         cpu = {"value": n / dt / 1e9, "unit": "Gbases/s", "cores": threads, "kind": "oracle",
@@ -472,7 +479,7 @@ def comparer_roof(plan, n_sm, sm_mhz, impl):
                      f"({alu_ops} LOP3 per 32 comparisons) x {n_sm} SMs x {sm_mhz:.0f} MHz"}
 
 
-def measure_e2e(wl, st, dev, args, world, genome_bases):
+def measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev=None):
     import torch
     import torch.distributed as dist
     from paper_conf_socc_jinv23_b200 import search
@@ -499,14 +506,15 @@ def measure_e2e(wl, st, dev, args, world, genome_bases):
     torch.cuda.synchronize(dev)
     dt = (time.perf_counter() - t0) / args.e2e_steps
     if world > 1:
-        t = torch.tensor([dt], dtype=torch.float64, device=dev)
+        t = torch.tensor([dt], dtype=torch.float64, device=coll_dev if coll_dev is not None else dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dt = float(t[0])
     return {"value": round(genome_bases / dt / 1e9, 4), "unit": "Gbases/s", "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "s_per_step": dt, "hits": nh,
-            "path": "Searcher.search_host: cof_load_chunk (copy stream, double-buffered) -> cof_find_pam -> "
-                    "cof_compare -> cof_sort_hits -> cof_decorate (device) -> D2H of the records into the "
-                    "caller's pinned buffer, from pinned packed host planes (wall clock)"}
+            "path": "Searcher.search_host: cof_load_chunk (copy stream, double-buffered) -> find/compare "
+                    "(fused masks path or item lists) -> cof_sort_hits -> cof_decorate (device) -> D2H of the "
+                    "records (D2H stream) into the caller's pinned buffer, from pinned packed host planes "
+                    "(wall clock)"}
 
 
 def main_reference(args, cfgname, metric):

@@ -284,7 +284,9 @@ class Searcher:
         if not hasattr(self, "d_planes2") or self.d_planes2.shape != self.d_planes.shape:
             self.d_planes2 = torch.empty_like(self.d_planes)
             self.copy_stream = torch.cuda.Stream(self.device)
+            self.d2h_stream = torch.cuda.Stream(self.device)
         planes = [self.d_planes, self.d_planes2]
+        rec_free = [None, None]
         ordered = all(a < b for a, b in zip(idx, idx[1:]))
         use_out = out is not None and ordered
         max_segs = max((len(host.chunks[i].pieces) for i in idx), default=1)
@@ -319,8 +321,10 @@ class Searcher:
                 _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned)
                 if nh > self._rec_cap:
                     self._reserve_records(nh)
-                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, self.d_records, ws[j],
-                                 self.stream)
+                recs = self.d_records[k]
+                if rec_free[k] is not None:          # the D2H of chunk j-2 from this buffer is done
+                    self.stream.wait_event(rec_free[k])
+                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, recs, ws[j], self.stream)
                 fr = torch.cuda.Event()
                 fr.record(self.stream)
                 freed[k] = fr
@@ -333,12 +337,17 @@ class Searcher:
                 if dst is None:
                     dst = torch.empty(max(nh, 1) * cof.HIT_DTYPE.itemsize, dtype=torch.uint8,
                                       pin_memory=True).numpy().view(cof.HIT_DTYPE)[:nh]
-                if nh:
-                    with torch.cuda.stream(self.stream):
-                        torch.from_numpy(dst.view(np.uint8)).copy_(self.d_records[: nh * cof.HIT_DTYPE.itemsize],
+                if nh:   # D2H on its own stream: overlaps the next chunk's kernels (and H2D)
+                    self.d2h_stream.wait_event(fr)
+                    with torch.cuda.stream(self.d2h_stream):
+                        torch.from_numpy(dst.view(np.uint8)).copy_(recs[: nh * cof.HIT_DTYPE.itemsize],
                                                                    non_blocking=True)
+                        ev = torch.cuda.Event()
+                        ev.record(self.d2h_stream)
+                    rec_free[k] = ev
                 results.append(dst)
                 total += nh
+            self.d2h_stream.synchronize()
             self.stream.synchronize()
             for j in range(len(idx)):
                 cof.cof_decorate_check(ws[j], self.stream)
@@ -347,9 +356,12 @@ class Searcher:
         return merge_hit_lists(results)
 
     def _reserve_records(self, n):
-        self.d_records = torch.empty(int(n * 1.25 + 1024) * cof.HIT_DTYPE.itemsize, dtype=torch.uint8,
-                                     device=self.device)
-        self._rec_cap = int(n * 1.25 + 1024)
+        # two device record buffers: chunk j decorates into one while chunk j-1's D2H drains the other
+        self.d2h_stream.synchronize() if hasattr(self, "d2h_stream") else None
+        cap = int(n * 1.25 + 1024)
+        self.d_records = [torch.empty(cap * cof.HIT_DTYPE.itemsize, dtype=torch.uint8, device=self.device)
+                          for _ in range(2)]
+        self._rec_cap = cap
 
     def _search_host_cpu_decorate(self, host: HostGenome, indices=None, out=None):
         """As search_host, decorating on CPU threads (cof_collect) overlapped with the GPU."""
