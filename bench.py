@@ -2,10 +2,11 @@
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl ours|reference]
 
-One *step* = one pass of the whole hot path over the synthetic genome: for every chunk
-(whole chromosome) the finder, the comparer and the device hit sort (SURVEY.md §8(a)
-rows a3-a7 on the device; a1 pack and a2 H2D are outside ``value`` because the inputs
-are resident in HBM, and inside ``e2e``).  ``value`` = genome bases of the whole job /
+One *step* = one pass of the whole hot path over the synthetic genome: the rank's
+chromosomes as one chunk through the finder, the comparer, the device hit sort and the
+device decoration into output records (SURVEY.md §8(a) rows a3-a7 on the device; a1 pack,
+a2 H2D and the D2H of the records are outside ``value`` because the inputs are resident
+in HBM, and inside ``e2e``).  ``value`` = genome bases of the whole job /
 max-over-ranks device time; comparisons/s are reported beside it.  Multi-GPU: chunks
 are LPT-sharded over ranks (no collective on the data path), strong scaling.
 
@@ -160,6 +161,10 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
     st.hits = [torch.empty(c, dtype=torch.int64, device=st.device) for c in st.caps]
     st.tmp = torch.empty(max(st.caps), dtype=torch.int64, device=st.device)
     st.sort_ws = torch.empty(cof.cof_sort_workspace_bytes(max(st.caps)), dtype=torch.uint8, device=st.device)
+    # device decoration (the device half of a7 collect): records per chunk
+    st.recs = [torch.empty(c * cof.HIT_DTYPE.itemsize, dtype=torch.uint8, device=st.device) for c in st.caps]
+    st.dec_ws = torch.empty((len(chunks), cof.cof_decorate_workspace_bytes(max(len(ch.pieces) for ch in chunks))),
+                            dtype=torch.uint8, device=st.device)
     st.max_owned = max_owned
     torch.cuda.synchronize(st.device)
     return wl, st
@@ -198,6 +203,7 @@ def run_device_pipeline(wl, st, collect=False, events=None, fevents=None):
         if events is not None:
             events.append((e0, ev()))
         cof.cof_sort_hits(st.plan, pd, dch, st.hits[i], st.tmp, st.caps[i], ON, st.sort_ws, s)
+        cof.cof_decorate(st.plan, pd, dch, st.hits[i], ON, st.recs[i], st.dec_ws[i], s, cap=st.caps[i])
     if not collect:
         return None
     out = []
@@ -213,6 +219,7 @@ def step_counts(st):
     from paper_conf_socc_jinv23_b200 import cof
     tot = [0, 0, 0]
     for i in range(len(st.chunks)):
+        cof.cof_decorate_check(st.dec_ws[i], st.stream)     # every key matched its chunk / plan
         c = cof.cof_read_counts(st.plan, st.plan_devs[i], st.stream)
         if c[2] > st.caps[i]:
             raise RuntimeError(f"chunk {i}: {c[2]} hits exceed capacity {st.caps[i]}")

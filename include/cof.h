@@ -236,14 +236,15 @@ cof_status cof_collect(const cof_plan *plan, const cof_chunk *host, const uint64
                        const uint64_t *host_keys, uint64_t n_hits, cof_hit *out, cof_stream s);
 
 /* The same decoration on the device: n_hits (sorted) keys of hits_dev -> n_hits records in
- * the DEVICE buffer out_dev (same order), one thread per hit, from the device planes of
+ * the DEVICE buffer out_dev (same order; n_hits = COF_COUNT_ON_DEVICE: the count of the
+ * last compare in plan_dev, clamped to cap), one thread per hit, from the device planes of
  * the chunk and the guide masks in plan_dev; dev->segs (host) is copied into workspace
  * (>= cof_decorate_workspace_bytes(dev->n_segs) device bytes).  Asynchronous; a key that
  * does not match the chunk/plan sets a flag that cof_decorate_check reports (COF_E_STATE,
  * synchronizes).  The caller copies the records to the host (pinned memory: no staging). */
 size_t     cof_decorate_workspace_bytes(uint32_t n_segs);
 cof_status cof_decorate(const cof_plan *plan, const void *plan_dev, const cof_chunk *dev,
-                        const uint64_t *hits_dev, uint64_t n_hits, cof_hit *out_dev,
+                        const uint64_t *hits_dev, uint64_t n_hits, uint64_t cap, cof_hit *out_dev,
                         void *workspace, cof_stream s);
 cof_status cof_decorate_check(const void *workspace, cof_stream s);
 

@@ -81,7 +81,7 @@ def _load():
         "cof_collect": (I32, [P, P, P, P, U64, P, P]),
         "cof_merge": (I32, [P, P, U32, P]),
         "cof_decorate_workspace_bytes": (SZ, [U32]),
-        "cof_decorate": (I32, [P, P, P, P, U64, P, P, P]),
+        "cof_decorate": (I32, [P, P, P, P, U64, U64, P, P, P]),
         "cof_decorate_check": (I32, [P, P]),
         "cof_find_compare_supported": (ctypes.c_int, [P]),
         "cof_find_compare_workspace_bytes": (SZ, [U64]),
@@ -334,10 +334,11 @@ def cof_decorate_workspace_bytes(n_segs: int) -> int:
     return int(lib.cof_decorate_workspace_bytes(int(n_segs)))
 
 
-def cof_decorate(plan, plan_dev, dev: cof_chunk, hits_dev, n_hits, out_dev, workspace, stream=None):
-    """Device decoration: n_hits keys -> n_hits cof_hit records in the device buffer out_dev."""
+def cof_decorate(plan, plan_dev, dev: cof_chunk, hits_dev, n_hits, out_dev, workspace, stream=None, cap=0):
+    """Device decoration: n_hits keys -> n_hits cof_hit records in the device buffer out_dev
+    (n_hits = COF_COUNT_ON_DEVICE: the device count clamped to ``cap``)."""
     _check(lib.cof_decorate(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(hits_dev), int(n_hits),
-                            _ptr(out_dev), _ptr(workspace), _stream(stream)))
+                            int(cap), _ptr(out_dev), _ptr(workspace), _stream(stream)))
 
 
 def cof_decorate_check(workspace, stream=None):

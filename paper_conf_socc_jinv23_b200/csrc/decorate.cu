@@ -21,7 +21,9 @@ struct DecorArgs {
     const uint32_t* hi;
     const uint32_t* nm;
     const unsigned long long* keys;
-    uint64_t n;
+    uint64_t n;                 // host count, or ON_DEVICE: min(*count, cap)
+    const unsigned long long* count;
+    uint64_t cap;
     cof_hit* out;
     const uint32_t* onehot;     // [2][n_guides][5]
     const cof_segment* segs;    // device copy, n_segs entries (0: single segment)
@@ -33,9 +35,19 @@ struct DecorArgs {
     unsigned int* bad;          // set to 1 if a key is inconsistent with the chunk / plan
 };
 
+__device__ __forceinline__ void decorate_one(const DecorArgs& a, uint64_t i);
+
 __global__ void __launch_bounds__(256) cof_decorate_kernel(const __grid_constant__ DecorArgs a) {
-    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= a.n) return;
+    uint64_t n = a.n;
+    if (a.count) {
+        n = *a.count;
+        if (n > a.cap) n = a.cap;
+    }
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        decorate_one(a, i);
+}
+
+__device__ __forceinline__ void decorate_one(const DecorArgs& a, uint64_t i) {
     const unsigned long long key = a.keys[i];
     const uint32_t pos = (uint32_t)(key >> 32);
     const uint32_t strand = (uint32_t)(key >> 31) & 1u;
@@ -106,7 +118,7 @@ size_t cof_decorate_workspace_bytes(uint32_t n_segs) {
 }
 
 cof_status cof_decorate(const cof_plan* plan, const void* plan_dev, const cof_chunk* dev, const uint64_t* hits_dev,
-                        uint64_t n_hits, cof_hit* out_dev, void* workspace, cof_stream s) {
+                        uint64_t n_hits, uint64_t cap, cof_hit* out_dev, void* workspace, cof_stream s) {
     static_assert(sizeof(cof_hit) == 56, "cof_hit layout");
     if (!plan || !plan_dev || !dev || !workspace || ((!hits_dev || !out_dev) && n_hits))
         return set_error(COF_E_ARG, "cof_decorate: NULL argument");
@@ -116,14 +128,17 @@ cof_status cof_decorate(const cof_plan* plan, const void* plan_dev, const cof_ch
     cof_segment* dsegs = (cof_segment*)((uint8_t*)workspace + 256);
     cudaError_t e = cudaMemsetAsync(bad, 0, sizeof(unsigned int), stream);   // also for n_hits == 0
     if (e != cudaSuccess) return cuda_error(e, "cof_decorate");
-    if (n_hits == 0) return COF_OK;
+    const bool on_dev = n_hits == COF_COUNT_ON_DEVICE;
+    if (on_dev ? cap == 0 : n_hits == 0) return COF_OK;
     if (e == cudaSuccess && dev->n_segs)
         e = cudaMemcpyAsync(dsegs, dev->segs, (size_t)dev->n_segs * sizeof(cof_segment), cudaMemcpyHostToDevice, stream);
     if (e != cudaSuccess) return cuda_error(e, "cof_decorate");
     DecorArgs a;
     a.lo = dev->lo; a.hi = dev->hi; a.nm = dev->nm;
     a.keys = (const unsigned long long*)hits_dev;
-    a.n = n_hits;
+    a.n = on_dev ? 0 : n_hits;
+    a.count = on_dev ? (const unsigned long long*)((const uint8_t*)plan_dev + plan->lay.counters + 16) : nullptr;
+    a.cap = cap;
     a.out = out_dev;
     a.onehot = (const uint32_t*)((const uint8_t*)plan_dev + plan->lay.onehot);
     a.segs = dsegs;
@@ -133,7 +148,8 @@ cof_status cof_decorate(const cof_plan* plan, const void* plan_dev, const cof_ch
     a.chrom = dev->chrom;
     a.start = dev->start;
     a.bad = bad;
-    const uint64_t blocks = (n_hits + 255) / 256;
+    uint64_t blocks = ((on_dev ? cap : n_hits) + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;   // grid-stride beyond that
     cof_decorate_kernel<<<(uint32_t)blocks, 256, 0, stream>>>(a);
     e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "cof_decorate launch");

@@ -319,12 +319,13 @@ class Searcher:
                 if j + 1 < len(idx):
                     dchs[(j + 1) & 1] = load(j + 1, (j + 1) & 1)
                 _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned)
-                if nh > self._rec_cap:
+                if self.d_records is None or nh > self._rec_cap:
                     self._reserve_records(nh)
                 recs = self.d_records[k]
                 if rec_free[k] is not None:          # the D2H of chunk j-2 from this buffer is done
                     self.stream.wait_event(rec_free[k])
-                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, recs, ws[j], self.stream)
+                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, recs, ws[j], self.stream,
+                                 cap=self._rec_cap)
                 fr = torch.cuda.Event()
                 fr.record(self.stream)
                 freed[k] = fr
