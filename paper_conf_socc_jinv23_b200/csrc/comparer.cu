@@ -167,23 +167,36 @@ __global__ void __launch_bounds__(CT) cof_comparer_popc(const __grid_constant__ 
 }
 
 // ============================================================================ v2 table
-// per-item, per-pair byte offset into a block's pair table: (pair * 25 + 5*b1 + b2) * 8
+// Shared-memory addressing of the pair tables: the entry of pair q for bases (b1, b2) of an
+// item is read at base[q] + OFF + q * 128, where OFF = the guide block's table offset and
+// q * 128 (pair q's 16 ACGT entries) are compile-time immediates of the LDS; base[q] is the
+// 128-byte-aligned table base plus the entry's offset relative to q * 128.
+// (wl, wh, wn: windows starting at window offset pl.p0, the first compared position)
 template <int NP>
-__device__ __forceinline__ void pair_offsets(const PairLayout& pl, uint32_t wl, uint32_t wh, uint32_t wn,
-                                             uint32_t (&off)[NP]) {
+__device__ __forceinline__ void pair_offsets(const PairLayout& pl, uint32_t s_base, uint32_t wl, uint32_t wh,
+                                             uint32_t wn, uint32_t (&base)[NP]) {
 #pragma unroll
     for (int q = 0; q < NP; q++) {
-        const uint32_t j1 = pl.j1[q], j2 = pl.j2[q];
+        const uint32_t j1 = pl.j1[q] - pl.p0, j2 = pl.j2[q] == 0xFFu ? 0xFFu : pl.j2[q] - pl.p0;
         const uint32_t b1 = ((wn >> j1) & 1u) ? 4u : (((wl >> j1) & 1u) | (((wh >> j1) & 1u) << 1));
         uint32_t b2 = 0;
         if (j2 != 0xFFu) b2 = ((wn >> j2) & 1u) ? 4u : (((wl >> j2) & 1u) | (((wh >> j2) & 1u) << 1));
-        off[q] = pair_entry(NP, (uint32_t)q, b1, b2) * 8u;
+        base[q] = s_base + pair_entry(NP, (uint32_t)q, b1, b2) * 8u - (uint32_t)q * 128u;
     }
 }
 
 template <uint32_t OFF>
 __device__ __forceinline__ void lds64(uint32_t addr, uint32_t& x, uint32_t& y) {
     asm volatile("ld.shared.v2.u32 {%0, %1}, [%2+%3];" : "=r"(x), "=r"(y) : "r"(addr), "n"(OFF));
+}
+
+// The NP pair-entry loads of one item and guide block: pair q at base[q] + OFF + q * 128.
+template <int NP, uint32_t OFF, int Q = 0>
+__device__ __forceinline__ void lds_pairs(const uint32_t (&base)[NP], uint32_t (&v0)[NP], uint32_t (&v1)[NP]) {
+    if constexpr (Q < NP) {
+        lds64<OFF + (uint32_t)Q * 128u>(base[Q], v0[Q], v1[Q]);
+        lds_pairs<NP, OFF, Q + 1>(base, v0, v1);
+    }
 }
 
 // Arguments of one table-comparer launch: ONE strand, up to MAX_TABLE_BLOCKS guide blocks.
@@ -218,8 +231,7 @@ template <int NP, uint32_t OFF, int TC>
 __device__ __forceinline__ uint32_t table_hits(const uint32_t (&base)[NP], const uint32_t* __restrict__ T,
                                                uint32_t (&s)[6]) {
     uint32_t v0[NP], v1[NP];
-#pragma unroll
-    for (int q = 0; q < NP; q++) lds64<OFF>(base[q], v0[q], v1[q]);
+    lds_pairs<NP, OFF>(base, v0, v1);
     if constexpr (TC >= 0) {
         const uint32_t Tl[6] = {0u - (TC & 1u), 0u - ((TC >> 1) & 1u), 0u - ((TC >> 2) & 1u),
                                 0u - ((TC >> 3) & 1u), 0u - ((TC >> 4) & 1u), 0u - ((TC >> 5) & 1u)};
@@ -276,8 +288,10 @@ __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base
                 if (h2) { table_hits<NP, 2 * BS, TC>(base[r], m + 16, sh); table_emit(a, idx, h2, sh, g0 + 64u); }
                 if (h3) { table_hits<NP, 3 * BS, TC>(base[r], m + 24, sh); table_emit(a, idx, h3, sh, g0 + 96u); }
             }
+            if (b + 4 < nb) {
 #pragma unroll
-            for (int q = 0; q < NP; q++) base[r][q] += 4 * BS;
+                for (int q = 0; q < NP; q++) base[r][q] += 4 * BS;
+            }
         }
     }
     for (; b < nb; b++) {
@@ -288,23 +302,25 @@ __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base
             uint32_t h0 = table_hits<NP, 0, TC>(base[r], m, s0);
             if (TAIL) h0 &= okm[r];
             if (h0) table_emit(a, pos0 + r * STRIDE, h0, s0, (a.block_base + gb0 + b) * 32u);
+            if (b + 1 < nb) {
 #pragma unroll
-            for (int q = 0; q < NP; q++) base[r][q] += BS;
+                for (int q = 0; q < NP; q++) base[r][q] += BS;
+            }
         }
     }
 }
 
-// Byte offsets (within a guide block's table) of the NP pair entries of the window at pos.
+// Table addresses (see pair_offsets) of the NP pair entries of one item, from its plane
+// windows taken at pos + pairs.p0 (every compared offset is >= p0 and < 32).
 template <int NP>
-__device__ __forceinline__ void item_offsets(const TableArgs& a, uint32_t pos, uint32_t (&off)[NP]) {
-    if (a.pairs.contig) {
-        // fast path: window starting at the first compared offset; with no N among the
-        // compared positions every pair index is one nibble of Y (even pairs) or Z (odd)
-        const uint32_t p = pos + a.pairs.p0;
-        const uint32_t wn = plane_window(a.nm, p);
-        const uint32_t cm = a.pairs.n_cmp >= 32 ? ~0u : ((1u << a.pairs.n_cmp) - 1u);
+__device__ __forceinline__ void window_bases(const PairLayout& pl, uint32_t s_base, uint32_t wl, uint32_t wh,
+                                             uint32_t wn, uint32_t (&base)[NP]) {
+    if (pl.contig) {
+        // fast path: with no N among the contiguous compared positions every pair index is
+        // one nibble of Y (even pairs) or Z (odd pairs); s_base is 128-aligned, so the
+        // entry offset ORs in (one SHF + one LOP3 per pair)
+        const uint32_t cm = pl.n_cmp >= 32 ? ~0u : ((1u << pl.n_cmp) - 1u);
         if ((wn & cm) == 0) {
-            const uint32_t wl = plane_window(a.lo, p), wh = plane_window(a.hi, p);
             const uint32_t Y = (wl & 0x33333333u) | ((wh & 0x33333333u) << 2);
             const uint32_t Z = ((wl >> 2) & 0x33333333u) | (wh & 0xCCCCCCCCu);
 #pragma unroll
@@ -312,76 +328,126 @@ __device__ __forceinline__ void item_offsets(const TableArgs& a, uint32_t pos, u
                 const uint32_t src = (q & 1) ? Z : Y;
                 const int k = q >> 1;
                 const uint32_t nib8 = k == 0 ? (src << 3) & 0x78u : (src >> (4 * k - 3)) & 0x78u;
-                off[q] = (uint32_t)q * 128u + nib8;
+                base[q] = s_base | nib8;
             }
             return;
         }
     }
-    pair_offsets<NP>(a.pairs, plane_window(a.lo, pos), plane_window(a.hi, pos), plane_window(a.nm, pos), off);
+    pair_offsets<NP>(pl, s_base, wl, wh, wn, base);
+}
+
+template <int NP>
+__device__ __forceinline__ void item_bases(const TableArgs& a, uint32_t s_base, uint32_t pos, uint32_t (&base)[NP]) {
+    const uint32_t p = pos + a.pairs.p0;
+    window_bases<NP>(a.pairs, s_base, plane_window(a.lo, p), plane_window(a.hi, p), plane_window(a.nm, p), base);
+}
+
+// Window prefetch of the table comparer: the 6 plane words (lo, hi, nm; two each) an item's
+// window needs are copied into this thread's shared-memory slots with cp.async one tile
+// ahead, so the dependent global loads of the next tile overlap this tile's table work.
+// Slot k of thread t lives at word k * CT + t (conflict-free).
+__device__ __forceinline__ void prefetch_window(const TableArgs& a, uint32_t slot, uint32_t pos) {
+    const uint32_t w = (pos + a.pairs.p0) >> 5;
+    cp_async4(slot + 0 * CT * 4, a.lo + w);
+    cp_async4(slot + 1 * CT * 4, a.lo + w + 1);
+    cp_async4(slot + 2 * CT * 4, a.hi + w);
+    cp_async4(slot + 3 * CT * 4, a.hi + w + 1);
+    cp_async4(slot + 4 * CT * 4, a.nm + w);
+    cp_async4(slot + 5 * CT * 4, a.nm + w + 1);
+}
+
+template <int NP>
+__device__ __forceinline__ void slot_bases(const TableArgs& a, uint32_t s_base, const uint32_t* slot, uint32_t sh,
+                                           uint32_t (&base)[NP]) {
+    const uint32_t wl = __funnelshift_r(slot[0 * CT], slot[1 * CT], sh);
+    const uint32_t wh = __funnelshift_r(slot[2 * CT], slot[3 * CT], sh);
+    const uint32_t wn = __funnelshift_r(slot[4 * CT], slot[5 * CT], sh);
+    window_bases<NP>(a.pairs, s_base, wl, wh, wn, base);
 }
 
 template <int NP, int R, int TC>
 __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constant__ TableArgs a) {
     extern __shared__ __align__(16) uint8_t s_raw[];
     // shared: [blocks_per_chunk][NP][25] uint2 pair table of the resident chunk of blocks
+    // (at the first 128-byte boundary), then the window slots
     constexpr uint32_t BS = NP * 25 * 8;
-    const uint32_t s_tab = smem_u32(s_raw);
-    uint64_t n = a.n == ON_DEVICE ? (uint64_t)a.counters[a.strand] : a.n;
-    if (n > a.items_cap) n = a.items_cap;
-    const uint64_t per_tile = (uint64_t)CT * R;
-    const uint64_t n_tiles = (n + per_tile - 1) / per_tile;
+    const uint32_t s_raw_a = smem_u32(s_raw);
+    const uint32_t s_base = (s_raw_a + 127u) & ~127u;
+    uint2* s_tab_p = reinterpret_cast<uint2*>(s_raw + (s_base - s_raw_a));
+    uint64_t n64 = a.n == ON_DEVICE ? (uint64_t)a.counters[a.strand] : a.n;
+    if (n64 > a.items_cap) n64 = a.items_cap;
+    // item indices fit 32 bits (n_bases < 2^32, checked by the host); an index past n that
+    // wraps in the look-ahead below lands inside the list and is never consumed
+    const uint32_t n = (uint32_t)n64;
+    constexpr uint32_t per_tile = (uint32_t)CT * R;
+    const uint32_t n_tiles = (uint32_t)((n64 + per_tile - 1) / per_tile);
     const uint32_t bpc = a.blocks_per_chunk;
     const uint32_t n_chunks = (a.n_blocks + bpc - 1) / bpc;
     uint32_t loaded = 0xFFFFFFFFu;
 
-    // item positions are prefetched one tile ahead (their load latency overlaps the
-    // previous tile's table work; only the dependent window loads remain exposed)
-    uint32_t pos_next[R];
-#pragma unroll
-    for (int r = 0; r < R; r++) {
-        const uint64_t idx = (uint64_t)blockIdx.x * per_tile + threadIdx.x + (uint64_t)r * CT;
-        pos_next[r] = (blockIdx.x < n_tiles && idx < n) ? __ldg(a.items + idx) : 0u;
-    }
-    for (uint64_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
-        const uint64_t t0 = tile * per_tile;
-        const uint64_t item0 = t0 + threadIdx.x;
-        const bool tail = t0 + per_tile > n;
-        uint32_t cur[R];
+    // Two-stage prefetch: positions two tiles ahead (registers), plane words one tile ahead
+    // (cp.async into per-thread shared slots after the resident table chunk).
+    const uint32_t slot_off = (s_base - s_raw_a) + ((bpc * BS + 15u) & ~15u);
+    const uint32_t slot_b = s_raw_a + slot_off;
+    const uint32_t* slot_p = reinterpret_cast<const uint32_t*>(s_raw + slot_off);
+    const uint32_t stride = gridDim.x * per_tile;
+    uint32_t pos_next[R], shf[R];   // shf: window shift of the item whose words are in flight
+    {
+        const uint32_t i0 = blockIdx.x * per_tile + threadIdx.x;
 #pragma unroll
         for (int r = 0; r < R; r++) {
-            cur[r] = pos_next[r];
-            const uint64_t nidx = item0 + (uint64_t)gridDim.x * per_tile + (uint64_t)r * CT;
+            const uint32_t idx = i0 + (uint32_t)r * CT;
+            const uint32_t p = idx < n ? __ldg(a.items + idx) : 0u;
+            prefetch_window(a, slot_b + (uint32_t)(r * 6 * CT + threadIdx.x) * 4u, p);
+            shf[r] = (p + a.pairs.p0) & 31u;
+            pos_next[r] = (idx + stride) < n ? __ldg(a.items + idx + stride) : 0u;
+        }
+        cp_async_commit();
+    }
+    for (uint32_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
+        const uint32_t t0 = tile * per_tile;
+        const uint32_t item0 = t0 + threadIdx.x;
+        const bool tail = n - t0 < per_tile;
+        uint32_t base[R][NP], okm[R];
+        cp_async_wait_all();
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            const uint32_t idx = item0 + (uint32_t)r * CT;
+            okm[r] = idx < n ? ~0u : 0u;
+            slot_bases<NP>(a, s_base, slot_p + r * 6 * CT + threadIdx.x, shf[r], base[r]);
+        }
+        // refill the slots for the next tile, then fetch the positions of the one after
+#pragma unroll
+        for (int r = 0; r < R; r++) {
+            prefetch_window(a, slot_b + (uint32_t)(r * 6 * CT + threadIdx.x) * 4u, pos_next[r]);
+            shf[r] = (pos_next[r] + a.pairs.p0) & 31u;
+            const uint32_t nidx = item0 + 2 * stride + (uint32_t)r * CT;
             pos_next[r] = nidx < n ? __ldg(a.items + nidx) : 0u;
         }
-        uint32_t off[R][NP], okm[R];
-#pragma unroll
-        for (int r = 0; r < R; r++) {
-            const uint64_t idx = item0 + (uint64_t)r * CT;
-            okm[r] = idx < n ? ~0u : 0u;
-            item_offsets<NP>(a, cur[r], off[r]);
-        }
+        cp_async_commit();
         for (uint32_t ch = 0; ch < n_chunks; ch++) {
             const uint32_t b0 = ch * bpc;
             const uint32_t nb = min(bpc, a.n_blocks - b0);
             if (loaded != ch) {
                 __syncthreads();
                 const uint2* src = a.ptab + (size_t)b0 * NP * 25;
-                uint2* dst = reinterpret_cast<uint2*>(s_raw);
                 const uint32_t n8 = nb * NP * 25;
-                for (uint32_t i = threadIdx.x; i < n8; i += CT) dst[i] = __ldg(src + i);
+                for (uint32_t i = threadIdx.x; i < n8; i += CT) s_tab_p[i] = __ldg(src + i);
                 __syncthreads();
                 loaded = ch;
             }
-            uint32_t base[R][NP];
-#pragma unroll
-            for (int r = 0; r < R; r++)
-#pragma unroll
-                for (int q = 0; q < NP; q++) base[r][q] = s_tab + off[r][q];
             if (tail) table_blocks<NP, R, true, TC>(a, base, nb, b0, a.items + item0, okm);
             else table_blocks<NP, R, false, TC>(a, base, nb, b0, a.items + item0, okm);
+            if (n_chunks > 1) {
+                // undo table_blocks' block-to-block advance (see its increments)
+                const uint32_t inc = (nb & 3u) ? (nb - 1u) * BS : (nb - 4u) * BS;
+#pragma unroll
+                for (int r = 0; r < R; r++)
+#pragma unroll
+                    for (int q = 0; q < NP; q++) base[r][q] -= inc;
+            }
         }
     }
-    (void)BS;
 }
 
 
@@ -404,12 +470,13 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_fused(const __grid_constan
     constexpr uint32_t BATCH = 32 * R;
     static_assert(FWQ % BATCH == 0 && FWQ >= 2 * BATCH, "ring");
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const uint32_t tab_bytes = (a.n_blocks * BS + 15u) & ~15u;
+    const uint32_t s_raw_a = smem_u32(s_raw);
+    const uint32_t s_base = (s_raw_a + 127u) & ~127u;   // table at the first 128-byte boundary
+    const uint32_t tab_bytes = (s_base - s_raw_a) + ((a.n_blocks * BS + 15u) & ~15u);
     uint32_t* queue = reinterpret_cast<uint32_t*>(s_raw + tab_bytes) + warp * FWQ;
-    const uint32_t s_tab = smem_u32(s_raw);
     {
         const uint2* src = a.ptab;
-        uint2* dst = reinterpret_cast<uint2*>(s_raw);
+        uint2* dst = reinterpret_cast<uint2*>(s_raw + (s_base - s_raw_a));
         const uint32_t n8 = a.n_blocks * NP * 25;
         for (uint32_t i = tid; i < n8; i += CT) dst[i] = __ldg(src + i);
     }
@@ -419,18 +486,13 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_fused(const __grid_constan
     uint32_t head = 0, q_n = 0;          // warp-uniform
     auto process = [&](uint32_t n_items) {   // ring[head, head + n_items), n_items <= BATCH
         const uint32_t* q = queue + head;
-        uint32_t off[R][NP], okm[R];
+        uint32_t base[R][NP], okm[R];
 #pragma unroll
         for (int r = 0; r < R; r++) {
             const uint32_t i = (uint32_t)r * 32 + lane;
             okm[r] = i < n_items ? ~0u : 0u;
-            item_offsets<NP>(a, i < n_items ? q[i] : 0u, off[r]);
+            item_bases<NP>(a, s_base, i < n_items ? q[i] : 0u, base[r]);
         }
-        uint32_t base[R][NP];
-#pragma unroll
-        for (int r = 0; r < R; r++)
-#pragma unroll
-            for (int qq = 0; qq < NP; qq++) base[r][qq] = s_tab + off[r][qq];
         if (n_items < BATCH) table_blocks<NP, R, true, TC, 32>(a, base, a.n_blocks, 0, q + lane, okm);
         else table_blocks<NP, R, false, TC, 32>(a, base, a.n_blocks, 0, q + lane, okm);
         __syncwarp();                     // the slots may be refilled after this
@@ -535,7 +597,7 @@ static cof_status launch_table_r(TableArgs& t, uint64_t n_hint, cudaStream_t str
     const uint32_t budget = table_smem_budget();
     if (bpc * per_block > budget) bpc = std::max<uint32_t>(1, budget / per_block);
     t.blocks_per_chunk = bpc;
-    const uint32_t smem = bpc * per_block;
+    const uint32_t smem = 128u + ((bpc * per_block + 15u) & ~15u) + (uint32_t)CT * R * 6u * 4u;   // table + window slots
     int bps = 0;
     auto fn = cof_comparer_table<NP, R, TC>;
     cof_status st = occupancy((const void*)fn, smem, &bps);
@@ -558,7 +620,7 @@ static cof_status launch_table_r(TableArgs& t, uint64_t n_hint, cudaStream_t str
 // per-guide-threshold kernel.
 template <int NP, int R, int TC>
 static cof_status launch_fused_r(TableArgs& t, cudaStream_t stream) {
-    const uint32_t smem = ((t.n_blocks * NP * 25 * 8 + 15u) & ~15u) + (CT / 32) * FWQ * 4;   // table + rings
+    const uint32_t smem = 128u + ((t.n_blocks * NP * 25 * 8 + 15u) & ~15u) + (CT / 32) * FWQ * 4;   // table + rings
     int bps = 0;
     auto fn = cof_comparer_fused<NP, R, TC>;
     cof_status st = occupancy((const void*)fn, smem, &bps);
@@ -608,6 +670,9 @@ static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs
     for (uint32_t i = 1; i < plan->n_guides && ut >= 0; i++)
         if (plan->max_mm[i] != plan->max_mm[0]) ut = -1;
     for (uint32_t sd = 0; sd < 2; sd++) {
+        if (!fused && a.n[sd] != ON_DEVICE && a.n[sd] >= (1ull << 32))
+            return set_error(COF_E_ARG, "cof_compare: %llu items (item lists index < 2^32 positions)",
+                             (unsigned long long)a.n[sd]);
         T.lo = a.lo; T.hi = a.hi; T.nm = a.nm;
         T.items = a.items[sd];
         T.n = a.n[sd];
