@@ -177,6 +177,17 @@ cof_status cof_compare(const cof_plan *plan, void *plan_dev, const cof_chunk *de
                        const uint32_t *items_rev, uint64_t n_rev,
                        uint64_t *hits, uint64_t hits_cap, uint64_t *n_hits, cof_stream s);
 
+/* Comparer implementation for cof_compare (process-wide): 0 = "popc" (POPC per
+ * comparison), 1 = "table" (bit-sliced pair tables on the ALU, default), 2 = "mma" (the
+ * comparison as an int8 GEMM on the tcgen05 tensor cores, comparer_mma.cu).  All three
+ * return the same hits.  COF_E_ARG for another value.  (Env COF_COMPARER=popc|table|mma
+ * sets the initial choice.)  The fused path (cof_find_compare) is the table comparer's. */
+cof_status cof_set_comparer(int impl);
+/* Contraction length K in bytes per int8 row of the plan's "mma" comparer: three sign
+ * bytes per position of the compared span (rounded to 4), two constant bytes and one byte
+ * per N-correction class, padded to 32.  0 for a NULL plan. */
+uint32_t   cof_plan_mma_kpad(const cof_plan *plan);
+
 /* ------------------------------------------------------------------ fused find + compare
  * the search and compare kernels of P:L29 without the host hand-off and
  * without the item lists: the finder (pass 1 only) writes per-word PAM masks into the

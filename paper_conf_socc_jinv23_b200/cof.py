@@ -88,6 +88,7 @@ def _load():
         "cof_find_compare": (I32, [P, P, P, P, P, U64, P, P]),
         "cof_find_masks": (I32, [P, P, P, P, P]),
         "cof_compare_masks": (I32, [P, P, P, P, P, U64, P, P]),
+        "cof_plan_mma_kpad": (U32, [P]),
         "cof_set_comparer": (I32, [ctypes.c_int]),
     }
     for name, (res, args) in sig.items():
@@ -110,7 +111,7 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_collect", "cof_merge", "cof_decorate_workspace_bytes", "cof_decorate",
                        "cof_decorate_check", "cof_find_compare_supported",
                        "cof_find_compare_workspace_bytes", "cof_find_compare", "cof_find_masks",
-                       "cof_compare_masks")]
+                       "cof_compare_masks", "cof_plan_mma_kpad", "cof_set_comparer")]
 
 
 def _check(st):
@@ -355,9 +356,15 @@ def cof_merge(lists) -> np.ndarray:
     return out
 
 
+def cof_plan_mma_kpad(plan) -> int:
+    """Contraction length K (bytes per int8 row) of the plan's tensor-core comparer."""
+    return int(lib.cof_plan_mma_kpad(plan.handle))
+
+
 def cof_set_comparer(impl: str):
-    """'table' (bit-sliced pair tables, default) or 'popc' (POPC per comparison)."""
-    _check(lib.cof_set_comparer({"popc": 0, "table": 1}[impl]))
+    """'table' (bit-sliced pair tables, default), 'popc' (POPC per comparison) or 'mma'
+    (int8 tcgen05 tensor-core GEMM, comparer_mma.cu)."""
+    _check(lib.cof_set_comparer({"popc": 0, "table": 1, "mma": 2}[impl]))
 
 
 class Fasta:

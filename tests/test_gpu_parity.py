@@ -14,7 +14,7 @@ from paper_conf_socc_jinv23_b200 import cof, search, synth
 from tests import golden_io
 
 pytestmark = pytest.mark.gpu
-IMPLS = ["table", "popc"]
+IMPLS = ["table", "popc", "mma"]
 
 
 @pytest.fixture(autouse=True)
@@ -86,6 +86,18 @@ def test_configs_scaled(name, scale, chunk, pack):
                     fused=False) == exp
     assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk, pack_bases=pack,
                     fused=True) == exp
+
+
+@pytest.mark.parametrize("name,scale,chunk,pack", [("C2", 0.1, None, None), ("C3", 0.004, 1_000_003, None),
+                                                   ("C4", 0.004, 333_333, 0), ("C5", 0.002, None, 0)])
+def test_configs_scaled_mma(name, scale, chunk, pack):
+    """The tensor-core comparer on the configs' shapes (incl. Cas12a TTTV with 23 compared
+    positions: three K steps) against the oracle."""
+    w = synth.make_workload(name, scale=scale, n_guides=None if name != "C5" else 1000)
+    cfg = w.cfg
+    exp = ref_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
+    assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk, pack_bases=pack,
+                    impl="mma") == exp
 
 
 def test_chunk_size_invariance():
@@ -218,9 +230,11 @@ def test_search_host_into_caller_buffer_and_chunk_pipeline(decorate):
     assert cof.hits_to_tuples(srch.search_host(packed, decorate=decorate)) == exp
 
 
-def test_many_guides_multiple_table_launches():
+@pytest.mark.parametrize("impl", ["table", "mma"])
+def test_many_guides_multiple_table_launches(impl):
     """> 4096 guides: the table comparer splits the guides into launches of 128 blocks
-    (thresholds in the parameter space) and tiles them through shared memory."""
+    (thresholds in the parameter space) and tiles them through shared memory; the mma
+    comparer into guide batches whose B image fits shared memory."""
     rng = np.random.default_rng(21)
     seq = synth.random_genome_text(rng, 30_000)
     n_g = 4096 + 300
@@ -228,6 +242,6 @@ def test_many_guides_multiple_table_launches():
     thr = [int(t) for t in rng.integers(4, 8, n_g)]
     exp = ref_hits([seq], "N" * 21 + "RG", guides, thr)
     assert len(exp) > 0
-    assert gpu_hits([seq], "N" * 21 + "RG", guides, thr) == exp
+    assert gpu_hits([seq], "N" * 21 + "RG", guides, thr, impl=impl) == exp
     thr_u = [7] * n_g
-    assert gpu_hits([seq], "N" * 21 + "RG", guides, thr_u) == ref_hits([seq], "N" * 21 + "RG", guides, thr_u)
+    assert gpu_hits([seq], "N" * 21 + "RG", guides, thr_u, impl=impl) == ref_hits([seq], "N" * 21 + "RG", guides, thr_u)
