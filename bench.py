@@ -100,22 +100,26 @@ class ClockSampler:
 
 
 # ----------------------------------------------------------------------------- workload
-def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
+def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl=None, query=None):
     """Synthetic workload + the device state the timed step runs on: resident planes of
     every chunk, one plan_dev per chunk (its counters), shared item buffers, per-chunk
-    hit buffers sized from a first (untimed) pass."""
+    hit buffers sized from a first (untimed) pass.  ``wl``: reuse a generated workload;
+    ``query``: (pattern, guides, thresholds) replacing the workload's (bulge variants)."""
     import torch
     from paper_conf_socc_jinv23_b200 import cof, search
 
-    wl = synth.make_workload(name, scale=scale, threads=max(1, min(16, os.cpu_count() or 1)))
-    L = wl.cfg.L
+    if wl is None:
+        wl = synth.make_workload(name, scale=scale, threads=max(1, min(16, os.cpu_count() or 1)))
+    pattern, guides, thresholds = query if query is not None else (wl.cfg.pattern, wl.guides, wl.thresholds)
+    L = len(pattern)
     if chunks is None:   # the whole genome as one multi-segment chunk (the bench's default)
         chunks = [search.pack_shard(search.plan_chunks([len(s) for s in wl.seqs], L, None))]
     st = type("State", (), {})()
     st.device = device or torch.device("cuda", torch.cuda.current_device())
     st.stream = torch.cuda.current_stream(st.device)
     st.chunks = chunks
-    st.plan = cof.cof_plan_create(wl.cfg.pattern, wl.guides, wl.thresholds)
+    st.plan = cof.cof_plan_create(pattern, guides, thresholds)
+    st.n_guides = len(guides)
     nbytes = cof.cof_plan_device_bytes(st.plan)
     st.host = search.HostGenome(wl.seqs, chunks)
     st.d_planes, st.d_chunks, st.plan_devs = [], [], []
@@ -132,7 +136,7 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None):
     max_owned = max(ch.n_owned for ch in chunks)
     # fused find+compare (finder masks -> comparer, no item lists) unless the guide table is
     # too large for it or COF_FUSED=0; the two-call path writes / reads ordered item lists
-    st.fused = search.use_fused(st.plan, len(wl.guides))
+    st.fused = search.use_fused(st.plan, len(guides))
     st.items = torch.empty((2, 1 if st.fused else max_owned), dtype=torch.int32, device=st.device)
     st.find_ws = torch.empty(cof.cof_find_compare_workspace_bytes(max(ch.n_bases for ch in chunks)),
                              dtype=torch.uint8, device=st.device)
@@ -266,6 +270,64 @@ def items_per_base_estimate(st, wl):
     return tot_items / max(1, sum(ch.n_owned for ch in st.chunks))
 
 
+# ----------------------------------------------------------------------------- bulge search
+def main_bulge(args, cfgname):
+    """--bulge D,R: the bulge search (bulge.py) of the config's genome on
+    one GPU: one device step = find -> compare -> sort -> decorate for every variant
+    pattern (X, DNA 1..D, RNA 1..R), each over all its guide variants; Gbases/s = genome
+    bases / device time of the whole step."""
+    import torch
+    from paper_conf_socc_jinv23_b200 import bulge, cof, search
+
+    dna, rna = (int(x) for x in args.bulge.split(","))
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    cof.cof_set_comparer(args.comparer)
+    wl = synth.make_workload(cfgname, scale=args.scale, threads=max(1, min(16, os.cpu_count() or 1)))
+    groups = bulge.variants(wl.cfg.pattern, wl.guides, wl.thresholds, dna, rna)
+    states = []
+    for pv, (gs, ts, ms) in groups.items():
+        chunks = [search.pack_shard(search.plan_chunks([len(x) for x in wl.seqs], len(pv), None))]
+        _, st = prepare_workload(cfgname, args.scale, chunks=chunks, device=dev, wl=wl, query=(pv, gs, ts))
+        states.append((pv, st))
+    for _ in range(max(args.warmup, 3)):
+        for _, st in states:
+            run_device_pipeline(wl, st)
+    torch.cuda.synchronize(dev)
+    s = states[0][1].stream
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    launches0 = cof.cof_launch_count()
+    t0.record(s)
+    for _ in range(args.steps):
+        for _, st in states:
+            run_device_pipeline(wl, st)
+    t1.record(s)
+    torch.cuda.synchronize(dev)
+    launches = cof.cof_launch_count() - launches0
+    ms = t0.elapsed_time(t1) / args.steps
+    comps = items = hits = 0
+    per = []
+    for pv, st in states:
+        c = step_counts(st)
+        items += c[0] + c[1]
+        comps += (c[0] + c[1]) * st.n_guides
+        hits += c[2]
+        per.append({"pattern": pv, "guide_variants": st.n_guides, "items": int(c[0] + c[1]), "hits": int(c[2])})
+    line = {"metric": "genome Gbases/s, bulge search (X + DNA<=%d + RNA<=%d)" % (dna, rna),
+            "value": round(wl.total_bases / (ms * 1e-3) / 1e9, 4), "unit": "Gbases/s", "n_gpus": 1,
+            "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": round(ms, 4),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32 bit-planes",
+            "data": "synthetic (seeded hg38-shaped genome, synth.py)", "comparisons_per_s": comps / (ms * 1e-3),
+            "hits_per_step": int(hits), "items_per_step": int(items),
+            "config": {"workload": cfgname, "genome_bases": wl.total_bases, "guides": len(wl.guides),
+                       "threshold": wl.cfg.threshold, "pattern": wl.cfg.pattern, "dna_bulge": dna, "rna_bulge": rna,
+                       "variant_searches": per, "comparer": args.comparer,
+                       "l2": "inputs larger than L2, no flush"},
+            "gpu_launches": int(launches // max(1, args.steps))}
+    print(json.dumps(line))
+    return 0
+
+
 # ----------------------------------------------------------------------------- main
 def main():
     ap = argparse.ArgumentParser()
@@ -279,6 +341,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--bulge", default=None, help="D,R: time the bulge search (max DNA, RNA bulge sizes)")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -291,6 +354,8 @@ def main():
         if rank != 0:
             return 0
         return main_reference(args, cfgname, metric)
+    if args.bulge:
+        return main_bulge(args, cfgname)
 
     import torch
     import torch.distributed as dist

@@ -6,7 +6,8 @@ INPUT follows the tool's input file ("the desired pattern, query sequences, and 
 mismatch number", P:L158 via [17]):
 
     /path/to/genome.fa            (a FASTA file, or a directory of .fa/.fasta/.fna files)
-    NNNNNNNNNNNNNNNNNNNNNRG       (pattern; N = any base, PAM letters in IUPAC)
+    NNNNNNNNNNNNNNNNNNNNNRG [D R] (pattern; N = any base, PAM letters in IUPAC; optional
+                                  maximum DNA / RNA bulge sizes)
     GGCCGACCTGTCGCTGACGCNNN 5     (query and its maximum mismatch count, one per line)
     ...
 
@@ -15,7 +16,8 @@ the number of mismatched bases and potential off-target DNA sequence with mismat
 bases"): query, chromosome name, 0-based position, site (mismatches lower-case),
 strand, mismatches — in (chromosome, position, strand, query) order (reading G13).
 The second positional argument (the original tool's C/G/A device letter) is accepted and
-ignored: the search always runs on the GPU.
+ignored: the search always runs on the GPU.  With bulges (D or R > 0) three columns follow:
+bulge type (X = none, DNA, RNA), bulge size and the guide offset of the bulge (bulge.py).
 """
 from __future__ import annotations
 
@@ -33,6 +35,8 @@ class InputSpec:
     pattern: str
     queries: list
     thresholds: list
+    dna_bulge: int = 0
+    rna_bulge: int = 0
 
 
 def parse_input(text: str, base_dir: str = ".") -> InputSpec:
@@ -43,7 +47,12 @@ def parse_input(text: str, base_dir: str = ".") -> InputSpec:
     genome = lines[0]
     if not os.path.isabs(genome):
         genome = os.path.join(base_dir, genome)
-    pattern = lines[1].split()[0]
+    pl = lines[1].split()
+    pattern = pl[0]
+    dna_b = int(pl[1]) if len(pl) > 1 else 0
+    rna_b = int(pl[2]) if len(pl) > 2 else 0
+    if dna_b < 0 or rna_b < 0:
+        raise ValueError(f"negative bulge size in {lines[1]!r}")
     queries, thr = [], []
     for ln in lines[2:]:
         parts = ln.split()
@@ -56,7 +65,7 @@ def parse_input(text: str, base_dir: str = ".") -> InputSpec:
             raise ValueError(f"negative mismatch count in {ln!r}")
         queries.append(q)
         thr.append(t)
-    return InputSpec(genome, pattern, queries, thr)
+    return InputSpec(genome, pattern, queries, thr, dna_b, rna_b)
 
 
 def genome_files(path: str):
@@ -73,6 +82,34 @@ def format_hits(hits, queries, names) -> str:
         out.append(f"{queries[int(h['guide'])]}\t{names[int(h['chrom'])]}\t{int(h['pos'])}\t"
                    f"{h['site'].decode()}\t{h['strand'].decode()}\t{int(h['mm'])}")
     return "\n".join(out) + ("\n" if out else "")
+
+
+def format_bulge_hits(hits, queries, names) -> str:
+    """TSV lines for a bulge.BULGE_DTYPE array (three bulge columns appended)."""
+    kinds = {b"X": "X", b"D": "DNA", b"R": "RNA"}
+    out = []
+    for h in hits:
+        out.append(f"{queries[int(h['guide'])]}\t{names[int(h['chrom'])]}\t{int(h['pos'])}\t"
+                   f"{h['site'].decode()}\t{h['strand'].decode()}\t{int(h['mm'])}\t"
+                   f"{kinds[h['kind']]}\t{int(h['size'])}\t{int(h['bpos'])}")
+    return "\n".join(out) + ("\n" if out else "")
+
+
+def run_bulge(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = None):
+    """Bulge search (bulge.py) of the genome of ``spec``; returns (hits, names)."""
+    import torch
+    from . import bulge, cof
+
+    names, seqs = [], []
+    for f in genome_files(spec.genome):
+        fa = cof.Fasta(f)
+        for i in range(len(fa)):
+            names.append(fa.name(i))
+            seqs.append(fa.read(i))
+    hits = bulge.search(seqs, spec.pattern, spec.queries, spec.thresholds, spec.dna_bulge, spec.rna_bulge,
+                        device=device, chunk_bases=chunk_bases)
+    torch.cuda.synchronize()
+    return hits, names
 
 
 def run(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = None):
@@ -106,8 +143,12 @@ def main(argv=None) -> int:
     output = a.args[-1]
     with open(a.input) as f:
         spec = parse_input(f.read(), os.path.dirname(os.path.abspath(a.input)))
-    hits, names = run(spec, a.device, a.chunk_bases)
-    text = format_hits(hits, spec.queries, names)
+    if spec.dna_bulge or spec.rna_bulge:
+        hits, names = run_bulge(spec, a.device, a.chunk_bases)
+        text = format_bulge_hits(hits, spec.queries, names)
+    else:
+        hits, names = run(spec, a.device, a.chunk_bases)
+        text = format_hits(hits, spec.queries, names)
     if output == "-":
         sys.stdout.write(text)
     else:

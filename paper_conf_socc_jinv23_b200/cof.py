@@ -385,6 +385,18 @@ class Fasta:
     def pack(self, i, first, n, lo, hi, nm):
         _check(lib.cof_fasta_pack(self.handle, i, int(first), int(n), _ptr(lo), _ptr(hi), _ptr(nm)))
 
+    def read(self, i) -> np.ndarray:
+        """Record i in canonical form (upper-case ACGT, N for anything else) as uint8 ASCII:
+        packed to planes and unpacked (the same canonicalisation as the device path)."""
+        n = self.length(i)
+        w = cof_plane_words(n)
+        planes = np.zeros((3, max(w, 1)), dtype=np.uint32)
+        out = np.empty(n, dtype=np.uint8)
+        if n:
+            self.pack(i, 0, n, planes[0], planes[1], planes[2])
+            cof_unpack(planes[0], planes[1], planes[2], 0, n, out)
+        return out
+
     def close(self):
         if self.handle:
             lib.cof_fasta_close(self.handle)

@@ -45,3 +45,32 @@ def test_cli_end_to_end(tmp_path):
                   f"{h['strand'].decode()}\t{int(h['mm'])}\n" for h in ref)
     assert len(ref) > 10
     assert out.read_text() == exp
+
+
+def test_parse_input_bulges():
+    spec = cli.parse_input("genome.fa\nNNNNNRG 2 1\nACGTANN 1\n")
+    assert (spec.dna_bulge, spec.rna_bulge) == (2, 1)
+    assert cli.parse_input("g\nNNRG\nACGN 0\n").dna_bulge == 0
+    with pytest.raises(ValueError):
+        cli.parse_input("g\nNNRG -1 0\nACGN 0\n")
+
+
+@pytest.mark.gpu
+def test_cli_bulge_end_to_end(tmp_path):
+    from oracle import bulge as obulge
+    rng = np.random.default_rng(32)
+    seqs = [synth.random_genome_text(rng, n) for n in (30_000, 12_345)]
+    names = ["chrA", "chrB"]
+    synth.write_fasta(tmp_path / "g.fa", names, seqs)
+    guides = ["".join(rng.choice(list("ACGT"), 20)) + "NNN" for _ in range(3)]
+    inp = tmp_path / "input.txt"
+    inp.write_text("g.fa\n" + "N" * 21 + "RG 1 1\n" + "".join(f"{g} 5\n" for g in guides))
+    out = tmp_path / "out.txt"
+    assert cli.main([str(inp), "G", str(out)]) == 0
+    ref = obulge.search(seqs, "N" * 21 + "RG", guides, [5] * 3, 1, 1)
+    kinds = {b"X": "X", b"D": "DNA", b"R": "RNA"}
+    exp = "".join(f"{guides[int(h['guide'])]}\t{names[int(h['chrom'])]}\t{int(h['pos'])}\t{h['site'].decode()}\t"
+                  f"{h['strand'].decode()}\t{int(h['mm'])}\t{kinds[h['kind']]}\t{int(h['size'])}\t{int(h['bpos'])}\n"
+                  for h in ref)
+    assert len(ref) > 0
+    assert out.read_text() == exp
