@@ -140,6 +140,22 @@ uint64_t   cof_fasta_length(const cof_fasta *fa, uint32_t i);
 cof_status cof_fasta_pack(const cof_fasta *fa, uint32_t i, uint64_t first, uint64_t n,
                           uint32_t *lo, uint32_t *hi, uint32_t *nm);
 
+/* ------------------------------------------------------------------ UCSC .2bit (f2)
+ * The packed genome format genomes are distributed in (hg38.2bit): 4 bases per byte, N
+ * and soft-mask runs as block lists.  Same interface as the FASTA reader: records are the
+ * file's sequences in index order; cof_2bit_pack writes bases [first, first+n) of record
+ * i into planes of cof_plane_words(n) words (N blocks -> nm = 1, lo = hi = 0; soft-mask
+ * ignored, reading G4).  COF_E_IO for a malformed or truncated file (checked at open),
+ * COF_E_ARG for a range past the record end. */
+typedef struct cof_twobit cof_twobit;
+cof_status cof_2bit_open(const char *path, cof_twobit **out);
+void       cof_2bit_close(cof_twobit *t);
+uint32_t   cof_2bit_count(const cof_twobit *t);
+const char *cof_2bit_name(const cof_twobit *t, uint32_t i);
+uint64_t   cof_2bit_length(const cof_twobit *t, uint32_t i);
+cof_status cof_2bit_pack(const cof_twobit *t, uint32_t i, uint64_t first, uint64_t n,
+                         uint32_t *lo, uint32_t *hi, uint32_t *nm);
+
 /* ------------------------------------------------------------------ finder (M5, M6)
  * The "search" kernel (signature Table VI): for every owned window
  * start p (single segment: p < n_owned; multi: vs bit set) with p+L <= n_bases, '+'

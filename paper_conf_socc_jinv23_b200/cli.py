@@ -5,7 +5,8 @@
 INPUT follows the tool's input file ("the desired pattern, query sequences, and maximum
 mismatch number", P:L158 via [17]):
 
-    /path/to/genome.fa            (a FASTA file, or a directory of .fa/.fasta/.fna files)
+    /path/to/genome.fa            (a FASTA or UCSC .2bit file, or a directory of
+                                  .fa/.fasta/.fna/.2bit files)
     NNNNNNNNNNNNNNNNNNNNNRG [D R] (pattern; N = any base, PAM letters in IUPAC; optional
                                   maximum DNA / RNA bulge sizes)
     GGCCGACCTGTCGCTGACGCNNN 5     (query and its maximum mismatch count, one per line)
@@ -70,7 +71,7 @@ def parse_input(text: str, base_dir: str = ".") -> InputSpec:
 
 def genome_files(path: str):
     if os.path.isdir(path):
-        ext = (".fa", ".fasta", ".fna", ".fa.txt")
+        ext = (".fa", ".fasta", ".fna", ".fa.txt", ".2bit")
         return sorted(os.path.join(path, f) for f in os.listdir(path) if f.lower().endswith(ext))
     return [path]
 
@@ -102,7 +103,7 @@ def run_bulge(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = N
 
     names, seqs = [], []
     for f in genome_files(spec.genome):
-        fa = cof.Fasta(f)
+        fa = cof.open_genome(f)
         for i in range(len(fa)):
             names.append(fa.name(i))
             seqs.append(fa.read(i))
@@ -117,7 +118,7 @@ def run(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = None):
     import torch
     from . import cof, search
 
-    fastas = [cof.Fasta(f) for f in genome_files(spec.genome)]
+    fastas = [cof.open_genome(f) for f in genome_files(spec.genome)]
     names, recs = [], []
     for fi, fa in enumerate(fastas):
         for i in range(len(fa)):

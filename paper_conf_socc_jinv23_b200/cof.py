@@ -89,6 +89,12 @@ def _load():
         "cof_find_masks": (I32, [P, P, P, P, P]),
         "cof_compare_masks": (I32, [P, P, P, P, P, U64, P, P]),
         "cof_plan_mma_kpad": (U32, [P]),
+        "cof_2bit_open": (I32, [ctypes.c_char_p, P]),
+        "cof_2bit_close": (None, [P]),
+        "cof_2bit_count": (U32, [P]),
+        "cof_2bit_name": (ctypes.c_char_p, [P, U32]),
+        "cof_2bit_length": (U64, [P, U32]),
+        "cof_2bit_pack": (I32, [P, U32, U64, U64, P, P, P]),
         "cof_set_comparer": (I32, [ctypes.c_int]),
     }
     for name, (res, args) in sig.items():
@@ -111,7 +117,9 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_collect", "cof_merge", "cof_decorate_workspace_bytes", "cof_decorate",
                        "cof_decorate_check", "cof_find_compare_supported",
                        "cof_find_compare_workspace_bytes", "cof_find_compare", "cof_find_masks",
-                       "cof_compare_masks", "cof_plan_mma_kpad", "cof_set_comparer")]
+                       "cof_compare_masks", "cof_plan_mma_kpad", "cof_set_comparer", "cof_2bit_open",
+                       "cof_2bit_close", "cof_2bit_count", "cof_2bit_name", "cof_2bit_length",
+                       "cof_2bit_pack")]
 
 
 def _check(st):
@@ -407,6 +415,37 @@ class Fasta:
             self.close()
         except Exception:
             pass
+
+
+class TwoBit(Fasta):
+    """UCSC .2bit genome (same interface as Fasta: len, name, length, pack, read)."""
+
+    def __init__(self, path):
+        out = ctypes.c_void_p()
+        _check(lib.cof_2bit_open(str(path).encode(), ctypes.addressof(out)))
+        self.handle = out.value
+
+    def __len__(self):
+        return int(lib.cof_2bit_count(self.handle))
+
+    def name(self, i):
+        return lib.cof_2bit_name(self.handle, i).decode()
+
+    def length(self, i):
+        return int(lib.cof_2bit_length(self.handle, i))
+
+    def pack(self, i, first, n, lo, hi, nm):
+        _check(lib.cof_2bit_pack(self.handle, i, int(first), int(n), _ptr(lo), _ptr(hi), _ptr(nm)))
+
+    def close(self):
+        if self.handle:
+            lib.cof_2bit_close(self.handle)
+            self.handle = None
+
+
+def open_genome(path):
+    """Fasta or TwoBit by file name (.2bit -> TwoBit)."""
+    return TwoBit(path) if str(path).lower().endswith(".2bit") else Fasta(path)
 
 
 def hits_to_tuples(arr):
