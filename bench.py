@@ -534,7 +534,7 @@ def comparer_roof(plan, n_sm, sm_mhz, impl):
     popc: 1 POPC per comparison, POPC = 16/clk/SM (measured, tools/microbench_pipes.cu).
     table: per item and 32-guide block, the minimal carry-save tree (FA/HA count from
     gen_csa for this plan's pair count) + 6-step borrow chain + 1 mask op, all LOP3 on
-    the ALU pipe (128 lanes/clk/SM, profiles/microbench_pipes_r1.txt); bound by shared memory: NP 64-bit lookups per item and
+    the 64/clk/SM ALU pipe (profiles/microbench_pipes_r1.txt); co-bound by shared memory: NP 64-bit lookups per item and
     block = 2*NP wavefronts per 32 items x 32 guides at 1 wavefront/clk/SM."""
     clk = sm_mhz * 1e6
     if impl == "popc":
@@ -559,7 +559,7 @@ def comparer_roof(plan, n_sm, sm_mhz, impl):
     fa = int(hdr.split(":")[1].split("full")[0])
     ha = int(hdr.split(",")[1].split("half")[0])
     alu_ops = 2 * fa + 2 * ha + 6 + 1
-    alu_rate = 128.0 * 32 / alu_ops          # comparisons / clk / SM (LOP3 full rate, measured)
+    alu_rate = 64.0 * 32 / alu_ops           # comparisons / clk / SM (64 LOP3/clk/SM, measured)
     lds_rate = 32.0 * 32 / (2 * npairs)      # comparisons / clk / SM
     per_clk = min(alu_rate, lds_rate)
     return {"peak": per_clk * n_sm * clk,
