@@ -100,7 +100,7 @@ class ClockSampler:
 
 
 # ----------------------------------------------------------------------------- workload
-def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl=None, query=None):
+def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl=None, query=None, n_guides=None):
     """Synthetic workload + the device state the timed step runs on: resident planes of
     every chunk, one plan_dev per chunk (its counters), shared item buffers, per-chunk
     hit buffers sized from a first (untimed) pass.  ``wl``: reuse a generated workload;
@@ -109,7 +109,7 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl
     from paper_conf_socc_jinv23_b200 import cof, search
 
     if wl is None:
-        wl = synth.make_workload(name, scale=scale, threads=max(1, min(16, os.cpu_count() or 1)))
+        wl = synth.make_workload(name, scale=scale, threads=max(1, min(16, os.cpu_count() or 1)), n_guides=n_guides)
     pattern, guides, thresholds = query if query is not None else (wl.cfg.pattern, wl.guides, wl.thresholds)
     L = len(pattern)
     if chunks is None:   # the whole genome as one multi-segment chunk (the bench's default)
@@ -342,6 +342,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--bulge", default=None, help="D,R: time the bulge search (max DNA, RNA bulge sizes)")
+    ap.add_argument("--n-guides", type=int, default=None, help="override the config's guide count (scaling study)")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -378,7 +379,7 @@ def main():
     all_chunks = search.plan_chunks([l for _, l in cfg.genome.chroms], L, None)
     shards = search.shard_lpt(all_chunks, world)
     mine = [search.pack_shard(shards[rank])]          # this rank's chromosomes as ONE chunk
-    wl, st = prepare_workload(cfgname, args.scale, chunks=mine, device=dev)
+    wl, st = prepare_workload(cfgname, args.scale, chunks=mine, device=dev, n_guides=args.n_guides)
     genome_bases = wl.total_bases
     my_items = sum(c[0] + c[1] for c in st.counts)
     comps_mine = my_items * len(wl.guides)
@@ -494,7 +495,8 @@ def main():
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32 bit-planes",
             "data": "synthetic (seeded hg38-shaped genome, synth.py)",
             "comparisons_per_s": comps_s, "hits_per_step": int(hits_all), "items_per_step": int(items_all),
-            "config": {"workload": cfgname, "description": cfg.description, "genome_bases": genome_bases,
+            "config": {"workload": cfgname if not args.n_guides else f"{cfgname} with {args.n_guides} guides",
+                       "description": cfg.description, "genome_bases": genome_bases,
                        "chromosomes": len(wl.seqs), "guides": len(wl.guides), "threshold": cfg.threshold,
                        "pattern": cfg.pattern,
                        "chunking": "device: this rank's chromosomes as one multi-segment chunk; "

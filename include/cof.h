@@ -209,8 +209,10 @@ uint32_t   cof_plan_mma_kpad(const cof_plan *plan);
  * without the item lists: the finder (pass 1 only) writes per-word PAM masks into the
  * workspace and the comparer expands them itself (shared-memory queue) before the table
  * comparison.  Same hits as cof_find_pam + cof_compare (same key format, unordered); the
- * item counts land in plan_dev (cof_read_counts).  Requires the whole guide table to fit
- * in shared memory (cof_find_compare_supported); otherwise COF_E_ARG.
+ * item counts land in plan_dev (cof_read_counts).  Each launch keeps its guide blocks
+ * resident in shared memory; larger guide sets run several launches per strand that
+ * re-expand the masks (up to 512 launches per strand, cof_find_compare_supported;
+ * otherwise COF_E_ARG).  Requires the table comparer (cof_set_comparer(1), the default).
  *  workspace  dev, >= cof_find_compare_workspace_bytes(dev->n_bases) bytes. */
 int        cof_find_compare_supported(const cof_plan *plan);
 size_t     cof_find_compare_workspace_bytes(uint64_t n_bases);

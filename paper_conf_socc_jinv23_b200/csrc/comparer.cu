@@ -32,6 +32,7 @@ namespace cof {
 constexpr int CT = 256;   // threads per CTA
 constexpr uint64_t ON_DEVICE = COF_COUNT_ON_DEVICE;
 constexpr uint32_t MAX_TABLE_BLOCKS = 128;   // 4096 guides per launch of the table comparer
+constexpr uint32_t FUSED_MAX_TICKETS = 1024; // grab counters (one per fused launch) after the finder workspace
 
 struct CompareArgs {
     const uint32_t* lo;
@@ -659,6 +660,8 @@ static cof_status launch_table(TableArgs& t, int uniform_t, uint64_t n_hint, cud
     return launch_any_r<NP, R_TABLE, -1>(t, fused, n_hint, stream);
 }
 
+static uint32_t fused_blocks_per_launch(const cof_plan* plan);
+
 // One launch per (strand, range of <= MAX_TABLE_BLOCKS guide blocks); thresholds travel in
 // the parameter space; hit counts accumulate on the device.
 static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs& a, cudaStream_t stream,
@@ -684,9 +687,11 @@ static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs
         T.n_wp = n_wp;
         T.ticket = tickets ? tickets + sd : nullptr;
         const uint32_t* pm = (const uint32_t*)(plan->image.data() + (sd == 0 ? plan->lay.pmeta_fwd : plan->lay.pmeta_rev));
-        for (uint32_t bb = 0; bb < plan->n_blocks; bb += MAX_TABLE_BLOCKS) {
+        const uint32_t batch = fused ? fused_blocks_per_launch(plan) : MAX_TABLE_BLOCKS;
+        for (uint32_t bb = 0, li = 0; bb < plan->n_blocks; bb += batch, li++) {
+            if (tickets) T.ticket = tickets + sd * ((plan->n_blocks + batch - 1) / batch) + li;
             T.block_base = bb;
-            T.n_blocks = std::min<uint32_t>(MAX_TABLE_BLOCKS, plan->n_blocks - bb);
+            T.n_blocks = std::min<uint32_t>(batch, plan->n_blocks - bb);
             T.ptab = (const uint2*)(pd + (sd == 0 ? plan->lay.ptab_fwd : plan->lay.ptab_rev)) + (size_t)bb * np * 25;
             for (uint32_t k = 0; k < T.n_blocks; k++)
                 for (int w = 0; w < 8; w++) T.meta[k][w] = pm[(size_t)(bb + k) * 8 + w];
@@ -756,10 +761,17 @@ cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* de
 const uint4* finder_masks(const void* workspace);
 uint64_t finder_word_pairs(const cof_plan* plan, const cof_chunk* dev);
 
+// Guide blocks per launch of the fused comparer: its whole launch table is resident in
+// shared memory (no re-loads between mask grabs), so a plan with more blocks runs several
+// launches per strand, each re-expanding the finder masks (0.25 B per base).
+static uint32_t fused_blocks_per_launch(const cof_plan* plan) {
+    const uint32_t per_block = plan->pairs[0].n_pairs * 25u * 8u;
+    const size_t avail = table_smem_budget() + 16u * 1024u - (CT / 32) * FWQ * 4u - 1024u;
+    return std::min<uint32_t>(MAX_TABLE_BLOCKS, (uint32_t)(avail / per_block));
+}
 static bool fusable(const cof_plan* plan) {
-    const uint32_t np = plan->pairs[0].n_pairs;
-    return plan->n_blocks <= MAX_TABLE_BLOCKS &&
-           (size_t)plan->n_blocks * np * 25 * 8 + (CT / 32) * FWQ * 4 + 1024 <= table_smem_budget() + 16 * 1024;
+    const uint32_t bpl = fused_blocks_per_launch(plan);
+    return bpl >= 1 && (plan->n_blocks + bpl - 1) / bpl * 2 <= FUSED_MAX_TICKETS;
 }
 
 }  // namespace cof
@@ -772,7 +784,9 @@ int cof_find_compare_supported(const cof_plan* plan) {
     return plan && comparer_impl() == 1 && fusable(plan) ? 1 : 0;
 }
 
-size_t cof_find_compare_workspace_bytes(uint64_t n_bases) { return cof_find_workspace_bytes(n_bases) + 256; }
+size_t cof_find_compare_workspace_bytes(uint64_t n_bases) {
+    return cof_find_workspace_bytes(n_bases) + FUSED_MAX_TICKETS * sizeof(unsigned int);
+}
 
 cof_status cof_find_masks(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace, cof_stream s) {
     if (!plan || !plan_dev || !dev || !workspace) return set_error(COF_E_ARG, "cof_find_masks: NULL argument");
@@ -797,7 +811,7 @@ cof_status cof_compare_masks(const cof_plan* plan, void* plan_dev, const cof_chu
     unsigned long long* counters = (unsigned long long*)(pd + plan->lay.counters);
     unsigned int* tickets = (unsigned int*)((uint8_t*)workspace + cof_find_workspace_bytes(dev->n_bases));
     cudaError_t e = cudaMemsetAsync(counters + 2, 0, sizeof(uint64_t), stream);
-    if (e == cudaSuccess) e = cudaMemsetAsync(tickets, 0, 2 * sizeof(unsigned int), stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(tickets, 0, FUSED_MAX_TICKETS * sizeof(unsigned int), stream);
     if (e != cudaSuccess) return cuda_error(e, "cof_compare_masks memset");
     CompareArgs a;
     a.lo = dev->lo; a.hi = dev->hi; a.nm = dev->nm;

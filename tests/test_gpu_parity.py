@@ -243,5 +243,8 @@ def test_many_guides_multiple_table_launches(impl):
     exp = ref_hits([seq], "N" * 21 + "RG", guides, thr)
     assert len(exp) > 0
     assert gpu_hits([seq], "N" * 21 + "RG", guides, thr, impl=impl) == exp
+    if impl == "table":   # fused (several launches per strand) and two-call paths
+        assert gpu_hits([seq], "N" * 21 + "RG", guides, thr, impl=impl, fused=True) == exp
+        assert gpu_hits([seq], "N" * 21 + "RG", guides, thr, impl=impl, fused=False) == exp
     thr_u = [7] * n_g
     assert gpu_hits([seq], "N" * 21 + "RG", guides, thr_u, impl=impl) == ref_hits([seq], "N" * 21 + "RG", guides, thr_u)
