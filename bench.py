@@ -166,7 +166,7 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl
     st.tmp = torch.empty(max(st.caps), dtype=torch.int64, device=st.device)
     st.sort_ws = torch.empty(cof.cof_sort_workspace_bytes(max(st.caps)), dtype=torch.uint8, device=st.device)
     # device decoration (the device half of a7 collect): records per chunk
-    st.recs = [torch.empty(c * cof.HIT_DTYPE.itemsize, dtype=torch.uint8, device=st.device) for c in st.caps]
+    st.recs = [torch.empty(c * cof.hit_dtype(st.plan.L).itemsize, dtype=torch.uint8, device=st.device) for c in st.caps]
     st.dec_ws = torch.empty((len(chunks), cof.cof_decorate_workspace_bytes(max(len(ch.pieces) for ch in chunks))),
                             dtype=torch.uint8, device=st.device)
     st.max_owned = max_owned
@@ -582,7 +582,8 @@ def measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev=None):
     n_out = int(len(hits0) * 1.05) + 1024
     # the caller's result buffer: pinned host memory, so the device-decorated records DMA
     # straight into it (allocated and touched once, outside the timed steps)
-    out = torch.zeros(n_out * cof.HIT_DTYPE.itemsize, dtype=torch.uint8, pin_memory=True).numpy().view(cof.HIT_DTYPE)
+    hd = srch.hit_dtype
+    out = torch.zeros(n_out * hd.itemsize, dtype=torch.uint8, pin_memory=True).numpy().view(hd)
     del hits0
     torch.cuda.synchronize(dev)
     if world > 1:

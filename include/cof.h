@@ -34,11 +34,17 @@ extern "C" {
 
 typedef int32_t cof_status;
 #define COF_OK          0
-#define COF_E_ARG      (-1)   /* bad argument: non-IUPAC letter, length mismatch, L>32, NULL, ... */
+#define COF_E_ARG      (-1)   /* bad argument: non-IUPAC letter, length mismatch, L>64, NULL, ... */
 #define COF_E_CAPACITY (-2)   /* output buffer too small; the needed count is returned */
 #define COF_E_CUDA     (-3)   /* CUDA runtime error (message has the CUDA error string) */
 #define COF_E_STATE    (-4)   /* plan / chunk / workspace mismatch */
 #define COF_E_IO       (-5)   /* file could not be read / parsed */
+
+/* Longest pattern / guide (two 32-bit plane words per window).  The
+ * paper fixes no bound (Listing 1 loops over plen).  Patterns with L <= 32 use
+ * one-word windows and the 56-byte cof_hit; 32 < L <= 64 use two-word windows and the
+ * 88-byte cof_hit64 (cof_collect64 / cof_decorate64 / cof_merge64). */
+#define COF_MAX_L 64
 
 /* Pass as a count to cof_compare / cof_sort_hits to use the count the previous call
  * left in the plan's device workspace (no host round trip between kernels). */
@@ -55,13 +61,15 @@ uint64_t cof_launch_count(void);
  * The input specification: a search pattern of length L (guide Ns + PAM, e.g.
  * "NNNNNNNNNNNNNNNNNNNNNRG") and n queries ("guides") of the same length, each with its
  * own maximum mismatch count (P:L158 via [17]; Listing 1 parameters P:L185-L188).
- *  pattern   NUL-terminated IUPAC string (ACGTRYSWKMBDHVN, case-insensitive), 1<=L<=32.
+ *  pattern   NUL-terminated IUPAC string (ACGTRYSWKMBDHVN, case-insensitive), 1<=L<=64.
  *  guides    n_guides NUL-terminated IUPAC strings of length L; 'N' positions are not
  *            compared (the -1-terminated index list; reading G7).
  *  max_mm    n_guides thresholds; a site is a hit iff #mismatches <= max_mm.
  *  out       receives a host-only, immutable plan (thread-safe to share read-only).
- * Errors: COF_E_ARG for a non-IUPAC letter (G18), guide length != L (G11), L>32,
- * n_guides == 0 or > 2^24, NULL pointers.  The plan reverse-complements pattern and
+ * Errors: COF_E_ARG for a non-IUPAC letter (G18), guide length != L (G11), L>64, a
+ * guide with 64 compared (non-N) letters, n_guides == 0 or > 2^24, NULL pointers.  For
+ * L > 32 the comparer is always the pair-table one (cof_set_comparer's popc / mma
+ * variants need L <= 32).  The plan reverse-complements pattern and
  * guides for the '-' strand and groups guides by compared-position mask. */
 typedef struct cof_plan cof_plan;
 cof_status cof_plan_create(const char *pattern, uint32_t n_guides, const char *const *guides,
@@ -257,12 +265,25 @@ typedef struct {
     char     site[34]; /* NUL-terminated */
 } cof_hit;
 
+/* The same record for patterns with 32 < L <= 64 (site up to 64 letters). */
+typedef struct {
+    uint32_t guide;
+    uint32_t chrom;
+    uint64_t pos;
+    char     strand;   /* '+' or '-' */
+    uint8_t  mm;
+    char     site[66]; /* NUL-terminated */
+} cof_hit64;
+
 /* D2H the n_hits keys from hits_dev (stream s), order them (host sort if they are not
  * already sorted), and decorate them from the HOST planes of the same chunk.
  * out must hold n_hits records; it is sorted by (pos, strand, guide).
  * If hits_dev is NULL, keys are read from host_keys instead (already on the host). */
 cof_status cof_collect(const cof_plan *plan, const cof_chunk *host, const uint64_t *hits_dev,
                        const uint64_t *host_keys, uint64_t n_hits, cof_hit *out, cof_stream s);
+/* cof_collect for plans with L > 32 (also accepts L <= 32). */
+cof_status cof_collect64(const cof_plan *plan, const cof_chunk *host, const uint64_t *hits_dev,
+                         const uint64_t *host_keys, uint64_t n_hits, cof_hit64 *out, cof_stream s);
 
 /* The same decoration on the device: n_hits (sorted) keys of hits_dev -> n_hits records in
  * the DEVICE buffer out_dev (same order; n_hits = COF_COUNT_ON_DEVICE: the count of the
@@ -275,12 +296,18 @@ size_t     cof_decorate_workspace_bytes(uint32_t n_segs);
 cof_status cof_decorate(const cof_plan *plan, const void *plan_dev, const cof_chunk *dev,
                         const uint64_t *hits_dev, uint64_t n_hits, uint64_t cap, cof_hit *out_dev,
                         void *workspace, cof_stream s);
+/* cof_decorate for plans with L > 32 (also accepts L <= 32): cof_hit64 records. */
+cof_status cof_decorate64(const cof_plan *plan, const void *plan_dev, const cof_chunk *dev,
+                          const uint64_t *hits_dev, uint64_t n_hits, uint64_t cap, cof_hit64 *out_dev,
+                          void *workspace, cof_stream s);
 cof_status cof_decorate_check(const void *workspace, cof_stream s);
 
 /* k-way merge of sorted lists into out (sum of lens records), order (chrom, pos,
  * strand, guide) (G13).  Lists from disjoint chunks merge by concatenation. */
 cof_status cof_merge(const cof_hit *const *lists, const uint64_t *lens, uint32_t n_lists,
                      cof_hit *out);
+cof_status cof_merge64(const cof_hit64 *const *lists, const uint64_t *lens, uint32_t n_lists,
+                       cof_hit64 *out);
 
 #ifdef __cplusplus
 }

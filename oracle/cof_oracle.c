@@ -37,13 +37,17 @@
 #include <omp.h>
 #endif
 
+/* Longest pattern the oracle accepts (reading G11: guide length = pattern length).  The
+ * paper fixes no bound; 64 covers the CUDA path's two-word windows. */
+#define COF_ORACLE_MAX_L 64
+
 typedef struct {
     int32_t guide;
     int32_t chrom;
     int64_t pos;      /* 0-based leftmost base of the window on the '+' strand (reading G5) */
     char strand;      /* '+' or '-' */
     int8_t mm;
-    char site[34];    /* NUL-terminated, length L */
+    char site[66];    /* NUL-terminated, length L (L <= COF_ORACLE_MAX_L) */
 } oracle_hit;
 
 /* ---- IUPAC nucleotide codes, written out as the nomenclature defines them ---- */
@@ -132,7 +136,7 @@ static int push(hitvec *h, const oracle_hit *x)
 /* Builds the strand-s reading S of the window at p: S = W ('+') or revcomp(W) ('-'). */
 static void window_reading(const char *seq, int64_t p, int L, char strand, char *S)
 {
-    char W[33];
+    char W[COF_ORACLE_MAX_L + 1];
     for (int j = 0; j < L; j++)
         W[j] = canon(seq[p + j]);
     if (strand == '+') {
@@ -155,7 +159,7 @@ static int validate(const char *pattern, int n_guides, const char *const *guides
                     const int32_t *max_mm, int *Lout)
 {
     int L = (int)strlen(pattern);
-    if (L < 1 || L > 32) return -1;
+    if (L < 1 || L > COF_ORACLE_MAX_L) return -1;
     for (int j = 0; j < L; j++)
         if (!is_iupac_code(upper(pattern[j]))) return -1;
     for (int i = 0; i < n_guides; i++) {
@@ -183,10 +187,10 @@ int64_t cof_oracle_search(int32_t n_chrom, const char *const *seqs, const int64_
     int L;
     *out = NULL;
     if (validate(pattern_in, n_guides, guides_in, max_mm, &L)) return -1;
-    char P[33];
+    char P[COF_ORACLE_MAX_L + 1];
     for (int j = 0; j < L; j++) P[j] = upper(pattern_in[j]);
     P[L] = 0;
-    char (*G)[33] = (char (*)[33])malloc((size_t)(n_guides ? n_guides : 1) * 33);
+    char (*G)[COF_ORACLE_MAX_L + 1] = (char (*)[COF_ORACLE_MAX_L + 1])malloc((size_t)(n_guides ? n_guides : 1) * (COF_ORACLE_MAX_L + 1));
     if (!G) return -2;
     for (int i = 0; i < n_guides; i++) {
         for (int j = 0; j < L; j++) G[i][j] = upper(guides_in[i][j]);
@@ -210,7 +214,7 @@ int64_t cof_oracle_search(int32_t n_chrom, const char *const *seqs, const int64_
 #endif
         for (int64_t b = 0; b < nblocks; b++) {
             int64_t p0 = lo + b * BLOCK, p1 = p0 + BLOCK < hi ? p0 + BLOCK : hi;
-            char S[33];
+            char S[COF_ORACLE_MAX_L + 1];
             for (int64_t p = p0; p < p1; p++) {
                 for (int s = 0; s < 2; s++) {
                     char strand = s == 0 ? '+' : '-';
@@ -263,8 +267,8 @@ int64_t cof_oracle_pam_sites(const char *seq, int64_t len, int64_t begin, int64_
 {
     int L = (int)strlen(pattern_in);
     *out = NULL;
-    if (L < 1 || L > 32 || (strand != '+' && strand != '-')) return -1;
-    char P[33];
+    if (L < 1 || L > COF_ORACLE_MAX_L || (strand != '+' && strand != '-')) return -1;
+    char P[COF_ORACLE_MAX_L + 1];
     for (int j = 0; j < L; j++) {
         P[j] = upper(pattern_in[j]);
         if (!is_iupac_code(P[j])) return -1;
@@ -274,7 +278,7 @@ int64_t cof_oracle_pam_sites(const char *seq, int64_t len, int64_t begin, int64_
     int64_t n = 0, cap = 1024;
     int64_t *v = (int64_t *)malloc((size_t)cap * sizeof(int64_t));
     if (!v) return -2;
-    char S[33];
+    char S[COF_ORACLE_MAX_L + 1];
     for (int64_t p = lo; p < hi; p++) {
         window_reading(seq, p, L, strand, S);
         if (!pam_ok(S, P, L)) continue;

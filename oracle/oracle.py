@@ -20,7 +20,7 @@ SRC = os.path.join(HERE, "cof_oracle.c")
 LIB = os.path.join(HERE, "liboracle.so")
 
 HIT_DTYPE = np.dtype([("guide", "<i4"), ("chrom", "<i4"), ("pos", "<i8"),
-                      ("strand", "S1"), ("mm", "i1"), ("site", "S34")], align=True)
+                      ("strand", "S1"), ("mm", "i1"), ("site", "S66")], align=True)
 
 
 def build(force: bool = False) -> str:

@@ -21,11 +21,12 @@ from __future__ import annotations
 
 import numpy as np
 
+from . import cof
 from . import search as _search
 
 BULGE_DTYPE = np.dtype([("guide", "<u4"), ("kind", "S1"), ("size", "u1"), ("bpos", "u1"),
                         ("chrom", "<u4"), ("pos", "<u8"), ("strand", "S1"), ("mm", "u1"),
-                        ("site", "S40")], align=True)
+                        ("site", "S66")], align=True)
 
 
 def compared_span(guide: str):
@@ -74,8 +75,8 @@ def search(seqs, pattern, guides, thresholds, dna: int = 0, rna: int = 0, device
             (np.frombuffer(s.encode(), dtype=np.uint8) if isinstance(s, str) else s) for s in seqs]
     parts = []
     for pv, (gs, ts, ms) in variants(pattern, guides, thresholds, dna, rna).items():
-        if len(pv) > 32:
-            raise ValueError(f"bulge variant pattern of length {len(pv)} exceeds 32")
+        if len(pv) > cof.COF_MAX_L:
+            raise ValueError(f"bulge variant pattern of length {len(pv)} exceeds {cof.COF_MAX_L}")
         chunks = _search.plan_chunks([len(a) for a in arrs], len(pv), chunk_bases, pack_bases)
         host = _search.HostGenome(arrs, chunks)
         srch = _search.Searcher(pv, gs, ts, device)

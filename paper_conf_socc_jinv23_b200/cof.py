@@ -25,6 +25,16 @@ COF_COUNT_ON_DEVICE = (1 << 64) - 1
 
 HIT_DTYPE = np.dtype([("guide", "<u4"), ("chrom", "<u4"), ("pos", "<u8"), ("strand", "S1"),
                       ("mm", "u1"), ("site", "S34")], align=True)
+# cof_hit64: the record of patterns with 32 < L <= COF_MAX_L
+HIT64_DTYPE = np.dtype([("guide", "<u4"), ("chrom", "<u4"), ("pos", "<u8"), ("strand", "S1"),
+                        ("mm", "u1"), ("site", "S66"), ("_pad", "V4")], align=True)
+COF_MAX_L = 64
+assert HIT_DTYPE.itemsize == 56 and HIT64_DTYPE.itemsize == 88
+
+
+def hit_dtype(L: int) -> np.dtype:
+    """Record dtype of a plan with pattern length L (cof_hit for L <= 32, else cof_hit64)."""
+    return HIT_DTYPE if L <= 32 else HIT64_DTYPE
 
 
 class CofError(RuntimeError):
@@ -79,9 +89,12 @@ def _load():
         "cof_sort_hits": (I32, [P, P, P, P, P, U64, U64, P, P]),
         "cof_read_counts": (I32, [P, P, P, P]),
         "cof_collect": (I32, [P, P, P, P, U64, P, P]),
+        "cof_collect64": (I32, [P, P, P, P, U64, P, P]),
         "cof_merge": (I32, [P, P, U32, P]),
+        "cof_merge64": (I32, [P, P, U32, P]),
         "cof_decorate_workspace_bytes": (SZ, [U32]),
         "cof_decorate": (I32, [P, P, P, P, U64, U64, P, P, P]),
+        "cof_decorate64": (I32, [P, P, P, P, U64, U64, P, P, P]),
         "cof_decorate_check": (I32, [P, P]),
         "cof_find_compare_supported": (ctypes.c_int, [P]),
         "cof_find_compare_workspace_bytes": (SZ, [U64]),
@@ -114,7 +127,8 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_fasta_count", "cof_fasta_name", "cof_fasta_length", "cof_fasta_pack",
                        "cof_find_workspace_bytes", "cof_find_pam", "cof_compare",
                        "cof_sort_workspace_bytes", "cof_sort_hits", "cof_read_counts",
-                       "cof_collect", "cof_merge", "cof_decorate_workspace_bytes", "cof_decorate",
+                       "cof_collect", "cof_collect64", "cof_merge", "cof_merge64",
+                       "cof_decorate_workspace_bytes", "cof_decorate", "cof_decorate64",
                        "cof_decorate_check", "cof_find_compare_supported",
                        "cof_find_compare_workspace_bytes", "cof_find_compare", "cof_find_masks",
                        "cof_compare_masks", "cof_plan_mma_kpad", "cof_set_comparer", "cof_2bit_open",
@@ -321,21 +335,26 @@ def cof_read_counts(plan, plan_dev, stream=None):
     return int(out[0]), int(out[1]), int(out[2])
 
 
+def _collect_fn(plan):
+    return lib.cof_collect if plan.L <= 32 else lib.cof_collect64
+
+
 def cof_collect(plan, host: cof_chunk, hits_dev, n_hits, stream=None, host_keys=None) -> np.ndarray:
-    out = np.empty(int(n_hits), dtype=HIT_DTYPE)
+    """cof_collect (L <= 32, cof_hit records) or cof_collect64 (L > 32, cof_hit64)."""
+    out = np.empty(int(n_hits), dtype=hit_dtype(plan.L))
     if n_hits:
-        _check(lib.cof_collect(plan.handle, ctypes.addressof(host), _ptr(hits_dev), _ptr(host_keys),
-                               int(n_hits), out.ctypes.data, _stream(stream)))
+        _check(_collect_fn(plan)(plan.handle, ctypes.addressof(host), _ptr(hits_dev), _ptr(host_keys),
+                                 int(n_hits), out.ctypes.data, _stream(stream)))
     return out
 
 
 def cof_collect_into(plan, host: cof_chunk, host_keys, n_hits, out: np.ndarray):
     """cof_collect from host keys into a caller-provided (contiguous) record array."""
-    if not out.flags["C_CONTIGUOUS"] or out.dtype != HIT_DTYPE or len(out) < n_hits:
-        raise ValueError("out must be a contiguous HIT_DTYPE array of >= n_hits records")
+    if not out.flags["C_CONTIGUOUS"] or out.dtype != hit_dtype(plan.L) or len(out) < n_hits:
+        raise ValueError("out must be a contiguous hit_dtype(L) array of >= n_hits records")
     if n_hits:
-        _check(lib.cof_collect(plan.handle, ctypes.addressof(host), None, _ptr(host_keys), int(n_hits),
-                               out.ctypes.data, None))
+        _check(_collect_fn(plan)(plan.handle, ctypes.addressof(host), None, _ptr(host_keys), int(n_hits),
+                                 out.ctypes.data, None))
     return out
 
 
@@ -345,8 +364,10 @@ def cof_decorate_workspace_bytes(n_segs: int) -> int:
 
 def cof_decorate(plan, plan_dev, dev: cof_chunk, hits_dev, n_hits, out_dev, workspace, stream=None, cap=0):
     """Device decoration: n_hits keys -> n_hits cof_hit records in the device buffer out_dev
-    (n_hits = COF_COUNT_ON_DEVICE: the device count clamped to ``cap``)."""
-    _check(lib.cof_decorate(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(hits_dev), int(n_hits),
+    (n_hits = COF_COUNT_ON_DEVICE: the device count clamped to ``cap``); cof_hit64 records
+    (cof_decorate64) when L > 32."""
+    fn = lib.cof_decorate if plan.L <= 32 else lib.cof_decorate64
+    _check(fn(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(hits_dev), int(n_hits),
                             int(cap), _ptr(out_dev), _ptr(workspace), _stream(stream)))
 
 
@@ -355,12 +376,16 @@ def cof_decorate_check(workspace, stream=None):
 
 
 def cof_merge(lists) -> np.ndarray:
-    lists = [np.ascontiguousarray(x, dtype=HIT_DTYPE) for x in lists]
+    """cof_merge (cof_hit lists) or cof_merge64 (cof_hit64 lists, any list of HIT64_DTYPE)."""
+    wide = any(getattr(x, "dtype", None) == HIT64_DTYPE for x in lists)
+    dt = HIT64_DTYPE if wide else HIT_DTYPE
+    lists = [np.ascontiguousarray(x, dtype=dt) for x in lists]
     total = sum(len(x) for x in lists)
-    out = np.empty(total, dtype=HIT_DTYPE)
+    out = np.empty(total, dtype=dt)
     ptrs = (ctypes.c_void_p * max(len(lists), 1))(*[x.ctypes.data for x in lists])
     lens = (ctypes.c_uint64 * max(len(lists), 1))(*[len(x) for x in lists])
-    _check(lib.cof_merge(ctypes.addressof(ptrs), ctypes.addressof(lens), len(lists), out.ctypes.data))
+    fn = lib.cof_merge64 if wide else lib.cof_merge
+    _check(fn(ctypes.addressof(ptrs), ctypes.addressof(lens), len(lists), out.ctypes.data))
     return out
 
 

@@ -28,8 +28,8 @@ inline int concrete_code(uint8_t m) {
 // ---- finder parameters (per strand, non-N pattern positions)
 struct PamStrand {
     uint32_t n;            // number of non-N positions
-    uint8_t j[32];         // window offset
-    uint8_t set[32];       // IUPAC set mask
+    uint8_t j[COF_MAX_L];      // window offset
+    uint8_t set[COF_MAX_L];    // IUPAC set mask
 };
 
 // ---- comparer guide tables (device image inside plan_dev)
@@ -64,10 +64,13 @@ COF_HD uint32_t pair_entry(uint32_t np, uint32_t q, uint32_t b1, uint32_t b2) {
 // Bit-sliced pair-table comparer (v2): per strand, per 32-guide block, per position pair,
 // 25 entries (base pair combos incl. N) of {bit0, bit1} mismatch-count planes.
 struct PairLayout {
-    uint32_t n_pairs;          // pairs covering the union of compared positions
-    uint8_t j1[16], j2[16];    // window offsets of the pair (j2 == 0xFF: single position)
+    uint32_t n_pairs;          // pairs covering the union of compared positions (+ padding)
+    uint8_t j1[32], j2[32];    // window offsets of the pair (j2 == 0xFF: single position,
+                               // 0xFE: padding pair, table entries all zero)
     uint32_t contig;           // 1: compared positions are the contiguous range [p0, p0 + n_cmp)
     uint32_t p0, n_cmp;        //    so pair q = window offsets (p0 + 2q, p0 + 2q + 1)
+    uint32_t wide;             // 1: compared span > 32: 64-bit windows, n_pairs a multiple of 4
+    uint32_t n_real;           // pairs before the padding
 };
 
 // Tensor-core comparer (comparer_mma.cu): the mismatch count of every (item, guide) pair
@@ -98,7 +101,7 @@ struct DevLayout {
     size_t recs_fwd, recs_rev;       // uint4[n_recs]
     size_t ptab_fwd, ptab_rev;       // pair tables: uint2[n_blocks][n_pairs][25]
     size_t pmeta_fwd, pmeta_rev;     // per block: uint32[8] = {T0..T5 threshold planes, valid, 0}
-    size_t onehot;                   // uint32[2][n_guides][5] decoration masks (see cof_plan::onehot)
+    size_t onehot;                   // uint64[2][n_guides][5] decoration masks (see cof_plan::onehot)
     size_t mma_b;                    // tensor-core comparer: int8 B images of all guide batches
     size_t mma_thr;                  // uint8[n_guides]: min(t_g, #compared positions)
     size_t total;
@@ -113,14 +116,14 @@ struct cof_plan {
     std::vector<std::string> guides;     // upper-case
     std::vector<uint8_t> max_mm;
     std::vector<uint8_t> gmask;          // [n_guides * L] IUPAC masks (forward orientation)
-    std::vector<uint32_t> onehot;        // [2][n_guides][5]: A, C, G, T membership + care, window offsets
+    std::vector<uint64_t> onehot;        // [2][n_guides][5]: A, C, G, T membership + care, window offsets
     cof::PamStrand pam[2];               // [0] '+', [1] '-' (reverse-complemented pattern)
     uint32_t n_groups = 0;
     uint32_t n_recs = 0;
     uint32_t n_blocks = 0;               // 32-guide blocks (pair-table comparer)
     cof::PairLayout pairs[2];
     cof::MmaPlan mma;
-    uint32_t union_care[2] = {0, 0};
+    uint64_t union_care[2] = {0, 0};
     bool any_degenerate = false;
     cof::DevLayout lay;
     std::vector<uint8_t> image;          // host copy of the device image (counters zeroed)

@@ -34,6 +34,12 @@ constexpr uint64_t ON_DEVICE = COF_COUNT_ON_DEVICE;
 constexpr uint32_t MAX_TABLE_BLOCKS = 128;   // 4096 guides per launch of the table comparer
 constexpr uint32_t FUSED_MAX_TICKETS = 1024; // grab counters (one per fused launch) after the finder workspace
 
+// Window word of the table comparer: one 32-bit slice, or 64 bits when the compared span
+// exceeds 32 positions (L > 32).
+template <bool W64> struct WinSel { using T = uint32_t; };
+template <> struct WinSel<true> { using T = unsigned long long; };
+template <bool W64> using WinT = typename WinSel<W64>::T;
+
 struct CompareArgs {
     const uint32_t* lo;
     const uint32_t* hi;
@@ -172,16 +178,17 @@ __global__ void __launch_bounds__(CT) cof_comparer_popc(const __grid_constant__ 
 // item is read at base[q] + OFF + q * 128, where OFF = the guide block's table offset and
 // q * 128 (pair q's 16 ACGT entries) are compile-time immediates of the LDS; base[q] is the
 // 128-byte-aligned table base plus the entry's offset relative to q * 128.
-// (wl, wh, wn: windows starting at window offset pl.p0, the first compared position)
-template <int NP>
-__device__ __forceinline__ void pair_offsets(const PairLayout& pl, uint32_t s_base, uint32_t wl, uint32_t wh,
-                                             uint32_t wn, uint32_t (&base)[NP]) {
+// (wl, wh, wn: windows starting at window offset pl.p0, the first compared position;
+// WT = uint32_t, or unsigned long long for compared spans > 32 (two-word windows, L > 32))
+template <int NP, typename WT>
+__device__ __forceinline__ void pair_offsets(const PairLayout& pl, uint32_t s_base, WT wl, WT wh,
+                                             WT wn, uint32_t (&base)[NP]) {
 #pragma unroll
     for (int q = 0; q < NP; q++) {
-        const uint32_t j1 = pl.j1[q] - pl.p0, j2 = pl.j2[q] == 0xFFu ? 0xFFu : pl.j2[q] - pl.p0;
-        const uint32_t b1 = ((wn >> j1) & 1u) ? 4u : (((wl >> j1) & 1u) | (((wh >> j1) & 1u) << 1));
+        const uint32_t j1 = pl.j1[q] - pl.p0, j2 = pl.j2[q] >= 0xFEu ? 0xFFu : pl.j2[q] - pl.p0;
+        const uint32_t b1 = ((wn >> j1) & 1u) ? 4u : (uint32_t)(((wl >> j1) & 1u) | (((wh >> j1) & 1u) << 1));
         uint32_t b2 = 0;
-        if (j2 != 0xFFu) b2 = ((wn >> j2) & 1u) ? 4u : (((wl >> j2) & 1u) | (((wh >> j2) & 1u) << 1));
+        if (j2 < 64u) b2 = ((wn >> j2) & 1u) ? 4u : (uint32_t)(((wl >> j2) & 1u) | (((wh >> j2) & 1u) << 1));
         base[q] = s_base + pair_entry(NP, (uint32_t)q, b1, b2) * 8u - (uint32_t)q * 128u;
     }
 }
@@ -312,62 +319,89 @@ __device__ __forceinline__ void table_blocks(const TableArgs& a, uint32_t (&base
 }
 
 // Table addresses (see pair_offsets) of the NP pair entries of one item, from its plane
-// windows taken at pos + pairs.p0 (every compared offset is >= p0 and < 32).
-template <int NP>
-__device__ __forceinline__ void window_bases(const PairLayout& pl, uint32_t s_base, uint32_t wl, uint32_t wh,
-                                             uint32_t wn, uint32_t (&base)[NP]) {
+// windows taken at pos + pairs.p0 (every compared offset is >= p0 and < p0 + 32, or
+// < p0 + 64 with W64 windows).
+template <int NP, bool W64>
+__device__ __forceinline__ void window_bases(const PairLayout& pl, uint32_t s_base, WinT<W64> wl, WinT<W64> wh,
+                                             WinT<W64> wn, uint32_t (&base)[NP]) {
+    using WT = WinT<W64>;
+    constexpr WT M33 = (WT)0x3333333333333333ull, MCC = (WT)0xCCCCCCCCCCCCCCCCull;
     if (pl.contig) {
         // fast path: with no N among the contiguous compared positions every pair index is
         // one nibble of Y (even pairs) or Z (odd pairs); s_base is 128-aligned, so the
         // entry offset ORs in (one SHF + one LOP3 per pair)
-        const uint32_t cm = pl.n_cmp >= 32 ? ~0u : ((1u << pl.n_cmp) - 1u);
+        const WT cm = pl.n_cmp >= 8 * sizeof(WT) ? ~(WT)0 : (((WT)1 << pl.n_cmp) - (WT)1);
         if ((wn & cm) == 0) {
-            const uint32_t Y = (wl & 0x33333333u) | ((wh & 0x33333333u) << 2);
-            const uint32_t Z = ((wl >> 2) & 0x33333333u) | (wh & 0xCCCCCCCCu);
+            const WT Y = (wl & M33) | ((wh & M33) << 2);
+            const WT Z = ((wl >> 2) & M33) | (wh & MCC);
 #pragma unroll
             for (int q = 0; q < NP; q++) {
-                const uint32_t src = (q & 1) ? Z : Y;
+                const WT src = (q & 1) ? Z : Y;
                 const int k = q >> 1;
-                const uint32_t nib8 = k == 0 ? (src << 3) & 0x78u : (src >> (4 * k - 3)) & 0x78u;
+                const uint32_t nib8 = (uint32_t)(k == 0 ? (src << 3) & 0x78u : (src >> (4 * k - 3)) & 0x78u);
                 base[q] = s_base | nib8;
             }
             return;
         }
     }
-    pair_offsets<NP>(pl, s_base, wl, wh, wn, base);
+    pair_offsets<NP, WT>(pl, s_base, wl, wh, wn, base);
 }
 
-template <int NP>
+// 64 consecutive bases from position p (bit j = base p+j): three plane words.
+__device__ __forceinline__ unsigned long long plane_window64(const uint32_t* __restrict__ plane, uint32_t p) {
+    const uint32_t w = p >> 5, sh = p & 31;
+    const uint32_t x = __ldg(plane + w), y = __ldg(plane + w + 1), z = __ldg(plane + w + 2);
+    return (unsigned long long)__funnelshift_r(x, y, sh) | ((unsigned long long)__funnelshift_r(y, z, sh) << 32);
+}
+
+template <bool W64>
+__device__ __forceinline__ WinT<W64> item_window(const uint32_t* __restrict__ plane, uint32_t p) {
+    if constexpr (W64) return plane_window64(plane, p);
+    else return plane_window(plane, p);
+}
+
+template <int NP, bool W64>
 __device__ __forceinline__ void item_bases(const TableArgs& a, uint32_t s_base, uint32_t pos, uint32_t (&base)[NP]) {
     const uint32_t p = pos + a.pairs.p0;
-    window_bases<NP>(a.pairs, s_base, plane_window(a.lo, p), plane_window(a.hi, p), plane_window(a.nm, p), base);
+    window_bases<NP, W64>(a.pairs, s_base, item_window<W64>(a.lo, p), item_window<W64>(a.hi, p),
+                          item_window<W64>(a.nm, p), base);
 }
 
-// Window prefetch of the table comparer: the 6 plane words (lo, hi, nm; two each) an item's
-// window needs are copied into this thread's shared-memory slots with cp.async one tile
-// ahead, so the dependent global loads of the next tile overlap this tile's table work.
-// Slot k of thread t lives at word k * CT + t (conflict-free).
+// Window prefetch of the table comparer: the plane words (lo, hi, nm; two each, three for
+// W64 windows) an item's window needs are copied into this thread's shared-memory slots
+// with cp.async one tile ahead, so the dependent global loads of the next tile overlap
+// this tile's table work.  Slot k of thread t lives at word k * CT + t (conflict-free).
+template <bool W64>
 __device__ __forceinline__ void prefetch_window(const TableArgs& a, uint32_t slot, uint32_t pos) {
+    constexpr uint32_t NWW = W64 ? 3 : 2;   // words per plane
     const uint32_t w = (pos + a.pairs.p0) >> 5;
-    cp_async4(slot + 0 * CT * 4, a.lo + w);
-    cp_async4(slot + 1 * CT * 4, a.lo + w + 1);
-    cp_async4(slot + 2 * CT * 4, a.hi + w);
-    cp_async4(slot + 3 * CT * 4, a.hi + w + 1);
-    cp_async4(slot + 4 * CT * 4, a.nm + w);
-    cp_async4(slot + 5 * CT * 4, a.nm + w + 1);
+#pragma unroll
+    for (uint32_t k = 0; k < NWW; k++) {
+        cp_async4(slot + (0 * NWW + k) * CT * 4, a.lo + w + k);
+        cp_async4(slot + (1 * NWW + k) * CT * 4, a.hi + w + k);
+        cp_async4(slot + (2 * NWW + k) * CT * 4, a.nm + w + k);
+    }
 }
 
-template <int NP>
+template <bool W64>
+__device__ __forceinline__ WinT<W64> slot_window(const uint32_t* slot, uint32_t sh) {
+    if constexpr (W64)
+        return (unsigned long long)__funnelshift_r(slot[0], slot[CT], sh) |
+               ((unsigned long long)__funnelshift_r(slot[CT], slot[2 * CT], sh) << 32);
+    else return __funnelshift_r(slot[0], slot[CT], sh);
+}
+
+template <int NP, bool W64>
 __device__ __forceinline__ void slot_bases(const TableArgs& a, uint32_t s_base, const uint32_t* slot, uint32_t sh,
                                            uint32_t (&base)[NP]) {
-    const uint32_t wl = __funnelshift_r(slot[0 * CT], slot[1 * CT], sh);
-    const uint32_t wh = __funnelshift_r(slot[2 * CT], slot[3 * CT], sh);
-    const uint32_t wn = __funnelshift_r(slot[4 * CT], slot[5 * CT], sh);
-    window_bases<NP>(a.pairs, s_base, wl, wh, wn, base);
+    constexpr uint32_t NWW = W64 ? 3 : 2;
+    window_bases<NP, W64>(a.pairs, s_base, slot_window<W64>(slot, sh), slot_window<W64>(slot + NWW * CT, sh),
+                          slot_window<W64>(slot + 2 * NWW * CT, sh), base);
 }
 
-template <int NP, int R, int TC>
-__global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constant__ TableArgs a) {
+template <int NP, int R, int TC, bool W64>
+__global__ void __launch_bounds__(CT, W64 ? 2 : 3) cof_comparer_table(const __grid_constant__ TableArgs a) {
+    constexpr uint32_t NSLOT = W64 ? 9 : 6;   // prefetched plane words per item
     extern __shared__ __align__(16) uint8_t s_raw[];
     // shared: [blocks_per_chunk][NP][25] uint2 pair table of the resident chunk of blocks
     // (at the first 128-byte boundary), then the window slots
@@ -399,7 +433,7 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constan
         for (int r = 0; r < R; r++) {
             const uint32_t idx = i0 + (uint32_t)r * CT;
             const uint32_t p = idx < n ? __ldg(a.items + idx) : 0u;
-            prefetch_window(a, slot_b + (uint32_t)(r * 6 * CT + threadIdx.x) * 4u, p);
+            prefetch_window<W64>(a, slot_b + (uint32_t)(r * NSLOT * CT + threadIdx.x) * 4u, p);
             shf[r] = (p + a.pairs.p0) & 31u;
             pos_next[r] = (idx + stride) < n ? __ldg(a.items + idx + stride) : 0u;
         }
@@ -415,12 +449,12 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_table(const __grid_constan
         for (int r = 0; r < R; r++) {
             const uint32_t idx = item0 + (uint32_t)r * CT;
             okm[r] = idx < n ? ~0u : 0u;
-            slot_bases<NP>(a, s_base, slot_p + r * 6 * CT + threadIdx.x, shf[r], base[r]);
+            slot_bases<NP, W64>(a, s_base, slot_p + r * NSLOT * CT + threadIdx.x, shf[r], base[r]);
         }
         // refill the slots for the next tile, then fetch the positions of the one after
 #pragma unroll
         for (int r = 0; r < R; r++) {
-            prefetch_window(a, slot_b + (uint32_t)(r * 6 * CT + threadIdx.x) * 4u, pos_next[r]);
+            prefetch_window<W64>(a, slot_b + (uint32_t)(r * NSLOT * CT + threadIdx.x) * 4u, pos_next[r]);
             shf[r] = (pos_next[r] + a.pairs.p0) & 31u;
             const uint32_t nidx = item0 + 2 * stride + (uint32_t)r * CT;
             pos_next[r] = nidx < n ? __ldg(a.items + nidx) : 0u;
@@ -464,8 +498,8 @@ constexpr uint32_t FWQ = 256;             // per-warp ring of queued positions (
 // Per-warp queues: each warp grabs its own word-pair ranges (dynamic ticket), expands its
 // strand's set bits into its ring (warp scan, ordered), and compares full batches of 32*R
 // positions; no CTA-wide barrier after the table load, so warps hide each other's latency.
-template <int NP, int R, int TC>
-__global__ void __launch_bounds__(CT, 3) cof_comparer_fused(const __grid_constant__ TableArgs a) {
+template <int NP, int R, int TC, bool W64>
+__global__ void __launch_bounds__(CT, W64 ? 2 : 3) cof_comparer_fused(const __grid_constant__ TableArgs a) {
     extern __shared__ __align__(16) uint8_t s_raw[];
     constexpr uint32_t BS = NP * 25 * 8;
     constexpr uint32_t BATCH = 32 * R;
@@ -492,7 +526,7 @@ __global__ void __launch_bounds__(CT, 3) cof_comparer_fused(const __grid_constan
         for (int r = 0; r < R; r++) {
             const uint32_t i = (uint32_t)r * 32 + lane;
             okm[r] = i < n_items ? ~0u : 0u;
-            item_bases<NP>(a, s_base, i < n_items ? q[i] : 0u, base[r]);
+            item_bases<NP, W64>(a, s_base, i < n_items ? q[i] : 0u, base[r]);
         }
         if (n_items < BATCH) table_blocks<NP, R, true, TC, 32>(a, base, a.n_blocks, 0, q + lane, okm);
         else table_blocks<NP, R, false, TC, 32>(a, base, a.n_blocks, 0, q + lane, okm);
@@ -590,17 +624,18 @@ static uint32_t table_smem_budget() {
 }
 static int table_r() { return R_TABLE; }
 
-template <int NP, int R, int TC>
+template <int NP, int R, int TC, bool W64>
 static cof_status launch_table_r(TableArgs& t, uint64_t n_hint, cudaStream_t stream) {
+    constexpr uint32_t NSLOT = W64 ? 9 : 6;
     // guide blocks resident in shared memory per pass (tiles over blocks if they do not fit)
     const uint32_t per_block = NP * 25 * 8;
     uint32_t bpc = t.n_blocks;
     const uint32_t budget = table_smem_budget();
     if (bpc * per_block > budget) bpc = std::max<uint32_t>(1, budget / per_block);
     t.blocks_per_chunk = bpc;
-    const uint32_t smem = 128u + ((bpc * per_block + 15u) & ~15u) + (uint32_t)CT * R * 6u * 4u;   // table + window slots
+    const uint32_t smem = 128u + ((bpc * per_block + 15u) & ~15u) + (uint32_t)CT * R * NSLOT * 4u;   // table + window slots
     int bps = 0;
-    auto fn = cof_comparer_table<NP, R, TC>;
+    auto fn = cof_comparer_table<NP, R, TC, W64>;
     cof_status st = occupancy((const void*)fn, smem, &bps);
     if (st != COF_OK) return st;
     uint64_t grid = (uint64_t)num_sms() * bps;
@@ -619,11 +654,11 @@ static cof_status launch_table_r(TableArgs& t, uint64_t n_hint, cudaStream_t str
 // Uniform-threshold specializations for the common guide shapes (20-nt SpCas9 guides:
 // 10 pairs; 23-nt Cas12a guides: 12 pairs) and t <= 7; everything else runs the generic
 // per-guide-threshold kernel.
-template <int NP, int R, int TC>
+template <int NP, int R, int TC, bool W64>
 static cof_status launch_fused_r(TableArgs& t, cudaStream_t stream) {
     const uint32_t smem = 128u + ((t.n_blocks * NP * 25 * 8 + 15u) & ~15u) + (CT / 32) * FWQ * 4;   // table + rings
     int bps = 0;
-    auto fn = cof_comparer_fused<NP, R, TC>;
+    auto fn = cof_comparer_fused<NP, R, TC, W64>;
     cof_status st = occupancy((const void*)fn, smem, &bps);
     if (st != COF_OK) return st;
     const uint64_t grabs = (t.n_wp + FGRAB - 1) / FGRAB;
@@ -637,9 +672,16 @@ static cof_status launch_fused_r(TableArgs& t, cudaStream_t stream) {
     return COF_OK;
 }
 
-template <int NP, int R, int TC>
+template <int NP, int R, int TC, bool W64 = false>
 static cof_status launch_any_r(TableArgs& t, bool fused, uint64_t n_hint, cudaStream_t stream) {
-    return fused ? launch_fused_r<NP, R, TC>(t, stream) : launch_table_r<NP, R, TC>(t, n_hint, stream);
+    return fused ? launch_fused_r<NP, R, TC, W64>(t, stream) : launch_table_r<NP, R, TC, W64>(t, n_hint, stream);
+}
+
+// Two-word windows (compared span > 32): generic thresholds, one item per thread (the NP
+// pair addresses and loaded entries of up to 32 pairs per item), NP a multiple of 4.
+template <int NP>
+static cof_status launch_table_wide(TableArgs& t, uint64_t n_hint, cudaStream_t stream, bool fused) {
+    return launch_any_r<NP, 1, -1, true>(t, fused, n_hint, stream);
 }
 
 template <int NP>
@@ -696,6 +738,21 @@ static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs
             for (uint32_t k = 0; k < T.n_blocks; k++)
                 for (int w = 0; w < 8; w++) T.meta[k][w] = pm[(size_t)(bb + k) * 8 + w];
             cof_status st;
+            if (T.pairs.wide) {
+                switch (np) {
+                    case 4: st = launch_table_wide<4>(T, T.n, stream, fused); break;
+                    case 8: st = launch_table_wide<8>(T, T.n, stream, fused); break;
+                    case 12: st = launch_table_wide<12>(T, T.n, stream, fused); break;
+                    case 16: st = launch_table_wide<16>(T, T.n, stream, fused); break;
+                    case 20: st = launch_table_wide<20>(T, T.n, stream, fused); break;
+                    case 24: st = launch_table_wide<24>(T, T.n, stream, fused); break;
+                    case 28: st = launch_table_wide<28>(T, T.n, stream, fused); break;
+                    case 32: st = launch_table_wide<32>(T, T.n, stream, fused); break;
+                    default: return set_error(COF_E_STATE, "cof_compare: %u pairs (wide)", np);
+                }
+                if (st != COF_OK) return st;
+                continue;
+            }
             switch (np) {
                 case 1: st = launch_table<1>(T, ut, T.n, stream, fused); break;
                 case 2: st = launch_table<2>(T, ut, T.n, stream, fused); break;
@@ -886,7 +943,7 @@ cof_status cof_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* de
     }
     if (tiles_hint != 0) {
         cof_status st;
-        if (comparer_impl() == 0) {
+        if (comparer_impl() == 0 && plan->L <= 32) {   // (v1 records are 32-bit windows)
             st = launch_popc(a, tiles_hint, stream);
         } else if (comparer_impl() == 2 && mma_supported(plan)) {
             st = run_mma(plan, pd, a.lo, a.hi, a.nm, items_fwd, n_fwd, items_rev, n_rev, a.items_cap, a.hits, a.cap,

@@ -24,8 +24,8 @@ struct DecorArgs {
     uint64_t n;                 // host count, or ON_DEVICE: min(*count, cap)
     const unsigned long long* count;
     uint64_t cap;
-    cof_hit* out;
-    const uint32_t* onehot;     // [2][n_guides][5]
+    void* out;                  // cof_hit[] (L <= 32) or cof_hit64[]
+    const unsigned long long* onehot;   // [2][n_guides][5] 64-bit window-offset masks
     const cof_segment* segs;    // device copy, n_segs entries (0: single segment)
     uint32_t n_segs;
     uint32_t n_guides;
@@ -35,8 +35,10 @@ struct DecorArgs {
     unsigned int* bad;          // set to 1 if a key is inconsistent with the chunk / plan
 };
 
+template <typename HIT>
 __device__ __forceinline__ void decorate_one(const DecorArgs& a, uint64_t i);
 
+template <typename HIT>
 __global__ void __launch_bounds__(256) cof_decorate_kernel(const __grid_constant__ DecorArgs a) {
     uint64_t n = a.n;
     if (a.count) {
@@ -44,10 +46,22 @@ __global__ void __launch_bounds__(256) cof_decorate_kernel(const __grid_constant
         if (n > a.cap) n = a.cap;
     }
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
-        decorate_one(a, i);
+        decorate_one<HIT>(a, i);
 }
 
+// 64 consecutive bases from position p (bit j = base p+j); the third word only when needed.
+__device__ __forceinline__ unsigned long long plane_window64(const uint32_t* __restrict__ plane, uint32_t p,
+                                                             bool wide) {
+    const uint32_t w = p >> 5, sh = p & 31;
+    const uint32_t a = __ldg(plane + w), b = __ldg(plane + w + 1);
+    const uint32_t c = wide ? __ldg(plane + w + 2) : 0u;
+    return (unsigned long long)__funnelshift_r(a, b, sh) | ((unsigned long long)__funnelshift_r(b, c, sh) << 32);
+}
+
+template <typename HIT>
 __device__ __forceinline__ void decorate_one(const DecorArgs& a, uint64_t i) {
+    constexpr int MAXL = (int)sizeof(((HIT*)nullptr)->site) - 2;   // 32 or 64
+    constexpr int NW = (int)sizeof(HIT) / 4;                          // record words
     const unsigned long long key = a.keys[i];
     const uint32_t pos = (uint32_t)(key >> 32);
     const uint32_t strand = (uint32_t)(key >> 31) & 1u;
@@ -56,12 +70,15 @@ __device__ __forceinline__ void decorate_one(const DecorArgs& a, uint64_t i) {
     const uint32_t L = a.L;
     bool ok = guide < a.n_guides;
     const uint32_t g = ok ? guide : 0u;
-    const uint32_t lo = plane_window(a.lo, pos), hi = plane_window(a.hi, pos), nm = plane_window(a.nm, pos);
-    const uint32_t* oh = a.onehot + ((size_t)strand * a.n_guides + g) * 5;
-    const uint32_t match = (~lo & ~hi & ~nm & __ldg(oh + 0)) | (lo & ~hi & ~nm & __ldg(oh + 1)) |
-                           (~lo & hi & ~nm & __ldg(oh + 2)) | (lo & hi & ~nm & __ldg(oh + 3));
-    const uint32_t mis = __ldg(oh + 4) & ~match;
-    ok = ok && (uint32_t)__popc(mis) == mm;
+    // (a one-word window suffices while the window ends inside the second word)
+    const bool wide = MAXL > 32 && (pos & 31u) + L > 32u;
+    const unsigned long long lo = plane_window64(a.lo, pos, wide), hi = plane_window64(a.hi, pos, wide),
+                             nm = plane_window64(a.nm, pos, wide);
+    const unsigned long long* oh = a.onehot + ((size_t)strand * a.n_guides + g) * 5;
+    const unsigned long long match = (~lo & ~hi & ~nm & __ldg(oh + 0)) | (lo & ~hi & ~nm & __ldg(oh + 1)) |
+                                     (~lo & hi & ~nm & __ldg(oh + 2)) | (lo & hi & ~nm & __ldg(oh + 3));
+    const unsigned long long mis = __ldg(oh + 4) & ~match;
+    ok = ok && (uint32_t)__popcll(mis) == mm;
     // chromosome and position
     uint32_t chrom = a.chrom;
     unsigned long long cpos = a.start + pos;
@@ -78,18 +95,18 @@ __device__ __forceinline__ void decorate_one(const DecorArgs& a, uint64_t i) {
         cpos = sg.chrom_off + (pos - sg.chunk_off);
     }
     if (!ok) atomicOr(a.bad, 1u);
-    // record: guide(4) chrom(4) pos(8) strand(1) mm(1) site(34) pad(4) = 56 bytes = 14 words
-    uint32_t w[14];
+    // record: guide(4) chrom(4) pos(8) strand(1) mm(1) site(34 | 66) pad(4 | 4) = 56 | 88 bytes
+    uint32_t w[NW];
     w[0] = guide;
     w[1] = chrom;
     w[2] = (uint32_t)cpos;
     w[3] = (uint32_t)(cpos >> 32);
     w[4] = (uint32_t)(strand ? '-' : '+') | (mm << 8);
 #pragma unroll
-    for (int k = 5; k < 14; k++) w[k] = 0;
+    for (int k = 5; k < NW; k++) w[k] = 0;
     // site bytes start at byte offset 18 (word 4, byte 2)
 #pragma unroll
-    for (int j = 0; j < 32; j++) {
+    for (int j = 0; j < MAXL; j++) {
         if ((uint32_t)j < L) {
             const uint32_t k = strand ? L - 1 - (uint32_t)j : (uint32_t)j;
             uint32_t c = (((lo >> k) & 1u) | (((hi >> k) & 1u) << 1));
@@ -102,9 +119,9 @@ __device__ __forceinline__ void decorate_one(const DecorArgs& a, uint64_t i) {
             w[byte >> 2] |= ch << (8 * (byte & 3));
         }
     }
-    uint2* dst = reinterpret_cast<uint2*>(a.out + i);
+    uint2* dst = reinterpret_cast<uint2*>(reinterpret_cast<HIT*>(a.out) + i);
 #pragma unroll
-    for (int k = 0; k < 7; k++) dst[k] = make_uint2(w[2 * k], w[2 * k + 1]);
+    for (int k = 0; k < NW / 2; k++) dst[k] = make_uint2(w[2 * k], w[2 * k + 1]);
 }
 
 }  // namespace cof
@@ -117,11 +134,17 @@ size_t cof_decorate_workspace_bytes(uint32_t n_segs) {
     return 256 + (size_t)n_segs * sizeof(cof_segment);
 }
 
-cof_status cof_decorate(const cof_plan* plan, const void* plan_dev, const cof_chunk* dev, const uint64_t* hits_dev,
-                        uint64_t n_hits, uint64_t cap, cof_hit* out_dev, void* workspace, cof_stream s) {
-    static_assert(sizeof(cof_hit) == 56, "cof_hit layout");
+}  // extern "C"
+
+template <typename HIT>
+static cof_status decorate_t(const char* fn, const cof_plan* plan, const void* plan_dev, const cof_chunk* dev,
+                             const uint64_t* hits_dev, uint64_t n_hits, uint64_t cap, HIT* out_dev, void* workspace,
+                             cof_stream s) {
+    static_assert(sizeof(cof_hit) == 56 && sizeof(cof_hit64) == 88, "cof_hit layout");
     if (!plan || !plan_dev || !dev || !workspace || ((!hits_dev || !out_dev) && n_hits))
-        return set_error(COF_E_ARG, "cof_decorate: NULL argument");
+        return set_error(COF_E_ARG, "%s: NULL argument", fn);
+    if (plan->L > sizeof out_dev->site - 2)   // cof_hit: L <= 32, cof_hit64: L <= 64
+        return set_error(COF_E_ARG, "%s: L = %u does not fit the record (use cof_decorate64)", fn, plan->L);
     if (dev->n_segs && !dev->segs) return set_error(COF_E_ARG, "cof_decorate: multi-segment chunk without segs");
     cudaStream_t stream = (cudaStream_t)s;
     unsigned int* bad = (unsigned int*)workspace;
@@ -140,7 +163,7 @@ cof_status cof_decorate(const cof_plan* plan, const void* plan_dev, const cof_ch
     a.count = on_dev ? (const unsigned long long*)((const uint8_t*)plan_dev + plan->lay.counters + 16) : nullptr;
     a.cap = cap;
     a.out = out_dev;
-    a.onehot = (const uint32_t*)((const uint8_t*)plan_dev + plan->lay.onehot);
+    a.onehot = (const unsigned long long*)((const uint8_t*)plan_dev + plan->lay.onehot);
     a.segs = dsegs;
     a.n_segs = dev->n_segs;
     a.n_guides = plan->n_guides;
@@ -150,11 +173,23 @@ cof_status cof_decorate(const cof_plan* plan, const void* plan_dev, const cof_ch
     a.bad = bad;
     uint64_t blocks = ((on_dev ? cap : n_hits) + 255) / 256;
     if (blocks > 148 * 16) blocks = 148 * 16;   // grid-stride beyond that
-    cof_decorate_kernel<<<(uint32_t)blocks, 256, 0, stream>>>(a);
+    cof_decorate_kernel<HIT><<<(uint32_t)blocks, 256, 0, stream>>>(a);
     e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "cof_decorate launch");
     count_launches(1);
     return COF_OK;
+}
+
+extern "C" {
+
+cof_status cof_decorate(const cof_plan* plan, const void* plan_dev, const cof_chunk* dev, const uint64_t* hits_dev,
+                        uint64_t n_hits, uint64_t cap, cof_hit* out_dev, void* workspace, cof_stream s) {
+    return decorate_t("cof_decorate", plan, plan_dev, dev, hits_dev, n_hits, cap, out_dev, workspace, s);
+}
+
+cof_status cof_decorate64(const cof_plan* plan, const void* plan_dev, const cof_chunk* dev, const uint64_t* hits_dev,
+                          uint64_t n_hits, uint64_t cap, cof_hit64* out_dev, void* workspace, cof_stream s) {
+    return decorate_t("cof_decorate64", plan, plan_dev, dev, hits_dev, n_hits, cap, out_dev, workspace, s);
 }
 
 cof_status cof_decorate_check(const void* workspace, cof_stream s) {

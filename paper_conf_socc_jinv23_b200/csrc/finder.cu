@@ -49,8 +49,8 @@ struct FinderArgs {
     unsigned long long* counters;  // plan_dev counters: [0] n_fwd, [1] n_rev
     uint32_t n_tiles;
     uint32_t ne;                 // non-N pattern letters per strand (same for both)
-    uint32_t pj[2][32];          // window offset of entry e
-    uint4 psel[2][32];           // entry e's IUPAC set as splat words {A, C, G, T} (0 / ~0)
+    uint32_t pj[2][COF_MAX_L];   // window offset of entry e
+    uint4 psel[2][COF_MAX_L];    // entry e's IUPAC set as splat words {A, C, G, T} (0 / ~0)
 };
 
 // Membership of each of 32 bases (bit-parallel) in the IUPAC set `set` (A=1 C=2 G=4 T=8):
@@ -63,19 +63,25 @@ __device__ __forceinline__ uint32_t member(uint32_t lo, uint32_t hi, uint32_t nm
 }
 
 // PAM masks of the 32 window starts of one plane word, both strands.  NE > 0: entry count
-// known at compile time (fully unrolled); NE < 0: generic loop.
-template <int NE>
-__device__ __forceinline__ void pam_masks(const FinderArgs& a, uint32_t valid, uint32_t lo0, uint32_t lo1,
-                                          uint32_t hi0, uint32_t hi1, uint32_t nm0, uint32_t nm1, uint32_t (&m)[2]) {
+// known at compile time (fully unrolled); NE < 0: generic loop.  WIDE: letters at window
+// offsets >= 32 (L > 32) select the plane word pair (w+1, w+2) instead of (w, w+1).
+template <int NE, bool WIDE>
+__device__ __forceinline__ void pam_masks(const FinderArgs& a, uint32_t valid, const uint32_t* lo,
+                                          const uint32_t* hi, const uint32_t* nm, uint32_t (&m)[2]) {
 #pragma unroll
     for (int st = 0; st < 2; st++) {
         uint32_t acc = valid;
         const uint32_t n = NE >= 0 ? (uint32_t)NE : a.ne;
 #pragma unroll
         for (uint32_t e = 0; e < (NE >= 0 ? (uint32_t)NE : n); e++) {
-            const uint32_t j = a.pj[st][e];
-            acc &= member(__funnelshift_r(lo0, lo1, j), __funnelshift_r(hi0, hi1, j), __funnelshift_r(nm0, nm1, j),
-                          a.psel[st][e]);
+            const uint32_t j = a.pj[st][e];   // funnel shifts use j & 31
+            if (WIDE && (j & 32u)) {
+                acc &= member(__funnelshift_r(lo[1], lo[2], j), __funnelshift_r(hi[1], hi[2], j),
+                              __funnelshift_r(nm[1], nm[2], j), a.psel[st][e]);
+            } else {
+                acc &= member(__funnelshift_r(lo[0], lo[1], j), __funnelshift_r(hi[0], hi[1], j),
+                              __funnelshift_r(nm[0], nm[1], j), a.psel[st][e]);
+            }
         }
         m[st] = acc;
     }
@@ -88,7 +94,7 @@ __device__ __forceinline__ void pam_masks(const FinderArgs& a, uint32_t valid, u
 //  offset) and pass 2 re-streams its range (mostly from L2) and writes the items in order.
 // One exchange per CTA replaces a decoupled look-back per tile, whose depth (all
 // concurrently running tiles) made it latency-bound.
-template <int NE, bool VS, bool MASKS_ONLY>
+template <int NE, bool VS, bool MASKS_ONLY, bool WIDE>
 __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ FinderArgs a) {
     extern __shared__ __align__(128) uint8_t smem[];
     uint32_t* stage = reinterpret_cast<uint32_t*>(smem);
@@ -132,9 +138,10 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
         const uint32_t* Shi = stage + (s * FPL + 1) * FLOAD + FWPT * tid;
         const uint32_t* Snm = stage + (s * FPL + 2) * FLOAD + FWPT * tid;
         const uint32_t* Svs = stage + (s * FPL + 3) * FLOAD + FWPT * tid;
-        uint32_t lo[FWPT + 1], hi[FWPT + 1], nm[FWPT + 1], vsw[FWPT];
+        constexpr int NWD = FWPT + (WIDE ? 2 : 1);   // plane words a thread's windows touch
+        uint32_t lo[FWPT + 2], hi[FWPT + 2], nm[FWPT + 2], vsw[FWPT];
 #pragma unroll
-        for (int w = 0; w <= FWPT; w++) { lo[w] = Slo[w]; hi[w] = Shi[w]; nm[w] = Snm[w]; }
+        for (int w = 0; w < NWD; w++) { lo[w] = Slo[w]; hi[w] = Shi[w]; nm[w] = Snm[w]; }
 #pragma unroll
         for (int w = 0; w < FWPT; w++) vsw[w] = VS ? Svs[w] : ~0u;
         __syncthreads();   // every thread has read stage s: refill it
@@ -150,7 +157,7 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
             uint32_t valid = vsw[w];
             if (pw + 32 > a.limit) valid &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
             uint32_t mw[2];
-            pam_masks<NE>(a, valid, lo[w], lo[w + 1], hi[w], hi[w + 1], nm[w], nm[w + 1], mw);
+            pam_masks<NE, WIDE>(a, valid, lo + w, hi + w, nm + w, mw);
             mk[2 * w] = mw[0];
             mk[2 * w + 1] = mw[1];
             cnt_f += (unsigned)__popc(mw[0]);
@@ -304,28 +311,29 @@ static int g_num_sms = -1;
 
 typedef void (*FinderFn)(FinderArgs);
 template <bool VS, bool MO>
-static FinderFn finder_fn_vs(uint32_t ne) {
+static FinderFn finder_fn_vs(uint32_t ne, bool wide) {
+    if (wide) return cof_finder_kernel<-1, VS, MO, true>;   // L > 32: generic letter loop
     switch (ne) {
-        case 0: return cof_finder_kernel<0, VS, MO>;
-        case 1: return cof_finder_kernel<1, VS, MO>;
-        case 2: return cof_finder_kernel<2, VS, MO>;
-        case 3: return cof_finder_kernel<3, VS, MO>;
-        case 4: return cof_finder_kernel<4, VS, MO>;
-        case 5: return cof_finder_kernel<5, VS, MO>;
-        case 6: return cof_finder_kernel<6, VS, MO>;
-        default: return cof_finder_kernel<-1, VS, MO>;
+        case 0: return cof_finder_kernel<0, VS, MO, false>;
+        case 1: return cof_finder_kernel<1, VS, MO, false>;
+        case 2: return cof_finder_kernel<2, VS, MO, false>;
+        case 3: return cof_finder_kernel<3, VS, MO, false>;
+        case 4: return cof_finder_kernel<4, VS, MO, false>;
+        case 5: return cof_finder_kernel<5, VS, MO, false>;
+        case 6: return cof_finder_kernel<6, VS, MO, false>;
+        default: return cof_finder_kernel<-1, VS, MO, false>;
     }
 }
-static FinderFn finder_fn(uint32_t ne, bool vs, bool masks_only = false) {
-    if (masks_only) return vs ? finder_fn_vs<true, true>(ne) : finder_fn_vs<false, true>(ne);
-    return vs ? finder_fn_vs<true, false>(ne) : finder_fn_vs<false, false>(ne);
+static FinderFn finder_fn(uint32_t ne, bool vs, bool masks_only = false, bool wide = false) {
+    if (masks_only) return vs ? finder_fn_vs<true, true>(ne, wide) : finder_fn_vs<false, true>(ne, wide);
+    return vs ? finder_fn_vs<true, false>(ne, wide) : finder_fn_vs<false, false>(ne, wide);
 }
 
 static cof_status finder_setup() {
     if (g_finder_blocks_per_sm > 0) return COF_OK;
     int bps_min = 1 << 30;
-    for (uint32_t k = 0; k < 32; k++) {
-        FinderFn fn = finder_fn(k & 7, (k >> 3) & 1, k >= 16);
+    for (uint32_t k = 0; k < 64; k++) {
+        FinderFn fn = finder_fn(k & 7, (k >> 3) & 1, (k >> 4) & 1, k >= 32);
         cudaError_t e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM);
         if (e != cudaSuccess) return cuda_error(e, "finder setup");
         int bps = 0;
@@ -434,6 +442,9 @@ cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* de
         a.counters = counters;
         a.n_tiles = n_tiles;
         a.ne = plan->pam[0].n;
+        bool wide = false;
+        for (int st = 0; st < 2; st++)
+            for (uint32_t k = 0; k < plan->pam[st].n; k++) wide |= plan->pam[st].j[k] >= 32;
         for (int st = 0; st < 2; st++)
             for (uint32_t k = 0; k < plan->pam[st].n; k++) {
                 const uint32_t set = plan->pam[st].set[k];
@@ -444,7 +455,7 @@ cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* de
         uint32_t grid = (uint32_t)g_num_sms * (uint32_t)g_finder_blocks_per_sm;
         if (grid > FMAX_CTAS) grid = FMAX_CTAS;
         if (grid > n_tiles) grid = n_tiles;
-        finder_fn(a.ne, a.vs != nullptr, masks_only)<<<grid, FT, FSMEM, stream>>>(a);
+        finder_fn(a.ne, a.vs != nullptr, masks_only, wide)<<<grid, FT, FSMEM, stream>>>(a);
         e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "cof_finder_kernel launch");
         count_launches(1);

@@ -306,11 +306,15 @@ cof_status cof_fasta_pack(const cof_fasta* fa, uint32_t i, uint64_t first, uint6
     return cof_pack(buf.data(), n, lo, hi, nm);
 }
 
+}  // extern "C"
+
 // ------------------------------------------------------------------ collect (M10) / merge
 // Decodes one hit key (see cof.h) into a record, building the site string from the host
 // planes: '+' reads the window, '-' reads its reverse complement (G6); a compared letter
 // is lower-cased where the genome base is not in the guide letter's IUPAC set (G19).
-static cof_status decorate(const cof_plan* plan, const cof_chunk* host, uint64_t key, cof_hit* h) {
+// HIT = cof_hit (L <= 32) or cof_hit64 (L <= 64); windows are 64-bit slices either way.
+template <typename HIT>
+static cof_status decorate(const cof_plan* plan, const cof_chunk* host, uint64_t key, HIT* h) {
     // char of a (code | N << 2 | mismatch << 3) index: ACGT/N, lower-cased when mismatched
     static const char CH[16] = {'A', 'C', 'G', 'T', 'N', 'N', 'N', 'N', 'a', 'c', 'g', 't', 'n', 'n', 'n', 'n'};
     const uint32_t L = plan->L;
@@ -318,21 +322,23 @@ static cof_status decorate(const cof_plan* plan, const cof_chunk* host, uint64_t
     const uint32_t strand = (uint32_t)(key >> 31) & 1u;
     const uint32_t guide = (uint32_t)(key >> 7) & 0xFFFFFFu;
     const uint32_t mm = (uint32_t)key & 127u;
-    if (guide >= plan->n_guides || pos + L > host->n_bases) return COF_E_STATE;
-    // the L-base window as 32-bit slices of the three planes (bit j = base pos + j)
+    if (guide >= plan->n_guides || pos + L > host->n_bases || L >= sizeof h->site) return COF_E_STATE;
+    // the L-base window as 64-bit slices of the three planes (bit j = base pos + j); the
+    // third word is read only when the window reaches into it
     const uint64_t w = pos >> 5;
     const uint32_t sh = (uint32_t)(pos & 31);
-    auto win = [&](const uint32_t* pl) -> uint32_t {
+    auto win = [&](const uint32_t* pl) -> uint64_t {
         const uint64_t v = ((uint64_t)pl[w + 1] << 32) | pl[w];
-        return (uint32_t)(v >> sh);
+        if (sh == 0 || sh + L <= 64) return v >> sh;
+        return (v >> sh) | ((uint64_t)pl[w + 2] << (64 - sh));
     };
-    const uint32_t lo = win(host->lo), hi = win(host->hi), nm = win(host->nm);
+    const uint64_t lo = win(host->lo), hi = win(host->hi), nm = win(host->nm);
     // mismatched window offsets against the guide in this strand's orientation (bit-parallel)
-    const uint32_t* oh = &plan->onehot[((size_t)strand * plan->n_guides + guide) * 5];
-    const uint32_t match = (~lo & ~hi & ~nm & oh[0]) | (lo & ~hi & ~nm & oh[1]) | (~lo & hi & ~nm & oh[2]) |
+    const uint64_t* oh = &plan->onehot[((size_t)strand * plan->n_guides + guide) * 5];
+    const uint64_t match = (~lo & ~hi & ~nm & oh[0]) | (lo & ~hi & ~nm & oh[1]) | (~lo & hi & ~nm & oh[2]) |
                            (lo & hi & ~nm & oh[3]);
-    const uint32_t mis = oh[4] & ~match;
-    if ((uint32_t)__builtin_popcount(mis) != mm) return COF_E_STATE;
+    const uint64_t mis = oh[4] & ~match;
+    if ((uint32_t)__builtin_popcountll(mis) != mm) return COF_E_STATE;
     // site read along the strand (G6): '+' = window offset j, '-' = complement of offset L-1-j
     if (strand == 0) {
         for (uint32_t j = 0; j < L; j++)
@@ -369,18 +375,21 @@ static cof_status decorate(const cof_plan* plan, const cof_chunk* host, uint64_t
 
 static inline uint64_t sort_key(uint64_t k) { return k >> 7; }   // (pos, strand, guide)
 
-cof_status cof_collect(const cof_plan* plan, const cof_chunk* host, const uint64_t* hits_dev,
-                       const uint64_t* host_keys, uint64_t n_hits, cof_hit* out, cof_stream s) {
+template <typename HIT>
+static cof_status collect_t(const char* fn, const cof_plan* plan, const cof_chunk* host, const uint64_t* hits_dev,
+                            const uint64_t* host_keys, uint64_t n_hits, HIT* out, cof_stream s) {
     if (!plan || !host || (!out && n_hits) || (!hits_dev && !host_keys && n_hits))
-        return set_error(COF_E_ARG, "cof_collect: NULL argument");
-    if (!host->lo || !host->hi || !host->nm) return set_error(COF_E_ARG, "cof_collect: host planes are NULL");
+        return set_error(COF_E_ARG, "%s: NULL argument", fn);
+    if (!host->lo || !host->hi || !host->nm) return set_error(COF_E_ARG, "%s: host planes are NULL", fn);
+    if (plan->L > sizeof out->site - 2)   // cof_hit: L <= 32, cof_hit64: L <= 64
+        return set_error(COF_E_ARG, "%s: L = %u does not fit the record (use cof_collect64)", fn, plan->L);
     if (n_hits == 0) return COF_OK;
     std::vector<uint64_t> keys(n_hits);
     if (hits_dev) {
         cudaStream_t st = (cudaStream_t)s;
         cudaError_t e = cudaMemcpyAsync(keys.data(), hits_dev, n_hits * 8, cudaMemcpyDeviceToHost, st);
         if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-        if (e != cudaSuccess) return cuda_error(e, "cof_collect");
+        if (e != cudaSuccess) return cuda_error(e, fn);
     } else {
         memcpy(keys.data(), host_keys, n_hits * 8);
     }
@@ -391,18 +400,20 @@ cof_status cof_collect(const cof_plan* plan, const cof_chunk* host, const uint64
 #pragma omp parallel for schedule(static) reduction(| : bad) if (n_hits > 4096)
     for (int64_t i = 0; i < (int64_t)n_hits; i++)
         if (decorate(plan, host, keys[i], &out[i]) != COF_OK) bad = 1;
-    if (bad) return set_error(COF_E_STATE, "cof_collect: a hit key does not match the plan/chunk (mismatch recount differs)");
+    if (bad) return set_error(COF_E_STATE, "%s: a hit key does not match the plan/chunk (mismatch recount differs)", fn);
     return COF_OK;
 }
 
-static inline bool hit_less(const cof_hit& a, const cof_hit& b) {
+template <typename HIT>
+static inline bool hit_less(const HIT& a, const HIT& b) {
     if (a.chrom != b.chrom) return a.chrom < b.chrom;
     if (a.pos != b.pos) return a.pos < b.pos;
     if (a.strand != b.strand) return a.strand == '+';
     return a.guide < b.guide;
 }
 
-cof_status cof_merge(const cof_hit* const* lists, const uint64_t* lens, uint32_t n_lists, cof_hit* out) {
+template <typename HIT>
+static cof_status merge_t(const HIT* const* lists, const uint64_t* lens, uint32_t n_lists, HIT* out) {
     if ((!lists || !lens) && n_lists) return set_error(COF_E_ARG, "cof_merge: NULL argument");
     uint64_t total = 0;
     for (uint32_t i = 0; i < n_lists; i++) {
@@ -415,7 +426,7 @@ cof_status cof_merge(const cof_hit* const* lists, const uint64_t* lens, uint32_t
     // fast path: non-empty lists already in global order (disjoint chunks in genome order)
     {
         bool ordered = true;
-        const cof_hit* prev = nullptr;
+        const HIT* prev = nullptr;
         for (uint32_t i = 0; i < n_lists && ordered; i++) {
             if (!lens[i]) continue;
             if (prev && !hit_less(*prev, lists[i][0])) ordered = false;
@@ -433,7 +444,7 @@ cof_status cof_merge(const cof_hit* const* lists, const uint64_t* lens, uint32_t
                 const uint32_t i = tasks[t].first;
                 const uint64_t k = tasks[t].second;
                 const uint64_t n = std::min<uint64_t>(CH, lens[i] - k);
-                memcpy(out + at[i] + k, lists[i] + k, n * sizeof(cof_hit));
+                memcpy(out + at[i] + k, lists[i] + k, n * sizeof(HIT));
             }
             return COF_OK;
         }
@@ -441,8 +452,8 @@ cof_status cof_merge(const cof_hit* const* lists, const uint64_t* lens, uint32_t
     // k-way merge with a min-heap of list heads (stable across lists for equal keys)
     typedef std::pair<uint32_t, uint64_t> Head;   // (list, index)
     auto cmp = [&](const Head& x, const Head& y) {
-        const cof_hit& a = lists[x.first][x.second];
-        const cof_hit& b = lists[y.first][y.second];
+        const HIT& a = lists[x.first][x.second];
+        const HIT& b = lists[y.first][y.second];
         if (hit_less(a, b)) return false;
         if (hit_less(b, a)) return true;
         return x.first > y.first;
@@ -457,6 +468,27 @@ cof_status cof_merge(const cof_hit* const* lists, const uint64_t* lens, uint32_t
         if (h.second + 1 < lens[h.first]) heap.push({h.first, h.second + 1});
     }
     return COF_OK;
+}
+
+
+extern "C" {
+
+cof_status cof_collect(const cof_plan* plan, const cof_chunk* host, const uint64_t* hits_dev,
+                       const uint64_t* host_keys, uint64_t n_hits, cof_hit* out, cof_stream s) {
+    return collect_t("cof_collect", plan, host, hits_dev, host_keys, n_hits, out, s);
+}
+
+cof_status cof_collect64(const cof_plan* plan, const cof_chunk* host, const uint64_t* hits_dev,
+                         const uint64_t* host_keys, uint64_t n_hits, cof_hit64* out, cof_stream s) {
+    return collect_t("cof_collect64", plan, host, hits_dev, host_keys, n_hits, out, s);
+}
+
+cof_status cof_merge(const cof_hit* const* lists, const uint64_t* lens, uint32_t n_lists, cof_hit* out) {
+    return merge_t(lists, lens, n_lists, out);
+}
+
+cof_status cof_merge64(const cof_hit64* const* lists, const uint64_t* lens, uint32_t n_lists, cof_hit64* out) {
+    return merge_t(lists, lens, n_lists, out);
 }
 
 }  // extern "C"

@@ -41,13 +41,13 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     *out = nullptr;
     if (!pattern || !guides || !max_mm) return set_error(COF_E_ARG, "cof_plan_create: NULL argument");
     size_t L = strlen(pattern);
-    if (L < 1 || L > 32) return set_error(COF_E_ARG, "pattern length %zu not in [1, 32]", L);
+    if (L < 1 || L > COF_MAX_L) return set_error(COF_E_ARG, "pattern length %zu not in [1, %d]", L, COF_MAX_L);
     if (n_guides == 0 || n_guides > (1u << 24))
         return set_error(COF_E_ARG, "n_guides %u not in [1, 2^24]", n_guides);
     cof_plan* p = new cof_plan();
     p->L = (uint32_t)L;
     p->n_guides = n_guides;
-    uint8_t pm[32];
+    uint8_t pm[COF_MAX_L];
     for (size_t j = 0; j < L; j++) {
         pm[j] = iupac_mask(pattern[j]);
         if (!pm[j]) { delete p; return set_error(COF_E_ARG, "pattern[%zu]='%c' is not an IUPAC code", j, pattern[j]); }
@@ -68,6 +68,11 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
             p->gmask[(size_t)i * L + j] = m;
             g.push_back((char)(guides[i][j] >= 'a' ? guides[i][j] - 32 : guides[i][j]));
         }
+        // the table comparer's 6-bit sums hold counts <= 63 (a 64-letter guide has no PAM)
+        if (std::count(g.begin(), g.end(), 'N') == 0 && L == 64) {
+            delete p;
+            return set_error(COF_E_ARG, "guide %u compares all 64 positions (at most 63 supported)", i);
+        }
         p->guides.push_back(g);
     }
 
@@ -87,20 +92,21 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     };
 
     // ---- host decoration: one-hot membership masks per guide and strand (window offsets)
-    p->onehot.assign((size_t)2 * n_guides * 5, 0u);
+    p->onehot.assign((size_t)2 * n_guides * 5, 0ull);
     for (int s = 0; s < 2; s++)
         for (uint32_t i = 0; i < n_guides; i++) {
-            uint32_t* oh = &p->onehot[((size_t)s * n_guides + i) * 5];
+            uint64_t* oh = &p->onehot[((size_t)s * n_guides + i) * 5];
             for (uint32_t j = 0; j < L; j++) {
                 const uint8_t m = gm(s, i, j);
-                for (int b = 0; b < 4; b++) oh[b] |= (uint32_t)((m >> b) & 1u) << j;
-                if (m != 15) oh[4] |= 1u << j;
+                for (int b = 0; b < 4; b++) oh[b] |= (uint64_t)((m >> b) & 1u) << j;
+                if (m != 15) oh[4] |= 1ull << j;
             }
         }
 
     // ---- v1 comparer: group guides by (care mask, kind); records per strand
+    // (32-bit care masks: built for L <= 32 only; longer patterns run the table comparer)
     std::map<std::pair<uint32_t, uint32_t>, std::vector<uint32_t>> groups;  // (care_fwd, kind) -> guides
-    for (uint32_t i = 0; i < n_guides; i++) {
+    for (uint32_t i = 0; i < n_guides && L <= 32; i++) {
         uint32_t care = 0, kind = GROUP_CONCRETE;
         for (uint32_t j = 0; j < L; j++) {
             uint8_t m = gm(0, i, j);
@@ -148,9 +154,9 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     // ---- v2 comparer: bit-sliced pair tables over the union of compared positions
     p->n_blocks = (n_guides + 31) / 32;
     for (int s = 0; s < 2; s++) {
-        uint32_t uc = 0;
+        uint64_t uc = 0;
         for (uint32_t i = 0; i < n_guides; i++)
-            for (uint32_t j = 0; j < L; j++) if (gm(s, i, j) != 15) uc |= 1u << j;
+            for (uint32_t j = 0; j < L; j++) if (gm(s, i, j) != 15) uc |= 1ull << j;
         p->union_care[s] = uc;
         PairLayout& pl = p->pairs[s];
         pl.n_pairs = 0;
@@ -165,10 +171,18 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
         if (pl.n_pairs == 0) {   // all guides all-N: one dummy pair that never counts
             pl.j1[0] = 0; pl.j2[0] = 0xFF; pl.n_pairs = 1;
         }
-        pl.n_cmp = (uint32_t)__builtin_popcount(uc);
-        pl.p0 = uc ? (uint32_t)__builtin_ctz(uc) : 0u;
-        pl.contig = uc != 0 && (uc >> pl.p0) == (pl.n_cmp >= 32 ? 0xFFFFFFFFu : ((1u << pl.n_cmp) - 1u)) &&
-                    pl.p0 + 2 * pl.n_pairs <= 32;
+        pl.n_real = pl.n_pairs;
+        pl.n_cmp = (uint32_t)__builtin_popcountll(uc);
+        pl.p0 = uc ? (uint32_t)__builtin_ctzll(uc) : 0u;
+        const uint32_t span = uc ? 64u - (uint32_t)__builtin_clzll(uc) - pl.p0 : 1u;
+        // two-word windows when the compared span exceeds one 32-bit word;
+        // the wide kernels exist for multiples of 4 pairs: pad with pairs whose table
+        // entries are all zero (they add nothing to any count)
+        pl.wide = span > 32 ? 1u : 0u;
+        if (pl.wide)
+            while (pl.n_pairs % 4) { pl.j1[pl.n_pairs] = (uint8_t)pl.p0; pl.j2[pl.n_pairs] = 0xFE; pl.n_pairs++; }
+        pl.contig = uc != 0 && (uc >> pl.p0) == (pl.n_cmp >= 64 ? ~0ull : ((1ull << pl.n_cmp) - 1ull)) &&
+                    (pl.wide ? 2 * pl.n_pairs <= 64 : pl.p0 + 2 * pl.n_pairs <= 32);
     }
     // (both strands have the same number of compared positions, hence of pairs)
     const uint32_t NPAIR = p->pairs[0].n_pairs;
@@ -176,8 +190,8 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
 
     // ---- tensor-core comparer: span, N-classes, guide batches (see MmaPlan)
     MmaPlan& mp = p->mma;
-    {
-        const uint32_t uc = p->union_care[0];
+    if (L <= 32) {   // the tensor-core comparer's span is one 32-bit word
+        const uint32_t uc = (uint32_t)p->union_care[0];
         mp.j0 = uc ? (uint32_t)__builtin_ctz(uc) : 0u;
         mp.npos = uc ? 32u - (uint32_t)__builtin_clz(uc) - mp.j0 : 1u;
         mp.pw = (mp.npos + 3) / 4;
@@ -231,7 +245,7 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     size_t pmeta_bytes = (size_t)p->n_blocks * 8 * 4;
     lay.pmeta_fwd = off; off = align256(off + pmeta_bytes);
     lay.pmeta_rev = off; off = align256(off + pmeta_bytes);
-    lay.onehot = off; off = align256(off + p->onehot.size() * 4);
+    lay.onehot = off; off = align256(off + p->onehot.size() * 8);
     size_t mma_b_bytes = 0;
     for (const MmaBatch& b : mp.batches) mma_b_bytes += (size_t)b.nt * b.tn * mp.kpad;
     lay.mma_b = off; off = align256(off + mma_b_bytes);
@@ -239,7 +253,7 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     lay.total = off;
     p->image.assign(lay.total, 0);
     uint8_t* img = p->image.data();
-    memcpy(img + lay.onehot, p->onehot.data(), p->onehot.size() * 4);
+    memcpy(img + lay.onehot, p->onehot.data(), p->onehot.size() * 8);
     memcpy(img + lay.groups_fwd, gd[0].data(), gd[0].size() * sizeof(GroupDesc));
     memcpy(img + lay.groups_rev, gd[1].data(), gd[1].size() * sizeof(GroupDesc));
     memcpy(img + lay.recs_fwd, recs[0].data(), recs[0].size() * 4);
@@ -272,6 +286,7 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
                             if (base == 4) return 1;                // genome N: always a mismatch (G2)
                             return (m >> base & 1) ? 0 : 1;
                         };
+                        if (q >= pl.n_real) break;             // padding pair: all zero
                         uint32_t cnt = mis(pl.j1[q], b1);
                         if (pl.j2[q] != 0xFF) cnt += mis(pl.j2[q], b2);
                         if (pl.j2[q] == 0xFF && p->union_care[s] == 0) cnt = 0;

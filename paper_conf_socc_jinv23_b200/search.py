@@ -129,11 +129,13 @@ def pack_shard(chunks):
     return Chunk(tuple(p for ch in chunks for p in ch.pieces))
 
 
-def merge_hit_lists(lists):
-    """Order (chrom, pos, strand, guide) across chunk / rank lists (cof_merge)."""
+def merge_hit_lists(lists, dtype=None):
+    """Order (chrom, pos, strand, guide) across chunk / rank lists (cof_merge / cof_merge64)."""
+    if dtype is None:
+        dtype = next((x.dtype for x in lists if hasattr(x, "dtype")), cof.HIT_DTYPE)
     lists = [x for x in lists if len(x)]
     if not lists:
-        return np.zeros(0, dtype=cof.HIT_DTYPE)
+        return np.zeros(0, dtype=dtype)
     return cof.cof_merge(lists)
 
 
@@ -196,6 +198,7 @@ class Searcher:
     def __init__(self, pattern, guides, thresholds, device="cuda", stream=None):
         self.device = torch.device(device)
         self.plan = cof.cof_plan_create(pattern, guides, thresholds)
+        self.hit_dtype = cof.hit_dtype(self.plan.L)   # cof_hit (L <= 32) or cof_hit64
         self.L = self.plan.L
         self.stream = stream or torch.cuda.current_stream(self.device)
         nbytes = cof.cof_plan_device_bytes(self.plan)
@@ -271,7 +274,7 @@ class Searcher:
         compare, device sort, device decoration (cof_decorate) and an async D2H of the
         finished records; nothing waits on the host except the item/hit counts.
 
-        Returns the sorted hit array.  If ``out`` (a ``cof.HIT_DTYPE`` array, ideally in
+        Returns the sorted hit array.  If ``out`` (a ``Searcher.hit_dtype`` array, ideally in
         pinned memory) is large enough, each chunk's records land straight in its slice of
         ``out`` (chunks are disjoint and in genome order, so no merge copy is needed) and a
         view of ``out`` is returned; otherwise per-chunk arrays are merged with cof_merge.
@@ -336,12 +339,12 @@ class Searcher:
                     else:
                         overflow = True
                 if dst is None:
-                    dst = torch.empty(max(nh, 1) * cof.HIT_DTYPE.itemsize, dtype=torch.uint8,
-                                      pin_memory=True).numpy().view(cof.HIT_DTYPE)[:nh]
+                    dst = torch.empty(max(nh, 1) * self.hit_dtype.itemsize, dtype=torch.uint8,
+                                      pin_memory=True).numpy().view(self.hit_dtype)[:nh]
                 if nh:   # D2H on its own stream: overlaps the next chunk's kernels (and H2D)
                     self.d2h_stream.wait_event(fr)
                     with torch.cuda.stream(self.d2h_stream):
-                        torch.from_numpy(dst.view(np.uint8)).copy_(recs[: nh * cof.HIT_DTYPE.itemsize],
+                        torch.from_numpy(dst.view(np.uint8)).copy_(recs[: nh * self.hit_dtype.itemsize],
                                                                    non_blocking=True)
                         ev = torch.cuda.Event()
                         ev.record(self.d2h_stream)
@@ -354,13 +357,13 @@ class Searcher:
                 cof.cof_decorate_check(ws[j], self.stream)
         if use_out and not overflow:
             return out[:total]
-        return merge_hit_lists(results)
+        return merge_hit_lists(results, self.hit_dtype)
 
     def _reserve_records(self, n):
         # two device record buffers: chunk j decorates into one while chunk j-1's D2H drains the other
         self.d2h_stream.synchronize() if hasattr(self, "d2h_stream") else None
         cap = int(n * 1.25 + 1024)
-        self.d_records = [torch.empty(cap * cof.HIT_DTYPE.itemsize, dtype=torch.uint8, device=self.device)
+        self.d_records = [torch.empty(cap * self.hit_dtype.itemsize, dtype=torch.uint8, device=self.device)
                           for _ in range(2)]
         self._rec_cap = cap
 
@@ -427,7 +430,7 @@ class Searcher:
             raise errors[0]
         if use_out and not overflow:
             return out[:total]
-        return merge_hit_lists([results[i] for i in idx])
+        return merge_hit_lists([results[i] for i in idx], self.hit_dtype)
 
 def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda", pack_bases=None, fused=None):
     """Convenience: whole search of ``seqs`` (list of uint8 ASCII arrays / bytes) on one GPU.
@@ -460,5 +463,5 @@ def gather_and_merge(local_hits: np.ndarray, group=None, dst: int = 0):
     dist.gather_object(local_hits.tobytes(), buf, dst=dst, group=group)
     if rank != dst:
         return None
-    lists = [np.frombuffer(b, dtype=cof.HIT_DTYPE) for b in buf]
-    return merge_hit_lists(lists)
+    lists = [np.frombuffer(b, dtype=local_hits.dtype) for b in buf]
+    return merge_hit_lists(lists, local_hits.dtype)

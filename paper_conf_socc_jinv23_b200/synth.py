@@ -125,10 +125,25 @@ def config(name: str, scale: float = 1.0) -> Config:
         return Config("C5", hg38, 303, 505, nrg, 1000, 20, "", "NNN",
                       ("AGG", "CAG", "GGG", "TAG"), 6,
                       "synthetic hg38-shaped genome, 1000 guides, <=6 mismatches, chromosome-sharded across 1/2/4/8 B200")
+    # Long-window parity cases (not BASELINE configs): patterns with
+    # 32 < L <= 64 on a chr22-shaped genome.
+    if name == "X1":   # 37-nt spacers + NGG: compared span 37 > 32 (two-word comparer windows)
+        g = GenomeSpec(_scaled([("chr22", 50_818_468)], scale), "chr22",
+                       rare_per_bp=1e-8 if scale == 1.0 else 2e-6)
+        return Config("X1", g, 202, 606, "N" * 38 + "GG", 20, 37, "", "NNN",
+                      ("AGG", "CGG", "GGG", "TGG"), 8,
+                      "synthetic chr22-sized genome, 37-nt guides + NGG (L = 40), 20 guides, <=8 mismatches")
+    if name == "X2":   # CjCas9-like 8-letter PAM after 30-nt spacers: L = 38, PAM offsets >= 32
+        g = GenomeSpec(_scaled([("chr22", 50_818_468)], scale), "chr22",
+                       rare_per_bp=1e-8 if scale == 1.0 else 2e-6)
+        return Config("X2", g, 202, 707, "N" * 34 + "RYAC", 20, 30, "", "NNNNNNNN",
+                      ("AGCTGCAC", "TTAAATAC", "CCGGACAC", "GATCGTAC"), 6,
+                      "synthetic chr22-sized genome, 30-nt guides + NNNNRYAC (L = 38), 20 guides, <=6 mismatches")
     raise KeyError(name)
 
 
 CONFIG_NAMES = ("C1", "C2", "C3", "C4", "C5")
+EXTRA_CONFIG_NAMES = ("X1", "X2")
 
 
 # --------------------------------------------------------------------------- genome

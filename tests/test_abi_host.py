@@ -72,7 +72,8 @@ def test_plan_validation():
         (good, ["ACGT" * 5 + "NN"], [3]),          # length mismatch (G11)
         ("N" * 21 + "RU", ["A" * 23], [3]),        # non-IUPAC pattern letter (G18)
         (good, ["ACGT" * 5 + "NNX"], [3]),         # non-IUPAC guide letter
-        ("N" * 33, ["N" * 33], [1]),               # L > 32
+        ("N" * 65, ["N" * 65], [1]),               # L > COF_MAX_L (64)
+        ("N" * 64, ["A" * 64], [1]),               # 64 compared letters (6-bit counts)
         ("", [""], [0]),                           # L = 0
         (good, [], []),                            # no guides
     ]
@@ -80,6 +81,9 @@ def test_plan_validation():
         with pytest.raises(cof.CofError) as ei:
             cof.cof_plan_create(pat, g, t)
         assert ei.value.status == cof.COF_E_ARG
+    # two-word windows: 32 < L <= 64
+    assert cof.cof_plan_create("N" * 60 + "NRG", ["A" * 62 + "N"], [5]).L == 63
+    assert cof.cof_plan_create("N" * 64, ["N" + "C" * 63], [5]).L == 64
     # lower case accepted (G4 / G18)
     assert cof.cof_plan_create(good.lower(), [("acgt" * 5) + "nnn"], [2]).L == 23
 
@@ -115,6 +119,39 @@ def test_collect_decorates_like_the_oracle():
     with pytest.raises(cof.CofError) as ei:
         cof.cof_collect(plan, host, None, len(badk), host_keys=badk)
     assert ei.value.status == cof.COF_E_STATE
+
+
+@pytest.mark.parametrize("L", [33, 41, 64])
+def test_collect64_decorates_like_the_oracle(L):
+    """cof_collect64 (L > 32: 64-bit windows, cof_hit64 records) against the oracle, incl.
+    windows whose start sits late in a plane word (three-word slices)."""
+    rng = np.random.default_rng(30 + L)
+    seq = synth.random_genome_text(rng, 30000, b"ACGTacgtN", p=[.22, .22, .22, .22, .02, .02, .02, .02, .04])
+    pat = "N" * (L - 3) + "NRG"
+    core = L - 4
+    guides = ["N" + "".join(rng.choice(list("ACGT"), core)) + "NNN" for _ in range(3)]
+    guides.append("N" + "RYNNKMSWAC" + "".join(rng.choice(list("ACGT"), core - 10)) + "NNN")
+    thr = [int(core * 0.6)] * 4
+    ref = oracle.search([seq], pat, guides, thr)
+    assert len(ref) > 20
+    plan = cof.cof_plan_create(pat, guides, thr)
+    w = cof.cof_plane_words(len(seq))
+    planes = np.zeros((3, w), np.uint32)
+    cof.cof_pack(seq, len(seq), planes[0], planes[1], planes[2])
+    host = cof.make_chunk(0, 0, len(seq), len(seq) - L + 1, planes[0], planes[1], planes[2])
+    keys = _keys_from_oracle(ref)
+    got = cof.cof_collect(plan, host, None, len(keys), host_keys=keys[rng.permutation(len(keys))])
+    assert got.dtype == cof.HIT64_DTYPE
+    assert cof.hits_to_tuples(got) == oracle.hits_to_tuples(ref)
+    # the 56-byte record cannot hold the site: cof_collect itself refuses
+    with pytest.raises(cof.CofError) as ei:
+        out = np.zeros(len(keys), dtype=cof.HIT_DTYPE)
+        cof._check(cof.lib.cof_collect(plan.handle, ctypes.addressof(host), None, keys.ctypes.data, len(keys),
+                                       out.ctypes.data, None))
+    assert ei.value.status == cof.COF_E_ARG
+    # cof_merge64 of the record halves gives the whole list back
+    m = cof.cof_merge([got[len(got) // 2:], got[:len(got) // 2]])
+    assert cof.hits_to_tuples(m) == cof.hits_to_tuples(got)
 
 
 def test_merge_orders_lists():

@@ -100,6 +100,54 @@ def test_configs_scaled_mma(name, scale, chunk, pack):
                     impl="mma") == exp
 
 
+@pytest.mark.parametrize("seed", range(6))
+def test_random_long(seed):
+    """32 < L <= 64: random long IUPAC patterns (PAM letters at window
+    offsets >= 32: the finder's three-word slices), guides whose compared span is either
+    <= 32 or up to 63 (two-word comparer windows, padded pair tables), degenerate letters,
+    genome N / lowercase; fused and two-call paths, one chunk and packed pieces; the popc
+    and mma selections fall back to the table comparer."""
+    rng = np.random.default_rng(900 + seed)
+    L = int(rng.integers(33, 65))
+    pat = "".join(rng.choice(list("N" * 24 + "ACGTRYSWKMBDHV"), L))
+    span = int(rng.integers(8, 33)) if seed % 2 else int(rng.integers(33, min(L, 63) + 1))
+    off = int(rng.integers(0, L - span + 1))
+    guides = []
+    for _ in range(int(rng.integers(1, 70))):
+        g = ["N"] * L
+        for j in range(off, off + span):
+            g[j] = str(rng.choice(list("ACGTACGTACGTNRYKMSWBDHV")))
+        g[off] = str(rng.choice(list("ACGT")))
+        g[off + span - 1] = str(rng.choice(list("ACGT")))
+        guides.append("".join(g))
+    thr = [int(rng.integers(span // 4, span // 2 + 2)) for _ in guides]
+    lens = [int(rng.integers(0, 3)) if i == 0 else int(rng.integers(L, 40_000)) for i in range(4)]
+    seqs = [synth.random_genome_text(rng, n, b"ACGTacgtNnRy",
+                                     p=[.22, .15, .15, .22, .05, .05, .05, .05, .04, .01, .005, .005]) for n in lens]
+    exp = ref_hits(seqs, pat, guides, thr)
+    assert gpu_hits(seqs, pat, guides, thr) == exp
+    assert gpu_hits(seqs, pat, guides, thr, pack_bases=0) == exp
+    assert gpu_hits(seqs, pat, guides, thr, chunk_bases=9973, pack_bases=30_000) == exp
+    assert gpu_hits(seqs, pat, guides, thr, fused=False) == exp
+    assert gpu_hits(seqs, pat, guides, thr, fused=True, pack_bases=0) == exp
+    assert gpu_hits(seqs, pat, guides, thr, impl="popc") == exp
+    assert gpu_hits(seqs, pat, guides, thr, impl="mma", fused=False) == exp
+
+
+@pytest.mark.parametrize("name,scale,n_guides", [("X1", 0.05, None), ("X2", 0.05, None), ("X1", 0.01, 300)])
+def test_long_configs(name, scale, n_guides):
+    """Long-window configs X1 (37-nt spacers + NGG, L = 40) and X2 (30-nt + NNNNRYAC,
+    L = 38) with planted sites, through the device decoration (cof_decorate64)."""
+    w = synth.make_workload(name, scale=scale, n_guides=n_guides)
+    cfg = w.cfg
+    exp = ref_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
+    assert len(exp) >= cfg.threshold + 1
+    for fused in (False, True):
+        assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, fused=fused) == exp
+        assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, fused=fused, pack_bases=0,
+                        chunk_bases=1_000_003) == exp
+
+
 def test_chunk_size_invariance():
     w = synth.make_workload("C2", scale=0.02)
     cfg = w.cfg
@@ -113,7 +161,7 @@ def test_finder_candidates_match_oracle():
     rng = np.random.default_rng(9)
     n = 300_001
     seq = synth.random_genome_text(rng, n, b"ACGTacgtN", p=[.23, .23, .23, .23, .02, .02, .02, .01, .01])
-    for pat in ("N" * 21 + "RG", "TTTV" + "N" * 23, "NGG", "N" * 8):
+    for pat in ("N" * 21 + "RG", "TTTV" + "N" * 23, "NGG", "N" * 8, "N" * 34 + "RYAC", "TTTV" + "N" * 40 + "GA"):
         L = len(pat)
         plan = cof.cof_plan_create(pat, ["N" * L], [0])
         s = torch.cuda.current_stream()

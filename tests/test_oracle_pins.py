@@ -225,7 +225,43 @@ def test_short_and_empty():
     with pytest.raises(ValueError):
         oracle.search(["ACGT"], "NNRU", ["ACNN"], [1])          # not an IUPAC letter (G18)
     with pytest.raises(ValueError):
-        oracle.search(["ACGT"], "N" * 33, ["N" * 33], [1])      # L > 32
+        oracle.search(["ACGT"], "N" * 65, ["N" * 65], [1])      # L > 64 (COF_ORACLE_MAX_L)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_long_patterns_two_oracles(seed):
+    """32 < L <= 64: the C oracle against the independent pure-Python
+    oracle on random long IUPAC patterns and guides (brute force on small genomes)."""
+    rng = np.random.default_rng(2000 + seed)
+    L = int(rng.integers(33, 65))
+    codes = "ACGTRYSWKMBDHV"
+    pat = "".join(rng.choice(list("N" * 30 + codes), L))
+    guides = ["".join(rng.choice(list("ACGTACGTN" + "RYKM"), L)) for _ in range(3)]
+    thr = [int(rng.integers(L // 3, L // 2)) for _ in guides]
+    chroms = [synth.random_genome_text(rng, int(rng.integers(0, 1500)), b"ACGTacgtNnRy",
+                                       p=[.2, .15, .15, .2, .06, .06, .06, .06, .03, .01, .01, .01]).tobytes().decode()
+              for _ in range(3)]
+    a = oracle.hits_to_tuples(oracle.search(chroms, pat, guides, thr))
+    b = pyoracle.search(chroms, pat, guides, thr)
+    assert a == b
+
+
+def test_planted_sites_long():
+    """Pin by construction at L = 40 (36-nt cores + NGG, a two-word compared span) and
+    L = 38 (CjCas9-like 8-letter PAM): every planted k <= t copy is found at mm == k."""
+    for name in ("X1", "X2"):
+        w = synth.make_workload(name, scale=0.01, n_guides=3)
+        cfg = w.cfg
+        assert cfg.L > 32
+        hits = oracle.search(w.seqs, cfg.pattern, w.guides, w.thresholds)
+        found = {(int(h["chrom"]), int(h["pos"]), h["strand"].decode(), int(h["guide"])): int(h["mm"])
+                 for h in hits}
+        for pl in w.plants:
+            key = (pl.chrom, pl.pos, pl.strand, pl.guide)
+            if pl.k <= cfg.threshold:
+                assert found.get(key) == pl.k, pl
+            else:
+                assert key not in found, pl
 
 
 def test_ranges_restrict_window_starts():
