@@ -64,17 +64,34 @@ class Chunk:
         return rows
 
 
-FUSED_MIN_GUIDES = 256   # measured crossover on B200: 100 guides two-call 12.4 ms vs fused 13.6 ms
-                         # (C3); 1000 guides fused 56.3 ms vs two-call 57.5 ms (C5)
+FUSED_MIN_GUIDES = 256     # fused path from this many guides on, whatever the PAM
+FUSED_MIN_DENSITY = 0.03   # ... and below it when PAM sites are at least this dense per strand
+_SET_SIZE = {c: len(v) for c, v in {"A": "A", "C": "C", "G": "G", "T": "T", "R": "AG", "Y": "CT", "S": "CG",
+                                    "W": "AT", "K": "GT", "M": "AC", "B": "CGT", "D": "AGT", "H": "ACT",
+                                    "V": "ACG", "N": "ACGT"}.items()}
+
+
+def pam_density(pattern: str) -> float:
+    """Expected PAM sites per window start and strand on a uniform random genome."""
+    d = 1.0
+    for c in pattern.upper():
+        d *= _SET_SIZE[c] / 4.0
+    return d
 
 
 def use_fused(plan, n_guides: int) -> bool:
+    """Fused find+compare (finder masks, no item lists) or the two-call path.  Measured on
+    B200 (round 1, final kernels): C3 (NRG, density 0.125, 100 guides) fused 9.67 ms vs
+    two-call 11.71 ms; C5 (1000 guides) 51.8 vs 57.5 ms; C2 (NGG 0.0625, 10 guides) 0.172 vs
+    0.180 ms; C4 (TTTV 0.0117, 100 guides) 3.82 vs 3.14 ms -- with sparse PAM sites the
+    per-strand mask expansion and the unprefetched window loads cost more than the item
+    lists save.  COF_FUSED=0/1 overrides."""
     env = os.environ.get("COF_FUSED")
     if not cof.cof_find_compare_supported(plan):
         return False
     if env is not None:
         return env != "0"
-    return n_guides >= FUSED_MIN_GUIDES
+    return n_guides >= FUSED_MIN_GUIDES or pam_density(plan.pattern) >= FUSED_MIN_DENSITY
 
 
 def plan_chunks(lengths, L: int, chunk_bases: int | None = None, pack_bases: int | None = None):

@@ -301,3 +301,13 @@ def test_plan_chunks_packed():
             iv = sorted(cover.get(c, []))
             assert sum(e - s for s, e in iv) == max(0, n - L + 1)
             assert all(a[1] == b[0] for a, b in zip(iv, iv[1:]))
+
+
+def test_path_selection_by_pam_density():
+    """search.use_fused: fused from 256 guides, or when PAM sites are dense (NRG, NGG);
+    the two-call path for sparse PAMs with few guides (TTTV)."""
+    assert search.pam_density("N" * 21 + "RG") == pytest.approx(0.125)
+    assert search.pam_density("TTTV" + "N" * 23) == pytest.approx(0.75 / 64)
+    nrg = cof.cof_plan_create("N" * 21 + "RG", ["A" * 20 + "NNN"] * 3, [3] * 3)
+    tttv = cof.cof_plan_create("TTTV" + "N" * 23, ["NNNN" + "A" * 23] * 3, [3] * 3)
+    assert search.use_fused(nrg, 3) and not search.use_fused(tttv, 100) and search.use_fused(tttv, 300)

@@ -100,6 +100,38 @@ def test_configs_scaled_mma(name, scale, chunk, pack):
                     impl="mma") == exp
 
 
+@pytest.mark.parametrize("shape", ["spcas9", "cas12a"])
+@pytest.mark.parametrize("n_guides", [1, 37, 512, 600])
+def test_uniform_threshold_paths(shape, n_guides):
+    """The uniform-threshold specializations (20-nt SpCas9 guides: 10 pairs; 23-nt Cas12a:
+    12 pairs) on genomes with N runs, lowercase and rare letters, one to 19 guide blocks
+    (one fused launch, or two for 600 guides of Cas12a), fused and two-call paths."""
+    rng = np.random.default_rng(77 + n_guides + (shape == "cas12a"))
+    if shape == "spcas9":
+        pat, mk = "N" * 21 + "RG", lambda: "".join(rng.choice(list("ACGT"), 20)) + "NNN"
+    else:
+        pat, mk = "TTTV" + "N" * 23, lambda: "NNNN" + "".join(rng.choice(list("ACGT"), 23))
+    guides = [mk() for _ in range(n_guides)]
+    t = 6 if shape == "spcas9" else 5
+    lens = [0, 5, 1_000_003 if n_guides < 100 else 200_003, 77_777]
+    seqs = [synth.random_genome_text(rng, n, b"ACGTacgtNnRy",
+                                     p=[.23, .17, .17, .23, .04, .04, .04, .04, .02, .01, .005, .005]) for n in lens]
+    # plant exact and near copies of every guide so every guide block sees hits
+    s2 = seqs[2]
+    for gi, g in enumerate(guides[:64]):
+        core = g.replace("N", "")
+        site = (core + "AGG") if shape == "spcas9" else ("TTTA" + core)
+        p = 1000 + gi * 997
+        s2[p:p + len(site)] = np.frombuffer(site.encode(), np.uint8)
+    thr = [t] * len(guides)
+    exp = ref_hits(seqs, pat, guides, thr)
+    assert len(exp) >= min(64, n_guides)
+    assert gpu_hits(seqs, pat, guides, thr, fused=True) == exp
+    assert gpu_hits(seqs, pat, guides, thr, fused=True, pack_bases=0) == exp
+    assert gpu_hits(seqs, pat, guides, thr, fused=True, chunk_bases=99_991, pack_bases=300_000) == exp
+    assert gpu_hits(seqs, pat, guides, thr, fused=False) == exp
+
+
 @pytest.mark.parametrize("seed", range(6))
 def test_random_long(seed):
     """32 < L <= 64: random long IUPAC patterns (PAM letters at window
