@@ -229,6 +229,7 @@ struct TableArgs {
     const uint4* masks;            // one {fwd0, rev0, fwd1, rev1} per word pair
     uint64_t n_wp;
     unsigned int* ticket;          // dynamic grab counter (zeroed per launch)
+    uint32_t grab_rounds;          // FGRAB-word-pair ranges per ticket
 };
 
 // Hit mask (bit k = guide k of the block) of one item against one 32-guide block whose
@@ -535,11 +536,16 @@ __global__ void __launch_bounds__(CT, W64 ? 2 : 3) cof_comparer_fused(const __gr
         q_n -= n_items;
     };
 
+    // one ticket = grab_rounds consecutive ranges of FGRAB word pairs (fewer atomics on the
+    // shared counter when PAM sites are sparse and a range holds few items)
+    uint32_t grab = 0, round = a.grab_rounds;
     for (;;) {
-        uint32_t grab = 0;
-        if (lane == 0) grab = atomicAdd(a.ticket, 1u);
-        grab = __shfl_sync(0xffffffffu, grab, 0);
-        const uint64_t wp0 = (uint64_t)grab * FGRAB;
+        if (round == a.grab_rounds) {
+            if (lane == 0) grab = atomicAdd(a.ticket, 1u);
+            grab = __shfl_sync(0xffffffffu, grab, 0);
+            round = 0;
+        }
+        const uint64_t wp0 = ((uint64_t)grab * a.grab_rounds + round++) * FGRAB;
         if (wp0 >= a.n_wp) break;
         const uint64_t wp = wp0 + lane;
         uint32_t m0 = 0, m1 = 0;
@@ -703,6 +709,7 @@ static cof_status launch_table(TableArgs& t, int uniform_t, uint64_t n_hint, cud
 }
 
 static uint32_t fused_blocks_per_launch(const cof_plan* plan);
+static uint32_t fused_grab_rounds(const cof_plan* plan);
 
 // One launch per (strand, range of <= MAX_TABLE_BLOCKS guide blocks); thresholds travel in
 // the parameter space; hit counts accumulate on the device.
@@ -728,6 +735,7 @@ static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs
         T.masks = masks;
         T.n_wp = n_wp;
         T.ticket = tickets ? tickets + sd : nullptr;
+        T.grab_rounds = fused_grab_rounds(plan);
         const uint32_t* pm = (const uint32_t*)(plan->image.data() + (sd == 0 ? plan->lay.pmeta_fwd : plan->lay.pmeta_rev));
         const uint32_t batch = fused ? fused_blocks_per_launch(plan) : MAX_TABLE_BLOCKS;
         for (uint32_t bb = 0, li = 0; bb < plan->n_blocks; bb += batch, li++) {
@@ -826,6 +834,23 @@ static uint32_t fused_blocks_per_launch(const cof_plan* plan) {
     const size_t avail = table_smem_budget() + 16u * 1024u - (CT / 32) * FWQ * 4u - 1024u;
     return std::min<uint32_t>(MAX_TABLE_BLOCKS, (uint32_t)(avail / per_block));
 }
+// Word-pair ranges per ticket of the fused comparer: ~16 PAM sites per lane and ticket
+// (1 range for NRG; more for sparse PAMs such as Cas12a TTTV), COF_GRAB_ROUNDS overrides.
+static uint32_t fused_grab_rounds(const cof_plan* plan) {
+    static int env = -2;
+    if (env == -2) {
+        const char* e = getenv("COF_GRAB_ROUNDS");
+        env = e ? atoi(e) : -1;
+    }
+    if (env > 0) return (uint32_t)std::min(env, 64);
+    double d = 1.0;   // expected PAM sites per start and strand on a uniform genome
+    for (uint32_t k = 0; k < plan->pam[0].n; k++) d *= __builtin_popcount(plan->pam[0].set[k]) / 4.0;
+    const double per_range = d * 64.0;   // per lane (64 starts) and strand
+    uint32_t r = 1;
+    while (r < 16 && per_range * r < 8.0) r *= 2;
+    return r;
+}
+
 static bool fusable(const cof_plan* plan) {
     const uint32_t bpl = fused_blocks_per_launch(plan);
     return bpl >= 1 && (plan->n_blocks + bpl - 1) / bpl * 2 <= FUSED_MAX_TICKETS;

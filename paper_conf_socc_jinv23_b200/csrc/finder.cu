@@ -13,9 +13,10 @@
 // funnel shift of each plane and a 3-LOP3 multiplexer select membership in the letter's
 // IUPAC set, AND-ed over letters.  Passing starts are compacted in order: each CTA owns
 // a contiguous tile range, counts it (pass 1), exchanges its total with all CTAs once
-// (grid barrier), then re-streams the range (pass 2: CTA scan of the per-thread popcounts,
-// staging in shared memory, coalesced stores).  Algorithmic bytes per base: 3/8 read +
-// 4 x items written (pass 2 re-reads the planes, largely from L2).
+// (grid barrier), then walks its pass-1 masks again (pass 2: one warp per tile, warp
+// scans of the masks' popcounts, one exchange of tile totals per 8 tiles, ordered direct
+// stores).  Algorithmic bytes per base: 3/8 read + 4 x items written (pass 2 re-reads the
+// 1/4 B/base of masks, largely from L2).
 #include <cuda_runtime.h>
 
 #include "cof_internal.h"
@@ -26,14 +27,15 @@ namespace cof {
 constexpr int FT = 256;          // threads per CTA
 constexpr int FWPT = 2;          // consecutive plane words (x 32 window starts) per thread
 constexpr int FW = FT * FWPT;    // words per tile (16384 window starts)
-constexpr int FSTAGE_ITEMS = 8192;   // shared staging capacity per output round
 constexpr int FSTAGES = 4;       // TMA ring depth
 constexpr int FLOAD = FW + 4;    // words per plane per stage: tile + halo, 16-byte multiple
 constexpr uint32_t FMAX_CTAS = 4096;                      // grid cap (co-residency)
 constexpr size_t FWS_BARRIER = 2 * FMAX_CTAS * sizeof(uint64_t);
 constexpr size_t FWS_MASKS = FWS_BARRIER + 256;
 constexpr int FPL = 4;           // planes per stage: lo, hi, nm, vs (valid starts; multi-segment chunks)
-constexpr uint32_t FSMEM = FSTAGES * FPL * FLOAD * 4 + FSTAGES * 8 + FSTAGE_ITEMS * 4;
+constexpr int FSTAGE_ITEMS = 8192;   // pass 2 (dense): items staged per round, in the idle TMA ring
+static_assert(FSTAGE_ITEMS <= FSTAGES * FPL * FLOAD, "pass-2 staging fits the TMA ring");
+constexpr uint32_t FSMEM = FSTAGES * FPL * FLOAD * 4 + FSTAGES * 8;
 
 struct FinderArgs {
     const uint32_t* lo;
@@ -48,6 +50,7 @@ struct FinderArgs {
     unsigned int* barrier;       // workspace: grid barrier counter (zeroed)
     unsigned long long* counters;  // plan_dev counters: [0] n_fwd, [1] n_rev
     uint32_t n_tiles;
+    uint32_t stage;              // pass 2 stages items in shared memory (dense PAM sites)
     uint32_t ne;                 // non-N pattern letters per strand (same for both)
     uint32_t pj[2][COF_MAX_L];   // window offset of entry e
     uint4 psel[2][COF_MAX_L];    // entry e's IUPAC set as splat words {A, C, G, T} (0 / ~0)
@@ -99,7 +102,6 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
     extern __shared__ __align__(128) uint8_t smem[];
     uint32_t* stage = reinterpret_cast<uint32_t*>(smem);
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + FSTAGES * FPL * FLOAD * 4);
-    uint32_t* items = reinterpret_cast<uint32_t*>(bars + FSTAGES);
     __shared__ uint32_t s_warp[FT / 32];
     __shared__ uint32_t s_tile_tot;
     __shared__ unsigned long long s_red[FT / 32][2];
@@ -222,87 +224,157 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
     }
 
     // ---------------- pass 2: masks (workspace, mostly L2) -> ordered item lists
-    unsigned long long run_f = 0, run_r = 0;
-    const uint4* mptr = reinterpret_cast<const uint4*>(a.masks);
-    uint4 mnext = n_mine ? __ldcg(mptr + (size_t)t_begin * FT + tid) : make_uint4(0, 0, 0, 0);
-    for (uint32_t k = 0; k < n_mine; k++) {
-        const uint32_t tile = t_begin + k;
-        const uint4 mv = mnext;
-        if (k + 1 < n_mine) mnext = __ldcg(mptr + (size_t)(tile + 1) * FT + tid);
-        const uint32_t m[2][FWPT] = {{mv.x, mv.z}, {mv.y, mv.w}};
-        const uint32_t cf = (uint32_t)(__popc(mv.x) + __popc(mv.z));
-        const uint32_t cr = (uint32_t)(__popc(mv.y) + __popc(mv.w));
-        const uint64_t p0 = ((uint64_t)tile * FW + FWPT * tid) * 32;
+    if (a.stage) {
+        // Dense PAM sites: CTA per tile -- thread t scans its 2 words, one CTA scan per
+        // tile, items staged in shared memory (the TMA ring, idle after pass 1) and written
+        // out coalesced.
+        uint32_t* items = stage;
+        unsigned long long run_f = 0, run_r = 0;
+        const uint4* mptr = reinterpret_cast<const uint4*>(a.masks);
+        uint4 mnext = n_mine ? __ldcg(mptr + (size_t)t_begin * FT + tid) : make_uint4(0, 0, 0, 0);
+        for (uint32_t k = 0; k < n_mine; k++) {
+            const uint32_t tile = t_begin + k;
+            const uint4 mv = mnext;
+            if (k + 1 < n_mine) mnext = __ldcg(mptr + (size_t)(tile + 1) * FT + tid);
+            const uint32_t m[2][FWPT] = {{mv.x, mv.z}, {mv.y, mv.w}};
+            const uint32_t cf = (uint32_t)(__popc(mv.x) + __popc(mv.z));
+            const uint32_t cr = (uint32_t)(__popc(mv.y) + __popc(mv.w));
+            const uint64_t p0 = ((uint64_t)tile * FW + FWPT * tid) * 32;
 
-        // CTA exclusive scan of packed counts (fwd bits 0..15, rev 16..31)
-        const uint32_t cnt = cf | (cr << 16);
-        uint32_t x = cnt;
+            // CTA exclusive scan of packed counts (fwd bits 0..15, rev 16..31)
+            const uint32_t cnt = cf | (cr << 16);
+            uint32_t x = cnt;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= o) x += y;
-        }
-        if (lane == 31) s_warp[warp] = x;
-        __syncthreads();
-        if (warp == 0) {
-            uint32_t wv = lane < FT / 32 ? s_warp[lane] : 0u;
-            uint32_t wi = wv;
-#pragma unroll
-            for (int o = 1; o < FT / 32; o <<= 1) {
-                uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
-                if (lane >= o) wi += y;
+            for (int o = 1; o < 32; o <<= 1) {
+                uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= o) x += y;
             }
-            if (lane < FT / 32) s_warp[lane] = wi - wv;
-            if (lane == FT / 32 - 1) s_tile_tot = wi;
-        }
-        __syncthreads();
-        const uint32_t local = s_warp[warp] + x - cnt;
-        const uint32_t tot = s_tile_tot;
-        const uint32_t pbase = (uint32_t)p0;
+            if (lane == 31) s_warp[warp] = x;
+            __syncthreads();
+            if (warp == 0) {
+                uint32_t wv = lane < FT / 32 ? s_warp[lane] : 0u;
+                uint32_t wi = wv;
 #pragma unroll
-        for (int st = 0; st < 2; st++) {
-            const uint32_t total = st == 0 ? (tot & 0xFFFFu) : (tot >> 16);
-            const uint32_t first = st == 0 ? (local & 0xFFFFu) : (local >> 16);
-            const unsigned long long base = s_base[st] + (st == 0 ? run_f : run_r);
-            uint32_t* out = a.out[st];
-            // staged in rounds of FSTAGE_ITEMS (one round unless the pattern is very permissive)
-            for (uint32_t r0 = 0; r0 < total; r0 += FSTAGE_ITEMS) {
-                if (total <= FSTAGE_ITEMS) {
-                    uint32_t off = first;
+                for (int o = 1; o < FT / 32; o <<= 1) {
+                    uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
+                    if (lane >= o) wi += y;
+                }
+                if (lane < FT / 32) s_warp[lane] = wi - wv;
+                if (lane == FT / 32 - 1) s_tile_tot = wi;
+            }
+            __syncthreads();
+            const uint32_t local = s_warp[warp] + x - cnt;
+            const uint32_t tot = s_tile_tot;
+            const uint32_t pbase = (uint32_t)p0;
 #pragma unroll
-                    for (int w = 0; w < FWPT; w++) {
-                        uint32_t mm = m[st][w];
-                        while (mm) {
-                            const int b = __ffs(mm) - 1;
-                            items[off++] = pbase + 32u * w + (uint32_t)b;
-                            mm &= mm - 1;
+            for (int st = 0; st < 2; st++) {
+                const uint32_t total = st == 0 ? (tot & 0xFFFFu) : (tot >> 16);
+                const uint32_t first = st == 0 ? (local & 0xFFFFu) : (local >> 16);
+                const unsigned long long base = s_base[st] + (st == 0 ? run_f : run_r);
+                uint32_t* out = a.out[st];
+                // staged in rounds of FSTAGE_ITEMS (one round unless the pattern is very permissive)
+                for (uint32_t r0 = 0; r0 < total; r0 += FSTAGE_ITEMS) {
+                    if (total <= FSTAGE_ITEMS) {
+                        uint32_t off = first;
+#pragma unroll
+                        for (int w = 0; w < FWPT; w++) {
+                            uint32_t mm = m[st][w];
+                            while (mm) {
+                                const int b = __ffs(mm) - 1;
+                                items[off++] = pbase + 32u * w + (uint32_t)b;
+                                mm &= mm - 1;
+                            }
+                        }
+                    } else {
+                        uint32_t rank = first;
+#pragma unroll
+                        for (int w = 0; w < FWPT; w++) {
+                            uint32_t mm = m[st][w];
+                            while (mm) {
+                                const int b = __ffs(mm) - 1;
+                                if (rank >= r0 && rank < r0 + FSTAGE_ITEMS) items[rank - r0] = pbase + 32u * w + (uint32_t)b;
+                                rank++;
+                                mm &= mm - 1;
+                            }
                         }
                     }
-                } else {
-                    uint32_t rank = first;
+                    __syncthreads();
+                    uint32_t n_round = min(total - r0, (uint32_t)FSTAGE_ITEMS);
+                    const unsigned long long o0 = base + r0;
+                    if (o0 >= a.cap) n_round = 0;
+                    else if (a.cap - o0 < n_round) n_round = (uint32_t)(a.cap - o0);
+                    uint32_t* __restrict__ dst = out + o0;
+                    for (uint32_t i = tid; i < n_round; i += FT) dst[i] = items[i];
+                    __syncthreads();
+                }
+            }
+            run_f += tot & 0xFFFFu;
+            run_r += tot >> 16;
+        }
+    } else {
+        // Sparse PAM sites: warp per tile.  The CTA's 8 warps take 8 consecutive tiles per
+        // round; each warp scans its tile's 256 word-pair masks (8 coalesced 16-byte loads
+        // per lane, one warp scan per load), the tile totals are exchanged once per round
+        // (two CTA barriers per 8 tiles instead of ~6 per tile), and every lane writes its
+        // items straight to their ordered slots (L2 merges the partial sectors).
+        constexpr int P2J = FT / 32;          // word-pair loads per lane and tile (8)
+        unsigned long long run_f = 0, run_r = 0;
+        const uint4* mptr = reinterpret_cast<const uint4*>(a.masks);
+        for (uint32_t k = 0; k < n_mine; k += FT / 32) {
+            const uint32_t tile = t_begin + k + (uint32_t)warp;
+            const bool mine = k + (uint32_t)warp < n_mine;
+            uint4 m[P2J];
+            uint32_t off[P2J];                 // lane's exclusive offset in the tile per load (fwd | rev << 16)
+            uint32_t acc = 0;                  // running tile total (fwd | rev << 16), warp-uniform
 #pragma unroll
-                    for (int w = 0; w < FWPT; w++) {
-                        uint32_t mm = m[st][w];
+            for (int j = 0; j < P2J; j++)
+                m[j] = mine ? __ldcg(mptr + (size_t)tile * FT + 32 * j + lane) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+            for (int j = 0; j < P2J; j++) {
+                const uint32_t c = (uint32_t)(__popc(m[j].x) + __popc(m[j].z)) |
+                                   ((uint32_t)(__popc(m[j].y) + __popc(m[j].w)) << 16);
+                uint32_t x = c;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                    if (lane >= o) x += y;
+                }
+                off[j] = acc + x - c;
+                acc += __shfl_sync(0xffffffffu, x, 31);
+            }
+            if (lane == 0) s_warp[warp] = acc;
+            __syncthreads();
+            unsigned long long bf = s_base[0] + run_f, br = s_base[1] + run_r;
+#pragma unroll
+            for (int w = 0; w < FT / 32; w++) {
+                const uint32_t t = s_warp[w];
+                if (w < warp) { bf += t & 0xFFFFu; br += t >> 16; }
+                run_f += t & 0xFFFFu;
+                run_r += t >> 16;
+            }
+            __syncthreads();   // s_warp is rewritten by the next round
+            if (!mine) continue;
+            const uint32_t pbase = tile * (uint32_t)FW * 32u + 64u * (uint32_t)lane;
+#pragma unroll
+            for (int j = 0; j < P2J; j++) {
+                const uint32_t pj = pbase + 2048u * j;   // 32 lanes x 64 starts per load
+#pragma unroll
+                for (int st = 0; st < 2; st++) {
+                    unsigned long long o = (st == 0 ? bf : br) + (st == 0 ? (off[j] & 0xFFFFu) : (off[j] >> 16));
+                    uint32_t* out = a.out[st];
+#pragma unroll
+                    for (int w = 0; w < 2; w++) {
+                        uint32_t mm = st == 0 ? (w ? m[j].z : m[j].x) : (w ? m[j].w : m[j].y);
                         while (mm) {
                             const int b = __ffs(mm) - 1;
-                            if (rank >= r0 && rank < r0 + FSTAGE_ITEMS) items[rank - r0] = pbase + 32u * w + (uint32_t)b;
-                            rank++;
+                            if (o < a.cap) out[o] = pj + 32u * w + (uint32_t)b;
+                            o++;
                             mm &= mm - 1;
                         }
                     }
                 }
-                __syncthreads();
-                uint32_t n_round = min(total - r0, (uint32_t)FSTAGE_ITEMS);
-                const unsigned long long o0 = base + r0;
-                if (o0 >= a.cap) n_round = 0;
-                else if (a.cap - o0 < n_round) n_round = (uint32_t)(a.cap - o0);
-                uint32_t* __restrict__ dst = out + o0;
-                for (uint32_t i = tid; i < n_round; i += FT) dst[i] = items[i];
-                __syncthreads();
             }
         }
-        run_f += tot & 0xFFFFu;
-        run_r += tot >> 16;
     }
 }
 
@@ -442,6 +514,11 @@ cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* de
         a.counters = counters;
         a.n_tiles = n_tiles;
         a.ne = plan->pam[0].n;
+        {   // expected PAM sites per start and strand on a uniform genome: stage when dense
+            double d = 1.0;
+            for (uint32_t k = 0; k < plan->pam[0].n; k++) d *= __builtin_popcount(plan->pam[0].set[k]) / 4.0;
+            a.stage = d >= 0.03 ? 1u : 0u;
+        }
         bool wide = false;
         for (int st = 0; st < 2; st++)
             for (uint32_t k = 0; k < plan->pam[st].n; k++) wide |= plan->pam[st].j[k] >= 32;
