@@ -223,7 +223,6 @@ struct TableArgs {
     uint32_t n_blocks;
     uint32_t block_base;
     uint32_t blocks_per_chunk;     // guide blocks resident in shared memory at a time
-    uint32_t prefetch;             // item-list comparer: cp.async window prefetch (1) or direct loads (0)
     PairLayout pairs;
     uint32_t meta[MAX_TABLE_BLOCKS][8];   // per block: T0..T5 threshold planes, valid mask
     // fused find+compare: the finder's PAM masks replace the item list
@@ -421,44 +420,6 @@ __global__ void __launch_bounds__(CT, W64 ? 2 : 3) cof_comparer_table(const __gr
     const uint32_t bpc = a.blocks_per_chunk;
     const uint32_t n_chunks = (a.n_blocks + bpc - 1) / bpc;
     uint32_t loaded = 0xFFFFFFFFu;
-
-    if (!a.prefetch) {
-        // no prefetch: each tile loads its positions and window words directly (latency
-        // hidden by the other resident warps), no cp.async traffic through shared memory
-        for (uint32_t tile = blockIdx.x; tile < n_tiles; tile += gridDim.x) {
-            const uint32_t item0 = tile * per_tile + threadIdx.x;
-            const bool tail = n - tile * per_tile < per_tile;
-            uint32_t base[R][NP], okm[R];
-#pragma unroll
-            for (int r = 0; r < R; r++) {
-                const uint32_t idx = item0 + (uint32_t)r * CT;
-                okm[r] = idx < n ? ~0u : 0u;
-                item_bases<NP, W64>(a, s_base, idx < n ? __ldg(a.items + idx) : 0u, base[r]);
-            }
-            for (uint32_t ch = 0; ch < n_chunks; ch++) {
-                const uint32_t b0 = ch * bpc;
-                const uint32_t nb = min(bpc, a.n_blocks - b0);
-                if (loaded != ch) {
-                    __syncthreads();
-                    const uint2* src = a.ptab + (size_t)b0 * NP * 25;
-                    const uint32_t n8 = nb * NP * 25;
-                    for (uint32_t i = threadIdx.x; i < n8; i += CT) s_tab_p[i] = __ldg(src + i);
-                    __syncthreads();
-                    loaded = ch;
-                }
-                if (tail) table_blocks<NP, R, true, TC>(a, base, nb, b0, a.items + item0, okm);
-                else table_blocks<NP, R, false, TC>(a, base, nb, b0, a.items + item0, okm);
-                if (n_chunks > 1) {
-                    const uint32_t inc = (nb & 3u) ? (nb - 1u) * BS : (nb - 4u) * BS;
-#pragma unroll
-                    for (int r = 0; r < R; r++)
-#pragma unroll
-                        for (int q = 0; q < NP; q++) base[r][q] -= inc;
-                }
-            }
-        }
-        return;
-    }
 
     // Two-stage prefetch: positions two tiles ahead (registers), plane words one tile ahead
     // (cp.async into per-thread shared slots after the resident table chunk).
@@ -658,8 +619,6 @@ constexpr int R_TABLE = 2;   // items per thread
 // Tuning knobs (defaults chosen from B200 measurements):
 //  COF_TABLE_SMEM_KB     shared-memory budget per CTA for resident guide blocks
 static bool g_uniform_t_enabled = getenv("COF_TABLE_GENERIC") == nullptr;
-//  COF_TABLE_PREFETCH=0  item-list comparer loads windows directly instead of cp.async slots
-static uint32_t g_table_prefetch = getenv("COF_TABLE_PREFETCH") == nullptr || atoi(getenv("COF_TABLE_PREFETCH")) != 0;
 static uint32_t table_smem_budget() {
     static uint32_t v = 0;
     if (!v) {
@@ -777,7 +736,6 @@ static cof_status run_table(const cof_plan* plan, uint8_t* pd, const CompareArgs
         T.n_wp = n_wp;
         T.ticket = tickets ? tickets + sd : nullptr;
         T.grab_rounds = fused_grab_rounds(plan);
-        T.prefetch = g_table_prefetch;
         const uint32_t* pm = (const uint32_t*)(plan->image.data() + (sd == 0 ? plan->lay.pmeta_fwd : plan->lay.pmeta_rev));
         const uint32_t batch = fused ? fused_blocks_per_launch(plan) : MAX_TABLE_BLOCKS;
         for (uint32_t bb = 0, li = 0; bb < plan->n_blocks; bb += batch, li++) {

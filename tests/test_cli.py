@@ -74,3 +74,34 @@ def test_cli_bulge_end_to_end(tmp_path):
                   for h in ref)
     assert len(ref) > 0
     assert out.read_text() == exp
+
+
+def test_format_hits_long():
+    """cof_hit64 records (L > 32) format like cof_hit ones."""
+    h = np.zeros(1, dtype=cof.HIT64_DTYPE)
+    site = b"ACGT" * 9 + b"AgG"
+    h[0]["guide"], h[0]["chrom"], h[0]["pos"], h[0]["strand"], h[0]["mm"], h[0]["site"] = 0, 0, 5, b"-", 1, site
+    txt = cli.format_hits(h, ["Q" * 39], ["chrA"])
+    assert txt == "Q" * 39 + "\tchrA\t5\t" + site.decode() + "\t-\t1\n"
+
+
+@pytest.mark.gpu
+def test_cli_long_pattern_end_to_end(tmp_path):
+    """A 40-letter pattern (two-word windows) through the CLI: .2bit-free FASTA input,
+    TSV output equal to the oracle's."""
+    rng = np.random.default_rng(33)
+    seqs = [synth.random_genome_text(rng, n, b"ACGTacgtN", p=[.23, .2, .2, .23, .03, .03, .03, .03, .02])
+            for n in (60_000, 9_001)]
+    names = ["chr1", "chr2"]
+    synth.write_fasta(tmp_path / "g.fa", names, seqs)
+    pat = "N" * 38 + "GG"
+    guides = ["".join(rng.choice(list("ACGT"), 37)) + "NNN" for _ in range(4)]
+    inp = tmp_path / "input.txt"
+    inp.write_text("g.fa\n" + pat + "\n" + "".join(f"{g} 21\n" for g in guides))
+    out = tmp_path / "out.txt"
+    assert cli.main([str(inp), "G", str(out)]) == 0
+    ref = oracle.search(seqs, pat, guides, [21] * 4)
+    exp = "".join(f"{guides[int(h['guide'])]}\t{names[int(h['chrom'])]}\t{int(h['pos'])}\t{h['site'].decode()}\t"
+                  f"{h['strand'].decode()}\t{int(h['mm'])}\n" for h in ref)
+    assert len(ref) > 10
+    assert out.read_text() == exp
