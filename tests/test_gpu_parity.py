@@ -257,12 +257,14 @@ def test_sorted_keys_and_determinism():
     assert a == sorted(a, key=lambda h: (h[0], h[1], h[2] == "-", h[3]))
 
 
-def test_full_size_sampled_c5():
-    """C5 at full size (the bench workload) on one GPU, in the bench's launch
-    configuration (whole-chromosome chunks, device-resident planes, counts on device);
-    the oracle recomputes sampled window ranges one by one."""
+@pytest.mark.parametrize("name", ["C5", "C3", "C4"])
+def test_full_size_sampled(name):
+    """C5 / C3 / C4 at full size on one GPU, in the bench's launch configuration (the whole
+    genome as one multi-segment chunk, device-resident planes, counts on device; fused
+    path for C5 and C3, two-call with the sparse-PAM finder pass 2 for C4); the oracle
+    recomputes sampled window ranges one by one."""
     from bench import run_device_pipeline, prepare_workload   # same code the bench times
-    wl, plan_obj = prepare_workload("C5")
+    wl, plan_obj = prepare_workload(name)
     res = run_device_pipeline(wl, plan_obj, collect=True)
     rng = np.random.default_rng(77)
     cfg = wl.cfg
