@@ -236,8 +236,8 @@ def run_e2e_step(wl, st, searcher, out=None):
     """Public-API end-to-end step from pinned host planes; returns (hits, h2d, d2h bytes).
     ``out``: the caller's result buffer (reused between steps, as an application would)."""
     hits = searcher.search_host(st.e2e_host, out=out)
-    h2d = st.e2e_host.bytes
-    d2h = len(hits) * 56 + 24 * len(st.e2e_host.chunks)     # decorated records + per-chunk counts
+    h2d = st.e2e_host.h2d_bytes
+    d2h = len(hits) * hits.dtype.itemsize + 24 * len(st.e2e_host.chunks)   # decorated records + per-chunk counts
     return hits, h2d, d2h
 
 

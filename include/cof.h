@@ -134,6 +134,19 @@ cof_status cof_valid_starts(const cof_segment *segs, uint32_t n_segs, uint64_t n
  * of dev (cof_plane_words(host->n_bases) words each); copies the metadata fields and the
  * segs pointer too.  (Table III.) */
 cof_status cof_load_chunk(const cof_chunk *host, cof_chunk *dev, cof_stream s);
+/* N runs of a chunk (host): the maximal [begin, end) intervals of N bases (nm bit set)
+ * among bases [0, n_bases), ascending, as pairs runs[2i], runs[2i+1].  *n_runs = the count;
+ * COF_E_CAPACITY (contents past cap unspecified) if it exceeds cap pairs. */
+cof_status cof_n_runs(const uint32_t *nm, uint64_t n_bases, uint64_t *runs, uint64_t cap,
+                      uint64_t *n_runs);
+/* cof_load_chunk with the sparse planes built on the device: H2D of lo/hi only (1/4 B per
+ * base), dev->nm rebuilt from the n_runs N runs (cof_n_runs of the chunk) and, for a
+ * multi-segment chunk, dev->vs from host->segs (the owned-start intervals) by small kernels
+ * on stream s.  host->nm / host->vs are not read.  The device planes equal what
+ * cof_load_chunk would copy.  COF_E_ARG for runs that are not ascending intervals inside
+ * the chunk or a segment that leaves it. */
+cof_status cof_load_chunk_runs(const cof_chunk *host, const uint64_t *runs, uint64_t n_runs,
+                               cof_chunk *dev, cof_stream s);
 
 /* ------------------------------------------------------------------ FASTA (M2)
  * Minimal indexed FASTA reader ("single- or multi-sequence data format"):

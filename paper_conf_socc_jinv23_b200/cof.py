@@ -88,6 +88,8 @@ def _load():
         "cof_sort_workspace_bytes": (SZ, [U64]),
         "cof_sort_hits": (I32, [P, P, P, P, P, U64, U64, P, P]),
         "cof_read_counts": (I32, [P, P, P, P]),
+        "cof_n_runs": (I32, [P, U64, P, U64, P]),
+        "cof_load_chunk_runs": (I32, [P, P, U64, P, P]),
         "cof_collect": (I32, [P, P, P, P, U64, P, P]),
         "cof_collect64": (I32, [P, P, P, P, U64, P, P]),
         "cof_merge": (I32, [P, P, U32, P]),
@@ -127,7 +129,7 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_fasta_count", "cof_fasta_name", "cof_fasta_length", "cof_fasta_pack",
                        "cof_find_workspace_bytes", "cof_find_pam", "cof_compare",
                        "cof_sort_workspace_bytes", "cof_sort_hits", "cof_read_counts",
-                       "cof_collect", "cof_collect64", "cof_merge", "cof_merge64",
+                       "cof_n_runs", "cof_load_chunk_runs", "cof_collect", "cof_collect64", "cof_merge", "cof_merge64",
                        "cof_decorate_workspace_bytes", "cof_decorate", "cof_decorate64",
                        "cof_decorate_check", "cof_find_compare_supported",
                        "cof_find_compare_workspace_bytes", "cof_find_compare", "cof_find_masks",
@@ -251,6 +253,27 @@ def cof_valid_starts(segs, n_segs, n_bases, vs):
 
 def cof_load_chunk(host: cof_chunk, dev: cof_chunk, stream=None):
     _check(lib.cof_load_chunk(ctypes.addressof(host), ctypes.addressof(dev), _stream(stream)))
+
+
+def cof_n_runs(nm, n_bases: int) -> np.ndarray:
+    """[begin, end) runs of N bases of an nm plane, as an (n, 2) uint64 array."""
+    cnt = ctypes.c_uint64(0)
+    cap = 64
+    while True:
+        runs = np.zeros((cap, 2), dtype=np.uint64)
+        st = lib.cof_n_runs(_ptr(nm), int(n_bases), runs.ctypes.data, cap, ctypes.byref(cnt))
+        if st == COF_E_CAPACITY:
+            cap = int(cnt.value)
+            continue
+        _check(st)
+        return runs[: int(cnt.value)]
+
+
+def cof_load_chunk_runs(host: cof_chunk, runs: np.ndarray, dev: cof_chunk, stream=None):
+    """cof_load_chunk with nm (from ``runs``) and vs (from the segments) built on the device."""
+    runs = np.ascontiguousarray(runs, dtype=np.uint64)
+    _check(lib.cof_load_chunk_runs(ctypes.addressof(host), runs.ctypes.data if len(runs) else None, len(runs),
+                                   ctypes.addressof(dev), _stream(stream)))
 
 
 def cof_find_workspace_bytes(n_bases: int) -> int:

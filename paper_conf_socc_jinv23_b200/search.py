@@ -158,12 +158,15 @@ def merge_hit_lists(lists, dtype=None):
 
 class HostGenome:
     """Packed bit-planes of every chunk in pinned host memory (a1: chunk & pack); multi-
-    segment chunks also get their valid-start plane and segment table."""
+    segment chunks also get their valid-start plane and segment table, every chunk the
+    list of its N runs (cof_n_runs: only lo/hi cross PCIe, nm and vs are rebuilt on the
+    device by cof_load_chunk_runs)."""
 
     def __init__(self, seqs, chunks, pin: bool = True):
         self.chunks = chunks
         self.planes = []
         self.segs = []
+        self.runs = []
         pin = pin and torch.cuda.is_available()
         for ch in chunks:
             words = cof.cof_plane_words(ch.n_bases)
@@ -180,13 +183,14 @@ class HostGenome:
             cof.cof_pack(text, ch.n_bases, buf[0], buf[1], buf[2])
             self.planes.append(buf)
             self.segs.append(segs)
+            self.runs.append(cof.cof_n_runs(buf[2], ch.n_bases))
 
     @classmethod
     def from_packer(cls, chunks, pack, pin: bool = True):
         """Single-segment chunks packed by ``pack(chrom, first, n, lo, hi, nm)`` (e.g. straight
         from an indexed FASTA file, cof_fasta_pack) without materialising the ASCII."""
         self = cls.__new__(cls)
-        self.chunks, self.planes, self.segs = chunks, [], []
+        self.chunks, self.planes, self.segs, self.runs = chunks, [], [], []
         pin = pin and torch.cuda.is_available()
         for ch in chunks:
             if ch.multi:
@@ -196,6 +200,7 @@ class HostGenome:
             pack(ch.chrom, ch.start, ch.n_bases, buf[0], buf[1], buf[2])
             self.planes.append(buf)
             self.segs.append(None)
+            self.runs.append(cof.cof_n_runs(buf[2], ch.n_bases))
         return self
 
     def chunk_struct(self, i) -> cof.cof_chunk:
@@ -207,6 +212,25 @@ class HostGenome:
     @property
     def bytes(self):
         return sum(p.numel() * 4 for p in self.planes)
+
+    def _use_runs(self, i) -> bool:
+        # the run list replaces the nm (and vs) planes when it is smaller than they are
+        return self.runs[i].nbytes < (self.planes[i].shape[0] - 2) * self.planes[i].shape[1] * 4
+
+    @property
+    def h2d_bytes(self):
+        """Bytes load() moves per pass over all chunks (lo, hi and the N runs, or all planes)."""
+        return sum(2 * p.shape[1] * 4 + r.nbytes if self._use_runs(i) else p.numel() * 4
+                   for i, (p, r) in enumerate(zip(self.planes, self.runs)))
+
+    def load(self, i, dev: cof.cof_chunk, stream):
+        """H2D of chunk i into the device chunk ``dev``: lo/hi copied and nm/vs rebuilt on the
+        device from the N runs / segments (cof_load_chunk_runs), or every plane copied
+        (cof_load_chunk) when the genome is so N-fragmented that the runs are larger."""
+        if self._use_runs(i):
+            cof.cof_load_chunk_runs(self.chunk_struct(i), self.runs[i], dev, stream)
+        else:
+            cof.cof_load_chunk(self.chunk_struct(i), dev, stream)
 
 
 class Searcher:
@@ -324,7 +348,7 @@ class Searcher:
                     if freed[k] is not None:
                         self.copy_stream.wait_event(freed[k])
                     dch = self.device_chunk(host.chunks[idx[j]], planes[k], host.segs[idx[j]])
-                    cof.cof_load_chunk(host.chunk_struct(idx[j]), dch, self.copy_stream)
+                    host.load(idx[j], dch, self.copy_stream)
                     ev = torch.cuda.Event()
                     ev.record(self.copy_stream)
                     loaded[k] = ev
@@ -423,7 +447,7 @@ class Searcher:
             with torch.cuda.device(self.device):
                 for i in idx:
                     dch = self.device_chunk(host.chunks[i], None, host.segs[i])
-                    cof.cof_load_chunk(host.chunk_struct(i), dch, self.stream)
+                    host.load(i, dch, self.stream)
                     _, _, nh = self.run_device_chunk(dch, host.chunks[i].n_owned)
                     keys = torch.empty(max(nh, 1), dtype=torch.int64, pin_memory=True)
                     with torch.cuda.stream(self.stream):

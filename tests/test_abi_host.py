@@ -311,3 +311,33 @@ def test_path_selection_by_pam_density():
     nrg = cof.cof_plan_create("N" * 21 + "RG", ["A" * 20 + "NNN"] * 3, [3] * 3)
     tttv = cof.cof_plan_create("TTTV" + "N" * 23, ["NNNN" + "A" * 23] * 3, [3] * 3)
     assert search.use_fused(nrg, 3) and not search.use_fused(tttv, 100) and search.use_fused(tttv, 300)
+
+
+@pytest.mark.parametrize("n", [0, 1, 31, 32, 33, 64, 1000, 70_001])
+def test_n_runs_match_numpy(n):
+    """cof_n_runs: maximal N intervals of the packed nm plane, checked against numpy
+    run boundaries of the canonical text (runs at 0, at the end, across words)."""
+    rng = np.random.default_rng(40 + n)
+    seq = synth.random_genome_text(rng, n, b"ACGTN", p=[.2, .2, .2, .2, .2]) if n else np.zeros(0, np.uint8)
+    if n > 40:
+        seq[:7] = ord("N")
+        seq[-5:] = ord("N")
+        seq[32:64] = ord("N")
+    w = cof.cof_plane_words(n)
+    lo, hi, nm = (np.zeros(w, np.uint32) for _ in range(3))
+    cof.cof_pack(seq, n, lo, hi, nm)
+    runs = cof.cof_n_runs(nm, n)
+    isn = np.frombuffer(_canon(seq.tobytes()), np.uint8) == ord("N") if n else np.zeros(0, bool)
+    d = np.diff(np.concatenate([[0], isn.astype(np.int8), [0]]))
+    exp = np.stack([np.flatnonzero(d == 1), np.flatnonzero(d == -1)], axis=1) if n else np.zeros((0, 2))
+    assert runs.shape == exp.shape and (runs == exp).all()
+
+
+def test_host_genome_h2d_bytes_with_runs():
+    """An assembly-shaped genome (few long N runs) crosses PCIe as lo/hi + its N runs:
+    about 2/3 of the plane bytes (3 planes; 1/2 of them with the valid-start plane)."""
+    w = synth.make_workload("C2", scale=0.05)
+    chunks = search.plan_chunks([len(s) for s in w.seqs], w.cfg.L, None, 0)
+    host = search.HostGenome(w.seqs, chunks, pin=False)
+    assert all(len(r) < 200 for r in host.runs)
+    assert host.h2d_bytes < 0.7 * host.bytes

@@ -330,3 +330,34 @@ def test_many_guides_multiple_table_launches(impl):
         assert gpu_hits([seq], "N" * 21 + "RG", guides, thr, impl=impl, fused=False) == exp
     thr_u = [7] * n_g
     assert gpu_hits([seq], "N" * 21 + "RG", guides, thr_u, impl=impl) == ref_hits([seq], "N" * 21 + "RG", guides, thr_u)
+
+
+@pytest.mark.parametrize("multi", [False, True])
+def test_load_chunk_runs_equals_copy(multi):
+    """cof_load_chunk_runs (lo/hi over PCIe, nm rebuilt from N runs and vs from the segment
+    table on the device) yields exactly the planes cof_load_chunk copies: runs at offset 0,
+    at the chunk end, within one word, whole words, and n_bases both a multiple of 32 and not."""
+    rng = np.random.default_rng(61 + multi)
+    lens = [64_000, 33, 5_001, 96] if multi else [100_003]
+    seqs = [synth.random_genome_text(rng, n, b"ACGTacgtNnRy",
+                                     p=[.23, .17, .17, .23, .04, .04, .04, .04, .02, .01, .005, .005]) for n in lens]
+    seqs[0][:40] = ord("N")
+    seqs[0][1000:1003] = ord("n")
+    seqs[0][2048:4096] = ord("N")
+    seqs[-1][-9:] = ord("N")
+    chunks = search.plan_chunks(lens, 23, None, 0 if multi else None)
+    host = search.HostGenome(seqs, chunks)
+    srch = search.Searcher("N" * 21 + "RG", ["A" * 20 + "NNN"], [3])
+    for i, ch in enumerate(chunks):
+        w = cof.cof_plane_words(ch.n_bases)
+        a = torch.zeros((4, w), dtype=torch.int32, device="cuda")
+        b = torch.full((4, w), -1, dtype=torch.int32, device="cuda")   # garbage the rebuild must overwrite
+        da = srch.device_chunk(ch, a, host.segs[i])
+        db = srch.device_chunk(ch, b, host.segs[i])
+        cof.cof_load_chunk(host.chunk_struct(i), da, srch.stream)
+        cof.cof_load_chunk_runs(host.chunk_struct(i), host.runs[i], db, srch.stream)
+        torch.cuda.synchronize()
+        n = 4 if ch.multi else 3
+        assert torch.equal(a[:n], b[:n]), i
+    # this genome is N-fragmented (4% scattered N letters): load() keeps copying its planes
+    assert host.h2d_bytes <= host.bytes
