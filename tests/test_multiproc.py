@@ -6,6 +6,7 @@ import os
 import socket
 
 import numpy as np
+import pytest
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
@@ -24,16 +25,16 @@ def _oracle_chunk_hits(wl, ch):
     ranges = [(0, 0)] * len(wl.seqs)
     ranges[ch.chrom] = (ch.start, ch.start + ch.n_owned)
     h = oracle.search(wl.seqs, cfg.pattern, wl.guides, wl.thresholds, ranges=ranges)
-    out = np.zeros(len(h), dtype=cof.HIT_DTYPE)
+    out = np.zeros(len(h), dtype=cof.hit_dtype(cfg.L))
     for f in ("guide", "chrom", "pos", "strand", "mm", "site"):
         out[f] = h[f]
     return out
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, name="C3"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    wl = synth.make_workload("C3", scale=0.0005, n_guides=8)
+    wl = synth.make_workload(name, scale=0.0005 if name == "C3" else 0.003, n_guides=8)
     chunks = search.plan_chunks([len(s) for s in wl.seqs], wl.cfg.L, 40_000)
     mine = search.shard_for_rank(chunks, rank, world)
     lists = [_oracle_chunk_hits(wl, ch) for ch in mine]
@@ -47,11 +48,13 @@ def _worker(rank, world, port, q):
     dist.destroy_process_group()
 
 
-def test_two_rank_shard_gather_merge():
+@pytest.mark.parametrize("name", ["C3", "X1"])
+def test_two_rank_shard_gather_merge(name):
+    """C3 (cof_hit records) and X1 (L = 40: cof_hit64 records, cof_merge64)."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    ps = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    ps = [ctx.Process(target=_worker, args=(r, 2, port, q, name)) for r in range(2)]
     for p in ps:
         p.start()
     res = [q.get(timeout=300) for _ in range(2)]
