@@ -395,9 +395,17 @@ def random_genome_text(rng, n, alphabet=b"ACGT", p=None):
 
 
 def write_fasta(path, names, seqs, width: int = 60):
+    """FASTA with ``width``-column lines (whole lines laid out with numpy: a 3 Gbp genome
+    in seconds)."""
     with open(path, "wb") as f:
         for n, s in zip(names, seqs):
             f.write(b">" + n.encode() + b"\n")
-            b = s.tobytes()
-            for i in range(0, len(b), width):
-                f.write(b[i:i + width] + b"\n")
+            a = np.frombuffer(s, dtype=np.uint8) if isinstance(s, (bytes, bytearray)) else np.asarray(s, np.uint8)
+            full = len(a) // width
+            if full:
+                lines = np.empty((full, width + 1), dtype=np.uint8)
+                lines[:, :width] = a[:full * width].reshape(full, width)
+                lines[:, width] = 10
+                f.write(lines.tobytes())
+            if len(a) % width:
+                f.write(a[full * width:].tobytes() + b"\n")
