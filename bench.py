@@ -34,7 +34,9 @@ sys.path.insert(0, ROOT)
 from paper_conf_socc_jinv23_b200 import synth  # noqa: E402
 
 
-E2E_CHUNK_BASES = 250_000_000   # e2e: chromosomes packed into chunks of <= this many bases
+E2E_CHUNK_BASES = int(os.environ.get("COF_E2E_CHUNK_BASES", 250_000_000))  # e2e: pieces packed into chunks of <= this
+# e2e: chromosomes cut into pieces of <= this many window starts first (0 = whole chromosomes)
+E2E_PIECE_BASES = int(os.environ.get("COF_E2E_PIECE_BASES", 0))
 SHARD_PIECE_BASES = 16_000_000   # N > 1: chromosome pieces LPT-assigned to ranks
 
 
@@ -546,7 +548,9 @@ def main():
                        "chromosomes": len(wl.seqs), "guides": len(wl.guides), "threshold": cfg.threshold,
                        "pattern": cfg.pattern,
                        "chunking": "device: this rank's chromosomes as one multi-segment chunk; "
-                                   "e2e: packed chunks of <= 250 Mbp, pipelined",
+                                   f"e2e: packed chunks of <= {E2E_CHUNK_BASES / 1e6:g} Mbp"
+                                   + (f" (pieces <= {E2E_PIECE_BASES / 1e6:g} Mbp)" if E2E_PIECE_BASES else "")
+                                   + ", pipelined",
                        "parallelism": (f"LPT shards of <= {SHARD_PIECE_BASES // 10**6} Mbp chromosome pieces over "
                                        f"{world} GPUs" if world > 1 else "one GPU, whole genome as one chunk"),
                        "comparer": args.comparer,
@@ -621,7 +625,10 @@ def measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev=None):
     import torch
     import torch.distributed as dist
     from paper_conf_socc_jinv23_b200 import search
-    chunks = search.pack_pieces([p for ch in st.chunks for p in ch.pieces], E2E_CHUNK_BASES)
+    pieces = [p for ch in st.chunks for p in ch.pieces]
+    if E2E_PIECE_BASES:
+        pieces = search.split_pieces(pieces, E2E_PIECE_BASES, len(wl.cfg.pattern))
+    chunks = search.pack_pieces(pieces, E2E_CHUNK_BASES)
     st.e2e_host = search.HostGenome(wl.seqs, chunks)
     srch = search.Searcher(wl.cfg.pattern, wl.guides, wl.thresholds, device=dev)
     srch.reserve(max(ch.n_bases for ch in chunks), max(st.caps))

@@ -114,6 +114,17 @@ def plan_chunks(lengths, L: int, chunk_bases: int | None = None, pack_bases: int
     return pack_pieces(pieces, pack_bases)
 
 
+def split_pieces(pieces, max_owned: int, L: int):
+    """Cut every piece into pieces of at most ``max_owned`` window starts (same ownership
+    rule as plan_chunks: consecutive pieces overlap by L-1 bases)."""
+    out = []
+    for p in pieces:
+        for s in range(0, p.n_owned, max_owned):
+            owned = min(max_owned, p.n_owned - s)
+            out.append(Piece(p.chrom, p.chrom_off + s, owned, owned + L - 1))
+    return out
+
+
 def pack_pieces(pieces, pack_bases: int):
     """Consecutive pieces -> multi-segment chunks of at most ``pack_bases`` bases (0: one)."""
     out, cur, cur_bases = [], [], 0

@@ -230,6 +230,17 @@ def test_plan_chunks_cover_every_window_once():
                 assert e0 == s1
 
 
+def test_split_pieces_matches_plan_chunks():
+    """Re-cutting whole-chromosome pieces gives exactly the pieces plan_chunks makes
+    directly at that size (same ownership, same L-1 overlap)."""
+    L = 23
+    lengths = [0, 10, 23, 24, 100_000, 77_777]
+    whole = [p for ch in search.plan_chunks(lengths, L, None) for p in ch.pieces]
+    for cb in (1, 1000, 7919, 10**6):
+        direct = [p for ch in search.plan_chunks(lengths, L, cb) for p in ch.pieces]
+        assert search.split_pieces(whole, cb, L) == direct
+
+
 def test_shard_lpt_assigns_each_chunk_once():
     chunks = search.plan_chunks([l for _, l in synth.HG38], 23, None)
     for world in (1, 2, 4, 8):
