@@ -258,9 +258,9 @@ def cof_load_chunk(host: cof_chunk, dev: cof_chunk, stream=None):
 def cof_n_runs(nm, n_bases: int) -> np.ndarray:
     """[begin, end) runs of N bases of an nm plane, as an (n, 2) uint64 array."""
     cnt = ctypes.c_uint64(0)
-    cap = 64
+    cap = 4096
     while True:
-        runs = np.zeros((cap, 2), dtype=np.uint64)
+        runs = np.empty((cap, 2), dtype=np.uint64)
         st = lib.cof_n_runs(_ptr(nm), int(n_bases), runs.ctypes.data, cap, ctypes.byref(cnt))
         if st == COF_E_CAPACITY:
             cap = int(cnt.value)

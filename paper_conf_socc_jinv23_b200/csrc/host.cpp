@@ -20,6 +20,7 @@
 #include <unistd.h>
 
 #include <cuda_runtime.h>
+#include <emmintrin.h>
 #include <omp.h>
 
 #include "cof_internal.h"
@@ -71,6 +72,24 @@ static inline void pack_word(const uint8_t* codes, int n, uint32_t& lo, uint32_t
     lo = l; hi = h; nm = m;
 }
 
+// Pack 32 ASCII bases (any case) into one word of each plane, SSE2 (baseline x86-64):
+// clearing bit 5 folds exactly {X, x} onto X, so the four byte compares against A/C/G/T
+// give the same codes as g_code; every other byte is N (lo = hi = 0).
+static inline void pack32_ascii(const char* s, uint32_t& lo, uint32_t& hi, uint32_t& nm) {
+    const __m128i fold = _mm_set1_epi8((char)0xDF);
+    const __m128i a = _mm_and_si128(_mm_loadu_si128((const __m128i*)s), fold);
+    const __m128i b = _mm_and_si128(_mm_loadu_si128((const __m128i*)(s + 16)), fold);
+    auto eq = [&](char ch) -> uint32_t {
+        const __m128i c = _mm_set1_epi8(ch);
+        return (uint32_t)_mm_movemask_epi8(_mm_cmpeq_epi8(a, c)) |
+               ((uint32_t)_mm_movemask_epi8(_mm_cmpeq_epi8(b, c)) << 16);
+    };
+    const uint32_t A = eq('A'), C = eq('C'), G = eq('G'), T = eq('T');
+    lo = C | T;
+    hi = G | T;
+    nm = ~(A | C | G | T);
+}
+
 }  // namespace cof
 
 using namespace cof;
@@ -93,12 +112,7 @@ cof_status cof_pack(const char* ascii, uint64_t n, uint32_t* lo, uint32_t* hi, u
     const uint64_t words = cof_plane_words(n);
     const int64_t full = (int64_t)(n / 32);
 #pragma omp parallel for schedule(static)
-    for (int64_t w = 0; w < full; w++) {
-        uint8_t codes[32];
-        const uint8_t* src = (const uint8_t*)ascii + w * 32;
-        for (int b = 0; b < 32; b++) codes[b] = g_code[src[b]];
-        pack_word(codes, 32, lo[w], hi[w], nm[w]);
-    }
+    for (int64_t w = 0; w < full; w++) pack32_ascii(ascii + w * 32, lo[w], hi[w], nm[w]);
     uint64_t w = (uint64_t)full;
     if (n % 32) {
         uint8_t codes[32];
@@ -201,6 +215,95 @@ struct cof_fasta {
     std::vector<Rec> recs;
 };
 
+}  // extern "C"
+
+// One record by a byte-wise line walk from its '>' at d[i] (the general reader: any line
+// lengths, blank lines, CR/LF).  Returns the offset of the next record's '>' (or n).
+static size_t scan_record(const char* d, size_t n, size_t i, cof_fasta::Rec& r) {
+    size_t e = i;
+    while (e < n && d[e] != '\n') e++;
+    size_t name_end = i + 1;
+    while (name_end < e && d[name_end] != ' ' && d[name_end] != '\t' && d[name_end] != '\r') name_end++;
+    r.name.assign(d + i + 1, name_end - i - 1);
+    r.seq_off = e < n ? e + 1 : n;
+    size_t j = r.seq_off;
+    r.length = 0; r.line_bases = 0; r.line_bytes = 0; r.regular = true;
+    bool seen_short = false;
+    while (j < n && d[j] != '>') {
+        size_t le = j;
+        while (le < n && d[le] != '\n') le++;
+        size_t content_end = le;
+        if (content_end > j && d[content_end - 1] == '\r') content_end--;
+        uint64_t nb = content_end - j;
+        size_t lb = (le < n ? le + 1 : le) - j;
+        if (r.line_bases == 0 && nb > 0) { r.line_bases = nb; r.line_bytes = lb; }
+        else if (nb > 0) {
+            if (seen_short || nb > r.line_bases || (nb == r.line_bases && lb != r.line_bytes)) r.regular = false;
+            if (nb < r.line_bases) seen_short = true;
+        }
+        r.length += nb;
+        j = le < n ? le + 1 : le;
+    }
+    r.seq_end = j;
+    return j;
+}
+
+// The same record by its line geometry alone, for the common layout (every line but the
+// last has the first line's length and ending, the last line is not longer, no blank
+// lines): the newline count of [seq_off, seq_end) and the byte before every line end are
+// checked in parallel instead of walking the bytes.  False: use scan_record.
+static bool fast_record(const char* d, size_t n, size_t i, size_t next, cof_fasta::Rec& r) {
+    const char* e = (const char*)memchr(d + i, '\n', next - i);
+    if (!e) return false;
+    size_t name_end = i + 1;
+    const size_t hdr_end = (size_t)(e - d);
+    while (name_end < hdr_end && d[name_end] != ' ' && d[name_end] != '\t' && d[name_end] != '\r') name_end++;
+    r.name.assign(d + i + 1, name_end - i - 1);
+    r.seq_off = hdr_end + 1;
+    r.seq_end = next;
+    r.regular = true;
+    const size_t R = r.seq_end - r.seq_off;
+    if (R == 0) { r.length = 0; r.line_bases = 0; r.line_bytes = 0; return true; }
+    const char* f = (const char*)memchr(d + r.seq_off, '\n', R);
+    if (!f) return false;                                   // single line without newline: rare
+    const size_t lb = (size_t)(f - d) - r.seq_off + 1;     // first line incl. its '\n'
+    const bool crlf = lb >= 2 && d[r.seq_off + lb - 2] == '\r';
+    const size_t nb = lb - 1 - (crlf ? 1 : 0);
+    if (nb == 0) return false;                              // blank first line
+    const size_t F = R / lb, rem = R % lb;
+    // the last (partial) line: content, then CR LF / LF, or nothing at the end of the file
+    size_t last = rem;
+    if (rem) {
+        if (d[r.seq_end - 1] == '\n') { last--; if (last && crlf && d[r.seq_end - 2] == '\r') last--; }
+        else if (r.seq_end != n) return false;
+        if (last == 0) return false;                        // blank line before the next header
+    }
+    const int64_t FF = (int64_t)F;
+    int64_t bad = 0, nl = 0;
+    const char* base = d + r.seq_off;
+#pragma omp parallel for schedule(static) reduction(+ : bad) if (F > (1u << 16))
+    for (int64_t k = 1; k <= FF; k++) {
+        const char* le = base + k * lb - 1;
+        bad += (*le != '\n') | (crlf && le[-1] != '\r');
+    }
+    if (bad) return false;
+    const int64_t RR = (int64_t)R;
+#pragma omp parallel for schedule(static) reduction(+ : nl) if (R > (1u << 22))
+    for (int64_t k0 = 0; k0 < RR; k0 += 1 << 16) {
+        const int64_t k1 = std::min(RR, k0 + (1 << 16));
+        int64_t c = 0;
+        for (int64_t k = k0; k < k1; k++) c += base[k] == '\n';
+        nl += c;
+    }
+    if ((uint64_t)nl != F + (rem && d[r.seq_end - 1] == '\n' ? 1 : 0)) return false;
+    r.line_bases = nb;
+    r.line_bytes = lb;
+    r.length = (uint64_t)F * nb + last;
+    return true;
+}
+
+extern "C" {
+
 cof_status cof_fasta_open(const char* path, cof_fasta** out) {
     if (!path || !out) return set_error(COF_E_ARG, "cof_fasta_open: NULL argument");
     *out = nullptr;
@@ -215,47 +318,38 @@ cof_status cof_fasta_open(const char* path, cof_fasta** out) {
         void* m = mmap(nullptr, fa->size, PROT_READ, MAP_PRIVATE, fd, 0);
         if (m == MAP_FAILED) { close(fd); delete fa; return set_error(COF_E_IO, "cannot mmap %s", path); }
         fa->data = (const char*)m;
+        madvise(m, fa->size, MADV_WILLNEED);
     }
     const char* d = fa->data;
-    size_t i = 0, n = fa->size;
-    while (i < n) {
-        if (d[i] != '>') {
-            if (d[i] == '\n' || d[i] == '\r') { i++; continue; }
-            cof_fasta_close(fa);
-            return set_error(COF_E_IO, "%s: expected '>' at byte %zu", path, i);
+    const size_t n = fa->size;
+    size_t i = 0;
+    while (i < n && (d[i] == '\n' || d[i] == '\r')) i++;
+    if (i < n && d[i] != '>') {
+        cof_fasta_close(fa);
+        return set_error(COF_E_IO, "%s: expected '>' at byte %zu", path, i);
+    }
+    // record starts: '>' at the start of a line, found in parallel blocks with memchr
+    const int nt = std::max(1, omp_get_max_threads());
+    std::vector<std::vector<size_t>> found(nt);
+    const size_t blk = (n - i + nt - 1) / nt;
+#pragma omp parallel num_threads(nt)
+    {
+        const int t = omp_get_thread_num();
+        size_t a = i + (size_t)t * blk, b = std::min(n, a + blk);
+        while (a < b) {
+            const char* g = (const char*)memchr(d + a, '>', b - a);
+            if (!g) break;
+            const size_t p = (size_t)(g - d);
+            if (p == i || d[p - 1] == '\n') found[t].push_back(p);
+            a = p + 1;
         }
-        size_t e = i;
-        while (e < n && d[e] != '\n') e++;
-        cof_fasta::Rec r;
-        size_t name_end = i + 1;
-        while (name_end < e && d[name_end] != ' ' && d[name_end] != '\t' && d[name_end] != '\r') name_end++;
-        r.name.assign(d + i + 1, name_end - i - 1);
-        r.seq_off = e < n ? e + 1 : n;
-        size_t j = r.seq_off;
-        r.length = 0; r.line_bases = 0; r.line_bytes = 0; r.regular = true;
-        uint64_t last_line_bases = 0;
-        bool seen_short = false;
-        while (j < n && d[j] != '>') {
-            size_t le = j;
-            while (le < n && d[le] != '\n') le++;
-            size_t content_end = le;
-            if (content_end > j && d[content_end - 1] == '\r') content_end--;
-            uint64_t nb = content_end - j;
-            size_t lb = (le < n ? le + 1 : le) - j;
-            if (r.line_bases == 0 && nb > 0) { r.line_bases = nb; r.line_bytes = lb; }
-            else if (nb > 0) {
-                if (seen_short || nb > r.line_bases || (nb == r.line_bases && lb != r.line_bytes)) r.regular = false;
-                if (nb < r.line_bases) seen_short = true;
-            }
-            if (nb == 0 && le < n && d[le + 1 < n ? le + 1 : le] != '>') { /* blank line inside */ }
-            r.length += nb;
-            last_line_bases = nb;
-            j = le < n ? le + 1 : le;
-        }
-        (void)last_line_bases;
-        r.seq_end = j;
-        fa->recs.push_back(r);
-        i = j;
+    }
+    std::vector<size_t> starts;
+    for (auto& v : found) starts.insert(starts.end(), v.begin(), v.end());
+    fa->recs.resize(starts.size());
+    for (size_t k = 0; k < starts.size(); k++) {
+        const size_t next = k + 1 < starts.size() ? starts[k + 1] : n;
+        if (!fast_record(d, n, starts[k], next, fa->recs[k])) scan_record(d, n, starts[k], fa->recs[k]);
     }
     *out = fa;
     return COF_OK;
@@ -282,26 +376,55 @@ cof_status cof_fasta_pack(const cof_fasta* fa, uint32_t i, uint64_t first, uint6
     if (i >= fa->recs.size()) return set_error(COF_E_ARG, "cof_fasta_pack: record %u out of range", i);
     const auto& r = fa->recs[i];
     if (first + n > r.length) return set_error(COF_E_ARG, "cof_fasta_pack: range past record end");
-    std::vector<char> buf(n);
     if (r.regular && r.line_bases) {
-        // random access: base k is at seq_off + (k / line_bases) * line_bytes + k % line_bases
-        const int64_t nn = (int64_t)n;
-#pragma omp parallel for schedule(static) if (n > (1u << 20))
-        for (int64_t k0 = 0; k0 < nn; k0 += 4096) {
-            int64_t k1 = std::min(nn, k0 + 4096);
-            for (int64_t k = k0; k < k1; k++) {
-                uint64_t b = first + (uint64_t)k;
-                buf[k] = fa->data[r.seq_off + (b / r.line_bases) * r.line_bytes + b % r.line_bases];
+        // straight from the mapped file: each thread walks its word range line by line
+        // (base k is at seq_off + (k / line_bases) * line_bytes + k % line_bases), gathers
+        // 32 bases per word and packs them (pack32_ascii); the tail word is N-padded
+        const uint64_t LB = r.line_bases, LBY = r.line_bytes;
+        const char* seq = fa->data + r.seq_off;
+        const int64_t nw = (int64_t)((n + 31) / 32);
+#pragma omp parallel if (n > (1u << 20))
+        {
+            const int nt = omp_get_num_threads(), t = omp_get_thread_num();
+            const int64_t per = (nw + nt - 1) / nt;
+            const int64_t w0 = std::min(nw, (int64_t)t * per), w1 = std::min(nw, w0 + per);
+            if (w0 < w1) {
+                uint64_t b = first + (uint64_t)w0 * 32;
+                uint64_t line = b / LB, off = b % LB;
+                char tmp[32];
+                for (int64_t w = w0; w < w1; w++) {
+                    const uint64_t want = std::min<uint64_t>(32, n - (uint64_t)w * 32);
+                    uint64_t got = 0;
+                    if (off + want <= LB) {
+                        memcpy(tmp, seq + line * LBY + off, want);
+                        got = want;
+                        off += want;
+                    } else {
+                        while (got < want) {
+                            const uint64_t take = std::min(want - got, LB - off);
+                            memcpy(tmp + got, seq + line * LBY + off, take);
+                            got += take;
+                            off += take;
+                            if (off == LB) { off = 0; line++; }
+                        }
+                    }
+                    if (off == LB) { off = 0; line++; }
+                    if (want < 32) memset(tmp + want, 'N', 32 - want);
+                    pack32_ascii(tmp, lo[w], hi[w], nm[w]);
+                }
             }
         }
-    } else {
-        uint64_t b = 0, o = 0;
-        for (size_t j = r.seq_off; j < r.seq_end && o < n; j++) {
-            char c = fa->data[j];
-            if (c == '\n' || c == '\r') continue;
-            if (b >= first) buf[o++] = c;
-            b++;
-        }
+        const uint64_t words = cof_plane_words(n);
+        for (uint64_t w = (uint64_t)nw; w < words; w++) { lo[w] = 0; hi[w] = 0; nm[w] = ~0u; }
+        return COF_OK;
+    }
+    std::vector<char> buf(n);
+    uint64_t b = 0, o = 0;
+    for (size_t j = r.seq_off; j < r.seq_end && o < n; j++) {
+        char c = fa->data[j];
+        if (c == '\n' || c == '\r') continue;
+        if (b >= first) buf[o++] = c;
+        b++;
     }
     return cof_pack(buf.data(), n, lo, hi, nm);
 }

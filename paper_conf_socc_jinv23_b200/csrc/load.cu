@@ -1,3 +1,5 @@
+#include <omp.h>
+#include <vector>
 // Chunk load with the sparse planes built on the device (a2, host -> device).
 //
 // Paper: the host splits the genome into chunks and hands each to the device before the
@@ -79,13 +81,13 @@ using namespace cof;
 
 extern "C" {
 
-cof_status cof_n_runs(const uint32_t* nm, uint64_t n_bases, uint64_t* runs, uint64_t cap, uint64_t* n_runs) {
-    if (!nm || !n_runs || (!runs && cap)) return set_error(COF_E_ARG, "cof_n_runs: NULL argument");
-    uint64_t n = 0;
+// N runs of words [w0, w1) of an nm plane (bases < n_bases only), appended to out.
+static void n_runs_range(const uint32_t* nm, uint64_t n_bases, uint64_t w0, uint64_t w1,
+                         std::vector<uint64_t>& out) {
     bool open = false;
     uint64_t begin = 0;
     const uint64_t words = (n_bases + 31) / 32;
-    for (uint64_t w = 0; w < words; w++) {
+    for (uint64_t w = w0; w < w1; w++) {
         uint32_t v = nm[w];
         if (w == words - 1 && (n_bases & 31)) v &= ~0u >> (32 - (n_bases & 31));   // bases only
         if (!open && v == 0) continue;
@@ -96,15 +98,40 @@ cof_status cof_n_runs(const uint32_t* nm, uint64_t n_bases, uint64_t* runs, uint
             const bool isn = (v >> bit) & 1u;
             if (isn && !open) { open = true; begin = p; }
             else if (!isn && open) {
-                if (n < cap) { runs[2 * n] = begin; runs[2 * n + 1] = p; }
-                n++;
+                out.push_back(begin);
+                out.push_back(p);
                 open = false;
             }
         }
     }
     if (open) {
-        if (n < cap) { runs[2 * n] = begin; runs[2 * n + 1] = n_bases; }
-        n++;
+        out.push_back(begin);
+        out.push_back(std::min<uint64_t>(w1 * 32, n_bases));
+    }
+}
+
+cof_status cof_n_runs(const uint32_t* nm, uint64_t n_bases, uint64_t* runs, uint64_t cap, uint64_t* n_runs) {
+    if (!nm || !n_runs || (!runs && cap)) return set_error(COF_E_ARG, "cof_n_runs: NULL argument");
+    // word ranges scanned in parallel; a run cut by a range boundary is joined afterwards
+    const uint64_t words = (n_bases + 31) / 32;
+    const int nt = words > (1u << 20) ? std::max(1, omp_get_max_threads()) : 1;
+    std::vector<std::vector<uint64_t>> part(nt);
+    const uint64_t per = (words + nt - 1) / nt;
+#pragma omp parallel for schedule(static) num_threads(nt) if (nt > 1)
+    for (int t = 0; t < nt; t++)
+        n_runs_range(nm, n_bases, std::min(words, t * per), std::min(words, (t + 1) * per), part[t]);
+    uint64_t n = 0, last_end = ~0ull;
+    for (int t = 0; t < nt; t++) {
+        for (size_t k = 0; k < part[t].size(); k += 2) {
+            const uint64_t b = part[t][k], e = part[t][k + 1];
+            if (n && b == last_end) {                  // continues the previous range's run
+                if (n <= cap) runs[2 * (n - 1) + 1] = e;
+            } else {
+                if (n < cap) { runs[2 * n] = b; runs[2 * n + 1] = e; }
+                n++;
+            }
+            last_end = e;
+        }
     }
     *n_runs = n;
     if (n > cap) return set_error(COF_E_CAPACITY, "cof_n_runs: %llu runs exceed capacity %llu",

@@ -210,6 +210,44 @@ def test_fasta_reader(tmp_path):
         cof.Fasta(tmp_path / "missing.fa")
 
 
+@pytest.mark.parametrize("eol", [b"\n", b"\r\n"])
+def test_fasta_layouts_against_plain_canonicalisation(tmp_path, eol):
+    """The line-geometry reader (regular records) and the byte-walk reader (everything else)
+    both give canon(sequence) for any (first, n): line widths around the 32-base word,
+    CR/LF, a missing final newline, blank lines, bytes that differ from ACGT in bit 5 only."""
+    rng = np.random.default_rng(11)
+    alphabet = np.frombuffer(b"ACGTacgtNnRy\xc1\xe3-*", np.uint8)
+    seqs = [rng.choice(alphabet, n).tobytes() for n in (0, 1, 31, 32, 33, 95, 1000, 2049)]
+    for width in (1, 31, 32, 33, 60):
+        for tail in (b"", b"nofinal", b"blank"):
+            text = b""
+            for k, s in enumerate(seqs):
+                text += b">r%d some description" % k + eol
+                text += b"".join(s[o:o + width] + eol for o in range(0, len(s), width))
+                if tail == b"blank" and k == 2:
+                    text += eol
+            if tail == b"nofinal" and text.endswith(eol):
+                text = text[: -len(eol)]
+            path = tmp_path / f"w{width}{tail.decode()}.fa"
+            path.write_bytes(text)
+            fa = cof.Fasta(path)
+            assert len(fa) == len(seqs)
+            for i, s in enumerate(seqs):
+                assert fa.name(i) == f"r{i}" and fa.length(i) == len(s)
+                for first, n in ((0, len(s)), (min(5, len(s)), max(0, len(s) - 7)), (len(s) // 3, len(s) // 2)):
+                    w = cof.cof_plane_words(n)
+                    a = np.zeros((3, w), np.uint32)
+                    fa.pack(i, first, n, a[0], a[1], a[2])
+                    out = np.zeros(n, np.uint8)
+                    cof.cof_unpack(a[0], a[1], a[2], 0, n, out)
+                    assert out.tobytes() == _canon(s[first:first + n]), (width, tail, i, first, n)
+                    full = (n + 31) // 32
+                    assert (a[2][full:] == 0xFFFFFFFF).all() and not a[0][full:].any()
+                    if n % 32:
+                        assert a[2][n // 32] >> (n % 32) == (1 << (32 - n % 32)) - 1
+            fa.close()
+
+
 def test_plan_chunks_cover_every_window_once():
     L = 23
     lengths = [0, 10, 23, 24, 100_000, 77_777]
@@ -341,6 +379,31 @@ def test_n_runs_match_numpy(n):
     isn = np.frombuffer(_canon(seq.tobytes()), np.uint8) == ord("N") if n else np.zeros(0, bool)
     d = np.diff(np.concatenate([[0], isn.astype(np.int8), [0]]))
     exp = np.stack([np.flatnonzero(d == 1), np.flatnonzero(d == -1)], axis=1) if n else np.zeros((0, 2))
+    assert runs.shape == exp.shape and (runs == exp).all()
+
+
+def test_n_runs_parallel_ranges_join():
+    """A plane long enough for the threaded scan (> 2^20 words): runs that straddle the
+    word-range boundaries of any thread count 2..64 come back whole."""
+    n = 40_000_003
+    seq = np.full(n, ord("A"), np.uint8)
+    words = (n + 31) // 32
+    for nt in range(2, 65):
+        per = -(-words // nt)
+        for t in range(1, nt):
+            b = t * per * 32
+            if b < n:
+                seq[max(0, b - 3 - nt):b + 2 * nt] = ord("N")
+    rng = np.random.default_rng(7)
+    for s0 in rng.integers(0, n, 300):
+        seq[s0:s0 + int(rng.integers(1, 5000))] = ord("n")
+    seq[-1] = ord("N")
+    w = cof.cof_plane_words(n)
+    lo, hi, nm = (np.zeros(w, np.uint32) for _ in range(3))
+    cof.cof_pack(seq, n, lo, hi, nm)
+    runs = cof.cof_n_runs(nm, n)
+    d = np.diff(np.concatenate([[0], ((seq | 0x20) == ord("n")).astype(np.int8), [0]]))
+    exp = np.stack([np.flatnonzero(d == 1), np.flatnonzero(d == -1)], axis=1)
     assert runs.shape == exp.shape and (runs == exp).all()
 
 
