@@ -244,6 +244,9 @@ class HostGenome:
             cof.cof_load_chunk(self.chunk_struct(i), dev, stream)
 
 
+PLANE_BUFS = int(os.environ.get("COF_PLANE_BUFS", 3))   # device plane sets in the search_host pipeline
+
+
 class Searcher:
     """One GPU's pipeline for a fixed (pattern, guides, thresholds) plan."""
 
@@ -336,11 +339,14 @@ class Searcher:
         idx = list(range(len(host.chunks)) if indices is None else indices)
         max_bases = max((host.chunks[i].n_bases for i in idx), default=1)
         self.reserve(max_bases, max(self._hits_cap, 1 << 16))
-        if not hasattr(self, "d_planes2") or self.d_planes2.shape != self.d_planes.shape:
-            self.d_planes2 = torch.empty_like(self.d_planes)
+        if not hasattr(self, "d_planes_more") or self.d_planes_more[0].shape != self.d_planes.shape:
+            # PLANE_BUFS device plane sets: the H2D of chunk j+1 waits only for the
+            # decoration of chunk j+1-PLANE_BUFS, not for the chunk just before it
+            self.d_planes_more = [torch.empty_like(self.d_planes) for _ in range(PLANE_BUFS - 1)]
             self.copy_stream = torch.cuda.Stream(self.device)
             self.d2h_stream = torch.cuda.Stream(self.device)
-        planes = [self.d_planes, self.d_planes2]
+        planes = [self.d_planes] + self.d_planes_more
+        nb = len(planes)
         rec_free = [None, None]
         ordered = all(a < b for a, b in zip(idx, idx[1:]))
         use_out = out is not None and ordered
@@ -351,8 +357,8 @@ class Searcher:
         total = 0
         overflow = False
         with torch.cuda.device(self.device):
-            loaded = [None, None]
-            freed = [None, None]
+            loaded = [None] * nb
+            freed = [None] * nb
 
             def load(j, k):
                 with torch.cuda.stream(self.copy_stream):
@@ -365,20 +371,20 @@ class Searcher:
                     loaded[k] = ev
                     return dch
 
-            dchs = [None, None]
+            dchs = [None] * nb
             if idx:
                 dchs[0] = load(0, 0)
             for j, i in enumerate(idx):
-                k = j & 1
+                k, kr = j % nb, j & 1
                 self.stream.wait_event(loaded[k])
                 if j + 1 < len(idx):
-                    dchs[(j + 1) & 1] = load(j + 1, (j + 1) & 1)
+                    dchs[(j + 1) % nb] = load(j + 1, (j + 1) % nb)
                 _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned)
                 if self.d_records is None or nh > self._rec_cap:
                     self._reserve_records(nh)
-                recs = self.d_records[k]
-                if rec_free[k] is not None:          # the D2H of chunk j-2 from this buffer is done
-                    self.stream.wait_event(rec_free[k])
+                recs = self.d_records[kr]
+                if rec_free[kr] is not None:         # the D2H of chunk j-2 from this buffer is done
+                    self.stream.wait_event(rec_free[kr])
                 cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, recs, ws[j], self.stream,
                                  cap=self._rec_cap)
                 fr = torch.cuda.Event()
@@ -400,7 +406,7 @@ class Searcher:
                                                                    non_blocking=True)
                         ev = torch.cuda.Event()
                         ev.record(self.d2h_stream)
-                    rec_free[k] = ev
+                    rec_free[kr] = ev
                 results.append(dst)
                 total += nh
             self.d2h_stream.synchronize()
