@@ -292,9 +292,10 @@ class Searcher:
                                   segs if segs is not None else cof.make_segments(ch.segments()))
         return cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, p[0], p[1], p[2])
 
-    def run_device_chunk(self, dchunk: cof.cof_chunk, items_cap: int):
-        """find -> compare -> sort on the device; returns (n_fwd, n_rev, n_hits).
-        Grows the hit buffer and re-runs compare on capacity overflow."""
+    def run_device_chunk(self, dchunk: cof.cof_chunk, items_cap: int, counts: bool = True):
+        """find -> compare -> sort on the device; returns (n_fwd, n_rev, n_hits) (item counts
+        None on the fused path with ``counts=False``).  Grows the hit buffer and re-runs
+        compare on capacity overflow."""
         s = self.stream
         if not self.fused and self.d_items.shape[1] < items_cap:   # path switched after reserve()
             self.d_items = torch.empty((2, items_cap), dtype=torch.int32, device=self.device)
@@ -317,10 +318,12 @@ class Searcher:
                     raise
                 _, _, need = cof.cof_read_counts(self.plan, self.plan_dev, s)
                 self.reserve(self._cap_bases, int(need * 1.25) + 1024)
+        if self.fused:
+            # item counts: compare's count read left the stream idle, so this sync is short;
+            # after the sort it would block the host until the sort is done (a pipeline bubble)
+            nf, nr = cof.cof_read_counts(self.plan, self.plan_dev, s)[:2] if counts else (None, None)
         cof.cof_sort_hits(self.plan, self.plan_dev, dchunk, self.d_hits, self.d_tmp, self._hits_cap, nh,
                           self.d_sort_ws, s)
-        if self.fused:
-            nf, nr, _ = cof.cof_read_counts(self.plan, self.plan_dev, s)
         return nf, nr, nh
 
     def search_host(self, host: HostGenome, indices=None, out=None, decorate="device"):
@@ -379,7 +382,7 @@ class Searcher:
                 self.stream.wait_event(loaded[k])
                 if j + 1 < len(idx):
                     dchs[(j + 1) % nb] = load(j + 1, (j + 1) % nb)
-                _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned)
+                _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned, counts=False)
                 if self.d_records is None or nh > self._rec_cap:
                     self._reserve_records(nh)
                 recs = self.d_records[kr]
