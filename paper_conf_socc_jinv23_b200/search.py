@@ -363,12 +363,22 @@ class Searcher:
             loaded = [None] * nb
             freed = [None] * nb
 
+            trace = [] if os.environ.get("COF_TRACE") else None   # (what, chunk, stream, event)
+
+            def mark(what, j, stream):
+                if trace is not None:
+                    e = torch.cuda.Event(enable_timing=True)
+                    e.record(stream)
+                    trace.append((what, j, e))
+
             def load(j, k):
                 with torch.cuda.stream(self.copy_stream):
                     if freed[k] is not None:
                         self.copy_stream.wait_event(freed[k])
+                    mark("h2d0", j, self.copy_stream)
                     dch = self.device_chunk(host.chunks[idx[j]], planes[k], host.segs[idx[j]])
                     host.load(idx[j], dch, self.copy_stream)
+                    mark("h2d1", j, self.copy_stream)
                     ev = torch.cuda.Event()
                     ev.record(self.copy_stream)
                     loaded[k] = ev
@@ -382,6 +392,7 @@ class Searcher:
                 self.stream.wait_event(loaded[k])
                 if j + 1 < len(idx):
                     dchs[(j + 1) % nb] = load(j + 1, (j + 1) % nb)
+                mark("dev0", j, self.stream)
                 _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned, counts=False)
                 if self.d_records is None or nh > self._rec_cap:
                     self._reserve_records(nh)
@@ -390,6 +401,7 @@ class Searcher:
                     self.stream.wait_event(rec_free[kr])
                 cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, recs, ws[j], self.stream,
                                  cap=self._rec_cap)
+                mark("dev1", j, self.stream)
                 fr = torch.cuda.Event()
                 fr.record(self.stream)
                 freed[k] = fr
@@ -414,6 +426,12 @@ class Searcher:
                 total += nh
             self.d2h_stream.synchronize()
             self.stream.synchronize()
+            if trace:   # COF_TRACE=1: per-chunk H2D / device intervals in ms from the first mark
+                import json
+                import sys
+                t0 = trace[0][2]
+                print(json.dumps({"search_host_trace": [(w, j, round(t0.elapsed_time(e), 3)) for w, j, e in trace]}),
+                      file=sys.stderr)
             for j in range(len(idx)):
                 cof.cof_decorate_check(ws[j], self.stream)
         if use_out and not overflow:
