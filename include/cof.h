@@ -147,6 +147,13 @@ cof_status cof_n_runs(const uint32_t *nm, uint64_t n_bases, uint64_t *runs, uint
  * the chunk or a segment that leaves it. */
 cof_status cof_load_chunk_runs(const cof_chunk *host, const uint64_t *runs, uint64_t n_runs,
                                cof_chunk *dev, cof_stream s);
+/* The same with the two halves on two streams: the lo/hi DMA on s_copy, the nm / vs fill
+ * kernels on s_fill (e.g. the stream that runs this chunk's kernels, so the fills are not
+ * queued behind a copy engine waiting on a persistent kernel, and the DMA queue holds
+ * DMA only).  The caller orders s_fill's later work after s_copy (an event) before
+ * reading lo/hi.  Arguments, ownership and errors as cof_load_chunk_runs. */
+cof_status cof_load_chunk_runs_split(const cof_chunk *host, const uint64_t *runs, uint64_t n_runs,
+                                     cof_chunk *dev, cof_stream s_copy, cof_stream s_fill);
 
 /* ------------------------------------------------------------------ FASTA (M2)
  * Minimal indexed FASTA reader ("single- or multi-sequence data format"):

@@ -90,6 +90,7 @@ def _load():
         "cof_read_counts": (I32, [P, P, P, P]),
         "cof_n_runs": (I32, [P, U64, P, U64, P]),
         "cof_load_chunk_runs": (I32, [P, P, U64, P, P]),
+        "cof_load_chunk_runs_split": (I32, [P, P, U64, P, P, P]),
         "cof_collect": (I32, [P, P, P, P, U64, P, P]),
         "cof_collect64": (I32, [P, P, P, P, U64, P, P]),
         "cof_merge": (I32, [P, P, U32, P]),
@@ -129,7 +130,7 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_fasta_count", "cof_fasta_name", "cof_fasta_length", "cof_fasta_pack",
                        "cof_find_workspace_bytes", "cof_find_pam", "cof_compare",
                        "cof_sort_workspace_bytes", "cof_sort_hits", "cof_read_counts",
-                       "cof_n_runs", "cof_load_chunk_runs", "cof_collect", "cof_collect64", "cof_merge", "cof_merge64",
+                       "cof_n_runs", "cof_load_chunk_runs", "cof_load_chunk_runs_split", "cof_collect", "cof_collect64", "cof_merge", "cof_merge64",
                        "cof_decorate_workspace_bytes", "cof_decorate", "cof_decorate64",
                        "cof_decorate_check", "cof_find_compare_supported",
                        "cof_find_compare_workspace_bytes", "cof_find_compare", "cof_find_masks",
@@ -274,6 +275,13 @@ def cof_load_chunk_runs(host: cof_chunk, runs: np.ndarray, dev: cof_chunk, strea
     runs = np.ascontiguousarray(runs, dtype=np.uint64)
     _check(lib.cof_load_chunk_runs(ctypes.addressof(host), runs.ctypes.data if len(runs) else None, len(runs),
                                    ctypes.addressof(dev), _stream(stream)))
+
+
+def cof_load_chunk_runs_split(host: cof_chunk, runs: np.ndarray, dev: cof_chunk, copy_stream, fill_stream):
+    """cof_load_chunk_runs with the lo/hi DMA on ``copy_stream`` and the fills on ``fill_stream``."""
+    runs = np.ascontiguousarray(runs, dtype=np.uint64)
+    _check(lib.cof_load_chunk_runs_split(ctypes.addressof(host), runs.ctypes.data if len(runs) else None, len(runs),
+                                         ctypes.addressof(dev), _stream(copy_stream), _stream(fill_stream)))
 
 
 def cof_find_workspace_bytes(n_bases: int) -> int:

@@ -139,8 +139,8 @@ cof_status cof_n_runs(const uint32_t* nm, uint64_t n_bases, uint64_t* runs, uint
     return COF_OK;
 }
 
-cof_status cof_load_chunk_runs(const cof_chunk* host, const uint64_t* runs, uint64_t n_runs, cof_chunk* dev,
-                               cof_stream s) {
+static cof_status load_runs(const cof_chunk* host, const uint64_t* runs, uint64_t n_runs, cof_chunk* dev,
+                            cudaStream_t st, cudaStream_t fs) {
     if (!host || !dev || !host->lo || !host->hi || !dev->lo || !dev->hi || !dev->nm || (!runs && n_runs))
         return set_error(COF_E_ARG, "cof_load_chunk_runs: NULL argument");
     if (host->n_segs && (!host->segs || !dev->vs))
@@ -151,17 +151,16 @@ cof_status cof_load_chunk_runs(const cof_chunk* host, const uint64_t* runs, uint
                              (unsigned long long)i);
     const uint64_t words = cof_plane_words(host->n_bases);
     const size_t bytes = words * sizeof(uint32_t);
-    cudaStream_t st = (cudaStream_t)s;
     cudaError_t e;
     if ((e = cudaMemcpyAsync(dev->lo, host->lo, bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess ||
         (e = cudaMemcpyAsync(dev->hi, host->hi, bytes, cudaMemcpyHostToDevice, st)) != cudaSuccess)
         return cuda_error(e, "cof_load_chunk_runs");
     FillArgs f{dev->nm, host->n_segs ? dev->vs : nullptr, words, host->n_bases};
     const uint64_t blocks = std::min<uint64_t>((words + 255) / 256, 148 * 8);
-    cof_fill_planes<<<(uint32_t)std::max<uint64_t>(blocks, 1), 256, 0, st>>>(f);
+    cof_fill_planes<<<(uint32_t)std::max<uint64_t>(blocks, 1), 256, 0, fs>>>(f);
     if ((e = cudaGetLastError()) != cudaSuccess) return cuda_error(e, "cof_fill_planes launch");
     count_launches(1);
-    cof_status r = set_runs(dev->nm, runs, n_runs, st);
+    cof_status r = set_runs(dev->nm, runs, n_runs, fs);
     if (r != COF_OK) return r;
     if (host->n_segs) {
         std::vector<uint64_t> own(2 * (size_t)host->n_segs);
@@ -172,7 +171,7 @@ cof_status cof_load_chunk_runs(const cof_chunk* host, const uint64_t* runs, uint
             own[2 * k] = g.chunk_off;
             own[2 * k + 1] = g.chunk_off + g.n_owned;
         }
-        r = set_runs(dev->vs, own.data(), host->n_segs, st);
+        r = set_runs(dev->vs, own.data(), host->n_segs, fs);
         if (r != COF_OK) return r;
     }
     dev->chrom = host->chrom;
@@ -183,6 +182,16 @@ cof_status cof_load_chunk_runs(const cof_chunk* host, const uint64_t* runs, uint
     dev->segs = host->segs;
     if (!host->n_segs) dev->vs = nullptr;
     return COF_OK;
+}
+
+cof_status cof_load_chunk_runs(const cof_chunk* host, const uint64_t* runs, uint64_t n_runs, cof_chunk* dev,
+                               cof_stream s) {
+    return load_runs(host, runs, n_runs, dev, (cudaStream_t)s, (cudaStream_t)s);
+}
+
+cof_status cof_load_chunk_runs_split(const cof_chunk* host, const uint64_t* runs, uint64_t n_runs, cof_chunk* dev,
+                                     cof_stream s_copy, cof_stream s_fill) {
+    return load_runs(host, runs, n_runs, dev, (cudaStream_t)s_copy, (cudaStream_t)s_fill);
 }
 
 }  // extern "C"

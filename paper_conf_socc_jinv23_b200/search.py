@@ -234,16 +234,20 @@ class HostGenome:
         return sum(2 * p.shape[1] * 4 + r.nbytes if self._use_runs(i) else p.numel() * 4
                    for i, (p, r) in enumerate(zip(self.planes, self.runs)))
 
-    def load(self, i, dev: cof.cof_chunk, stream):
+    def load(self, i, dev: cof.cof_chunk, stream, fill_stream=None):
         """H2D of chunk i into the device chunk ``dev``: lo/hi copied and nm/vs rebuilt on the
-        device from the N runs / segments (cof_load_chunk_runs), or every plane copied
-        (cof_load_chunk) when the genome is so N-fragmented that the runs are larger."""
-        if self._use_runs(i):
+        device from the N runs / segments (cof_load_chunk_runs; the fill kernels on
+        ``fill_stream`` if given), or every plane copied (cof_load_chunk) when the genome is
+        so N-fragmented that the runs are larger."""
+        if self._use_runs(i) and fill_stream is not None:
+            cof.cof_load_chunk_runs_split(self.chunk_struct(i), self.runs[i], dev, stream, fill_stream)
+        elif self._use_runs(i):
             cof.cof_load_chunk_runs(self.chunk_struct(i), self.runs[i], dev, stream)
         else:
             cof.cof_load_chunk(self.chunk_struct(i), dev, stream)
 
 
+SPLIT_FILL = os.environ.get("COF_SPLIT_FILL", "1") != "0"
 PLANE_BUFS = int(os.environ.get("COF_PLANE_BUFS", 2))   # device plane sets in the search_host pipeline (3 measured no faster)
 
 
@@ -377,7 +381,10 @@ class Searcher:
                         self.copy_stream.wait_event(freed[k])
                     mark("h2d0", j, self.copy_stream)
                     dch = self.device_chunk(host.chunks[idx[j]], planes[k], host.segs[idx[j]])
-                    host.load(idx[j], dch, self.copy_stream)
+                    # fills on the compute stream: that stream last used this plane set, and on
+                    # the copy stream they would queue behind the running persistent kernels
+                    # (COF_TRACE showed H2D intervals ~40% longer than the bytes need)
+                    host.load(idx[j], dch, self.copy_stream, fill_stream=self.stream if SPLIT_FILL else None)
                     mark("h2d1", j, self.copy_stream)
                     ev = torch.cuda.Event()
                     ev.record(self.copy_stream)
