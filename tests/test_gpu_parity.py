@@ -354,10 +354,17 @@ def test_load_chunk_runs_equals_copy(multi):
         b = torch.full((4, w), -1, dtype=torch.int32, device="cuda")   # garbage the rebuild must overwrite
         da = srch.device_chunk(ch, a, host.segs[i])
         db = srch.device_chunk(ch, b, host.segs[i])
+        c = torch.full((4, w), -1, dtype=torch.int32, device="cuda")
+        dc = srch.device_chunk(ch, c, host.segs[i])
         cof.cof_load_chunk(host.chunk_struct(i), da, srch.stream)
         cof.cof_load_chunk_runs(host.chunk_struct(i), host.runs[i], db, srch.stream)
+        side = torch.cuda.Stream()
+        torch.cuda.synchronize()
+        # the two halves on two streams (DMA on a side stream, fills on the main one)
+        cof.cof_load_chunk_runs_split(host.chunk_struct(i), host.runs[i], dc, side, srch.stream)
         torch.cuda.synchronize()
         n = 4 if ch.multi else 3
         assert torch.equal(a[:n], b[:n]), i
+        assert torch.equal(a[:n], c[:n]), i
     # this genome is N-fragmented (4% scattered N letters): load() keeps copying its planes
     assert host.h2d_bytes <= host.bytes
