@@ -247,7 +247,7 @@ class HostGenome:
             cof.cof_load_chunk(self.chunk_struct(i), dev, stream)
 
 
-SPLIT_FILL = os.environ.get("COF_SPLIT_FILL", "1") != "0"
+SPLIT_FILL = os.environ.get("COF_SPLIT_FILL", "0") == "1"   # measured slower end to end
 PLANE_BUFS = int(os.environ.get("COF_PLANE_BUFS", 2))   # device plane sets in the search_host pipeline (3 measured no faster)
 
 
