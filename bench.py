@@ -140,6 +140,7 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl
     # fused find+compare (finder masks -> comparer, no item lists) unless the guide table is
     # too large for it or COF_FUSED=0; the two-call path writes / reads ordered item lists
     st.fused = search.use_fused(st.plan, len(guides))
+    st.path_name = "fused" if st.fused else "twocall"
     st.items = torch.empty((2, 1 if st.fused else max_owned), dtype=torch.int32, device=st.device)
     st.find_ws = torch.empty(cof.cof_find_compare_workspace_bytes(max(ch.n_bases for ch in chunks)),
                              dtype=torch.uint8, device=st.device)
@@ -281,6 +282,50 @@ def measure_from_fasta(wl, dev, runs: int = 2):
                     "decoration, D2H of the records); wall clock, best of runs"}
 
 
+def input_sha256(wl):
+    """SHA-256 over the synthetic input exactly as the search sees it: every chromosome's
+    name and ASCII bases, then the pattern and each (guide, threshold)."""
+    import hashlib
+    h = hashlib.sha256()
+    for name, seq in zip(wl.names, wl.seqs):
+        h.update(name.encode() + b"\n")
+        h.update(memoryview(np.ascontiguousarray(seq)))
+        h.update(b"\n")
+    h.update(wl.cfg.pattern.encode() + b"\n")
+    for g, t in zip(wl.guides, wl.thresholds):
+        h.update(f"{g} {int(t)}\n".encode())
+    return h.hexdigest()
+
+
+def host_info():
+    """CPU model and core counts of the box (record the lscpu model)."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    model = ln.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"cpu_model": model, "cpus": os.cpu_count(), "affinity_cpus": len(os.sched_getaffinity(0))}
+
+
+def oracle_single_thread():
+    """the oracle on ONE thread over the whole C1 and C2 workloads (seconds
+    each), wall clock, with the hit counts it found."""
+    from oracle import oracle as orc
+    out = {}
+    for name in ("C1", "C2"):
+        w = synth.make_workload(name)
+        t = time.perf_counter()
+        h = orc.search(w.seqs, w.cfg.pattern, w.guides, w.thresholds, threads=1)
+        dt = time.perf_counter() - t
+        out[name] = {"s": round(dt, 3), "Gbases_per_s": round(w.total_bases / dt / 1e9, 6), "hits": int(len(h)),
+                     "genome_bases": int(w.total_bases), "guides": len(w.guides)}
+    return out
+
+
 # ----------------------------------------------------------------------------- oracle arm
 def oracle_sample(wl, target_s: float, threads: int):
     """Bounded sample for the CPU oracle: the first B window starts after the leading
@@ -381,8 +426,12 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
-    ap.add_argument("--from-fasta", action="store_true",
-                    help="also time the search from a FASTA file (SURVEY §8(d) (iii); writes it under /tmp)")
+    ap.add_argument("--no-fasta", action="store_true",
+                    help="skip the search from a FASTA file (SURVEY §8(d) (iii), fasta_e2e; it writes the "
+                         "genome as FASTA under /tmp first)")
+    ap.add_argument("--from-fasta", action="store_true", help=argparse.SUPPRESS)   # the default now
+    ap.add_argument("--no-single-thread", action="store_true",
+                    help="skip the single-thread oracle times of C1 and C2 (SURVEY §8(d))")
     ap.add_argument("--bulge", default=None, help="D,R: time the bulge search (max DNA, RNA bulge sizes)")
     ap.add_argument("--n-guides", type=int, default=None, help="override the config's guide count (scaling study)")
     args = ap.parse_args()
@@ -425,6 +474,10 @@ def main():
     mine = [search.pack_shard(shards[rank])]          # this rank's pieces as ONE chunk
     wl, st = prepare_workload(cfgname, args.scale, chunks=mine, device=dev, n_guides=args.n_guides)
     genome_bases = wl.total_bases
+    sha = None
+    if rank == 0:   # SHA-256 of the input (genome text, pattern, guides, thresholds), off the timed path
+        import concurrent.futures
+        sha = concurrent.futures.ThreadPoolExecutor(1).submit(input_sha256, wl)
     my_items = sum(c[0] + c[1] for c in st.counts)
     comps_mine = my_items * len(wl.guides)
 
@@ -488,7 +541,7 @@ def main():
         achieved = ops / (cmp_ms * 1e-3) / 1e12 if cmp_ms > 0 else 0.0
         pk = 2.0 * float(peaks.get("bf16_tflops", 2250.0 / 2))
         roofline = {"bound": "tensor", "kernel": "cof_comparer_mma", "achieved": achieved, "peak": pk,
-                    "unit": "TFLOP/s", "frac": achieved / pk, "traffic": traffic_for("cof_comparer_mma", st),
+                    "unit": "TFLOP/s", "frac": achieved / pk, "traffic": traffic_for("cof_comparer_mma", st, cfgname),
                     "peak_basis": f"int8 dense = 2 x measured bf16 dense ({peaks.get('bf16_tflops')} TFLOP/s); "
                                   f"ops = 2 x items x guides x K={kpad} (int8 OPs)",
                     "comparisons_per_s": cmp_rate, "alu_table_roof_comparisons_per_s": roof["peak"],
@@ -497,9 +550,12 @@ def main():
         roofline = {"bound": "alu", "kernel": f"cof_comparer_{'fused' if st.fused else args.comparer}",
                     "achieved": cmp_rate, "peak": roof["peak"], "unit": "comparisons/s",
                     "frac": cmp_rate / roof["peak"] if roof["peak"] else None,
-                    "traffic": traffic_for("cof_comparer", st),
+                    "traffic": traffic_for("cof_comparer", st, cfgname),
                     "peak_basis": roof["basis"], "launches": n_cmp_launch,
-                    "share_of_step": cmp_ms_max / ms_total if ms_total else None}
+                    "share_of_step": cmp_ms_max / ms_total if ms_total else None,
+                    # the same rate against SURVEY §8(d)'s roof (one POPC per comparison)
+                    "frac_popc_roof": cmp_rate / popc_roof(n_sm, sm_max),
+                    "popc_roof": popc_roof(n_sm, sm_max)}
 
     # finder roofline (HBM): algorithmic bytes of the search kernel per step
     plane_bytes = sum(cof.cof_plane_words(ch.n_bases) * 4 * (4 if ch.multi else 3) for ch in st.chunks)
@@ -515,15 +571,19 @@ def main():
     finder_roof = {"bound": "hbm", "kernel": "cof_finder_kernel", "achieved": round(find_gbs, 1),
                    "peak": hbm_peak, "unit": "GB/s", "frac": find_gbs / hbm_peak,
                    "bytes_per_step": int(find_bytes), "basis": find_basis,
-                   "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_finder_kernel", st)}
+                   "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_finder_kernel", st, cfgname)}
 
     e2e = None
     if not args.no_e2e:
         e2e = measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev)
 
     fasta = None
-    if rank == 0 and world == 1 and args.from_fasta:
+    if rank == 0 and world == 1 and not args.no_fasta:
         fasta = measure_from_fasta(wl, dev)
+
+    single = None
+    if rank == 0 and world == 1 and not args.no_cpu and not args.no_single_thread:
+        single = oracle_single_thread()
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -563,7 +623,10 @@ def main():
             "e2e": e2e,
             "fasta_e2e": fasta,
             "cpu_baseline": cpu,
+            "oracle_single_thread": single,
             "peaks_source": peak_src,
+            "host": host_info(),
+            "input_sha256": sha.result() if sha is not None else None,
         }
         print(json.dumps(line))
     if world > 1:
@@ -571,16 +634,25 @@ def main():
     return 0
 
 
-def traffic_for(kernel, st):
-    """DRAM bytes per launch of ``kernel`` from the committed ncu --set full capture
-    (profiles/roofline_traffic.json), or None."""
+def traffic_for(kernel, st, cfgname):
+    """DRAM bytes per launch of ``kernel`` on THIS config and path from a committed ncu
+    --set full capture (profiles/roofline_traffic.json, keyed "<config>:<kernel>_<path>"),
+    or None when no capture of that config and path is committed."""
     try:
         with open(os.path.join(ROOT, "profiles", "roofline_traffic.json")) as f:
             d = json.load(f)
-        key = f"{kernel}_{'fused' if st.fused else 'twocall'}"
-        return d.get(key, {}).get("dram_bytes_per_launch")
+        key = f"{cfgname}:{kernel}_{st.path_name}"
+        e = d.get(key)
+        return None if e is None else {"dram_bytes_per_launch": e["dram_bytes_per_launch"], "capture": e.get("capture")}
     except Exception:
         return None
+
+
+def popc_roof(n_sm, sm_mhz):
+    """SURVEY §8(d)'s comparer roof: one POPC per comparison on the quarter-rate POPC pipe,
+    16/clk/SM (measured 4.54e12 POPC/s = 15.6/clk/SM at 1965 MHz,
+    profiles/microbench_pipes_r1.txt)."""
+    return 16.0 * n_sm * sm_mhz * 1e6
 
 
 def comparer_roof(plan, n_sm, sm_mhz, impl):
@@ -592,7 +664,7 @@ def comparer_roof(plan, n_sm, sm_mhz, impl):
     block = 2*NP wavefronts per 32 items x 32 guides at 1 wavefront/clk/SM."""
     clk = sm_mhz * 1e6
     if impl == "popc":
-        return {"peak": 16 * n_sm * clk, "basis": "POPC pipe 16/clk/SM x SMs x max SM clock"}
+        return {"peak": popc_roof(n_sm, sm_mhz), "basis": "POPC pipe 16/clk/SM x SMs x max SM clock"}
     # (mma: the table comparer's ALU roof is reported beside the tensor roofline)
     import importlib.util
     spec = importlib.util.spec_from_file_location(
@@ -613,7 +685,10 @@ def comparer_roof(plan, n_sm, sm_mhz, impl):
     fa = int(hdr.split(":")[1].split("full")[0])
     ha = int(hdr.split(",")[1].split("half")[0])
     alu_ops = 2 * fa + 2 * ha + 6 + 1
-    alu_rate = 64.0 * 32 / alu_ops           # comparisons / clk / SM (64 LOP3/clk/SM, measured)
+    # 64 LOP3/clk/SM: the ALU pipe issues one warp instruction per 2 cycles per SMSP
+    # (B300_MICROARCH.md "Pipe rates"); measured 1.855e13 LOP3/s = 63.8/clk/SM at the
+    # 1965 MHz max clock (profiles/microbench_pipes_r1.txt; its own clock column is wrong)
+    alu_rate = 64.0 * 32 / alu_ops           # comparisons / clk / SM
     lds_rate = 32.0 * 32 / (2 * npairs)      # comparisons / clk / SM
     per_clk = min(alu_rate, lds_rate)
     return {"peak": per_clk * n_sm * clk,
@@ -622,17 +697,58 @@ def comparer_roof(plan, n_sm, sm_mhz, impl):
 
 
 def measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev=None):
+    """``e2e``: the same search through the public API from pinned packed HOST planes,
+    wall clock, H2D + kernels + D2H of the decorated records inside the timed region.
+    N = 1: Searcher.search_host over packed chunks of <= 250 Mbp into the caller's pinned
+    result buffer.  N > 1: search.search_dist's path -- the genome cut into <= 64 Mbp work
+    units (genome order), LPT-assigned to the ranks, each rank's search_host pipeline, then
+    merge_dist (per-chunk counts all-reduced -> offsets -> every rank writes its records
+    into one shared-memory result): the merge is inside the timed step."""
     import torch
     import torch.distributed as dist
     from paper_conf_socc_jinv23_b200 import search
+    L = len(wl.cfg.pattern)
+    if world > 1:
+        rank = dist.get_rank()
+        gchunks = search.plan_chunks([len(x) for x in wl.seqs], L, search.MULTI_CHUNK_BASES)
+        mine = search.shard_indices(gchunks, world)[rank]
+        host = search.HostGenome(wl.seqs, [gchunks[i] for i in mine])
+        srch = search.Searcher(wl.cfg.pattern, wl.guides, wl.thresholds, device=dev)
+        srch.reserve(max(ch.n_bases for ch in host.chunks), max(st.caps))
+
+        def step():
+            per = {}
+            srch.search_host(host, sink=lambda j, r: per.__setitem__(mine[j], r))
+            merged = search.merge_dist(per, len(gchunks), srch.hit_dtype)
+            d2h = sum(len(r) for r in per.values()) * srch.hit_dtype.itemsize + 24 * len(mine)
+            return merged, host.h2d_bytes, d2h
+
+        step()                                   # warm-up
+        torch.cuda.synchronize(dev)
+        dist.barrier()
+        t0 = time.perf_counter()
+        nh = 0
+        for _ in range(args.e2e_steps):
+            merged, h2d, d2h = step()
+            nh = len(merged) if merged is not None else 0
+        torch.cuda.synchronize(dev)
+        dt = (time.perf_counter() - t0) / args.e2e_steps
+        t = torch.tensor([dt], dtype=torch.float64, device=coll_dev if coll_dev is not None else dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dt = float(t[0])
+        return {"value": round(genome_bases / dt / 1e9, 4), "unit": "Gbases/s", "h2d_bytes_per_step": int(h2d),
+                "d2h_bytes_per_step": int(d2h), "s_per_step": dt, "hits": nh, "bytes_per_step_per_rank": "rank 0",
+                "path": "search_dist: <= 64 Mbp work units LPT-assigned to ranks -> per-rank Searcher.search_host "
+                        "(H2D lo/hi + N runs, find/compare, sort, device decoration, D2H of the records) -> "
+                        "merge_dist (per-chunk counts all-reduced, each rank writes its records at their "
+                        "genome-order offsets into one shared-memory result); wall clock, max over ranks"}
     pieces = [p for ch in st.chunks for p in ch.pieces]
     if E2E_PIECE_BASES:
-        pieces = search.split_pieces(pieces, E2E_PIECE_BASES, len(wl.cfg.pattern))
+        pieces = search.split_pieces(pieces, E2E_PIECE_BASES, L)
     chunks = search.pack_pieces(pieces, E2E_CHUNK_BASES)
     st.e2e_host = search.HostGenome(wl.seqs, chunks)
     srch = search.Searcher(wl.cfg.pattern, wl.guides, wl.thresholds, device=dev)
     srch.reserve(max(ch.n_bases for ch in chunks), max(st.caps))
-    from paper_conf_socc_jinv23_b200 import cof
     hits0, _, _ = run_e2e_step(wl, st, srch)     # warm-up; sizes the caller's result buffer
     n_out = int(len(hits0) * 1.05) + 1024
     # the caller's result buffer: pinned host memory, so the device-decorated records DMA
@@ -641,8 +757,6 @@ def measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev=None):
     out = torch.zeros(n_out * hd.itemsize, dtype=torch.uint8, pin_memory=True).numpy().view(hd)
     del hits0
     torch.cuda.synchronize(dev)
-    if world > 1:
-        dist.barrier()
     t0 = time.perf_counter()
     h2d = d2h = 0
     nh = 0
@@ -651,10 +765,6 @@ def measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev=None):
         h2d, d2h, nh = a, b, len(hits)
     torch.cuda.synchronize(dev)
     dt = (time.perf_counter() - t0) / args.e2e_steps
-    if world > 1:
-        t = torch.tensor([dt], dtype=torch.float64, device=coll_dev if coll_dev is not None else dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dt = float(t[0])
     return {"value": round(genome_bases / dt / 1e9, 4), "unit": "Gbases/s", "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "s_per_step": dt, "hits": nh,
             "path": "Searcher.search_host: cof_load_chunk (copy stream, double-buffered) -> find/compare "

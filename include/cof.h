@@ -64,9 +64,10 @@ uint64_t cof_launch_count(void);
  *  pattern   NUL-terminated IUPAC string (ACGTRYSWKMBDHVN, case-insensitive), 1<=L<=64.
  *  guides    n_guides NUL-terminated IUPAC strings of length L; 'N' positions are not
  *            compared (the -1-terminated index list; reading G7).
- *  max_mm    n_guides thresholds; a site is a hit iff #mismatches <= max_mm.
+ *  max_mm    n_guides thresholds, each <= L; a site is a hit iff #mismatches <= max_mm
+ *            (P:L225).
  *  out       receives a host-only, immutable plan (thread-safe to share read-only).
- * Errors: COF_E_ARG for a non-IUPAC letter (G18), guide length != L (G11), L>64, a
+ * Errors: COF_E_ARG for a non-IUPAC letter (G18), guide length != L (G11), L>64, max_mm > L, a
  * guide with 64 compared (non-N) letters, n_guides == 0 or > 2^24, NULL pointers.  For
  * L > 32 the comparer is always the pair-table one (cof_set_comparer's popc / mma
  * variants need L <= 32).  The plan reverse-complements pattern and

@@ -49,7 +49,7 @@ def variants(pattern: str, guides, thresholds, dna: int = 0, rna: int = 0):
     def put(pv, gv, t, meta):
         gs, ts, ms = groups.setdefault(pv, ([], [], []))
         gs.append(gv)
-        ts.append(t)
+        ts.append(min(t, len(pv)))   # a threshold >= the variant length admits every PAM site either way
         ms.append(meta)
 
     for gi, (g0, t) in enumerate(zip(guides, thresholds)):

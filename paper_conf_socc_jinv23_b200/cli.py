@@ -65,7 +65,7 @@ def parse_input(text: str, base_dir: str = ".") -> InputSpec:
         if t < 0:
             raise ValueError(f"negative mismatch count in {ln!r}")
         queries.append(q)
-        thr.append(t)
+        thr.append(min(t, len(pattern)))   # t >= L admits every PAM site; the C ABI wants t <= L
     return InputSpec(genome, pattern, queries, thr, dna_b, rna_b)
 
 

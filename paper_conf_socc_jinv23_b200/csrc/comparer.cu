@@ -254,15 +254,28 @@ __device__ __forceinline__ uint32_t table_hits(const uint32_t (&base)[NP], const
 __device__ __noinline__ void table_emit_v(const TableArgs& a, const uint32_t* pos_ptr, uint32_t hitm, uint32_t s0,
                                           uint32_t s1, uint32_t s2, uint32_t s3, uint32_t s4, uint32_t s5,
                                           uint32_t guide0) {
+    // Warp-aggregated append (P:L226 `old = atomic_inc(entrycount)` once per WARP and round):
+    // every lane that reached here holds >= 1 hit; each round, every lane with hits left
+    // emits one key, and one elected lane reserves the round's slots with a single atomic.
     const uint32_t pos = *pos_ptr;   // item list (global) or the fused kernel's queue (shared)
-    do {
-        const int k = __ffs(hitm) - 1;
-        hitm &= hitm - 1;
-        const uint32_t mm = ((s0 >> k) & 1u) | (((s1 >> k) & 1u) << 1) | (((s2 >> k) & 1u) << 2) |
-                            (((s3 >> k) & 1u) << 3) | (((s4 >> k) & 1u) << 4) | (((s5 >> k) & 1u) << 5);
-        const unsigned long long o = atomicAdd(&a.counters[2], 1ull);
-        if (o < a.cap) a.hits[o] = hit_key(pos, a.strand, guide0 + (uint32_t)k, mm);
-    } while (hitm);
+    const unsigned act = __activemask();
+    const int lane = threadIdx.x & 31;
+    for (;;) {
+        const unsigned m = __ballot_sync(act, hitm != 0u);
+        if (!m) break;
+        const int leader = __ffs(m) - 1;
+        unsigned long long base = 0;
+        if (lane == leader) base = atomicAdd(&a.counters[2], (unsigned long long)__popc(m));
+        base = __shfl_sync(act, base, leader);
+        if (hitm) {
+            const int k = __ffs(hitm) - 1;
+            hitm &= hitm - 1;
+            const uint32_t mm = ((s0 >> k) & 1u) | (((s1 >> k) & 1u) << 1) | (((s2 >> k) & 1u) << 2) |
+                                (((s3 >> k) & 1u) << 3) | (((s4 >> k) & 1u) << 4) | (((s5 >> k) & 1u) << 5);
+            const unsigned long long o = base + (unsigned)__popc(m & lanemask_lt());
+            if (o < a.cap) a.hits[o] = hit_key(pos, a.strand, guide0 + (uint32_t)k, mm);
+        }
+    }
 }
 
 __device__ __forceinline__ void table_emit(const TableArgs& a, const uint32_t* pos_ptr, uint32_t hitm,

@@ -17,6 +17,8 @@
 // scans of the masks' popcounts, one exchange of tile totals per 8 tiles, ordered direct
 // stores).  Algorithmic bytes per base: 3/8 read + 4 x items written (pass 2 re-reads the
 // 1/4 B/base of masks, largely from L2).
+#include <mutex>
+
 #include <cuda_runtime.h>
 
 #include "cof_internal.h"
@@ -93,7 +95,7 @@ __device__ __forceinline__ void pam_masks(const FinderArgs& a, uint32_t valid, c
 // Two passes over a contiguous tile range per CTA with one grid-wide exchange in between:
 //  pass 1 counts the passing starts of the CTA's range (no writes), publishes the CTA
 //  total and waits at a grid barrier (all CTAs are co-resident: the grid is sized from the
-//  occupancy calculator); every CTA then sums the totals of the CTAs before it (its global
+//  occupancy calculator and launched cooperatively); every CTA then sums the totals of the CTAs before it (its global
 //  offset) and pass 2 re-streams its range (mostly from L2) and writes the items in order.
 // One exchange per CTA replaces a decoupled look-back per tile, whose depth (all
 // concurrently running tiles) made it latency-bound.
@@ -378,8 +380,12 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
     }
 }
 
-static int g_finder_blocks_per_sm = -1;
-static int g_num_sms = -1;
+// per device (function attributes and occupancy are per-device state; several host threads
+// may drive several GPUs, search_multi)
+constexpr int FMAX_DEVICES = 64;
+static int g_finder_blocks_per_sm[FMAX_DEVICES];
+static int g_num_sms[FMAX_DEVICES];
+static std::mutex g_finder_mu;
 
 typedef void (*FinderFn)(FinderArgs);
 template <bool VS, bool MO>
@@ -401,23 +407,30 @@ static FinderFn finder_fn(uint32_t ne, bool vs, bool masks_only = false, bool wi
     return vs ? finder_fn_vs<true, false>(ne, wide) : finder_fn_vs<false, false>(ne, wide);
 }
 
-static cof_status finder_setup() {
-    if (g_finder_blocks_per_sm > 0) return COF_OK;
-    int bps_min = 1 << 30;
-    for (uint32_t k = 0; k < 64; k++) {
-        FinderFn fn = finder_fn(k & 7, (k >> 3) & 1, (k >> 4) & 1, k >= 32);
-        cudaError_t e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM);
-        if (e != cudaSuccess) return cuda_error(e, "finder setup");
-        int bps = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, (const void*)fn, FT, FSMEM);
-        if (e != cudaSuccess) return cuda_error(e, "finder occupancy");
-        if (bps < bps_min) bps_min = bps;
+static cof_status finder_setup(int* bps_out, int* sms_out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_error(e, "finder setup");
+    if (dev < 0 || dev >= FMAX_DEVICES) return set_error(COF_E_CUDA, "finder setup: device %d out of range", dev);
+    std::lock_guard<std::mutex> lk(g_finder_mu);
+    if (g_finder_blocks_per_sm[dev] <= 0) {
+        int bps_min = 1 << 30;
+        for (uint32_t k = 0; k < 64; k++) {
+            FinderFn fn = finder_fn(k & 7, (k >> 3) & 1, (k >> 4) & 1, k >= 32);
+            e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize, FSMEM);
+            if (e != cudaSuccess) return cuda_error(e, "finder setup");
+            int bps = 0;
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, (const void*)fn, FT, FSMEM);
+            if (e != cudaSuccess) return cuda_error(e, "finder occupancy");
+            if (bps < bps_min) bps_min = bps;
+        }
+        int sms = 0;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        g_num_sms[dev] = sms;
+        g_finder_blocks_per_sm[dev] = bps_min > 0 ? bps_min : 1;
     }
-    int dev = 0, sms = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    g_num_sms = sms;
-    g_finder_blocks_per_sm = bps_min > 0 ? bps_min : 1;
+    *bps_out = g_finder_blocks_per_sm[dev];
+    *sms_out = g_num_sms[dev];
     return COF_OK;
 }
 
@@ -488,7 +501,8 @@ cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* de
     if (!dev->lo || !dev->hi || !dev->nm) return set_error(COF_E_ARG, "cof_find_pam: chunk planes are NULL");
     if (((uintptr_t)dev->lo | (uintptr_t)dev->hi | (uintptr_t)dev->nm | (uintptr_t)dev->vs) & 15)
         return set_error(COF_E_ARG, "cof_find_pam: planes must be 16-byte aligned");
-    cof_status st = finder_setup();
+    int f_bps = 0, f_sms = 0;
+    cof_status st = finder_setup(&f_bps, &f_sms);
     if (st != COF_OK) return st;
     const uint64_t L = plan->L;
     if (dev->n_segs && !dev->vs) return set_error(COF_E_ARG, "cof_find_pam: multi-segment chunk without vs plane");
@@ -529,11 +543,21 @@ cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* de
                 a.psel[st][k] = make_uint4(0u - (set & 1u), 0u - ((set >> 1) & 1u), 0u - ((set >> 2) & 1u),
                                            0u - ((set >> 3) & 1u));
             }
-        uint32_t grid = (uint32_t)g_num_sms * (uint32_t)g_finder_blocks_per_sm;
+        uint32_t grid = (uint32_t)f_sms * (uint32_t)f_bps;
         if (grid > FMAX_CTAS) grid = FMAX_CTAS;
         if (grid > n_tiles) grid = n_tiles;
-        finder_fn(a.ne, a.vs != nullptr, masks_only, wide)<<<grid, FT, FSMEM, stream>>>(a);
-        e = cudaGetLastError();
+        FinderFn fn = finder_fn(a.ne, a.vs != nullptr, masks_only, wide);
+        if (masks_only) {   // pass 1 only: no grid-wide exchange, a plain launch
+            fn<<<grid, FT, FSMEM, stream>>>(a);
+            e = cudaGetLastError();
+        } else {
+            // the grid exchange between pass 1 and pass 2 needs every CTA resident at once:
+            // a cooperative launch guarantees it (or fails with
+            // cudaErrorCooperativeLaunchTooLarge -> COF_E_CUDA) instead of hanging when other
+            // work holds SMs; the grid never exceeds the occupancy limit computed above
+            void* args[] = {(void*)&a};
+            e = cudaLaunchCooperativeKernel((const void*)fn, dim3(grid), dim3(FT), args, FSMEM, stream);
+        }
         if (e != cudaSuccess) return cuda_error(e, "cof_finder_kernel launch");
         count_launches(1);
     }

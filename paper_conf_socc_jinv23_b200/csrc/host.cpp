@@ -279,7 +279,7 @@ static bool fast_record(const char* d, size_t n, size_t i, size_t next, cof_fast
         if (last == 0) return false;                        // blank line before the next header
     }
     const int64_t FF = (int64_t)F;
-    int64_t bad = 0, nl = 0;
+    int64_t bad = 0, nl = 0, cr = 0;
     const char* base = d + r.seq_off;
 #pragma omp parallel for schedule(static) reduction(+ : bad) if (F > (1u << 16))
     for (int64_t k = 1; k <= FF; k++) {
@@ -288,14 +288,18 @@ static bool fast_record(const char* d, size_t n, size_t i, size_t next, cof_fast
     }
     if (bad) return false;
     const int64_t RR = (int64_t)R;
-#pragma omp parallel for schedule(static) reduction(+ : nl) if (R > (1u << 22))
+    // newline count (every line break where the geometry puts it) and carriage returns: in an
+    // LF record a CR anywhere (e.g. one CRLF line) would be packed as a base -> slow path
+#pragma omp parallel for schedule(static) reduction(+ : nl, cr) if (R > (1u << 22))
     for (int64_t k0 = 0; k0 < RR; k0 += 1 << 16) {
         const int64_t k1 = std::min(RR, k0 + (1 << 16));
-        int64_t c = 0;
-        for (int64_t k = k0; k < k1; k++) c += base[k] == '\n';
+        int64_t c = 0, c2 = 0;
+        for (int64_t k = k0; k < k1; k++) { c += base[k] == '\n'; c2 += base[k] == '\r'; }
         nl += c;
+        cr += c2;
     }
     if ((uint64_t)nl != F + (rem && d[r.seq_end - 1] == '\n' ? 1 : 0)) return false;
+    if (cr != (crlf ? nl : 0)) return false;
     r.line_bases = nb;
     r.line_bytes = lb;
     r.length = (uint64_t)F * nb + last;

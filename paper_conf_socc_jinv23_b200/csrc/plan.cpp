@@ -57,6 +57,10 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     p->max_mm.assign(max_mm, max_mm + n_guides);
     for (uint32_t i = 0; i < n_guides; i++) {
         if (!guides[i]) { delete p; return set_error(COF_E_ARG, "guide %u is NULL", i); }
+        if (max_mm[i] > L) {   // max_mm <= L (a larger threshold means the same: every PAM site)
+            delete p;
+            return set_error(COF_E_ARG, "guide %u: max_mm %u exceeds the pattern length %zu", i, (unsigned)max_mm[i], L);
+        }
         if (strlen(guides[i]) != L) {
             delete p;
             return set_error(COF_E_ARG, "guide %u has length %zu, pattern has %zu", i, strlen(guides[i]), L);

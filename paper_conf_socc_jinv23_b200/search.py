@@ -249,6 +249,9 @@ class HostGenome:
 
 SPLIT_FILL = os.environ.get("COF_SPLIT_FILL", "0") == "1"   # measured slower end to end
 PLANE_BUFS = int(os.environ.get("COF_PLANE_BUFS", 2))   # device plane sets in the search_host pipeline (3 measured no faster)
+if PLANE_BUFS < 2:
+    # with one plane set chunk j+1's H2D would overwrite the planes chunk j is searched on
+    raise ValueError(f"COF_PLANE_BUFS={PLANE_BUFS}: the search_host pipeline needs at least 2 device plane sets")
 
 
 class Searcher:
@@ -330,39 +333,49 @@ class Searcher:
                           self.d_sort_ws, s)
         return nf, nr, nh
 
-    def search_host(self, host: HostGenome, indices=None, out=None, decorate="device"):
+    def search_host(self, host: HostGenome, indices=None, out=None, decorate="device", sink=None):
         """End-to-end over host-resident packed chunks.  Per chunk: H2D on a copy stream
         (double-buffered device planes, overlapping the previous chunk's kernels), find,
         compare, device sort, device decoration (cof_decorate) and an async D2H of the
         finished records; nothing waits on the host except the item/hit counts.
 
-        Returns the sorted hit array.  If ``out`` (a ``Searcher.hit_dtype`` array, ideally in
-        pinned memory) is large enough, each chunk's records land straight in its slice of
-        ``out`` (chunks are disjoint and in genome order, so no merge copy is needed) and a
-        view of ``out`` is returned; otherwise per-chunk arrays are merged with cof_merge.
-        ``decorate="host"`` decorates on CPU threads instead (cof_collect)."""
+        ``indices``: the chunks to search, in order -- a list, or any iterable (e.g. a shared
+        work queue that several Searchers on several GPUs pop from, search_multi); it is
+        consumed one chunk ahead of the device.  Returns the sorted hit array.  If ``out``
+        (a ``Searcher.hit_dtype`` array, ideally in pinned memory) is large enough and the
+        chunks come in genome order, each chunk's records land straight in its slice of
+        ``out`` and a view of ``out`` is returned; otherwise per-chunk arrays are merged
+        with cof_merge.  ``sink(i, records)``: called once per chunk with its sorted records
+        (after the final synchronisation); then the merged array is not built and None is
+        returned.  ``decorate="host"`` decorates on CPU threads instead (cof_collect)."""
         if decorate == "host":
+            if sink is not None:
+                raise ValueError("sink needs device decoration")
             return self._search_host_cpu_decorate(host, indices, out)
-        idx = list(range(len(host.chunks)) if indices is None else indices)
-        max_bases = max((host.chunks[i].n_bases for i in idx), default=1)
+        listed = indices is None or isinstance(indices, (list, tuple, range))
+        it = iter(range(len(host.chunks)) if indices is None else indices)
+        # device buffers: sized for every chunk this call may see (an iterator may yield any)
+        cand = list(indices) if listed and indices is not None else range(len(host.chunks))
+        max_bases = max((host.chunks[i].n_bases for i in cand), default=1)
+        max_segs = max((len(host.chunks[i].pieces) for i in cand), default=1)
         self.reserve(max_bases, max(self._hits_cap, 1 << 16))
-        if not hasattr(self, "d_planes_more") or self.d_planes_more[0].shape != self.d_planes.shape:
+        if getattr(self, "_planes_more_shape", None) != tuple(self.d_planes.shape):
             # PLANE_BUFS device plane sets: the H2D of chunk j+1 waits only for the
             # decoration of chunk j+1-PLANE_BUFS, not for the chunk just before it
             self.d_planes_more = [torch.empty_like(self.d_planes) for _ in range(PLANE_BUFS - 1)]
+            self._planes_more_shape = tuple(self.d_planes.shape)
             self.copy_stream = torch.cuda.Stream(self.device)
             self.d2h_stream = torch.cuda.Stream(self.device)
         planes = [self.d_planes] + self.d_planes_more
         nb = len(planes)
         rec_free = [None, None]
-        ordered = all(a < b for a, b in zip(idx, idx[1:]))
-        use_out = out is not None and ordered
-        max_segs = max((len(host.chunks[i].pieces) for i in idx), default=1)
-        ws = torch.empty((len(idx), cof.cof_decorate_workspace_bytes(max_segs)), dtype=torch.uint8,
-                         device=self.device)
-        results = []
+        use_out = out is not None and sink is None
+        ws_bytes = cof.cof_decorate_workspace_bytes(max_segs)
+        ws = []                    # one decoration workspace (key-check flag) per chunk
+        results = []               # (chunk index, records)
         total = 0
         overflow = False
+        last_i = -1
         with torch.cuda.device(self.device):
             loaded = [None] * nb
             freed = [None] * nb
@@ -375,16 +388,16 @@ class Searcher:
                     e.record(stream)
                     trace.append((what, j, e))
 
-            def load(j, k):
+            def load(j, i, k):
                 with torch.cuda.stream(self.copy_stream):
                     if freed[k] is not None:
                         self.copy_stream.wait_event(freed[k])
                     mark("h2d0", j, self.copy_stream)
-                    dch = self.device_chunk(host.chunks[idx[j]], planes[k], host.segs[idx[j]])
+                    dch = self.device_chunk(host.chunks[i], planes[k], host.segs[i])
                     # fills on the compute stream: that stream last used this plane set, and on
                     # the copy stream they would queue behind the running persistent kernels
                     # (COF_TRACE showed H2D intervals ~40% longer than the bytes need)
-                    host.load(idx[j], dch, self.copy_stream, fill_stream=self.stream if SPLIT_FILL else None)
+                    host.load(i, dch, self.copy_stream, fill_stream=self.stream if SPLIT_FILL else None)
                     mark("h2d1", j, self.copy_stream)
                     ev = torch.cuda.Event()
                     ev.record(self.copy_stream)
@@ -392,13 +405,19 @@ class Searcher:
                     return dch
 
             dchs = [None] * nb
-            if idx:
-                dchs[0] = load(0, 0)
-            for j, i in enumerate(idx):
+            cur = next(it, None)
+            if cur is not None:
+                dchs[0] = load(0, cur, 0)
+            j = 0
+            while cur is not None:
+                i = cur
+                nxt = next(it, None)
                 k, kr = j % nb, j & 1
                 self.stream.wait_event(loaded[k])
-                if j + 1 < len(idx):
-                    dchs[(j + 1) % nb] = load(j + 1, (j + 1) % nb)
+                if nxt is not None:
+                    if host.chunks[nxt].n_bases > self._cap_bases:
+                        raise ValueError(f"chunk {nxt} is larger than the chunks this call was sized for")
+                    dchs[(j + 1) % nb] = load(j + 1, nxt, (j + 1) % nb)
                 mark("dev0", j, self.stream)
                 _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned, counts=False)
                 if self.d_records is None or nh > self._rec_cap:
@@ -406,7 +425,8 @@ class Searcher:
                 recs = self.d_records[kr]
                 if rec_free[kr] is not None:         # the D2H of chunk j-2 from this buffer is done
                     self.stream.wait_event(rec_free[kr])
-                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, recs, ws[j], self.stream,
+                ws.append(torch.empty(ws_bytes, dtype=torch.uint8, device=self.device))
+                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, recs, ws[-1], self.stream,
                                  cap=self._rec_cap)
                 mark("dev1", j, self.stream)
                 fr = torch.cuda.Event()
@@ -414,7 +434,7 @@ class Searcher:
                 freed[k] = fr
                 dst = None
                 if use_out and not overflow:
-                    if total + nh <= len(out):
+                    if i > last_i and total + nh <= len(out):
                         dst = out[total:total + nh]
                     else:
                         overflow = True
@@ -429,21 +449,28 @@ class Searcher:
                         ev = torch.cuda.Event()
                         ev.record(self.d2h_stream)
                     rec_free[kr] = ev
-                results.append(dst)
+                results.append((i, dst))
                 total += nh
+                last_i = i
+                cur = nxt
+                j += 1
             self.d2h_stream.synchronize()
             self.stream.synchronize()
             if trace:   # COF_TRACE=1: per-chunk H2D / device intervals in ms from the first mark
                 import json
                 import sys
                 t0 = trace[0][2]
-                print(json.dumps({"search_host_trace": [(w, j, round(t0.elapsed_time(e), 3)) for w, j, e in trace]}),
+                print(json.dumps({"search_host_trace": [(w, jj, round(t0.elapsed_time(e), 3)) for w, jj, e in trace]}),
                       file=sys.stderr)
-            for j in range(len(idx)):
-                cof.cof_decorate_check(ws[j], self.stream)
+            for w in ws:
+                cof.cof_decorate_check(w, self.stream)
+        if sink is not None:
+            for i, r in results:
+                sink(i, r)
+            return None
         if use_out and not overflow:
             return out[:total]
-        return merge_hit_lists(results, self.hit_dtype)
+        return merge_hit_lists([r for _, r in sorted(results, key=lambda x: x[0])], self.hit_dtype)
 
     def _reserve_records(self, n):
         # two device record buffers: chunk j decorates into one while chunk j-1's D2H drains the other
@@ -518,13 +545,17 @@ class Searcher:
             return out[:total]
         return merge_hit_lists([results[i] for i in idx], self.hit_dtype)
 
+def _as_arrays(seqs):
+    return [np.frombuffer(s, dtype=np.uint8) if isinstance(s, (bytes, bytearray)) else
+            (np.frombuffer(s.encode(), dtype=np.uint8) if isinstance(s, str) else s) for s in seqs]
+
+
 def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda", pack_bases=None, fused=None):
     """Convenience: whole search of ``seqs`` (list of uint8 ASCII arrays / bytes) on one GPU.
     ``pack_bases`` packs chromosome pieces into multi-segment chunks (0 = one chunk);
     ``fused`` False forces the two-call path (item lists) even when the fused one fits."""
     L = len(pattern)
-    arrs = [np.frombuffer(s, dtype=np.uint8) if isinstance(s, (bytes, bytearray)) else
-            (np.frombuffer(s.encode(), dtype=np.uint8) if isinstance(s, str) else s) for s in seqs]
+    arrs = _as_arrays(seqs)
     chunks = plan_chunks([len(a) for a in arrs], L, chunk_bases, pack_bases)
     host = HostGenome(arrs, chunks)
     srch = Searcher(pattern, guides, thresholds, device)
@@ -533,15 +564,163 @@ def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda", p
     return srch.search_host(host)
 
 
+# ----------------------------------------------------------------------------- multi-GPU
+# The path shards: chromosomes -- and pieces of a chromosome that overlap by L-1 bases --
+# are independent (reading G12), and the global order (chrom, pos, strand, guide) is a
+# property of the records, so results do not depend on which GPU searched which piece.
+# The host concatenates per-chunk lists in genome order (the host collects the
+# results; the paper ran one GPU).  No collective touches the data path.
+
+MULTI_CHUNK_BASES = 64_000_000   # owned window starts per work unit (<= 64 Mbp chunk queue)
+
+
+class ChunkQueue:
+    """Thread-safe iterator over chunk indices in genome order: the shared work queue the
+    per-GPU pipelines of search_multi pop from (dynamic balance: a GPU that finishes early
+    takes the next chunk)."""
+
+    def __init__(self, n: int):
+        import threading
+        self._it = iter(range(n))
+        self._lock = threading.Lock()
+
+    def __iter__(self):
+        return self
+
+    def __next__(self):
+        with self._lock:
+            return next(self._it)
+
+
+def search_multi(seqs, pattern, guides, thresholds, devices=None, chunk_bases=MULTI_CHUNK_BASES, host=None,
+                 streams_per_device: int = 1):
+    """Single-process multi-GPU search: the genome cut into chunks of <= ``chunk_bases``
+    owned window starts, one host thread per GPU (``devices``; default every visible GPU;
+    a device may repeat) running its own Searcher pipeline over chunks popped from one
+    shared queue in genome order; the merge is the concatenation of the per-chunk lists in
+    chunk order (cof_merge's parallel fast path).  ``host``: a prebuilt HostGenome."""
+    import threading
+    if host is None:
+        arrs = _as_arrays(seqs)
+        host = HostGenome(arrs, plan_chunks([len(a) for a in arrs], len(pattern), chunk_bases))
+    if devices is None:
+        devices = [f"cuda:{k}" for k in range(torch.cuda.device_count())]
+    devices = [torch.device(d) for d in devices for _ in range(max(1, streams_per_device))]
+    if not devices:
+        raise RuntimeError("search_multi: no CUDA device")
+    queue = ChunkQueue(len(host.chunks))
+    per_chunk = [None] * len(host.chunks)
+    errors = []
+
+    def sink(i, recs):
+        per_chunk[i] = recs
+
+    def worker(dev):
+        try:
+            torch.cuda.set_device(dev)
+            srch = Searcher(pattern, guides, thresholds, device=dev, stream=torch.cuda.Stream(dev))
+            srch.search_host(host, indices=queue, sink=sink)
+        except BaseException as e:   # surfaced after the join
+            errors.append(e)
+
+    threads = [threading.Thread(target=worker, args=(d,), daemon=True) for d in devices]
+    for t in threads:
+        t.start()
+    for t in threads:
+        t.join()
+    if errors:
+        raise errors[0]
+    missing = [i for i, r in enumerate(per_chunk) if r is None]
+    if missing:
+        raise RuntimeError(f"search_multi: chunks {missing[:5]} were not searched")
+    return merge_hit_lists(per_chunk, cof.hit_dtype(len(pattern)))
+
+
 def shard_for_rank(chunks, rank: int, world: int):
     """This rank's chunks (LPT over owned window starts; ranks are independent)."""
     return shard_lpt(chunks, world)[rank]
 
 
+def shard_indices(chunks, world: int):
+    """LPT shards as chunk INDEX lists (genome order inside each shard)."""
+    idx = {id(c): i for i, c in enumerate(chunks)}
+    return [[idx[id(c)] for c in sh] for sh in shard_lpt(chunks, world)]
+
+
+def _coll_device(group=None):
+    import torch.distributed as dist
+    return torch.device("cuda", torch.cuda.current_device()) if dist.get_backend(group) == "nccl" else torch.device("cpu")
+
+
+def merge_dist(per_chunk: dict, n_chunks: int, dtype, group=None, dst: int = 0, shm_dir=None):
+    """Host merge of a torchrun job (one process per GPU): ``per_chunk`` maps this rank's
+    global chunk indices to their sorted records.  Per-chunk hit counts are summed over
+    the ranks (one small all-reduce), their exclusive prefix gives every chunk's offset in
+    the genome-ordered result, and every rank copies its records straight into that slice
+    of one shared-memory file (all ranks of a torchrun job share the node) -- the merge is
+    a parallel concatenation, no record crosses the process group.  Returns the merged
+    array (a read-only view of the mapping) on ``dst`` and None elsewhere."""
+    import tempfile
+    import uuid
+    import torch.distributed as dist
+    rank = dist.get_rank(group)
+    cd = _coll_device(group)
+    counts = torch.zeros(n_chunks, dtype=torch.int64)
+    for i, r in per_chunk.items():
+        counts[i] = len(r)
+    counts = counts.to(cd)
+    dist.all_reduce(counts, group=group)
+    counts = counts.cpu().numpy()
+    offs = np.zeros(n_chunks + 1, dtype=np.int64)
+    np.cumsum(counts, out=offs[1:])
+    total = int(offs[-1])
+    name = [None]
+    if rank == dst:
+        d = shm_dir or ("/dev/shm" if os.path.isdir("/dev/shm") else tempfile.gettempdir())
+        name[0] = os.path.join(d, f"cof_merge_{uuid.uuid4().hex}.bin")
+        with open(name[0], "wb") as f:
+            f.truncate(max(1, total) * dtype.itemsize)
+    dist.broadcast_object_list(name, src=dst, group=group)
+    path = name[0]
+    dist.barrier(group=group)
+    mine = [(i, r) for i, r in per_chunk.items() if len(r)]
+    if mine:
+        mm = np.memmap(path, dtype=dtype, mode="r+", shape=(max(1, total),))
+        for i, r in mine:
+            mm[offs[i]:offs[i] + len(r)] = r
+        mm.flush()
+        del mm
+    dist.barrier(group=group)
+    if rank != dst:
+        return None
+    out = np.memmap(path, dtype=dtype, mode="r", shape=(max(1, total),))[:total]
+    os.unlink(path)          # the mapping stays valid; the name goes away
+    return out
+
+
+def search_dist(seqs, pattern, guides, thresholds, chunk_bases=MULTI_CHUNK_BASES, group=None, device=None,
+                dst: int = 0):
+    """Multi-process multi-GPU search (torchrun, one rank per GPU): every rank plans the
+    same chunks, packs and searches its LPT share (search_host pipeline on its GPU) and
+    the ranks merge through merge_dist.  Returns the merged list on ``dst``, None elsewhere."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    arrs = _as_arrays(seqs)
+    chunks = plan_chunks([len(a) for a in arrs], len(pattern), chunk_bases)
+    mine = shard_indices(chunks, world)[rank]
+    dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+    per = {}
+    if mine:
+        host = HostGenome(arrs, [chunks[i] for i in mine])
+        srch = Searcher(pattern, guides, thresholds, device=dev)
+        srch.search_host(host, sink=lambda j, r: per.__setitem__(mine[j], r))
+    return merge_dist(per, len(chunks), cof.hit_dtype(len(pattern)), group=group, dst=dst)
+
+
 def gather_and_merge(local_hits: np.ndarray, group=None, dst: int = 0):
-    """Collect every rank's sorted hit list on ``dst`` (host objects over the process
-    group; the data path itself has no collective) and merge them there.  Returns the
-    merged array on ``dst`` and None elsewhere."""
+    """Merge of per-rank hit lists that each cover whole genome-ordered chunks (host
+    objects over the process group; kept for callers with one list per rank -- the
+    product path is merge_dist)."""
     import torch.distributed as dist
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)

@@ -76,6 +76,7 @@ def test_plan_validation():
         ("N" * 64, ["A" * 64], [1]),               # 64 compared letters (6-bit counts)
         ("", [""], [0]),                           # L = 0
         (good, [], []),                            # no guides
+        (good, ["ACGT" * 5 + "NNN"], [24]),        # max_mm > L
     ]
     for pat, g, t in bad:
         with pytest.raises(cof.CofError) as ei:
@@ -246,6 +247,22 @@ def test_fasta_layouts_against_plain_canonicalisation(tmp_path, eol):
                     if n % 32:
                         assert a[2][n // 32] >> (n % 32) == (1 << (32 - n % 32)) - 1
             fa.close()
+
+
+def test_fasta_mixed_line_endings(tmp_path):
+    """One CRLF line inside an LF record: its newline still sits where the line geometry
+    expects one, so the fast reader must notice the CR and hand the record to the byte
+    walk (otherwise the CR is packed as an N and every later coordinate shifts by one)."""
+    rng = np.random.default_rng(12)
+    s = rng.choice(np.frombuffer(b"ACGT", np.uint8), 49).tobytes()
+    lines = [s[0:10], s[10:19], s[19:29], s[29:39], s[39:49]]
+    text = b">m\n" + lines[0] + b"\n" + lines[1] + b"\r\n" + b"".join(x + b"\n" for x in lines[2:])
+    path = tmp_path / "mixed.fa"
+    path.write_bytes(text)
+    fa = cof.Fasta(path)
+    assert fa.length(0) == len(s)
+    assert fa.read(0).tobytes() == s
+    fa.close()
 
 
 def test_plan_chunks_cover_every_window_once():

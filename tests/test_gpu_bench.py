@@ -47,9 +47,12 @@ def test_bench_two_ranks_share_one_gpu():
     d1 = _last_json(one.stdout)
     env = dict(os.environ, COF_DIST_BACKEND="gloo")
     two = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
-                          "--master-addr=127.0.0.1", f"--master-port={_port()}", "bench.py", "--gpus", "2", *ARGS,
-                          "--no-e2e"], cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
+                          "--master-addr=127.0.0.1", f"--master-port={_port()}", "bench.py", "--gpus", "2", *ARGS],
+                         cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
     assert two.returncode == 0, two.stderr[-3000:]
     d2 = _last_json(two.stdout)
     assert d2["n_gpus"] == 2 and d2["scaling"] == "strong"
     assert d2["hits_per_step"] == d1["hits_per_step"] and d2["items_per_step"] == d1["items_per_step"]
+    # N > 1 e2e: per-rank pipelines + merge_dist; the merged list has every hit
+    assert d2["e2e"]["hits"] == d1["hits_per_step"] and d2["e2e"]["value"] > 0
+    assert "merge_dist" in d2["e2e"]["path"]

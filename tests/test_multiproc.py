@@ -1,7 +1,8 @@
 """World-size-2 (gloo, CPU) test of the multi-GPU host logic: LPT sharding of chunks over
-ranks, per-rank independent search, gather + merge on rank 0 == single-process search.
-The per-rank search is the oracle here (no GPU on this box); the sharding, gather and
-merge code is the product's (search.shard_for_rank / gather_and_merge / cof_merge)."""
+ranks, per-rank independent search, merge on rank 0 == single-process search.  The
+per-rank search is the oracle here (no GPU on this box); the sharding and merge code is
+the product's (search.shard_indices / merge_dist / gather_and_merge / cof_merge).  The
+GPU twins are in tests/test_gpu_multi.py."""
 import os
 import socket
 
@@ -36,14 +37,20 @@ def _worker(rank, world, port, q, name="C3"):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     wl = synth.make_workload(name, scale=0.0005 if name == "C3" else 0.003, n_guides=8)
     chunks = search.plan_chunks([len(s) for s in wl.seqs], wl.cfg.L, 40_000)
-    mine = search.shard_for_rank(chunks, rank, world)
-    lists = [_oracle_chunk_hits(wl, ch) for ch in mine]
-    local = search.merge_hit_lists(lists)
-    merged = search.gather_and_merge(local)
+    # the product's merge (merge_dist): per-chunk lists of this rank's LPT share -> offsets
+    # from the summed per-chunk counts -> slices of one shared-memory file
+    mine = search.shard_indices(chunks, world)[rank]
+    per = {i: _oracle_chunk_hits(wl, chunks[i]) for i in mine}
+    merged = search.merge_dist(per, len(chunks), cof.hit_dtype(wl.cfg.L))
+    # the older per-rank-list gather (host objects) gives the same list
+    local = search.merge_hit_lists([per[i] for i in mine], cof.hit_dtype(wl.cfg.L))
+    merged2 = search.gather_and_merge(local)
     if rank == 0:
         ref = oracle.search(wl.seqs, wl.cfg.pattern, wl.guides, wl.thresholds)
-        q.put((cof.hits_to_tuples(merged), oracle.hits_to_tuples(ref), len(mine), len(chunks)))
+        q.put((cof.hits_to_tuples(merged), oracle.hits_to_tuples(ref), len(mine), len(chunks),
+               cof.hits_to_tuples(merged2)))
     else:
+        assert merged is None and merged2 is None
         q.put(("rank1", len(mine)))
     dist.destroy_process_group()
 
@@ -63,6 +70,26 @@ def test_two_rank_shard_gather_merge(name):
         assert p.exitcode == 0
     r0 = [r for r in res if r[0] != "rank1"][0]
     r1 = [r for r in res if r[0] == "rank1"][0]
-    got, exp, n0, n_all = r0
+    got, exp, n0, n_all, got2 = r0
     assert got == exp and len(exp) > 0
+    assert got2 == exp
     assert n0 + r1[1] == n_all and n0 > 0 and r1[1] > 0
+
+
+def test_chunk_queue_hands_out_each_index_once():
+    import threading
+    qq = search.ChunkQueue(5000)
+    seen = []
+    lock = threading.Lock()
+
+    def pop():
+        for i in qq:
+            with lock:
+                seen.append(i)
+
+    ts = [threading.Thread(target=pop) for _ in range(6)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    assert sorted(seen) == list(range(5000))
