@@ -139,8 +139,8 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl
     max_owned = max(ch.n_owned for ch in chunks)
     # fused find+compare (finder masks -> comparer, no item lists) unless the guide table is
     # too large for it or COF_FUSED=0; the two-call path writes / reads ordered item lists
-    st.fused = search.use_fused(st.plan, len(guides))
-    st.path_name = "fused" if st.fused else "twocall"
+    st.path_name = search.choose_path(st.plan, len(guides))   # single pass / fused masks / two-call
+    st.fused = st.path_name != "twocall"
     st.items = torch.empty((2, 1 if st.fused else max_owned), dtype=torch.int32, device=st.device)
     st.find_ws = torch.empty(cof.cof_find_compare_workspace_bytes(max(ch.n_bases for ch in chunks)),
                              dtype=torch.uint8, device=st.device)
@@ -150,7 +150,10 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl
     tmp_hits = torch.empty(tmp_cap, dtype=torch.int64, device=st.device)
     for i, ch in enumerate(chunks):
         try:
-            if st.fused:
+            if st.path_name == "single":
+                nh = cof.cof_search_single(st.plan, st.plan_devs[i], st.d_chunks[i], st.find_ws, tmp_hits, tmp_cap,
+                                           st.stream)
+            elif st.fused:
                 cof.cof_find_masks(st.plan, st.plan_devs[i], st.d_chunks[i], st.find_ws, st.stream)
                 nh = cof.cof_compare_masks(st.plan, st.plan_devs[i], st.d_chunks[i], st.find_ws, tmp_hits, tmp_cap,
                                            st.stream)
@@ -196,15 +199,18 @@ def run_device_pipeline(wl, st, collect=False, events=None, fevents=None):
 
     for i in range(len(st.chunks)):
         dch, pd = st.d_chunks[i], st.plan_devs[i]
-        f0 = ev() if fevents is not None else None
-        if st.fused:
-            cof.cof_find_masks(st.plan, pd, dch, st.find_ws, s)
-        else:
-            cof.cof_find_pam(st.plan, pd, dch, st.find_ws, st.items[0], st.items[1], st.max_owned, s, sync=False)
-        if fevents is not None:
-            fevents.append((f0, ev()))
+        if st.path_name != "single":   # (the single pass has no separate search kernel)
+            f0 = ev() if fevents is not None else None
+            if st.fused:
+                cof.cof_find_masks(st.plan, pd, dch, st.find_ws, s)
+            else:
+                cof.cof_find_pam(st.plan, pd, dch, st.find_ws, st.items[0], st.items[1], st.max_owned, s, sync=False)
+            if fevents is not None:
+                fevents.append((f0, ev()))
         e0 = ev() if events is not None else None
-        if st.fused:
+        if st.path_name == "single":
+            cof.cof_search_single(st.plan, pd, dch, st.find_ws, st.hits[i], st.caps[i], s, sync=False)
+        elif st.fused:
             cof.cof_compare_masks(st.plan, pd, dch, st.find_ws, st.hits[i], st.caps[i], s, sync=False)
         else:
             cof.cof_compare(st.plan, pd, dch, st.items[0], ON, st.items[1], ON, st.hits[i], st.caps[i], s, sync=False)
@@ -530,7 +536,7 @@ def main():
     peaks, peak_src = _peaks()
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     n_sm = torch.cuda.get_device_properties(dev).multi_processor_count
-    roof = comparer_roof(st.plan, n_sm, sm_max, args.comparer)
+    roof = comparer_roof(st.plan, n_sm, sm_max, args.comparer, st.path_name)
     cmp_rate = comps_mine * args.steps / (cmp_ms * 1e-3) if cmp_ms > 0 else 0.0
     n_cmp_launch = len(events)
     if args.comparer == "mma":
@@ -547,10 +553,13 @@ def main():
                     "comparisons_per_s": cmp_rate, "alu_table_roof_comparisons_per_s": roof["peak"],
                     "launches": n_cmp_launch, "share_of_step": cmp_ms_max / ms_total if ms_total else None}
     else:
-        roofline = {"bound": "alu", "kernel": f"cof_comparer_{'fused' if st.fused else args.comparer}",
+        kname = {"single": "cof_single_kernel", "fused": "cof_comparer_fused"}.get(st.path_name,
+                                                                                  f"cof_comparer_{args.comparer}")
+        roofline = {"bound": "alu", "kernel": kname,
                     "achieved": cmp_rate, "peak": roof["peak"], "unit": "comparisons/s",
                     "frac": cmp_rate / roof["peak"] if roof["peak"] else None,
-                    "traffic": traffic_for("cof_comparer", st, cfgname),
+                    "traffic": traffic_for("cof_single_kernel" if st.path_name == "single" else "cof_comparer",
+                                           st, cfgname),
                     "peak_basis": roof["basis"], "launches": n_cmp_launch,
                     "share_of_step": cmp_ms_max / ms_total if ms_total else None,
                     # the same rate against SURVEY §8(d)'s roof (one POPC per comparison)
@@ -560,7 +569,13 @@ def main():
     # finder roofline (HBM): algorithmic bytes of the search kernel per step
     plane_bytes = sum(cof.cof_plane_words(ch.n_bases) * 4 * (4 if ch.multi else 3) for ch in st.chunks)
     words = sum(cof.cof_plane_words(ch.n_bases) for ch in st.chunks)
-    if st.fused:      # planes (+ valid-start plane) read, {fwd, rev} masks written
+    if st.path_name == "single":   # planes streamed once per launch by the single-pass kernel
+        n_launch = max(1, len(events) // max(1, args.steps))
+        find_bytes = plane_bytes * n_launch
+        find_basis = ("single pass: no separate search kernel; planes (+ valid-start plane) streamed once per "
+                      "launch by cof_single_kernel (PAM test fused into it) -- bytes / that kernel's time")
+        find_ms = cmp_ms
+    elif st.fused:      # planes (+ valid-start plane) read, {fwd, rev} masks written
         find_bytes = plane_bytes + words * 8
         find_basis = "planes read + 8 B of PAM masks per plane word written (fused path)"
     else:             # planes read, 4 B per item written
@@ -568,7 +583,8 @@ def main():
         find_basis = "planes read + 4 B per item written (two-call path)"
     find_gbs = find_bytes * args.steps / (find_ms * 1e-3) / 1e9 if find_ms > 0 else 0.0
     hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
-    finder_roof = {"bound": "hbm", "kernel": "cof_finder_kernel", "achieved": round(find_gbs, 1),
+    finder_roof = {"bound": "hbm", "kernel": "cof_single_kernel" if st.path_name == "single" else "cof_finder_kernel",
+                   "achieved": round(find_gbs, 1),
                    "peak": hbm_peak, "unit": "GB/s", "frac": find_gbs / hbm_peak,
                    "bytes_per_step": int(find_bytes), "basis": find_basis,
                    "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_finder_kernel", st, cfgname)}
@@ -655,7 +671,43 @@ def popc_roof(n_sm, sm_mhz):
     return 16.0 * n_sm * sm_mhz * 1e6
 
 
-def comparer_roof(plan, n_sm, sm_mhz, impl):
+def single_roof(plan, n_sm, sm_mhz):
+    """Peak comparisons/s of the single-pass kernel's filter: per site and
+    32-guide block, NP one-word shared-memory lookups (one wavefront per warp each, 1 per
+    clk per SM) and the nz_count carry-save tree (gen_csa.gen_count: FA / HA counts for
+    this plan's NP) + a 4-step comparator + the valid mask, all LOP3 at 64 /clk/SM.
+    Verification of the filter's survivors, site setup and queueing are not in this roof."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "gen_csa", os.path.join(ROOT, "paper_conf_socc_jinv23_b200", "csrc", "gen_csa.py"))
+    g = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(g)
+    care = 0
+    for gs in plan.guides:
+        for j, ch in enumerate(gs):
+            if ch.upper() != "N":
+                care |= 1 << j
+    npairs = max(1, (bin(care).count("1") + 1) // 2)
+    hdr = g.gen_count(npairs).splitlines()[0]
+    fa = int(hdr.split(":")[1].split("full")[0])
+    ha = int(hdr.split(",")[1].split("half")[0])
+    alu_ops = 2 * fa + 2 * ha + 4 + 1
+    alu_rate = 64.0 * 32 / alu_ops
+    lds_rate = 32.0 * 32 / npairs
+    per_clk = min(alu_rate, lds_rate)
+    return {"peak": per_clk * n_sm * sm_mhz * 1e6,
+            "basis": f"single-pass filter: min(ALU {alu_rate:.1f}, LDS {lds_rate:.1f}) comparisons/clk/SM for "
+                     f"{npairs} pairs ({alu_ops} LOP3 and {npairs} one-word lookups per 32 comparisons; survivor "
+                     f"verification excluded) x {n_sm} SMs x {sm_mhz:.0f} MHz"}
+
+
+def comparer_roof(plan, n_sm, sm_mhz, impl, path="fused"):
+    if path == "single":
+        return single_roof(plan, n_sm, sm_mhz)
+    return table_roof(plan, n_sm, sm_mhz, impl)
+
+
+def table_roof(plan, n_sm, sm_mhz, impl):
     """Peak comparisons/s of the comparer's binding pipe.
     popc: 1 POPC per comparison, POPC = 16/clk/SM (measured, tools/microbench_pipes.cu).
     table: per item and 32-guide block, the minimal carry-save tree (FA/HA count from

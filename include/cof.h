@@ -245,9 +245,27 @@ uint32_t   cof_plan_mma_kpad(const cof_plan *plan);
  *  workspace  dev, >= cof_find_compare_workspace_bytes(dev->n_bases) bytes. */
 int        cof_find_compare_supported(const cof_plan *plan);
 size_t     cof_find_compare_workspace_bytes(uint64_t n_bases);
-/* = cof_find_masks + cof_compare_masks */
+/* = cof_search_single when cof_single_supported(plan), else cof_find_masks +
+ * cof_compare_masks.  Same arguments as cof_compare_masks. */
 cof_status cof_find_compare(const cof_plan *plan, void *plan_dev, const cof_chunk *dev, void *workspace,
                             uint64_t *hits, uint64_t hits_cap, uint64_t *n_hits, cof_stream s);
+/* Single pass (SURVEY §8(f) f1 as one streaming kernel, single.cu): the planes stream
+ * through shared memory once; each tile's PAM test (both strands) feeds per-warp queues
+ * of sites with their 32-base windows, which are compared against all guides of the
+ * launch: a necessary-condition filter (number of mismatched position pairs <= t, from
+ * one 32-bit shared-memory lookup per pair and 32 guides) and the exact count of every
+ * survivor, hits appended warp-aggregated.  No item list,
+ * no mask array, no window gather.  Same hits as cof_find_pam + cof_compare (same key
+ * format, unordered); item counts land in plan_dev.  Needs every compared position of
+ * both strands inside one 31-position window (L <= 32 patterns) and the table comparer;
+ * COF_E_ARG otherwise.  Guide sets larger than one launch's shared-memory tables (~1,500
+ * 20-nt guides) run several launches, each re-streaming the planes.
+ * cof_single_supported(plan) = 1 when the shape fits AND the filter is selective (every
+ * threshold at least 3 below the number of position pairs); COF_SINGLE=1 / 0 overrides.
+ *  workspace  dev, >= cof_find_compare_workspace_bytes(dev->n_bases) bytes (tile tickets). */
+int        cof_single_supported(const cof_plan *plan);
+cof_status cof_search_single(const cof_plan *plan, void *plan_dev, const cof_chunk *dev, void *workspace,
+                             uint64_t *hits, uint64_t hits_cap, uint64_t *n_hits, cof_stream s);
 /* The search kernel's pass 1 alone: PAM masks of every plane word, both strands, into the
  * workspace ({fwd, rev} 32-bit masks per plane word, bit b = window start 32w + b);
  * item counts into plan_dev.  Asynchronous. */

@@ -1,6 +1,6 @@
 """Cas-OFFinder-style command line (I/O compatibility).
 
-    python -m paper_conf_socc_jinv23_b200 INPUT [G] OUTPUT [--chunk-bases N] [--device cuda:0]
+    python -m paper_conf_socc_jinv23_b200 INPUT [G] OUTPUT [--chunk-bases N] [--device cuda:0] [--gpus N]
 
 INPUT follows the tool's input file ("the desired pattern, query sequences, and maximum
 mismatch number", P:L158 via [17]):
@@ -113,8 +113,10 @@ def run_bulge(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = N
     return hits, names
 
 
-def run(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = None):
-    """Search the genome of ``spec`` on one GPU; returns (hits, chromosome names)."""
+def run(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = None, gpus: int = 1):
+    """Search the genome of ``spec``; returns (hits, chromosome names).  ``gpus`` > 1: the
+    single-process multi-GPU path (search.search_multi: one pipeline per GPU over a shared
+    queue of <= 64 Mbp work units, merge by concatenation in genome order)."""
     import torch
     from . import cof, search
 
@@ -125,11 +127,18 @@ def run(spec: InputSpec, device: str = "cuda", chunk_bases: int | None = None):
             names.append(fa.name(i))
             recs.append((fi, i, fa.length(i)))
     L = len(spec.pattern)
+    if gpus > 1 and chunk_bases is None:
+        chunk_bases = search.MULTI_CHUNK_BASES
     chunks = search.plan_chunks([r[2] for r in recs], L, chunk_bases)
     host = search.HostGenome.from_packer(chunks, lambda c, first, n, lo, hi, nm:
                                          fastas[recs[c][0]].pack(recs[c][1], first, n, lo, hi, nm))
-    srch = search.Searcher(spec.pattern, spec.queries, spec.thresholds, device=device)
-    hits = srch.search_host(host)
+    if gpus > 1:
+        n_dev = torch.cuda.device_count()
+        devices = [f"cuda:{k % n_dev}" for k in range(gpus)]
+        hits = search.search_multi(None, spec.pattern, spec.queries, spec.thresholds, devices=devices, host=host)
+    else:
+        srch = search.Searcher(spec.pattern, spec.queries, spec.thresholds, device=device)
+        hits = srch.search_host(host)
     torch.cuda.synchronize()
     return hits, names
 
@@ -140,6 +149,8 @@ def main(argv=None) -> int:
     ap.add_argument("args", nargs="+", help="[C|G|A] OUTPUT")
     ap.add_argument("--chunk-bases", type=int, default=None)
     ap.add_argument("--device", default="cuda")
+    ap.add_argument("--gpus", type=int, default=1,
+                    help="GPUs of this node to shard the genome over (one pipeline per GPU, one process)")
     a = ap.parse_args(argv)
     output = a.args[-1]
     with open(a.input) as f:
@@ -148,7 +159,7 @@ def main(argv=None) -> int:
         hits, names = run_bulge(spec, a.device, a.chunk_bases)
         text = format_bulge_hits(hits, spec.queries, names)
     else:
-        hits, names = run(spec, a.device, a.chunk_bases)
+        hits, names = run(spec, a.device, a.chunk_bases, gpus=a.gpus)
         text = format_hits(hits, spec.queries, names)
     if output == "-":
         sys.stdout.write(text)

@@ -100,6 +100,8 @@ def _load():
         "cof_decorate64": (I32, [P, P, P, P, U64, U64, P, P, P]),
         "cof_decorate_check": (I32, [P, P]),
         "cof_find_compare_supported": (ctypes.c_int, [P]),
+        "cof_single_supported": (ctypes.c_int, [P]),
+        "cof_search_single": (I32, [P, P, P, P, P, U64, P, P]),
         "cof_find_compare_workspace_bytes": (SZ, [U64]),
         "cof_find_compare": (I32, [P, P, P, P, P, U64, P, P]),
         "cof_find_masks": (I32, [P, P, P, P, P]),
@@ -134,7 +136,7 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_decorate_workspace_bytes", "cof_decorate", "cof_decorate64",
                        "cof_decorate_check", "cof_find_compare_supported",
                        "cof_find_compare_workspace_bytes", "cof_find_compare", "cof_find_masks",
-                       "cof_compare_masks", "cof_plan_mma_kpad", "cof_set_comparer", "cof_2bit_open",
+                       "cof_compare_masks", "cof_single_supported", "cof_search_single", "cof_plan_mma_kpad", "cof_set_comparer", "cof_2bit_open",
                        "cof_2bit_close", "cof_2bit_count", "cof_2bit_name", "cof_2bit_length",
                        "cof_2bit_pack")]
 
@@ -333,6 +335,22 @@ def cof_find_compare(plan, plan_dev, dev: cof_chunk, workspace, hits, hits_cap, 
         return int(n.value)
     _check(lib.cof_find_compare(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
                                 _ptr(hits), int(hits_cap), None, _stream(stream)))
+    return None
+
+
+def cof_single_supported(plan) -> bool:
+    return bool(lib.cof_single_supported(plan.handle))
+
+
+def cof_search_single(plan, plan_dev, dev: cof_chunk, workspace, hits, hits_cap, stream=None, sync=True):
+    """Single-pass find + compare (one streaming kernel); returns n_hits if ``sync`` else None."""
+    if sync:
+        n = ctypes.c_uint64()
+        _check(lib.cof_search_single(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
+                                     _ptr(hits), int(hits_cap), ctypes.addressof(n), _stream(stream)))
+        return int(n.value)
+    _check(lib.cof_search_single(plan.handle, _ptr(plan_dev), ctypes.addressof(dev), _ptr(workspace),
+                                 _ptr(hits), int(hits_cap), None, _stream(stream)))
     return None
 
 

@@ -61,6 +61,12 @@ COF_HD uint32_t pair_entry(uint32_t np, uint32_t q, uint32_t b1, uint32_t b2) {
     return np * 16u + q * 9u + (b1 == 4 ? b2 : 5u + b1);
 }
 
+// Single-pass comparer filter table (single.cu): per strand and 32-guide block, per
+// position pair, 25 one-word entries (bit k = guide k's pair has >= 1 mismatch for that
+// base pair), indexed like pair_entry; blocks padded to a 64-byte multiple so the
+// 16 ACGT entries of a pair (64 bytes) can be addressed by OR-ing the pair nibble in.
+COF_HD uint32_t filter_block_words(uint32_t np) { return (np * 25u + 15u) & ~15u; }
+
 // Bit-sliced pair-table comparer (v2): per strand, per 32-guide block, per position pair,
 // 25 entries (base pair combos incl. N) of {bit0, bit1} mismatch-count planes.
 struct PairLayout {
@@ -104,6 +110,8 @@ struct DevLayout {
     size_t onehot;                   // uint64[2][n_guides][5] decoration masks (see cof_plan::onehot)
     size_t mma_b;                    // tensor-core comparer: int8 B images of all guide batches
     size_t mma_thr;                  // uint8[n_guides]: min(t_g, #compared positions)
+    size_t ftab_fwd, ftab_rev;       // single-pass filter tables: uint32[n_blocks][filter_block_words(np)]
+    size_t vrec_fwd, vrec_rev;       // single-pass verification records: uint4[n_blocks * 32][2]
     size_t total;
 };
 

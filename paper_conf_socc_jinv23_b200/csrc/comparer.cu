@@ -838,6 +838,10 @@ cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* de
                        cudaStream_t stream);
 const uint4* finder_masks(const void* workspace);
 uint64_t finder_word_pairs(const cof_plan* plan, const cof_chunk* dev);
+bool single_supported(const cof_plan* plan, bool strict);
+uint32_t single_launches(const cof_plan* plan);
+cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, unsigned int* tickets,
+                      uint64_t* hits, uint64_t hits_cap, cudaStream_t stream);
 
 // Guide blocks per launch of the fused comparer: its whole launch table is resident in
 // shared memory (no re-loads between mask grabs), so a plan with more blocks runs several
@@ -934,8 +938,45 @@ cof_status cof_compare_masks(const cof_plan* plan, void* plan_dev, const cof_chu
     return COF_OK;
 }
 
+int cof_single_supported(const cof_plan* plan) {
+    return plan && comparer_impl() == 1 && single_supported(plan, true) &&
+           single_launches(plan) <= FUSED_MAX_TICKETS ? 1 : 0;
+}
+
+cof_status cof_search_single(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
+                             uint64_t* hits, uint64_t hits_cap, uint64_t* n_hits, cof_stream s) {
+    if (!plan || !plan_dev || !dev || !workspace || (!hits && hits_cap))
+        return set_error(COF_E_ARG, "cof_search_single: NULL argument");
+    if (!dev->lo || !dev->hi || !dev->nm) return set_error(COF_E_ARG, "cof_search_single: chunk planes are NULL");
+    if (!single_supported(plan, false) || single_launches(plan) > FUSED_MAX_TICKETS)
+        return set_error(COF_E_ARG, "cof_search_single: the plan's compared span exceeds one 31-position window "
+                                    "(use cof_find_compare / cof_find_pam + cof_compare)");
+    cudaStream_t stream = (cudaStream_t)s;
+    uint8_t* pd = (uint8_t*)plan_dev;
+    unsigned long long* counters = (unsigned long long*)(pd + plan->lay.counters);
+    unsigned int* tickets = (unsigned int*)((uint8_t*)workspace + cof_find_workspace_bytes(dev->n_bases));
+    cudaError_t e = cudaMemsetAsync(counters, 0, 3 * sizeof(uint64_t), stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(tickets, 0, FUSED_MAX_TICKETS * sizeof(unsigned int), stream);
+    if (e != cudaSuccess) return cuda_error(e, "cof_search_single memset");
+    cof_status st = run_single(plan, pd, dev, tickets, hits, hits_cap, stream);
+    if (st != COF_OK) return st;
+    if (n_hits) {
+        uint64_t c = 0;
+        e = cudaMemcpyAsync(&c, counters + 2, sizeof c, cudaMemcpyDeviceToHost, stream);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(stream);
+        if (e != cudaSuccess) return cuda_error(e, "cof_search_single count");
+        *n_hits = c;
+        if (c > hits_cap)
+            return set_error(COF_E_CAPACITY, "cof_search_single: %llu hits exceed capacity %llu",
+                             (unsigned long long)c, (unsigned long long)hits_cap);
+    }
+    return COF_OK;
+}
+
 cof_status cof_find_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
                             uint64_t* hits, uint64_t hits_cap, uint64_t* n_hits, cof_stream s) {
+    if (plan && cof_single_supported(plan))   // one streaming kernel
+        return cof_search_single(plan, plan_dev, dev, workspace, hits, hits_cap, n_hits, s);
     if (plan && !fusable(plan))
         return set_error(COF_E_ARG, "cof_find_compare: guide table too large for the fused kernel "
                                     "(use cof_find_pam + cof_compare)");

@@ -254,6 +254,13 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     for (const MmaBatch& b : mp.batches) mma_b_bytes += (size_t)b.nt * b.tn * mp.kpad;
     lay.mma_b = off; off = align256(off + mma_b_bytes);
     lay.mma_thr = off; off = align256(off + n_guides);
+    // (rounded up to whole groups of 4 blocks: the single-pass kernel reads blocks four at a time)
+    const size_t ftab_bytes = (size_t)((p->n_blocks + 3) & ~3u) * filter_block_words(NPAIR) * 4;
+    lay.ftab_fwd = off; off = align256(off + ftab_bytes);
+    lay.ftab_rev = off; off = align256(off + ftab_bytes);
+    const size_t vrec_bytes = (size_t)((p->n_blocks + 3) & ~3u) * 32 * 2 * 16;
+    lay.vrec_fwd = off; off = align256(off + vrec_bytes);
+    lay.vrec_rev = off; off = align256(off + vrec_bytes);
     lay.total = off;
     p->image.assign(lay.total, 0);
     uint8_t* img = p->image.data();
@@ -300,7 +307,31 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
                     size_t e = (size_t)b * NPAIR * 25 + pair_entry(NPAIR, q, b1, b2);
                     tab[e * 2 + 0] = w0;
                     tab[e * 2 + 1] = w1;
+                    // single-pass filter: the pair has at least one mismatch (count 1 or 2)
+                    uint32_t* ft = (uint32_t*)(img + (s == 0 ? lay.ftab_fwd : lay.ftab_rev));
+                    ft[(size_t)b * filter_block_words(NPAIR) + pair_entry(NPAIR, q, b1, b2)] = w0 | w1;
                 }
+            }
+        }
+        // single-pass verification records, window offsets relative to p0 (compared spans
+        // <= 32 only): {lo, hi, care, t} of the concrete letters and the one-hot {A, C, G, T}
+        // membership of every letter
+        if (!pl.wide) {
+            uint32_t* vr = (uint32_t*)(img + (s == 0 ? lay.vrec_fwd : lay.vrec_rev));
+            for (uint32_t i = 0; i < n_guides; i++) {
+                uint32_t lo = 0, hi = 0, care = 0, oh[4] = {0, 0, 0, 0};
+                for (uint32_t j = pl.p0; j < L && j < pl.p0 + 32; j++) {
+                    const uint8_t m = gm(s, i, j);
+                    if (m == 15) continue;
+                    const uint32_t bit = 1u << (j - pl.p0);
+                    care |= bit;
+                    for (int bb = 0; bb < 4; bb++) if (m >> bb & 1) oh[bb] |= bit;
+                    const int c = concrete_code(m);
+                    if (c >= 0) { lo |= (c & 1) ? bit : 0u; hi |= (c >> 1) ? bit : 0u; }
+                }
+                uint32_t* r = vr + (size_t)i * 8;
+                r[0] = lo; r[1] = hi; r[2] = care; r[3] = p->max_mm[i];
+                r[4] = oh[0]; r[5] = oh[1]; r[6] = oh[2]; r[7] = oh[3];
             }
         }
     }

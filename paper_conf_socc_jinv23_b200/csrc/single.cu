@@ -1,0 +1,601 @@
+// Single-pass find + compare for sm_100a: ONE streaming kernel tests the
+// PAM on both strands and compares every passing site against every guide of the launch,
+// so neither item lists (4 B per item, written and re-read) nor PAM masks ever reach HBM.
+//
+// Paper: the host hands the search kernel's PAM sites to the compare kernel; the
+// compare kernel (Listing 1) counts, per site and query, the mismatched bases
+// over the query's non-N positions and appends a hit when the count is
+// <= the threshold through an atomic counter.
+//
+// B200 design (DESIGN.md §5 "Single pass"):
+//  * persistent CTAs, one per SM, streaming tiles of the lo / hi / nm (/ vs) planes
+//    through a 4-stage shared-memory ring filled by the TMA engine (cp.async.bulk +
+//    mbarrier); tiles are grabbed dynamically (one global atomic per tile), and the
+//    refill of a stage is issued by whichever warp releases it last (a shared-memory
+//    counter per stage) -- no producer warp, no blocking on an "empty" barrier;
+//  * 16 warps, one plane word (32 window starts) per lane: the lane copies its three
+//    words of each plane into registers, releases the stage at once, evaluates the
+//    pattern and its reverse complement bit-parallel (the finder's multiplexer test), and
+//    appends every passing start to its warp's ring queue together with the start's three
+//    32-bit window slices (funnel shifts of the registers: no global window gathers);
+//  * full batches of 64 queued sites (2 per lane) are compared against the launch's guide
+//    blocks in two steps:
+//      filter -- per site, position pair q and 32-guide block, one 32-bit shared-memory
+//        lookup indexed by the pair's two genome bases gives "the pair holds >= 1
+//        mismatch" for all 32 guides; a carry-save tree counts those bits, and a guide
+//        survives iff the count of mismatched pairs is <= its threshold.  Every mismatch
+//        lies in some pair, so #mismatched pairs <= #mismatches: a hit always survives
+//        (necessary condition), while on a random genome only ~0.3% of (site, guide)
+//        comparisons do at t = 6 (about 70x the hit rate);
+//      verify -- each survivor's exact count from its record: popc over the compared
+//        positions of (window != guide) | N (Listing 1's rows, bit-parallel), or the
+//        one-hot IUPAC form for degenerate letters; hits are appended warp-aggregated
+//        (one atomic per warp and round).
+//    Per comparison that is ~0.5 ALU op + 0.3 shared-memory lookups of the filter plus the
+//    rare verifications, against ~1.2 + 0.3 (64-bit lookups) for the exact pair-table sum.
+#include <algorithm>
+#include <mutex>
+
+#include <cuda_runtime.h>
+
+#include "cof_internal.h"
+#include "dev_common.cuh"
+#include "csa_gen.cuh"
+
+namespace cof {
+
+constexpr int SW = 16;                    // warps per CTA (4 per SM sub-partition: <= 128 registers)
+constexpr int STHREADS = 32 * SW;
+constexpr int STW = 32 * SW;              // plane words per tile (one per lane)
+constexpr int SLOAD = STW + 4;            // words per plane and stage: tile + halo (16-byte multiple)
+constexpr int SSTAGES = 4;
+constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
+constexpr uint32_t SQ = 128;              // queued sites per warp (16-byte entries)
+constexpr int SR = 2;                     // sites per lane and batch
+constexpr uint32_t SBATCH = 32 * SR;
+constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
+constexpr uint32_t S_END = 0xFFFFFFFFu;   // tile id: no more tiles
+static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH, "ring");
+
+struct SingleArgs {
+    const uint32_t* lo;
+    const uint32_t* hi;
+    const uint32_t* nm;
+    const uint32_t* vs;               // valid-start plane (multi-segment chunks) or nullptr
+    uint64_t limit;                   // no window start >= limit is valid
+    uint32_t n_tiles;
+    unsigned int* ticket;             // dynamic tile counter (zeroed per launch)
+    unsigned long long* hits;
+    uint64_t cap;
+    unsigned long long* counters;     // [0] n_fwd, [1] n_rev (PAM sites), [2] n_hits
+    const uint32_t* ftab[2];          // filter tables of this launch's blocks, per strand
+    const uint4* vrec[2];             // verification records of this launch's guides, per strand
+    uint32_t n_blocks;                // guide blocks in this launch
+    uint32_t block_base;              // first block of this launch (global guide = (base + b) * 32 + k)
+    uint32_t count_items;             // count PAM sites (one launch per search does)
+    uint32_t ne;                      // non-N pattern letters per strand
+    uint32_t pj[2][32];               // their window offsets
+    uint4 psel[2][32];                // their IUPAC sets as splat words {A, C, G, T}
+    uint32_t p0[2];                   // first compared window offset per strand
+    uint32_t contig;                  // compared positions contiguous from p0 (both strands)
+    uint32_t cmp_mask;                // n_cmp low bits: the compared positions of a window at p0
+    uint32_t j1[2][16], j2[2][16];    // pair offsets relative to p0 (j2 = 0xFF: single position)
+    uint32_t meta[SMAX_BLOCKS][8];    // per block: threshold planes T0..T5, valid guide mask
+};
+
+// Membership of 32 bases in an IUPAC set given as splat words (the finder's multiplexer);
+// a genome N is in no set (reading G2).
+__device__ __forceinline__ uint32_t s_member(uint32_t lo, uint32_t hi, uint32_t nm, uint4 sel) {
+    const uint32_t t0 = (hi & sel.z) | (~hi & sel.x);
+    const uint32_t t1 = (hi & sel.w) | (~hi & sel.y);
+    return ((lo & t1) | (~lo & t0)) & ~nm;
+}
+
+// Filter: bit k of the result = guide k of the block survives (its number of pairs with a
+// mismatch is <= its threshold).  TC >= 0: one threshold for every guide of the launch.
+template <int NP, int TC>
+__device__ __forceinline__ uint32_t filter_pass(const uint32_t (&v)[NP], const uint32_t* __restrict__ m) {
+    uint32_t c[5];
+    nz_count<NP>(v, c);
+    uint32_t bw;                       // borrow out of (t - count): set where count > t
+    if constexpr (TC >= 0) {
+        bw = (TC & 1) ? 0u : c[0];
+#pragma unroll
+        for (int w = 1; w < 5; w++) bw = ((TC >> w) & 1) ? (c[w] & bw) : (c[w] | bw);
+    } else {
+        bw = c[0] & ~m[0];
+#pragma unroll
+        for (int w = 1; w < 6; w++) {
+            const uint32_t cw = w < 5 ? c[w] : 0u;
+            bw = (~m[w] & cw) | (~m[w] & bw) | (cw & bw);
+        }
+    }
+    return m[6] & ~bw;
+}
+
+template <uint32_t OFF>
+__device__ __forceinline__ uint32_t lds32(uint32_t addr) {
+    uint32_t x;
+    asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(x) : "r"(addr), "n"(OFF));
+    return x;
+}
+
+// The NP filter lookups of one site in block b: pair q at base[q] + OFF + q * 64.
+template <int NP, uint32_t OFF, int Q = 0>
+__device__ __forceinline__ void lds_filter(const uint32_t (&base)[NP], uint32_t (&v)[NP]) {
+    if constexpr (Q < NP) {
+        v[Q] = lds32<OFF + (uint32_t)Q * 64u>(base[Q]);
+        lds_filter<NP, OFF, Q + 1>(base, v);
+    }
+}
+
+// Shared-memory addresses of the NP filter entries of a site (pair q's entry read at
+// base[q] + q * 64 + block offset); tbase = the strand's table (64-byte aligned).
+template <int NP>
+__device__ __forceinline__ void site_bases(const SingleArgs& a, uint32_t tbase, uint32_t sd, uint32_t wl,
+                                           uint32_t wh, uint32_t wn, uint32_t (&base)[NP]) {
+    if (a.contig && (wn & a.cmp_mask) == 0) {
+        // pair q = window offsets (2q, 2q + 1): its 4-bit entry index lo(b1) | lo(b2) << 1 |
+        // hi(b1) << 2 | hi(b2) << 3 is nibble q/2 of Y (even q) or Z (odd q)
+        const uint32_t Y = (wl & 0x33333333u) | ((wh & 0x33333333u) << 2);
+        const uint32_t Z = ((wl >> 2) & 0x33333333u) | (wh & 0xCCCCCCCCu);
+#pragma unroll
+        for (int q = 0; q < NP; q++) {
+            const uint32_t src = (q & 1) ? Z : Y;
+            const int k = q >> 1;
+            const uint32_t off = k == 0 ? (src << 2) & 0x3Cu : (src >> (4 * k - 2)) & 0x3Cu;
+            base[q] = tbase | off;
+        }
+        return;
+    }
+#pragma unroll
+    for (int q = 0; q < NP; q++) {
+        const uint32_t j1 = a.j1[sd][q], j2 = a.j2[sd][q];
+        const uint32_t b1 = ((wn >> j1) & 1u) ? 4u : (((wl >> j1) & 1u) | (((wh >> j1) & 1u) << 1));
+        uint32_t b2 = 0;
+        if (j2 < 32u) b2 = ((wn >> j2) & 1u) ? 4u : (((wl >> j2) & 1u) | (((wh >> j2) & 1u) << 1));
+        base[q] = tbase + pair_entry(NP, (uint32_t)q, b1, b2) * 4u - (uint32_t)q * 64u;
+    }
+}
+
+__device__ __forceinline__ unsigned long long s_key(uint32_t pos, uint32_t strand, uint32_t guide, uint32_t mm) {
+    return ((unsigned long long)pos << 32) | ((unsigned long long)strand << 31) | ((unsigned long long)guide << 7) |
+           (unsigned long long)mm;
+}
+
+template <int NP, int TC, bool CONCRETE>
+__global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_constant__ SingleArgs a) {
+    extern __shared__ __align__(128) uint8_t smem[];
+    // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise][verification
+    //         records: '+' n_blocks*32 x 32 B, 64 B, '-'][ring: SSTAGES x SPL x SLOAD words]
+    //         [queues: SW x SQ x uint4][tile ids, release counters][full mbarriers]
+    constexpr uint32_t FBW = (NP * 25u + 15u) & ~15u;
+    const uint32_t nb = a.n_blocks;
+    uint32_t* s_ftab = reinterpret_cast<uint32_t*>(smem);
+    uint4* s_vrec = reinterpret_cast<uint4*>(smem + 2 * nb * FBW * 4 + 64);
+    uint32_t* ring = reinterpret_cast<uint32_t*>(smem + 2 * nb * FBW * 4 + 64 + 2 * nb * 32 * 32 + 64);
+    uint4* queues = reinterpret_cast<uint4*>(ring + SSTAGES * SPL * SLOAD);
+    uint32_t* s_tile = reinterpret_cast<uint32_t*>(queues + SW * SQ);
+    uint32_t* s_rel = s_tile + SSTAGES;
+    uint64_t* full = reinterpret_cast<uint64_t*>(s_tile + 2 * SSTAGES);
+
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const bool vsp = a.vs != nullptr;
+    // grab the next tile and stream it into stage st (or mark the stage as the end)
+    auto refill = [&](int st) {
+        const uint32_t tile = atomicAdd(a.ticket, 1u);
+        if (tile >= a.n_tiles) {
+            s_tile[st] = S_END;
+            mbar_arrive(&full[st]);
+            return;
+        }
+        s_tile[st] = tile;
+        const size_t w0 = (size_t)tile * STW;
+        uint32_t* S = ring + st * SPL * SLOAD;
+        fence_proxy_async_smem();
+        mbar_arrive_expect_tx(&full[st], (vsp ? 4 : 3) * SLOAD * 4);
+        bulk_g2s(S + 0 * SLOAD, a.lo + w0, SLOAD * 4, &full[st]);
+        bulk_g2s(S + 1 * SLOAD, a.hi + w0, SLOAD * 4, &full[st]);
+        bulk_g2s(S + 2 * SLOAD, a.nm + w0, SLOAD * 4, &full[st]);
+        if (vsp) bulk_g2s(S + 3 * SLOAD, a.vs + w0, SLOAD * 4, &full[st]);
+    };
+    {   // guide tables -> shared memory (both strands)
+        const uint32_t nf = nb * FBW;
+        for (uint32_t i = tid; i < nf; i += STHREADS) {
+            s_ftab[i] = __ldg(a.ftab[0] + i);
+            s_ftab[nf + 16 + i] = __ldg(a.ftab[1] + i);
+        }
+        const uint32_t nv = nb * 32 * 2;
+        for (uint32_t i = tid; i < nv; i += STHREADS) {
+            s_vrec[i] = __ldg(a.vrec[0] + i);
+            s_vrec[nv + 4 + i] = __ldg(a.vrec[1] + i);
+        }
+    }
+    if (tid == 0) {
+        for (int s = 0; s < SSTAGES; s++) {
+            mbar_init(&full[s], 1);
+            s_rel[s] = 0;
+        }
+        fence_mbar_init();
+        for (int s = 0; s < SSTAGES; s++) refill(s);
+    }
+    __syncthreads();
+
+    uint4* queue = queues + warp * SQ;
+    // strand 1's tables start 64 bytes past a 128-byte boundary: the 16 entries of a pair
+    // then sit in the other 16 banks than strand 0's, so a batch mixing '+' and '-' sites
+    // never has two lanes in one bank (see single_smem)
+    const uint32_t tb0 = smem_u32(s_ftab), tb1 = tb0 + nb * FBW * 4 + 64;
+    const uint4* vrec1 = s_vrec + nb * 64 + 4;
+    uint32_t head = 0, q_n = 0;           // warp-uniform ring state
+    unsigned long long cnt_f = 0, cnt_r = 0;
+
+    // per-lane state of the tile being expanded: its plane words and the PAM bits not yet queued
+    uint32_t lo0 = 0, lo1 = 0, lo2 = 0, hi0 = 0, hi1 = 0, hi2 = 0, nm0 = 0, nm1 = 0, nm2 = 0;
+    uint32_t pend0 = 0u, pend1 = 0u, pbase = 0;
+    const int w = warp * 32 + lane;
+    uint32_t k = 0;
+    bool tiles_done = false;
+    // One loop, one call site each for the batch comparison and the queue append (the
+    // kernel's code stays small): compare while a full batch is queued, else append the
+    // pending sites of the current tile, else take the next tile.
+    for (;;) {
+        if (q_n >= SBATCH || (tiles_done && q_n > 0)) {
+            // ---------------- compare a batch: ring[head, head + n_items)
+            const uint32_t n_items = min(q_n, SBATCH);
+            uint32_t base[SR][NP], wl[SR], wh[SR], wn[SR], pos[SR], sd[SR];
+#pragma unroll
+            for (int r = 0; r < SR; r++) {
+                const uint32_t i = (uint32_t)r * 32 + lane;
+                // a missing site gets an all-N window (every pair mismatches) and is masked below
+                const uint4 e = i < n_items ? queue[(head + i) & (SQ - 1)] : make_uint4(0u, 0u, 0u, 0x7FFFFFFFu);
+                pos[r] = e.x;
+                wl[r] = e.y;
+                wh[r] = e.z;
+                sd[r] = e.w >> 31;
+                wn[r] = e.w & 0x7FFFFFFFu;
+                site_bases<NP>(a, sd[r] ? tb1 : tb0, sd[r], wl[r], wh[r], wn[r], base[r]);
+            }
+            const uint32_t okm0 = (uint32_t)lane < n_items ? ~0u : 0u, okm1 = 32u + lane < n_items ? ~0u : 0u;
+            for (uint32_t b = 0; b < nb; b += 4) {
+                const uint32_t* m = a.meta[b];
+                uint32_t p[SR][4];
+#pragma unroll
+                for (int r = 0; r < SR; r++) {
+                    uint32_t v[NP];
+                    lds_filter<NP, 0 * FBW * 4>(base[r], v);
+                    p[r][0] = filter_pass<NP, TC>(v, m);
+                    lds_filter<NP, 1 * FBW * 4>(base[r], v);
+                    p[r][1] = filter_pass<NP, TC>(v, m + 8);
+                    lds_filter<NP, 2 * FBW * 4>(base[r], v);
+                    p[r][2] = filter_pass<NP, TC>(v, m + 16);
+                    lds_filter<NP, 3 * FBW * 4>(base[r], v);
+                    p[r][3] = filter_pass<NP, TC>(v, m + 24);
+                    const uint32_t ok = r == 0 ? okm0 : okm1;
+                    p[r][0] &= ok; p[r][1] &= ok; p[r][2] &= ok; p[r][3] &= ok;
+                }
+                // ---- verify the survivors (blocks past the plan have valid mask 0): warp-
+                // uniform rounds, every lane with a survivor left takes one per round; the
+                // round's hits are appended with one atomic
+#pragma unroll
+                for (int r = 0; r < SR; r++) {
+                    uint32_t m0 = p[r][0], m1 = p[r][1], m2 = p[r][2], m3 = p[r][3];
+                    while (__any_sync(0xFFFFFFFFu, (m0 | m1 | m2 | m3) != 0u)) {
+                        bool hit = false;
+                        uint32_t g = 0, mm = 0;
+                        if (m0 | m1 | m2 | m3) {
+                            uint32_t bi, kk;
+                            if (m0) { kk = __ffs(m0) - 1; m0 &= m0 - 1; bi = 0; }
+                            else if (m1) { kk = __ffs(m1) - 1; m1 &= m1 - 1; bi = 1; }
+                            else if (m2) { kk = __ffs(m2) - 1; m2 &= m2 - 1; bi = 2; }
+                            else { kk = __ffs(m3) - 1; m3 &= m3 - 1; bi = 3; }
+                            g = (b + bi) * 32u + kk;                       // launch-local guide
+                            const uint4* rec = (sd[r] ? vrec1 : s_vrec) + 2u * g;
+                            const uint4 r0 = rec[0];                       // {lo, hi, care, t}
+                            uint32_t mis;
+                            if constexpr (CONCRETE) {
+                                mis = ((wl[r] ^ r0.x) | (wh[r] ^ r0.y) | wn[r]) & r0.z;
+                            } else {
+                                const uint4 oh = rec[1];                   // one-hot {A, C, G, T}
+                                const uint32_t nn = ~wn[r];
+                                const uint32_t match = (oh.x & ~wl[r] & ~wh[r] & nn) | (oh.y & wl[r] & ~wh[r] & nn) |
+                                                       (oh.z & ~wl[r] & wh[r] & nn) | (oh.w & wl[r] & wh[r] & nn);
+                                mis = r0.z & ~match;
+                            }
+                            mm = (uint32_t)__popc(mis);
+                            hit = mm <= r0.w;
+                        }
+                        const unsigned hm = __ballot_sync(0xFFFFFFFFu, hit);
+                        if (hm) {
+                            const int leader = __ffs(hm) - 1;
+                            unsigned long long o = 0;
+                            if (lane == leader) o = atomicAdd(&a.counters[2], (unsigned long long)__popc(hm));
+                            o = __shfl_sync(0xFFFFFFFFu, o, leader) + (unsigned)__popc(hm & lanemask_lt());
+                            if (hit && o < a.cap) a.hits[o] = s_key(pos[r], sd[r], a.block_base * 32u + g, mm);
+                        }
+                    }
+                }
+                if (b + 4 < nb) {
+#pragma unroll
+                    for (int r = 0; r < SR; r++)
+#pragma unroll
+                        for (int q = 0; q < NP; q++) base[r][q] += 4 * FBW * 4;
+                }
+            }
+            __syncwarp();
+            head = (head + SBATCH) & (SQ - 1);
+            q_n -= n_items;
+            continue;
+        }
+        if (tiles_done) break;
+        if (__any_sync(0xFFFFFFFFu, (pend0 | pend1) != 0u)) {
+            // ---------------- append pending sites of one strand (all '+' first, then '-')
+            const bool any0 = __any_sync(0xFFFFFFFFu, pend0 != 0u);
+            const uint32_t sdw = any0 ? 0u : 1u;          // warp-uniform strand of this append
+            uint32_t m = any0 ? pend0 : pend1;
+            const uint32_t p0 = a.p0[sdw];
+            const uint32_t Al = __funnelshift_r(lo0, lo1, p0), Bl = __funnelshift_r(lo1, lo2, p0);
+            const uint32_t Ah = __funnelshift_r(hi0, hi1, p0), Bh = __funnelshift_r(hi1, hi2, p0);
+            const uint32_t An = __funnelshift_r(nm0, nm1, p0), Bn = __funnelshift_r(nm1, nm2, p0);
+            const uint32_t c = (uint32_t)__popc(m);
+            uint32_t x = c;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+                if (lane >= o) x += y;
+            }
+            const uint32_t total = __shfl_sync(0xFFFFFFFFu, x, 31);
+            const uint32_t take = min(SQ - q_n, total);
+            const uint32_t tail = head + q_n;
+            uint32_t rank = x - c;
+            while (m && rank < take) {
+                const int bit = __ffs(m) - 1;
+                m &= m - 1;
+                const uint32_t wl = __funnelshift_r(Al, Bl, bit), wh = __funnelshift_r(Ah, Bh, bit);
+                const uint32_t wn = __funnelshift_r(An, Bn, bit);
+                queue[(tail + rank) & (SQ - 1)] = make_uint4(pbase + (uint32_t)bit, wl, wh,
+                                                               (wn & 0x7FFFFFFFu) | (sdw << 31));
+                rank++;
+            }
+            if (any0) pend0 = m; else pend1 = m;
+            __syncwarp();
+            q_n += take;
+            continue;
+        }
+        // ---------------- next tile: words -> registers, release the stage, PAM test
+        const int st = (int)(k % SSTAGES);
+        mbar_wait_parity(&full[st], (k / SSTAGES) & 1u);
+        k++;
+        const uint32_t tile = s_tile[st];
+        if (tile == S_END) {
+            tiles_done = true;
+            continue;
+        }
+        const uint32_t* S = ring + st * SPL * SLOAD;
+        lo0 = S[w]; lo1 = S[w + 1]; lo2 = S[w + 2];
+        hi0 = S[SLOAD + w]; hi1 = S[SLOAD + w + 1]; hi2 = S[SLOAD + w + 2];
+        nm0 = S[2 * SLOAD + w]; nm1 = S[2 * SLOAD + w + 1]; nm2 = S[2 * SLOAD + w + 2];
+        uint32_t valid = vsp ? S[3 * SLOAD + w] : ~0u;
+        __syncwarp();
+        if (lane == 0) {   // this warp is done with the stage; the last of the SW warps refills it
+            __threadfence_block();
+            if (atomicAdd(&s_rel[st], 1u) == SW - 1) {
+                s_rel[st] = 0;
+                __threadfence_block();
+                refill(st);
+            }
+        }
+        const uint64_t pw = ((uint64_t)tile * STW + (uint32_t)w) * 32u;   // first start of this word
+        if (pw + 32 > a.limit) valid &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
+        pend0 = pend1 = valid;
+        for (uint32_t e = 0; e < a.ne; e++) {
+            const uint32_t j0 = a.pj[0][e], j1 = a.pj[1][e];
+            pend0 &= s_member(__funnelshift_r(lo0, lo1, j0), __funnelshift_r(hi0, hi1, j0),
+                              __funnelshift_r(nm0, nm1, j0), a.psel[0][e]);
+            pend1 &= s_member(__funnelshift_r(lo0, lo1, j1), __funnelshift_r(hi0, hi1, j1),
+                              __funnelshift_r(nm0, nm1, j1), a.psel[1][e]);
+        }
+        if (a.count_items) {
+            cnt_f += (unsigned)__popc(pend0);
+            cnt_r += (unsigned)__popc(pend1);
+        }
+        pbase = (uint32_t)pw;
+    }
+    if (a.count_items) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            cnt_f += __shfl_xor_sync(0xFFFFFFFFu, cnt_f, o);
+            cnt_r += __shfl_xor_sync(0xFFFFFFFFu, cnt_r, o);
+        }
+        if (lane == 0) {
+            atomicAdd(&a.counters[0], cnt_f);
+            atomicAdd(&a.counters[1], cnt_r);
+        }
+    }
+}
+
+// ============================================================================ host side
+typedef void (*SingleFn)(SingleArgs);
+
+template <int NP, int TC, bool CONCRETE>
+static SingleFn single_fn_t() { return cof_single_kernel<NP, TC, CONCRETE>; }
+
+template <int NP>
+static SingleFn single_fn_np(int tc, bool concrete) {
+    if constexpr (NP == 10 || NP == 12) {
+        if (concrete) {
+            switch (tc) {
+                case 0: return single_fn_t<NP, 0, true>();
+                case 1: return single_fn_t<NP, 1, true>();
+                case 2: return single_fn_t<NP, 2, true>();
+                case 3: return single_fn_t<NP, 3, true>();
+                case 4: return single_fn_t<NP, 4, true>();
+                case 5: return single_fn_t<NP, 5, true>();
+                case 6: return single_fn_t<NP, 6, true>();
+                case 7: return single_fn_t<NP, 7, true>();
+                default: break;
+            }
+        }
+    }
+    return single_fn_t<NP, -1, false>();
+}
+
+static SingleFn single_fn(uint32_t np, int tc, bool concrete) {
+    switch (np) {
+        case 1: return single_fn_np<1>(tc, concrete);
+        case 2: return single_fn_np<2>(tc, concrete);
+        case 3: return single_fn_np<3>(tc, concrete);
+        case 4: return single_fn_np<4>(tc, concrete);
+        case 5: return single_fn_np<5>(tc, concrete);
+        case 6: return single_fn_np<6>(tc, concrete);
+        case 7: return single_fn_np<7>(tc, concrete);
+        case 8: return single_fn_np<8>(tc, concrete);
+        case 9: return single_fn_np<9>(tc, concrete);
+        case 10: return single_fn_np<10>(tc, concrete);
+        case 11: return single_fn_np<11>(tc, concrete);
+        case 12: return single_fn_np<12>(tc, concrete);
+        case 13: return single_fn_np<13>(tc, concrete);
+        case 14: return single_fn_np<14>(tc, concrete);
+        case 15: return single_fn_np<15>(tc, concrete);
+        case 16: return single_fn_np<16>(tc, concrete);
+        default: return nullptr;
+    }
+}
+
+static size_t single_smem(uint32_t np, uint32_t nb) {
+    const size_t fbw = filter_block_words(np);
+    // (+ 64 bytes after the '+' filter tables and 64 after the '+' records: bank offsets)
+    return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * 32 + 64 + (size_t)SSTAGES * SPL * SLOAD * 4 +
+           (size_t)SW * SQ * 16 + 2 * SSTAGES * 4 + SSTAGES * 8;
+}
+
+static constexpr size_t SMEM_MAX = 227 * 1024;
+
+// Guide blocks per launch: as many as fit the shared-memory budget (a multiple of 4).
+static uint32_t single_blocks_per_launch(uint32_t np) {
+    uint32_t nb = SMAX_BLOCKS;
+    while (nb > 4 && single_smem(np, nb) > SMEM_MAX) nb -= 4;
+    return nb;
+}
+
+// The single-pass kernel handles one-word windows: every compared offset of both strands
+// within [p0, p0 + 31) (bit 31 of the queued N-window carries the strand), <= 16 pairs.
+static bool single_shape_ok(const cof_plan* plan) {
+    if (plan->L > 32) return false;
+    for (int s = 0; s < 2; s++) {
+        const PairLayout& pl = plan->pairs[s];
+        if (pl.wide || pl.n_pairs > 16) return false;
+        const uint64_t uc = plan->union_care[s];
+        if (!uc) continue;
+        const uint32_t span = 64u - (uint32_t)__builtin_clzll(uc) - pl.p0;
+        if (span > 31) return false;
+    }
+    return plan->pairs[0].n_pairs == plan->pairs[1].n_pairs;
+}
+
+// The filter pays when few (site, guide) pairs survive it: thresholds well below the pair
+// count (COF_SINGLE=1 forces the single pass whenever the shape allows, 0 disables it).
+bool single_supported(const cof_plan* plan, bool strict) {
+    static int env = -2;
+    if (env == -2) {
+        const char* e = getenv("COF_SINGLE");
+        env = e ? atoi(e) : -1;
+    }
+    if (env == 0 || !single_shape_ok(plan)) return false;
+    if (env == 1 || !strict) return true;
+    const uint32_t np = plan->pairs[0].n_pairs;
+    uint32_t tmax = 0;
+    for (uint32_t i = 0; i < plan->n_guides; i++) tmax = std::max<uint32_t>(tmax, plan->max_mm[i]);
+    return tmax + 3 <= np;
+}
+
+static std::mutex g_single_mu;
+
+cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, unsigned int* tickets,
+                      uint64_t* hits, uint64_t hits_cap, cudaStream_t stream) {
+    const uint64_t L = plan->L;
+    if (dev->n_bases >= (1ull << 32)) return set_error(COF_E_ARG, "single pass: n_bases must be < 2^32");
+    if (((uintptr_t)dev->lo | (uintptr_t)dev->hi | (uintptr_t)dev->nm | (uintptr_t)dev->vs) & 15)
+        return set_error(COF_E_ARG, "single pass: planes must be 16-byte aligned");
+    if (dev->n_segs && !dev->vs) return set_error(COF_E_ARG, "single pass: multi-segment chunk without vs plane");
+    uint64_t limit = dev->n_bases >= L ? dev->n_bases - L + 1 : 0;
+    if (!dev->n_segs && limit > dev->n_owned) limit = dev->n_owned;
+    const uint32_t n_tiles = (uint32_t)((limit + (uint64_t)STW * 32 - 1) / ((uint64_t)STW * 32));
+    const uint32_t np = plan->pairs[0].n_pairs;
+    int ut = (int)plan->max_mm[0];
+    for (uint32_t i = 1; i < plan->n_guides && ut >= 0; i++)
+        if (plan->max_mm[i] != plan->max_mm[0]) ut = -1;
+    const bool concrete = !plan->any_degenerate;
+    SingleFn fn = single_fn(np, ut, concrete);
+    if (!fn) return set_error(COF_E_STATE, "single pass: %u pairs", np);
+    int dev_id = 0;
+    cudaGetDevice(&dev_id);
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev_id);
+    static thread_local SingleArgs A;
+    A.lo = dev->lo; A.hi = dev->hi; A.nm = dev->nm;
+    A.vs = dev->n_segs ? dev->vs : nullptr;
+    A.limit = limit;
+    A.n_tiles = n_tiles;
+    A.hits = (unsigned long long*)hits;
+    A.cap = hits_cap;
+    A.counters = (unsigned long long*)(pd + plan->lay.counters);
+    A.ne = plan->pam[0].n;
+    if (plan->pam[1].n != A.ne || A.ne > 32) return set_error(COF_E_STATE, "single pass: PAM letter counts");
+    for (int s = 0; s < 2; s++) {
+        for (uint32_t k = 0; k < A.ne; k++) {
+            const uint32_t set = plan->pam[s].set[k];
+            A.pj[s][k] = plan->pam[s].j[k];
+            A.psel[s][k] = make_uint4(0u - (set & 1u), 0u - ((set >> 1) & 1u), 0u - ((set >> 2) & 1u),
+                                      0u - ((set >> 3) & 1u));
+        }
+        const PairLayout& pl = plan->pairs[s];
+        A.p0[s] = pl.p0;
+        for (uint32_t q = 0; q < 16; q++) {
+            A.j1[s][q] = q < pl.n_pairs ? pl.j1[q] - pl.p0 : 0u;
+            A.j2[s][q] = q < pl.n_pairs && pl.j2[q] < 0xFE ? pl.j2[q] - pl.p0 : 0xFFu;
+        }
+    }
+    A.contig = plan->pairs[0].contig && plan->pairs[1].contig && plan->pairs[0].n_cmp == plan->pairs[1].n_cmp;
+    A.cmp_mask = plan->pairs[0].n_cmp >= 32 ? ~0u : ((1u << plan->pairs[0].n_cmp) - 1u);
+    const uint32_t bpl = single_blocks_per_launch(np);
+    const uint32_t fbw = filter_block_words(np);
+    const uint32_t* pm = (const uint32_t*)(plan->image.data() + plan->lay.pmeta_fwd);
+    {
+        std::lock_guard<std::mutex> lk(g_single_mu);   // (per device state; cheap, set every call)
+        cudaError_t e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)single_smem(np, bpl));
+        if (e != cudaSuccess) return cuda_error(e, "single pass smem attribute");
+    }
+    uint32_t li = 0;
+    for (uint32_t bb = 0; bb < plan->n_blocks; bb += bpl, li++) {
+        const uint32_t nbl = std::min(bpl, plan->n_blocks - bb);
+        // whole groups of 4 blocks: padding blocks (zero tables in the plan image) have no valid guide
+        const uint32_t nb4 = (nbl + 3) & ~3u;
+        A.n_blocks = nb4;
+        A.block_base = bb;
+        A.count_items = li == 0;
+        A.ticket = tickets + li;
+        A.ftab[0] = (const uint32_t*)(pd + plan->lay.ftab_fwd) + (size_t)bb * fbw;
+        A.ftab[1] = (const uint32_t*)(pd + plan->lay.ftab_rev) + (size_t)bb * fbw;
+        A.vrec[0] = (const uint4*)(pd + plan->lay.vrec_fwd) + (size_t)bb * 64;
+        A.vrec[1] = (const uint4*)(pd + plan->lay.vrec_rev) + (size_t)bb * 64;
+        for (uint32_t k = 0; k < SMAX_BLOCKS; k++)
+            for (int w = 0; w < 8; w++) A.meta[k][w] = k < nbl ? pm[(size_t)(bb + k) * 8 + w] : 0u;
+        if (n_tiles == 0) continue;
+        uint32_t grid = (uint32_t)sms;
+        if (grid > n_tiles) grid = n_tiles;
+        fn<<<grid, STHREADS, single_smem(np, nb4), stream>>>(A);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_error(e, "cof_single_kernel launch");
+        count_launches(1);
+    }
+    return COF_OK;
+}
+
+uint32_t single_launches(const cof_plan* plan) {
+    const uint32_t bpl = single_blocks_per_launch(plan->pairs[0].n_pairs);
+    return (plan->n_blocks + bpl - 1) / bpl;
+}
+
+}  // namespace cof

@@ -94,6 +94,24 @@ def use_fused(plan, n_guides: int) -> bool:
     return n_guides >= FUSED_MIN_GUIDES or pam_density(plan.pattern) >= FUSED_MIN_DENSITY
 
 
+PATHS = ("single", "fused", "twocall")
+
+
+def choose_path(plan, n_guides: int) -> str:
+    """The device path of a plan: "single" (one streaming find + compare kernel, filter +
+    verify comparer; cof_single_supported), else "fused" (finder masks -> mask-expanding
+    pair-table comparer) or "twocall" (ordered item lists, the paper's two kernels).
+    COF_PATH=single|fused|twocall overrides (falling back when unsupported)."""
+    env = os.environ.get("COF_PATH")
+    if env == "twocall":
+        return "twocall"
+    if env in (None, "single") and cof.cof_single_supported(plan):
+        return "single"
+    if env == "fused" or use_fused(plan, n_guides):
+        return "fused" if cof.cof_find_compare_supported(plan) else "twocall"
+    return "twocall"
+
+
 def plan_chunks(lengths, L: int, chunk_bases: int | None = None, pack_bases: int | None = None):
     """Split chromosomes into pieces of at most ``chunk_bases`` owned window starts (whole
     chromosomes if None): every valid start 0 <= p <= len-L belongs to exactly one piece.
@@ -270,9 +288,18 @@ class Searcher:
         self._hits_cap = 0
         self._rec_cap = 0
         self.d_records = None
-        # fused find+compare (no item lists) when the guide table fits the fused kernel and there
-        # are enough guides to amortise the in-kernel expansion (COF_FUSED=0/1 overrides)
-        self.fused = use_fused(self.plan, len(guides))
+        # single pass, fused (masks) or two-call (item lists): choose_path
+        self.path = choose_path(self.plan, len(guides))
+
+    @property
+    def fused(self) -> bool:
+        """No item lists (single pass or the masks path)."""
+        return self.path != "twocall"
+
+    @fused.setter
+    def fused(self, on: bool):
+        # True: the masks path (the single pass is chosen with .path = "single")
+        self.path = "fused" if on and cof.cof_find_compare_supported(self.plan) else "twocall"
 
     # ---- device buffers sized for the largest chunk seen so far
     def reserve(self, max_bases: int, hits_cap: int):
@@ -306,14 +333,17 @@ class Searcher:
         s = self.stream
         if not self.fused and self.d_items.shape[1] < items_cap:   # path switched after reserve()
             self.d_items = torch.empty((2, items_cap), dtype=torch.int32, device=self.device)
-        if self.fused:
+        if self.path == "fused":
             cof.cof_find_masks(self.plan, self.plan_dev, dchunk, self.d_find_ws, s)
-        else:
+        elif self.path == "twocall":
             nf, nr = cof.cof_find_pam(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_items[0],
                                       self.d_items[1], items_cap, s)
         while True:
             try:
-                if self.fused:
+                if self.path == "single":
+                    nh = cof.cof_search_single(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_hits,
+                                               self._hits_cap, s)
+                elif self.fused:
                     nh = cof.cof_compare_masks(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_hits,
                                                self._hits_cap, s)
                 else:
@@ -550,17 +580,22 @@ def _as_arrays(seqs):
             (np.frombuffer(s.encode(), dtype=np.uint8) if isinstance(s, str) else s) for s in seqs]
 
 
-def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda", pack_bases=None, fused=None):
+def search(seqs, pattern, guides, thresholds, chunk_bases=None, device="cuda", pack_bases=None, fused=None,
+           path=None):
     """Convenience: whole search of ``seqs`` (list of uint8 ASCII arrays / bytes) on one GPU.
     ``pack_bases`` packs chromosome pieces into multi-segment chunks (0 = one chunk);
-    ``fused`` False forces the two-call path (item lists) even when the fused one fits."""
+    ``fused`` False forces the two-call path (item lists), True the masks path;
+    ``path`` = "single" | "fused" | "twocall" picks the device path explicitly (the single
+    pass is then run even when its filter is not selective, if the plan's shape allows)."""
     L = len(pattern)
     arrs = _as_arrays(seqs)
     chunks = plan_chunks([len(a) for a in arrs], L, chunk_bases, pack_bases)
     host = HostGenome(arrs, chunks)
     srch = Searcher(pattern, guides, thresholds, device)
     if fused is not None:
-        srch.fused = bool(fused) and cof.cof_find_compare_supported(srch.plan)
+        srch.fused = bool(fused)
+    if path is not None:
+        srch.path = path
     return srch.search_host(host)
 
 

@@ -45,6 +45,10 @@ def test_cli_end_to_end(tmp_path):
                   f"{h['strand'].decode()}\t{int(h['mm'])}\n" for h in ref)
     assert len(ref) > 10
     assert out.read_text() == exp
+    # --gpus 2: one pipeline per GPU (both on the one GPU of the test box), same TSV
+    out2 = tmp_path / "out2.txt"
+    assert cli.main([str(inp), "G", str(out2), "--chunk-bases", "7777", "--gpus", "2"]) == 0
+    assert out2.read_text() == exp
 
 
 def test_parse_input_bulges():
