@@ -41,6 +41,7 @@
 #include "cof_internal.h"
 #include "dev_common.cuh"
 #include "csa_gen.cuh"
+#include "filter_circuit.cuh"
 
 namespace cof {
 
@@ -53,6 +54,7 @@ constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
 constexpr uint32_t SQ = 128;              // queued sites per warp (16-byte entries)
 constexpr int SR = 2;                     // sites per lane and batch
 constexpr uint32_t SBATCH = 32 * SR;
+constexpr uint32_t SVC = 64;              // survivor entries per warp (ring)
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
 constexpr uint32_t S_END = 0xFFFFFFFFu;   // tile id: no more tiles
 static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH, "ring");
@@ -89,28 +91,6 @@ __device__ __forceinline__ uint32_t s_member(uint32_t lo, uint32_t hi, uint32_t 
     const uint32_t t0 = (hi & sel.z) | (~hi & sel.x);
     const uint32_t t1 = (hi & sel.w) | (~hi & sel.y);
     return ((lo & t1) | (~lo & t0)) & ~nm;
-}
-
-// Filter: bit k of the result = guide k of the block survives (its number of pairs with a
-// mismatch is <= its threshold).  TC >= 0: one threshold for every guide of the launch.
-template <int NP, int TC>
-__device__ __forceinline__ uint32_t filter_pass(const uint32_t (&v)[NP], const uint32_t* __restrict__ m) {
-    uint32_t c[5];
-    nz_count<NP>(v, c);
-    uint32_t bw;                       // borrow out of (t - count): set where count > t
-    if constexpr (TC >= 0) {
-        bw = (TC & 1) ? 0u : c[0];
-#pragma unroll
-        for (int w = 1; w < 5; w++) bw = ((TC >> w) & 1) ? (c[w] & bw) : (c[w] | bw);
-    } else {
-        bw = c[0] & ~m[0];
-#pragma unroll
-        for (int w = 1; w < 6; w++) {
-            const uint32_t cw = w < 5 ? c[w] : 0u;
-            bw = (~m[w] & cw) | (~m[w] & bw) | (cw & bw);
-        }
-    }
-    return m[6] & ~bw;
 }
 
 template <uint32_t OFF>
@@ -166,16 +146,21 @@ __device__ __forceinline__ unsigned long long s_key(uint32_t pos, uint32_t stran
 template <int NP, int TC, bool CONCRETE>
 __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_constant__ SingleArgs a) {
     extern __shared__ __align__(128) uint8_t smem[];
-    // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise][verification
-    //         records: '+' n_blocks*32 x 32 B, 64 B, '-'][ring: SSTAGES x SPL x SLOAD words]
-    //         [queues: SW x SQ x uint4][tile ids, release counters][full mbarriers]
+    // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
+    //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
+    //         [ring: SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
+    //         [append owners: SW x SQ words][survivor lists: SW x SVC x 5 words]
+    //         [tile ids, release counters][full mbarriers]
     constexpr uint32_t FBW = (NP * 25u + 15u) & ~15u;
+    constexpr uint32_t VSTR = CONCRETE ? 1u : 2u;     // uint4 per verification record in shared memory
     const uint32_t nb = a.n_blocks;
     uint32_t* s_ftab = reinterpret_cast<uint32_t*>(smem);
     uint4* s_vrec = reinterpret_cast<uint4*>(smem + 2 * nb * FBW * 4 + 64);
-    uint32_t* ring = reinterpret_cast<uint32_t*>(smem + 2 * nb * FBW * 4 + 64 + 2 * nb * 32 * 32 + 64);
+    uint32_t* ring = reinterpret_cast<uint32_t*>(reinterpret_cast<uint8_t*>(s_vrec) + 2 * nb * 32 * VSTR * 16 + 64);
     uint4* queues = reinterpret_cast<uint4*>(ring + SSTAGES * SPL * SLOAD);
-    uint32_t* s_tile = reinterpret_cast<uint32_t*>(queues + SW * SQ);
+    uint32_t* owners = reinterpret_cast<uint32_t*>(queues + SW * SQ);
+    uint32_t* svl = owners + SW * SQ;
+    uint32_t* s_tile = svl + SW * SVC * 5;
     uint32_t* s_rel = s_tile + SSTAGES;
     uint64_t* full = reinterpret_cast<uint64_t*>(s_tile + 2 * SSTAGES);
 
@@ -199,16 +184,17 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
         bulk_g2s(S + 2 * SLOAD, a.nm + w0, SLOAD * 4, &full[st]);
         if (vsp) bulk_g2s(S + 3 * SLOAD, a.vs + w0, SLOAD * 4, &full[st]);
     };
-    {   // guide tables -> shared memory (both strands)
+    {   // guide tables -> shared memory (both strands; strand '-' 64 bytes further: other banks)
         const uint32_t nf = nb * FBW;
         for (uint32_t i = tid; i < nf; i += STHREADS) {
             s_ftab[i] = __ldg(a.ftab[0] + i);
             s_ftab[nf + 16 + i] = __ldg(a.ftab[1] + i);
         }
-        const uint32_t nv = nb * 32 * 2;
-        for (uint32_t i = tid; i < nv; i += STHREADS) {
-            s_vrec[i] = __ldg(a.vrec[0] + i);
-            s_vrec[nv + 4 + i] = __ldg(a.vrec[1] + i);
+        const uint32_t nv = nb * 32;
+        for (uint32_t i = tid; i < nv * VSTR; i += STHREADS) {
+            const uint32_t g = i / VSTR, h = i % VSTR;
+            s_vrec[i] = __ldg(a.vrec[0] + 2 * g + h);
+            s_vrec[nv * VSTR + 4 + i] = __ldg(a.vrec[1] + 2 * g + h);
         }
     }
     if (tid == 0) {
@@ -222,15 +208,88 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
     __syncthreads();
 
     uint4* queue = queues + warp * SQ;
-    // strand 1's tables start 64 bytes past a 128-byte boundary: the 16 entries of a pair
-    // then sit in the other 16 banks than strand 0's, so a batch mixing '+' and '-' sites
-    // never has two lanes in one bank (see single_smem)
+    uint32_t* owner = owners + warp * SQ;
+    uint32_t* sv_x = svl + warp * SVC * 5;               // survivor entries: slot | group << 8
+    uint32_t* sv_m = sv_x + SVC;                          // and the group's 4 survivor masks
     const uint32_t tb0 = smem_u32(s_ftab), tb1 = tb0 + nb * FBW * 4 + 64;
-    const uint4* vrec1 = s_vrec + nb * 64 + 4;
-    uint32_t head = 0, q_n = 0;           // warp-uniform ring state
+    const uint4* vrec1 = s_vrec + nb * 32 * VSTR + 4;
+    uint32_t head = 0, q_n = 0;           // warp-uniform site ring state
     unsigned long long cnt_f = 0, cnt_r = 0;
 
-    // per-lane state of the tile being expanded: its plane words and the PAM bits not yet queued
+    // Verify up to 32 survivor entries [sv_h, sv_h + n) (one site and the four 32-guide
+    // survivor masks of one group of blocks each), in two warp-wide steps per pass:
+    // (1) lane i lists the survivors of entry i -- (queue slot, launch-local guide) -- into
+    // the warp's index list (the owner list: not in use during a batch), at most SQ per
+    // pass; (2) the warp verifies the list 32 survivors per round, one per lane: exact count
+    // from the guide's record, hits appended with one atomic per round.
+    auto flush = [&](uint32_t sv_h, uint32_t n) {
+        uint32_t m0 = 0, m1 = 0, m2 = 0, m3 = 0, xs = 0;
+        if ((uint32_t)lane < n) {
+            const uint32_t e = (sv_h + lane) & (SVC - 1);
+            const uint32_t x = sv_x[e];
+            m0 = sv_m[e]; m1 = sv_m[SVC + e]; m2 = sv_m[2 * SVC + e]; m3 = sv_m[3 * SVC + e];
+            xs = (x & (SQ - 1)) | ((x >> 8) << 14);          // slot | group << 14 (guide = group*128 + ...)
+        }
+        for (;;) {
+            const uint32_t c = (uint32_t)(__popc(m0) + __popc(m1) + __popc(m2) + __popc(m3));
+            uint32_t x = c;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+                if (lane >= o) x += y;
+            }
+            const uint32_t total = __shfl_sync(0xFFFFFFFFu, x, 31);
+            if (total == 0) break;
+            const uint32_t take = min(total, SQ);
+            uint32_t rank = x - c;
+            // codes: slot (7 bits) | launch-local guide << 7
+            const uint32_t slot = xs & (SQ - 1), gbase = (xs >> 14) * 128u;
+            while (m0 && rank < take) { const uint32_t lw = m0 & (0u - m0); m0 ^= lw; owner[rank++] = slot | ((gbase + (uint32_t)(__ffs(lw) - 1)) << 7); }
+            while (m1 && rank < take) { const uint32_t lw = m1 & (0u - m1); m1 ^= lw; owner[rank++] = slot | ((gbase + 32u + (uint32_t)(__ffs(lw) - 1)) << 7); }
+            while (m2 && rank < take) { const uint32_t lw = m2 & (0u - m2); m2 ^= lw; owner[rank++] = slot | ((gbase + 64u + (uint32_t)(__ffs(lw) - 1)) << 7); }
+            while (m3 && rank < take) { const uint32_t lw = m3 & (0u - m3); m3 ^= lw; owner[rank++] = slot | ((gbase + 96u + (uint32_t)(__ffs(lw) - 1)) << 7); }
+            __syncwarp();
+            for (uint32_t j0 = 0; j0 < take; j0 += 32) {
+                const uint32_t j = j0 + lane;
+                bool hit = false;
+                uint32_t g = 0, mm = 0, pos = 0, sd = 0;
+                if (j < take) {
+                    const uint32_t code = owner[j];
+                    g = code >> 7;
+                    const uint4 it = queue[code & (SQ - 1)];
+                    pos = it.x;
+                    sd = it.w >> 31;
+                    const uint32_t wl = it.y, wh = it.z, wn = it.w & 0x7FFFFFFFu;
+                    const uint4* rec = (sd ? vrec1 : s_vrec) + g * VSTR;
+                    const uint4 r0 = rec[0];                          // {lo, hi, care, t}
+                    uint32_t mis;
+                    if constexpr (CONCRETE) {
+                        mis = ((wl ^ r0.x) | (wh ^ r0.y) | wn) & r0.z;
+                    } else {
+                        const uint4 oh = rec[1];                      // one-hot {A, C, G, T}
+                        const uint32_t nn = ~wn;
+                        const uint32_t match = (oh.x & ~wl & ~wh & nn) | (oh.y & wl & ~wh & nn) |
+                                               (oh.z & ~wl & wh & nn) | (oh.w & wl & wh & nn);
+                        mis = r0.z & ~match;
+                    }
+                    mm = (uint32_t)__popc(mis);
+                    hit = mm <= r0.w;
+                }
+                const unsigned hm = __ballot_sync(0xFFFFFFFFu, hit);
+                if (hm) {
+                    const int leader = __ffs(hm) - 1;
+                    unsigned long long o = 0;
+                    if (lane == leader) o = atomicAdd(&a.counters[2], (unsigned long long)__popc(hm));
+                    o = __shfl_sync(0xFFFFFFFFu, o, leader) + (unsigned)__popc(hm & lanemask_lt());
+                    if (hit && o < a.cap) a.hits[o] = s_key(pos, sd, a.block_base * 32u + g, mm);
+                }
+            }
+            __syncwarp();
+            if (total <= SQ) break;
+        }
+    };
+
+    // per-lane state of the tile being appended: its plane words and the PAM bits not yet queued
     uint32_t lo0 = 0, lo1 = 0, lo2 = 0, hi0 = 0, hi1 = 0, hi2 = 0, nm0 = 0, nm1 = 0, nm2 = 0;
     uint32_t pend0 = 0u, pend1 = 0u, pbase = 0;
     const int w = warp * 32 + lane;
@@ -243,75 +302,48 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
         if (q_n >= SBATCH || (tiles_done && q_n > 0)) {
             // ---------------- compare a batch: ring[head, head + n_items)
             const uint32_t n_items = min(q_n, SBATCH);
-            uint32_t base[SR][NP], wl[SR], wh[SR], wn[SR], pos[SR], sd[SR];
+            uint32_t base[SR][NP];
 #pragma unroll
             for (int r = 0; r < SR; r++) {
                 const uint32_t i = (uint32_t)r * 32 + lane;
                 // a missing site gets an all-N window (every pair mismatches) and is masked below
                 const uint4 e = i < n_items ? queue[(head + i) & (SQ - 1)] : make_uint4(0u, 0u, 0u, 0x7FFFFFFFu);
-                pos[r] = e.x;
-                wl[r] = e.y;
-                wh[r] = e.z;
-                sd[r] = e.w >> 31;
-                wn[r] = e.w & 0x7FFFFFFFu;
-                site_bases<NP>(a, sd[r] ? tb1 : tb0, sd[r], wl[r], wh[r], wn[r], base[r]);
+                const uint32_t sd = e.w >> 31;
+                site_bases<NP>(a, sd ? tb1 : tb0, sd, e.y, e.z, e.w & 0x7FFFFFFFu, base[r]);
             }
             const uint32_t okm0 = (uint32_t)lane < n_items ? ~0u : 0u, okm1 = 32u + lane < n_items ? ~0u : 0u;
+            uint32_t sv_h = 0, sv_n = 0;                    // warp-uniform survivor list state
             for (uint32_t b = 0; b < nb; b += 4) {
                 const uint32_t* m = a.meta[b];
-                uint32_t p[SR][4];
 #pragma unroll
                 for (int r = 0; r < SR; r++) {
-                    uint32_t v[NP];
+                    uint32_t v[NP], p0, p1, p2, p3;
                     lds_filter<NP, 0 * FBW * 4>(base[r], v);
-                    p[r][0] = filter_pass<NP, TC>(v, m);
+                    p0 = filter_pass<NP, TC>(v, m);
                     lds_filter<NP, 1 * FBW * 4>(base[r], v);
-                    p[r][1] = filter_pass<NP, TC>(v, m + 8);
+                    p1 = filter_pass<NP, TC>(v, m + 8);
                     lds_filter<NP, 2 * FBW * 4>(base[r], v);
-                    p[r][2] = filter_pass<NP, TC>(v, m + 16);
+                    p2 = filter_pass<NP, TC>(v, m + 16);
                     lds_filter<NP, 3 * FBW * 4>(base[r], v);
-                    p[r][3] = filter_pass<NP, TC>(v, m + 24);
+                    p3 = filter_pass<NP, TC>(v, m + 24);
                     const uint32_t ok = r == 0 ? okm0 : okm1;
-                    p[r][0] &= ok; p[r][1] &= ok; p[r][2] &= ok; p[r][3] &= ok;
-                }
-                // ---- verify the survivors (blocks past the plan have valid mask 0): warp-
-                // uniform rounds, every lane with a survivor left takes one per round; the
-                // round's hits are appended with one atomic
-#pragma unroll
-                for (int r = 0; r < SR; r++) {
-                    uint32_t m0 = p[r][0], m1 = p[r][1], m2 = p[r][2], m3 = p[r][3];
-                    while (__any_sync(0xFFFFFFFFu, (m0 | m1 | m2 | m3) != 0u)) {
-                        bool hit = false;
-                        uint32_t g = 0, mm = 0;
-                        if (m0 | m1 | m2 | m3) {
-                            uint32_t bi, kk;
-                            if (m0) { kk = __ffs(m0) - 1; m0 &= m0 - 1; bi = 0; }
-                            else if (m1) { kk = __ffs(m1) - 1; m1 &= m1 - 1; bi = 1; }
-                            else if (m2) { kk = __ffs(m2) - 1; m2 &= m2 - 1; bi = 2; }
-                            else { kk = __ffs(m3) - 1; m3 &= m3 - 1; bi = 3; }
-                            g = (b + bi) * 32u + kk;                       // launch-local guide
-                            const uint4* rec = (sd[r] ? vrec1 : s_vrec) + 2u * g;
-                            const uint4 r0 = rec[0];                       // {lo, hi, care, t}
-                            uint32_t mis;
-                            if constexpr (CONCRETE) {
-                                mis = ((wl[r] ^ r0.x) | (wh[r] ^ r0.y) | wn[r]) & r0.z;
-                            } else {
-                                const uint4 oh = rec[1];                   // one-hot {A, C, G, T}
-                                const uint32_t nn = ~wn[r];
-                                const uint32_t match = (oh.x & ~wl[r] & ~wh[r] & nn) | (oh.y & wl[r] & ~wh[r] & nn) |
-                                                       (oh.z & ~wl[r] & wh[r] & nn) | (oh.w & wl[r] & wh[r] & nn);
-                                mis = r0.z & ~match;
-                            }
-                            mm = (uint32_t)__popc(mis);
-                            hit = mm <= r0.w;
+                    p0 &= ok; p1 &= ok; p2 &= ok; p3 &= ok;
+                    // a site with a survivor in this group of 4 blocks -> one survivor entry
+                    // (ballot append: no per-bit loop here; blocks past the plan have valid 0)
+                    const bool has = (p0 | p1 | p2 | p3) != 0u;
+                    const unsigned hb = __ballot_sync(0xFFFFFFFFu, has);
+                    if (hb) {
+                        if (has) {
+                            const uint32_t e = (sv_h + sv_n + (uint32_t)__popc(hb & lanemask_lt())) & (SVC - 1);
+                            sv_x[e] = ((head + (uint32_t)r * 32 + lane) & (SQ - 1)) | ((b >> 2) << 8);
+                            sv_m[e] = p0; sv_m[SVC + e] = p1; sv_m[2 * SVC + e] = p2; sv_m[3 * SVC + e] = p3;
                         }
-                        const unsigned hm = __ballot_sync(0xFFFFFFFFu, hit);
-                        if (hm) {
-                            const int leader = __ffs(hm) - 1;
-                            unsigned long long o = 0;
-                            if (lane == leader) o = atomicAdd(&a.counters[2], (unsigned long long)__popc(hm));
-                            o = __shfl_sync(0xFFFFFFFFu, o, leader) + (unsigned)__popc(hm & lanemask_lt());
-                            if (hit && o < a.cap) a.hits[o] = s_key(pos[r], sd[r], a.block_base * 32u + g, mm);
+                        sv_n += (uint32_t)__popc(hb);
+                        if (sv_n >= 32) {
+                            __syncwarp();
+                            flush(sv_h, 32);
+                            sv_h = (sv_h + 32) & (SVC - 1);
+                            sv_n -= 32;
                         }
                     }
                 }
@@ -322,6 +354,10 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
                         for (int q = 0; q < NP; q++) base[r][q] += 4 * FBW * 4;
                 }
             }
+            if (sv_n) {
+                __syncwarp();
+                flush(sv_h, sv_n);
+            }
             __syncwarp();
             head = (head + SBATCH) & (SQ - 1);
             q_n -= n_items;
@@ -329,14 +365,13 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
         }
         if (tiles_done) break;
         if (__any_sync(0xFFFFFFFFu, (pend0 | pend1) != 0u)) {
-            // ---------------- append pending sites of one strand (all '+' first, then '-')
+            // ---------------- append pending sites of one strand (all '+' first, then '-'):
+            // (1) each lane writes (lane, bit) of its sites into the warp's owner list (a short
+            // per-lane loop), (2) the warp builds the queue entries cooperatively, 32 per round:
+            // lane i takes owner i and shuffles the owner's strand-shifted words
             const bool any0 = __any_sync(0xFFFFFFFFu, pend0 != 0u);
             const uint32_t sdw = any0 ? 0u : 1u;          // warp-uniform strand of this append
             uint32_t m = any0 ? pend0 : pend1;
-            const uint32_t p0 = a.p0[sdw];
-            const uint32_t Al = __funnelshift_r(lo0, lo1, p0), Bl = __funnelshift_r(lo1, lo2, p0);
-            const uint32_t Ah = __funnelshift_r(hi0, hi1, p0), Bh = __funnelshift_r(hi1, hi2, p0);
-            const uint32_t An = __funnelshift_r(nm0, nm1, p0), Bn = __funnelshift_r(nm1, nm2, p0);
             const uint32_t c = (uint32_t)__popc(m);
             uint32_t x = c;
 #pragma unroll
@@ -346,18 +381,35 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
             }
             const uint32_t total = __shfl_sync(0xFFFFFFFFu, x, 31);
             const uint32_t take = min(SQ - q_n, total);
-            const uint32_t tail = head + q_n;
-            uint32_t rank = x - c;
-            while (m && rank < take) {
-                const int bit = __ffs(m) - 1;
-                m &= m - 1;
-                const uint32_t wl = __funnelshift_r(Al, Bl, bit), wh = __funnelshift_r(Ah, Bh, bit);
-                const uint32_t wn = __funnelshift_r(An, Bn, bit);
-                queue[(tail + rank) & (SQ - 1)] = make_uint4(pbase + (uint32_t)bit, wl, wh,
-                                                               (wn & 0x7FFFFFFFu) | (sdw << 31));
-                rank++;
+            const uint32_t first = x - c;
+            // this lane's sites with rank < take: a count-bounded loop (one test per site)
+            const int n_mine = (int)min(c, take > first ? take - first : 0u);
+            uint32_t* ow = owner + first;
+            const uint32_t lane5 = (uint32_t)lane << 5;
+            for (int i = 0; i < n_mine; i++) {
+                const uint32_t low = m & (0u - m);
+                ow[i] = lane5 | (uint32_t)(__ffs(low) - 1);
+                m ^= low;
             }
             if (any0) pend0 = m; else pend1 = m;
+            __syncwarp();
+            const uint32_t p0s = a.p0[sdw];
+            const uint32_t Al = __funnelshift_r(lo0, lo1, p0s), Bl = __funnelshift_r(lo1, lo2, p0s);
+            const uint32_t Ah = __funnelshift_r(hi0, hi1, p0s), Bh = __funnelshift_r(hi1, hi2, p0s);
+            const uint32_t An = __funnelshift_r(nm0, nm1, p0s), Bn = __funnelshift_r(nm1, nm2, p0s);
+            const uint32_t tail = head + q_n;
+            for (uint32_t j0 = 0; j0 < take; j0 += 32) {
+                const uint32_t j = j0 + lane;
+                const uint32_t o = j < take ? owner[j] : 0u;
+                const int src = (int)(o >> 5), bit = (int)(o & 31u);
+                const uint32_t al = __shfl_sync(0xFFFFFFFFu, Al, src), bl = __shfl_sync(0xFFFFFFFFu, Bl, src);
+                const uint32_t ah = __shfl_sync(0xFFFFFFFFu, Ah, src), bh = __shfl_sync(0xFFFFFFFFu, Bh, src);
+                const uint32_t an = __shfl_sync(0xFFFFFFFFu, An, src), bn = __shfl_sync(0xFFFFFFFFu, Bn, src);
+                if (j < take)
+                    queue[(tail + j) & (SQ - 1)] =
+                        make_uint4(pbase + 32u * (uint32_t)src + (uint32_t)bit, __funnelshift_r(al, bl, bit),
+                                   __funnelshift_r(ah, bh, bit), (__funnelshift_r(an, bn, bit) & 0x7FFFFFFFu) | (sdw << 31));
+            }
             __syncwarp();
             q_n += take;
             continue;
@@ -399,7 +451,7 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
             cnt_f += (unsigned)__popc(pend0);
             cnt_r += (unsigned)__popc(pend1);
         }
-        pbase = (uint32_t)pw;
+        pbase = (uint32_t)(((uint64_t)tile * STW + (uint32_t)warp * 32u) * 32u);   // first start of lane 0's word
     }
     if (a.count_items) {
 #pragma unroll
@@ -440,6 +492,13 @@ static SingleFn single_fn_np(int tc, bool concrete) {
     return single_fn_t<NP, -1, false>();
 }
 
+// The kernel variant a plan runs: uniform-threshold, concrete-letter specialisations for
+// the configs' shapes (10 pairs: 20-nt SpCas9 guides; 12: 23-nt Cas12a) with t <= 7,
+// else the generic one (per-guide thresholds, one-hot IUPAC verification).
+static bool single_uses_concrete(uint32_t np, int tc, bool concrete) {
+    return (np == 10 || np == 12) && concrete && tc >= 0 && tc <= 7;
+}
+
 static SingleFn single_fn(uint32_t np, int tc, bool concrete) {
     switch (np) {
         case 1: return single_fn_np<1>(tc, concrete);
@@ -462,19 +521,20 @@ static SingleFn single_fn(uint32_t np, int tc, bool concrete) {
     }
 }
 
-static size_t single_smem(uint32_t np, uint32_t nb) {
+static size_t single_smem(uint32_t np, uint32_t nb, bool concrete) {
     const size_t fbw = filter_block_words(np);
     // (+ 64 bytes after the '+' filter tables and 64 after the '+' records: bank offsets)
-    return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * 32 + 64 + (size_t)SSTAGES * SPL * SLOAD * 4 +
-           (size_t)SW * SQ * 16 + 2 * SSTAGES * 4 + SSTAGES * 8;
+    return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * (concrete ? 16 : 32) + 64 +
+           (size_t)SSTAGES * SPL * SLOAD * 4 + (size_t)SW * SQ * 16 + (size_t)SW * SQ * 4 + (size_t)SW * SVC * 20 +
+           2 * SSTAGES * 4 + SSTAGES * 8;
 }
 
 static constexpr size_t SMEM_MAX = 227 * 1024;
 
 // Guide blocks per launch: as many as fit the shared-memory budget (a multiple of 4).
-static uint32_t single_blocks_per_launch(uint32_t np) {
+static uint32_t single_blocks_per_launch(uint32_t np, bool concrete) {
     uint32_t nb = SMAX_BLOCKS;
-    while (nb > 4 && single_smem(np, nb) > SMEM_MAX) nb -= 4;
+    while (nb > 4 && single_smem(np, nb, concrete) > SMEM_MAX) nb -= 4;
     return nb;
 }
 
@@ -525,7 +585,7 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     int ut = (int)plan->max_mm[0];
     for (uint32_t i = 1; i < plan->n_guides && ut >= 0; i++)
         if (plan->max_mm[i] != plan->max_mm[0]) ut = -1;
-    const bool concrete = !plan->any_degenerate;
+    const bool concrete = single_uses_concrete(np, ut, !plan->any_degenerate);
     SingleFn fn = single_fn(np, ut, concrete);
     if (!fn) return set_error(COF_E_STATE, "single pass: %u pairs", np);
     int dev_id = 0;
@@ -558,13 +618,13 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     }
     A.contig = plan->pairs[0].contig && plan->pairs[1].contig && plan->pairs[0].n_cmp == plan->pairs[1].n_cmp;
     A.cmp_mask = plan->pairs[0].n_cmp >= 32 ? ~0u : ((1u << plan->pairs[0].n_cmp) - 1u);
-    const uint32_t bpl = single_blocks_per_launch(np);
+    const uint32_t bpl = single_blocks_per_launch(np, concrete);
     const uint32_t fbw = filter_block_words(np);
     const uint32_t* pm = (const uint32_t*)(plan->image.data() + plan->lay.pmeta_fwd);
     {
         std::lock_guard<std::mutex> lk(g_single_mu);   // (per device state; cheap, set every call)
         cudaError_t e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)single_smem(np, bpl));
+                                             (int)single_smem(np, bpl, concrete));
         if (e != cudaSuccess) return cuda_error(e, "single pass smem attribute");
     }
     uint32_t li = 0;
@@ -585,7 +645,7 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
         if (n_tiles == 0) continue;
         uint32_t grid = (uint32_t)sms;
         if (grid > n_tiles) grid = n_tiles;
-        fn<<<grid, STHREADS, single_smem(np, nb4), stream>>>(A);
+        fn<<<grid, STHREADS, single_smem(np, nb4, concrete), stream>>>(A);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "cof_single_kernel launch");
         count_launches(1);
@@ -594,7 +654,11 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
 }
 
 uint32_t single_launches(const cof_plan* plan) {
-    const uint32_t bpl = single_blocks_per_launch(plan->pairs[0].n_pairs);
+    int ut = (int)plan->max_mm[0];
+    for (uint32_t i = 1; i < plan->n_guides && ut >= 0; i++)
+        if (plan->max_mm[i] != plan->max_mm[0]) ut = -1;
+    const uint32_t np = plan->pairs[0].n_pairs;
+    const uint32_t bpl = single_blocks_per_launch(np, single_uses_concrete(np, ut, !plan->any_degenerate));
     return (plan->n_blocks + bpl - 1) / bpl;
 }
 
