@@ -692,6 +692,11 @@ def single_roof(plan, n_sm, sm_mhz):
     fa = int(hdr.split(":")[1].split("full")[0])
     ha = int(hdr.split(",")[1].split("half")[0])
     alu_ops = 2 * fa + 2 * ha + 4 + 1
+    # hand-reduced count-vs-threshold circuits (csrc/filter_circuit.cuh; LOP3 per 32 comparisons,
+    # incl. the survivor mask): uniform thresholds of the configs' shapes
+    ts = set(int(t) for t in plan.max_mm)
+    if len(ts) == 1:
+        alu_ops = {(10, 4): 16, (10, 5): 15, (10, 6): 16, (12, 5): 18}.get((npairs, ts.pop()), alu_ops)
     alu_rate = 64.0 * 32 / alu_ops
     lds_rate = 32.0 * 32 / npairs
     per_clk = min(alu_rate, lds_rate)

@@ -49,25 +49,30 @@ def _generate():
             f.write(text)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
+    """Build libcof.so (or, with ``defines`` such as "COF_SINGLE_SW=20", a variant library at
+    ``out`` for A/B measurements, loaded through COF_LIB)."""
     _generate()
     cu, cpp, hdr = _sources()
-    digest = _digest(cu + cpp + hdr + [__file__])
-    stamp = os.path.join(BUILD, "stamp")
-    if not force and os.path.exists(LIB) and os.path.exists(stamp) and open(stamp).read() == digest:
-        return LIB
-    os.makedirs(BUILD, exist_ok=True)
+    lib = out or LIB
+    digest = _digest(cu + cpp + hdr + [__file__]) + "".join(defines)
+    build_dir = BUILD if not defines else BUILD + "_" + "_".join(d.replace("=", "") for d in defines)
+    stamp = os.path.join(build_dir, "stamp")
+    if not force and os.path.exists(lib) and os.path.exists(stamp) and open(stamp).read() == digest:
+        return lib
+    os.makedirs(build_dir, exist_ok=True)
+    dflags = [f"-D{d}" for d in defines]
     objs = []
     procs = []
     for src in cu:
-        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fopenmp",
-               "-Xptxas", "-v" if verbose else "-O3", "-I", INCLUDE, "-c", src, "-o", obj]
+               "-Xptxas", "-v" if verbose else "-O3", *dflags, "-I", INCLUDE, "-c", src, "-o", obj]
         procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
         objs.append(obj)
     for src in cpp:
-        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-        cmd = ["g++", "-O3", "-std=c++17", "-fPIC", "-fopenmp", "-Wall", "-I", INCLUDE,
+        obj = os.path.join(build_dir, os.path.basename(src) + ".o")
+        cmd = ["g++", "-O3", "-std=c++17", "-fPIC", "-fopenmp", "-Wall", *dflags, "-I", INCLUDE,
                "-I", os.path.join(CUDA, "include"), "-c", src, "-o", obj]
         procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
         objs.append(obj)
@@ -78,15 +83,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
             raise RuntimeError("build failed: " + " ".join(cmd))
         if verbose and out:
             sys.stderr.write(out.decode(errors="replace"))
-    tmp = LIB + f".{os.getpid()}.tmp"
+    tmp = lib + f".{os.getpid()}.tmp"
     cmd = ["g++", "-shared", "-fopenmp", "-o", tmp, *objs, "-L", os.path.join(CUDA, "lib64"),
            "-lcudart_static", "-ldl", "-lrt", "-lpthread", "-Wl,--no-undefined"]
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
+    os.replace(tmp, lib)
     with open(stamp, "w") as f:
         f.write(digest)
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, defines=defs, out=outs[0] if outs else None))

@@ -13,7 +13,8 @@ import os
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libcof.so")
+# (COF_LIB: an alternative build of the same library, for A/B measurements of kernel variants)
+LIB_PATH = os.environ.get("COF_LIB") or os.path.join(HERE, "libcof.so")
 
 COF_OK = 0
 COF_E_ARG = -1

@@ -45,7 +45,10 @@
 
 namespace cof {
 
-constexpr int SW = 16;                    // warps per CTA (4 per SM sub-partition: <= 128 registers)
+#ifndef COF_SINGLE_SW
+#define COF_SINGLE_SW 16
+#endif
+constexpr int SW = COF_SINGLE_SW;         // warps per CTA (16: 4 per SM sub-partition, <= 128 registers)
 constexpr int STHREADS = 32 * SW;
 constexpr int STW = 32 * SW;              // plane words per tile (one per lane)
 constexpr int SLOAD = STW + 4;            // words per plane and stage: tile + halo (16-byte multiple)
@@ -54,10 +57,12 @@ constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
 constexpr uint32_t SQ = 128;              // queued sites per warp (16-byte entries)
 constexpr int SR = 2;                     // sites per lane and batch
 constexpr uint32_t SBATCH = 32 * SR;
-constexpr uint32_t SVC = 64;              // survivor entries per warp (ring)
+constexpr uint32_t SVC = 128;             // survivor entries per warp (ring; shares the owner list's space)
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
 constexpr uint32_t S_END = 0xFFFFFFFFu;   // tile id: no more tiles
 static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH, "ring");
+static_assert(5 * SVC >= SQ, "the owner list shares the survivor ring's space");
+static_assert(SVC >= 31 + 32 * SR, "a group of blocks appends at most 32 entries per site row");
 
 struct SingleArgs {
     const uint32_t* lo;
@@ -66,6 +71,7 @@ struct SingleArgs {
     const uint32_t* vs;               // valid-start plane (multi-segment chunks) or nullptr
     uint64_t limit;                   // no window start >= limit is valid
     uint32_t n_tiles;
+    uint64_t words;                   // plane words allocated (cof_plane_words(n_bases)): TMA bound
     unsigned int* ticket;             // dynamic tile counter (zeroed per launch)
     unsigned long long* hits;
     uint64_t cap;
@@ -149,7 +155,7 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
     // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
     //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
     //         [ring: SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
-    //         [append owners: SW x SQ words][survivor lists: SW x SVC x 5 words]
+    //         [per warp: append owner list (SQ words) / survivor ring (SVC x 5 words)]
     //         [tile ids, release counters][full mbarriers]
     constexpr uint32_t FBW = (NP * 25u + 15u) & ~15u;
     constexpr uint32_t VSTR = CONCRETE ? 1u : 2u;     // uint4 per verification record in shared memory
@@ -158,9 +164,8 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
     uint4* s_vrec = reinterpret_cast<uint4*>(smem + 2 * nb * FBW * 4 + 64);
     uint32_t* ring = reinterpret_cast<uint32_t*>(reinterpret_cast<uint8_t*>(s_vrec) + 2 * nb * 32 * VSTR * 16 + 64);
     uint4* queues = reinterpret_cast<uint4*>(ring + SSTAGES * SPL * SLOAD);
-    uint32_t* owners = reinterpret_cast<uint32_t*>(queues + SW * SQ);
-    uint32_t* svl = owners + SW * SQ;
-    uint32_t* s_tile = svl + SW * SVC * 5;
+    uint32_t* owners = reinterpret_cast<uint32_t*>(queues + SW * SQ);   // per warp: 5 x SVC words
+    uint32_t* s_tile = owners + SW * 5 * SVC;
     uint32_t* s_rel = s_tile + SSTAGES;
     uint64_t* full = reinterpret_cast<uint64_t*>(s_tile + 2 * SSTAGES);
 
@@ -176,13 +181,16 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
         }
         s_tile[st] = tile;
         const size_t w0 = (size_t)tile * STW;
+        // (a tile size that does not divide the planes' 512-word padding: the last tile's
+        // copy stops at the allocation; the words past it only feed invalid starts)
+        const uint32_t nbytes = (uint32_t)min((uint64_t)SLOAD, a.words - w0) * 4u;
         uint32_t* S = ring + st * SPL * SLOAD;
         fence_proxy_async_smem();
-        mbar_arrive_expect_tx(&full[st], (vsp ? 4 : 3) * SLOAD * 4);
-        bulk_g2s(S + 0 * SLOAD, a.lo + w0, SLOAD * 4, &full[st]);
-        bulk_g2s(S + 1 * SLOAD, a.hi + w0, SLOAD * 4, &full[st]);
-        bulk_g2s(S + 2 * SLOAD, a.nm + w0, SLOAD * 4, &full[st]);
-        if (vsp) bulk_g2s(S + 3 * SLOAD, a.vs + w0, SLOAD * 4, &full[st]);
+        mbar_arrive_expect_tx(&full[st], (vsp ? 4 : 3) * nbytes);
+        bulk_g2s(S + 0 * SLOAD, a.lo + w0, nbytes, &full[st]);
+        bulk_g2s(S + 1 * SLOAD, a.hi + w0, nbytes, &full[st]);
+        bulk_g2s(S + 2 * SLOAD, a.nm + w0, nbytes, &full[st]);
+        if (vsp) bulk_g2s(S + 3 * SLOAD, a.vs + w0, nbytes, &full[st]);
     };
     {   // guide tables -> shared memory (both strands; strand '-' 64 bytes further: other banks)
         const uint32_t nf = nb * FBW;
@@ -208,65 +216,46 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
     __syncthreads();
 
     uint4* queue = queues + warp * SQ;
-    uint32_t* owner = owners + warp * SQ;
-    uint32_t* sv_x = svl + warp * SVC * 5;               // survivor entries: slot | group << 8
-    uint32_t* sv_m = sv_x + SVC;                          // and the group's 4 survivor masks
+    uint32_t* owner = owners + warp * 5 * SVC;           // append: (lane, bit) of queued sites
+    uint32_t* sv_x = owner;                              // batch: survivor entries: slot | group << 8
+    uint32_t* sv_m = owner + SVC;                        //        and the group's 4 survivor masks
     const uint32_t tb0 = smem_u32(s_ftab), tb1 = tb0 + nb * FBW * 4 + 64;
     const uint4* vrec1 = s_vrec + nb * 32 * VSTR + 4;
     uint32_t head = 0, q_n = 0;           // warp-uniform site ring state
     unsigned long long cnt_f = 0, cnt_r = 0;
 
-    // Verify up to 32 survivor entries [sv_h, sv_h + n) (one site and the four 32-guide
-    // survivor masks of one group of blocks each), in two warp-wide steps per pass:
-    // (1) lane i lists the survivors of entry i -- (queue slot, launch-local guide) -- into
-    // the warp's index list (the owner list: not in use during a batch), at most SQ per
-    // pass; (2) the warp verifies the list 32 survivors per round, one per lane: exact count
-    // from the guide's record, hits appended with one atomic per round.
+    // Verify up to 32 survivor entries [sv_h, sv_h + n): lane i takes entry i -- one site
+    // (its queue slot) and the four 32-guide survivor masks of one group of blocks -- and the
+    // warp walks the set bits block by block in warp-uniform rounds (a round per bit of the
+    // fullest lane; most masks are empty or hold one bit): exact count from the guide's
+    // record, the round's hits appended with one atomic.
     auto flush = [&](uint32_t sv_h, uint32_t n) {
-        uint32_t m0 = 0, m1 = 0, m2 = 0, m3 = 0, xs = 0;
+        uint32_t mk[4] = {0u, 0u, 0u, 0u}, g0 = 0, pos = 0, wl = 0, wh = 0, wn = 0, sd = 0;
         if ((uint32_t)lane < n) {
             const uint32_t e = (sv_h + lane) & (SVC - 1);
             const uint32_t x = sv_x[e];
-            m0 = sv_m[e]; m1 = sv_m[SVC + e]; m2 = sv_m[2 * SVC + e]; m3 = sv_m[3 * SVC + e];
-            xs = (x & (SQ - 1)) | ((x >> 8) << 14);          // slot | group << 14 (guide = group*128 + ...)
-        }
-        for (;;) {
-            const uint32_t c = (uint32_t)(__popc(m0) + __popc(m1) + __popc(m2) + __popc(m3));
-            uint32_t x = c;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
-                if (lane >= o) x += y;
-            }
-            const uint32_t total = __shfl_sync(0xFFFFFFFFu, x, 31);
-            if (total == 0) break;
-            const uint32_t take = min(total, SQ);
-            uint32_t rank = x - c;
-            // codes: slot (7 bits) | launch-local guide << 7
-            const uint32_t slot = xs & (SQ - 1), gbase = (xs >> 14) * 128u;
-            while (m0 && rank < take) { const uint32_t lw = m0 & (0u - m0); m0 ^= lw; owner[rank++] = slot | ((gbase + (uint32_t)(__ffs(lw) - 1)) << 7); }
-            while (m1 && rank < take) { const uint32_t lw = m1 & (0u - m1); m1 ^= lw; owner[rank++] = slot | ((gbase + 32u + (uint32_t)(__ffs(lw) - 1)) << 7); }
-            while (m2 && rank < take) { const uint32_t lw = m2 & (0u - m2); m2 ^= lw; owner[rank++] = slot | ((gbase + 64u + (uint32_t)(__ffs(lw) - 1)) << 7); }
-            while (m3 && rank < take) { const uint32_t lw = m3 & (0u - m3); m3 ^= lw; owner[rank++] = slot | ((gbase + 96u + (uint32_t)(__ffs(lw) - 1)) << 7); }
-            __syncwarp();
-            for (uint32_t j0 = 0; j0 < take; j0 += 32) {
-                const uint32_t j = j0 + lane;
+            for (int q = 0; q < 4; q++) mk[q] = sv_m[q * SVC + e];
+            const uint4 it = queue[x & (SQ - 1)];
+            pos = it.x; wl = it.y; wh = it.z; sd = it.w >> 31; wn = it.w & 0x7FFFFFFFu;
+            g0 = (x >> 8) * 128u;                                 // first guide of the group
+        }
+        const uint4* vr = sd ? vrec1 : s_vrec;
+#pragma unroll 1
+        for (int q = 0; q < 4; q++) {
+            uint32_t msk = q == 0 ? mk[0] : q == 1 ? mk[1] : q == 2 ? mk[2] : mk[3];
+            while (__any_sync(0xFFFFFFFFu, msk != 0u)) {
                 bool hit = false;
-                uint32_t g = 0, mm = 0, pos = 0, sd = 0;
-                if (j < take) {
-                    const uint32_t code = owner[j];
-                    g = code >> 7;
-                    const uint4 it = queue[code & (SQ - 1)];
-                    pos = it.x;
-                    sd = it.w >> 31;
-                    const uint32_t wl = it.y, wh = it.z, wn = it.w & 0x7FFFFFFFu;
-                    const uint4* rec = (sd ? vrec1 : s_vrec) + g * VSTR;
-                    const uint4 r0 = rec[0];                          // {lo, hi, care, t}
+                uint32_t g = 0, mm = 0;
+                if (msk) {
+                    g = g0 + 32u * q + (uint32_t)(__ffs(msk) - 1);   // launch-local guide
+                    msk &= msk - 1;
+                    const uint4 r0 = vr[g * VSTR];                    // {lo, hi, care, t}
                     uint32_t mis;
                     if constexpr (CONCRETE) {
                         mis = ((wl ^ r0.x) | (wh ^ r0.y) | wn) & r0.z;
                     } else {
-                        const uint4 oh = rec[1];                      // one-hot {A, C, G, T}
+                        const uint4 oh = vr[g * VSTR + 1];            // one-hot {A, C, G, T}
                         const uint32_t nn = ~wn;
                         const uint32_t match = (oh.x & ~wl & ~wh & nn) | (oh.y & wl & ~wh & nn) |
                                                (oh.z & ~wl & wh & nn) | (oh.w & wl & wh & nn);
@@ -284,8 +273,6 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
                     if (hit && o < a.cap) a.hits[o] = s_key(pos, sd, a.block_base * 32u + g, mm);
                 }
             }
-            __syncwarp();
-            if (total <= SQ) break;
         }
     };
 
@@ -313,50 +300,51 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
             }
             const uint32_t okm0 = (uint32_t)lane < n_items ? ~0u : 0u, okm1 = 32u + lane < n_items ? ~0u : 0u;
             uint32_t sv_h = 0, sv_n = 0;                    // warp-uniform survivor list state
-            for (uint32_t b = 0; b < nb; b += 4) {
-                const uint32_t* m = a.meta[b];
+            // groups of 4 blocks; one extra pass (b >= nb) drains the survivor list, so the
+            // verification code exists once in the kernel (its size decides the I-cache hit rate)
+            for (uint32_t b = 0;; b += 4) {
+                const bool drain = b >= nb;
+                if (!drain) {
+                    const uint32_t* m = a.meta[b];
 #pragma unroll
-                for (int r = 0; r < SR; r++) {
-                    uint32_t v[NP], p0, p1, p2, p3;
-                    lds_filter<NP, 0 * FBW * 4>(base[r], v);
-                    p0 = filter_pass<NP, TC>(v, m);
-                    lds_filter<NP, 1 * FBW * 4>(base[r], v);
-                    p1 = filter_pass<NP, TC>(v, m + 8);
-                    lds_filter<NP, 2 * FBW * 4>(base[r], v);
-                    p2 = filter_pass<NP, TC>(v, m + 16);
-                    lds_filter<NP, 3 * FBW * 4>(base[r], v);
-                    p3 = filter_pass<NP, TC>(v, m + 24);
-                    const uint32_t ok = r == 0 ? okm0 : okm1;
-                    p0 &= ok; p1 &= ok; p2 &= ok; p3 &= ok;
-                    // a site with a survivor in this group of 4 blocks -> one survivor entry
-                    // (ballot append: no per-bit loop here; blocks past the plan have valid 0)
-                    const bool has = (p0 | p1 | p2 | p3) != 0u;
-                    const unsigned hb = __ballot_sync(0xFFFFFFFFu, has);
-                    if (hb) {
+                    for (int r = 0; r < SR; r++) {
+                        uint32_t v[NP], p0, p1, p2, p3;
+                        lds_filter<NP, 0 * FBW * 4>(base[r], v);
+                        p0 = filter_pass<NP, TC>(v, m);
+                        lds_filter<NP, 1 * FBW * 4>(base[r], v);
+                        p1 = filter_pass<NP, TC>(v, m + 8);
+                        lds_filter<NP, 2 * FBW * 4>(base[r], v);
+                        p2 = filter_pass<NP, TC>(v, m + 16);
+                        lds_filter<NP, 3 * FBW * 4>(base[r], v);
+                        p3 = filter_pass<NP, TC>(v, m + 24);
+                        const uint32_t ok = r == 0 ? okm0 : okm1;
+                        p0 &= ok; p1 &= ok; p2 &= ok; p3 &= ok;
+                        // a site with a survivor in this group of 4 blocks -> one survivor
+                        // entry (ballot append; blocks past the plan have valid 0)
+                        const bool has = (p0 | p1 | p2 | p3) != 0u;
+                        const unsigned hb = __ballot_sync(0xFFFFFFFFu, has);
+                        const uint32_t e = (sv_h + sv_n + (uint32_t)__popc(hb & lanemask_lt())) & (SVC - 1);
                         if (has) {
-                            const uint32_t e = (sv_h + sv_n + (uint32_t)__popc(hb & lanemask_lt())) & (SVC - 1);
                             sv_x[e] = ((head + (uint32_t)r * 32 + lane) & (SQ - 1)) | ((b >> 2) << 8);
                             sv_m[e] = p0; sv_m[SVC + e] = p1; sv_m[2 * SVC + e] = p2; sv_m[3 * SVC + e] = p3;
                         }
                         sv_n += (uint32_t)__popc(hb);
-                        if (sv_n >= 32) {
-                            __syncwarp();
-                            flush(sv_h, 32);
-                            sv_h = (sv_h + 32) & (SVC - 1);
-                            sv_n -= 32;
-                        }
+                    }
+                    if (b + 4 < nb) {
+#pragma unroll
+                        for (int r = 0; r < SR; r++)
+#pragma unroll
+                            for (int q = 0; q < NP; q++) base[r][q] += 4 * FBW * 4;
                     }
                 }
-                if (b + 4 < nb) {
-#pragma unroll
-                    for (int r = 0; r < SR; r++)
-#pragma unroll
-                        for (int q = 0; q < NP; q++) base[r][q] += 4 * FBW * 4;
-                }
-            }
-            if (sv_n) {
                 __syncwarp();
-                flush(sv_h, sv_n);
+                while (sv_n >= 32 || (drain && sv_n > 0)) {   // (<= 31 + SR x 32 entries: SVC holds them)
+                    const uint32_t nf = min(sv_n, 32u);
+                    flush(sv_h, nf);
+                    sv_h = (sv_h + nf) & (SVC - 1);
+                    sv_n -= nf;
+                }
+                if (drain) break;
             }
             __syncwarp();
             head = (head + SBATCH) & (SQ - 1);
@@ -525,7 +513,7 @@ static size_t single_smem(uint32_t np, uint32_t nb, bool concrete) {
     const size_t fbw = filter_block_words(np);
     // (+ 64 bytes after the '+' filter tables and 64 after the '+' records: bank offsets)
     return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * (concrete ? 16 : 32) + 64 +
-           (size_t)SSTAGES * SPL * SLOAD * 4 + (size_t)SW * SQ * 16 + (size_t)SW * SQ * 4 + (size_t)SW * SVC * 20 +
+           (size_t)SSTAGES * SPL * SLOAD * 4 + (size_t)SW * SQ * 16 + (size_t)SW * 5 * SVC * 4 +
            2 * SSTAGES * 4 + SSTAGES * 8;
 }
 
@@ -597,6 +585,7 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     A.vs = dev->n_segs ? dev->vs : nullptr;
     A.limit = limit;
     A.n_tiles = n_tiles;
+    A.words = cof_plane_words(dev->n_bases);
     A.hits = (unsigned long long*)hits;
     A.cap = hits_cap;
     A.counters = (unsigned long long*)(pd + plan->lay.counters);
