@@ -52,12 +52,18 @@ constexpr int SW = COF_SINGLE_SW;         // warps per CTA (16: 4 per SM sub-par
 constexpr int STHREADS = 32 * SW;
 constexpr int STW = 32 * SW;              // plane words per tile (one per lane)
 constexpr int SLOAD = STW + 4;            // words per plane and stage: tile + halo (16-byte multiple)
-constexpr int SSTAGES = 4;
+#ifndef COF_SINGLE_STAGES
+#define COF_SINGLE_STAGES 4
+#endif
+constexpr int SSTAGES = COF_SINGLE_STAGES;
 constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
-constexpr uint32_t SQ = 128;              // queued sites per warp (16-byte entries)
-constexpr int SR = 2;                     // sites per lane and batch
+#ifndef COF_SINGLE_R
+#define COF_SINGLE_R 2
+#endif
+constexpr int SR = COF_SINGLE_R;          // sites per lane and batch
+constexpr uint32_t SQ = 64u * SR;           // queued sites per warp (16-byte entries): two batches
 constexpr uint32_t SBATCH = 32 * SR;
-constexpr uint32_t SVC = 128;             // survivor entries per warp (ring; shares the owner list's space)
+constexpr uint32_t SVC = SR == 1 ? 64u : 128u;   // survivor entries per warp (ring; shares the owner list's space)
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
 constexpr uint32_t S_END = 0xFFFFFFFFu;   // tile id: no more tiles
 static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH, "ring");
@@ -106,12 +112,14 @@ __device__ __forceinline__ uint32_t lds32(uint32_t addr) {
     return x;
 }
 
-// The NP filter lookups of one site in block b: pair q at base[q] + OFF + q * 64.
+// The NP filter lookups of one site in block b: pair q at base[q] + boff + OFF + q * 64.
+// boff (the group's block offset) is warp-uniform: the address add can live in the
+// uniform datapath instead of NP vector adds per site and group.
 template <int NP, uint32_t OFF, int Q = 0>
-__device__ __forceinline__ void lds_filter(const uint32_t (&base)[NP], uint32_t (&v)[NP]) {
+__device__ __forceinline__ void lds_filter(const uint32_t (&base)[NP], uint32_t boff, uint32_t (&v)[NP]) {
     if constexpr (Q < NP) {
-        v[Q] = lds32<OFF + (uint32_t)Q * 64u>(base[Q]);
-        lds_filter<NP, OFF, Q + 1>(base, v);
+        v[Q] = lds32<OFF + (uint32_t)Q * 64u>(base[Q] + boff);
+        lds_filter<NP, OFF, Q + 1>(base, boff, v);
     }
 }
 
@@ -298,7 +306,7 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
                 const uint32_t sd = e.w >> 31;
                 site_bases<NP>(a, sd ? tb1 : tb0, sd, e.y, e.z, e.w & 0x7FFFFFFFu, base[r]);
             }
-            const uint32_t okm0 = (uint32_t)lane < n_items ? ~0u : 0u, okm1 = 32u + lane < n_items ? ~0u : 0u;
+
             uint32_t sv_h = 0, sv_n = 0;                    // warp-uniform survivor list state
             // groups of 4 blocks; one extra pass (b >= nb) drains the survivor list, so the
             // verification code exists once in the kernel (its size decides the I-cache hit rate)
@@ -306,18 +314,19 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
                 const bool drain = b >= nb;
                 if (!drain) {
                     const uint32_t* m = a.meta[b];
+                    const uint32_t boff = b * FBW * 4;
 #pragma unroll
                     for (int r = 0; r < SR; r++) {
                         uint32_t v[NP], p0, p1, p2, p3;
-                        lds_filter<NP, 0 * FBW * 4>(base[r], v);
+                        lds_filter<NP, 0 * FBW * 4>(base[r], boff, v);
                         p0 = filter_pass<NP, TC>(v, m);
-                        lds_filter<NP, 1 * FBW * 4>(base[r], v);
+                        lds_filter<NP, 1 * FBW * 4>(base[r], boff, v);
                         p1 = filter_pass<NP, TC>(v, m + 8);
-                        lds_filter<NP, 2 * FBW * 4>(base[r], v);
+                        lds_filter<NP, 2 * FBW * 4>(base[r], boff, v);
                         p2 = filter_pass<NP, TC>(v, m + 16);
-                        lds_filter<NP, 3 * FBW * 4>(base[r], v);
+                        lds_filter<NP, 3 * FBW * 4>(base[r], boff, v);
                         p3 = filter_pass<NP, TC>(v, m + 24);
-                        const uint32_t ok = r == 0 ? okm0 : okm1;
+                        const uint32_t ok = (uint32_t)r * 32u + lane < n_items ? ~0u : 0u;
                         p0 &= ok; p1 &= ok; p2 &= ok; p3 &= ok;
                         // a site with a survivor in this group of 4 blocks -> one survivor
                         // entry (ballot append; blocks past the plan have valid 0)
@@ -330,12 +339,7 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
                         }
                         sv_n += (uint32_t)__popc(hb);
                     }
-                    if (b + 4 < nb) {
-#pragma unroll
-                        for (int r = 0; r < SR; r++)
-#pragma unroll
-                            for (int q = 0; q < NP; q++) base[r][q] += 4 * FBW * 4;
-                    }
+
                 }
                 __syncwarp();
                 while (sv_n >= 32 || (drain && sv_n > 0)) {   // (<= 31 + SR x 32 entries: SVC holds them)

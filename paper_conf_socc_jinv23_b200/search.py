@@ -265,6 +265,32 @@ class HostGenome:
             cof.cof_load_chunk(self.chunk_struct(i), dev, stream)
 
 
+class ResidentGenome:
+    """A genome's packed chunks resident in one GPU's memory (all planes, incl. the N and
+    valid-start planes), uploaded once from a HostGenome: searches with different guide
+    sets then move no genome bytes over PCIe (Searcher.search_resident)."""
+
+    def __init__(self, host: HostGenome, device="cuda", stream=None):
+        self.device = torch.device(device)
+        self.chunks = host.chunks
+        self.segs = host.segs
+        self.d_planes, self.d_chunks = [], []
+        stream = stream or torch.cuda.current_stream(self.device)
+        with torch.cuda.device(self.device):
+            for i, ch in enumerate(host.chunks):
+                d = torch.empty((4, host.planes[i].shape[1]), dtype=torch.int32, device=self.device)
+                dch = (cof.make_chunk(0, 0, ch.n_bases, ch.n_owned, d[0], d[1], d[2], d[3], host.segs[i]) if ch.multi
+                       else cof.make_chunk(ch.chrom, ch.start, ch.n_bases, ch.n_owned, d[0], d[1], d[2]))
+                host.load(i, dch, stream)                       # the chunk's one H2D
+                self.d_planes.append(d)
+                self.d_chunks.append(dch)
+            stream.synchronize()
+
+    @property
+    def bytes(self):
+        return sum(d.numel() * 4 for d in self.d_planes)
+
+
 SPLIT_FILL = os.environ.get("COF_SPLIT_FILL", "0") == "1"   # measured slower end to end (DESIGN §6)
 PLANE_BUFS = int(os.environ.get("COF_PLANE_BUFS", 2))   # device plane sets in the search_host pipeline (3 measured no faster)
 if PLANE_BUFS < 2:
@@ -501,6 +527,63 @@ class Searcher:
         if use_out and not overflow:
             return out[:total]
         return merge_hit_lists([r for _, r in sorted(results, key=lambda x: x[0])], self.hit_dtype)
+
+    def search_resident(self, rg: "ResidentGenome", out=None):
+        """The search over a genome already resident in this GPU's memory (ResidentGenome:
+        planes uploaded once, then searched with any number of guide sets -- the usual
+        CRISPR-design loop): per chunk find / compare, device sort and decoration, and the
+        records' D2H on a second stream that overlaps the next chunk's kernels.  ``out``:
+        as in search_host.  Returns the sorted hit array."""
+        if rg.device != self.device:
+            raise ValueError(f"resident genome on {rg.device}, searcher on {self.device}")
+        max_bases = max((ch.n_bases for ch in rg.chunks), default=1)
+        self.reserve(max_bases, max(self._hits_cap, 1 << 16))
+        if not hasattr(self, "d2h_stream"):
+            self.d2h_stream = torch.cuda.Stream(self.device)
+        ws_bytes = cof.cof_decorate_workspace_bytes(max((len(ch.pieces) for ch in rg.chunks), default=1))
+        ws, results = [], []
+        rec_free = [None, None]
+        total, overflow = 0, False
+        with torch.cuda.device(self.device):
+            for j, (ch, dch) in enumerate(zip(rg.chunks, rg.d_chunks)):
+                kr = j & 1
+                _, _, nh = self.run_device_chunk(dch, ch.n_owned, counts=False)
+                if self.d_records is None or nh > self._rec_cap:
+                    self._reserve_records(nh)
+                recs = self.d_records[kr]
+                if rec_free[kr] is not None:
+                    self.stream.wait_event(rec_free[kr])
+                ws.append(torch.empty(ws_bytes, dtype=torch.uint8, device=self.device))
+                cof.cof_decorate(self.plan, self.plan_dev, dch, self.d_hits, nh, recs, ws[-1], self.stream,
+                                 cap=self._rec_cap)
+                fr = torch.cuda.Event()
+                fr.record(self.stream)
+                dst = None
+                if out is not None and not overflow:
+                    if total + nh <= len(out):
+                        dst = out[total:total + nh]
+                    else:
+                        overflow = True
+                if dst is None:
+                    dst = torch.empty(max(nh, 1) * self.hit_dtype.itemsize, dtype=torch.uint8,
+                                      pin_memory=True).numpy().view(self.hit_dtype)[:nh]
+                if nh:
+                    self.d2h_stream.wait_event(fr)
+                    with torch.cuda.stream(self.d2h_stream):
+                        torch.from_numpy(dst.view(np.uint8)).copy_(recs[: nh * self.hit_dtype.itemsize],
+                                                                   non_blocking=True)
+                        ev = torch.cuda.Event()
+                        ev.record(self.d2h_stream)
+                    rec_free[kr] = ev
+                results.append(dst)
+                total += nh
+            self.d2h_stream.synchronize()
+            self.stream.synchronize()
+            for w in ws:
+                cof.cof_decorate_check(w, self.stream)
+        if out is not None and not overflow:
+            return out[:total]
+        return merge_hit_lists(results, self.hit_dtype)
 
     def _reserve_records(self, n):
         # two device record buffers: chunk j decorates into one while chunk j-1's D2H drains the other
