@@ -57,6 +57,21 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity)
         : "memory");
 }
 
+// As mbar_wait_parity, but each try_wait may suspend the warp in hardware until the phase
+// completes (time hint ~1 ms): a warp that waits for a tile does not keep re-issuing.
+__device__ __forceinline__ void mbar_wait_parity_sleep(uint64_t* bar, uint32_t parity) {
+    uint32_t addr = smem_u32(bar);
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "WAITS_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n"
+        "@!P1 bra WAITS_%=;\n"
+        "}\n" ::"r"(addr),
+        "r"(parity), "r"(1000000u)
+        : "memory");
+}
+
 // 1-D bulk copy global -> shared through the TMA engine (cp.async.bulk, SASS UBLKCP);
 // completion is signalled on the mbarrier as transaction bytes.
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {

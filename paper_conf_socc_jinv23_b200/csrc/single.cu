@@ -45,30 +45,32 @@
 
 namespace cof {
 
-#ifndef COF_SINGLE_SW
-#define COF_SINGLE_SW 16
-#endif
-constexpr int SW = COF_SINGLE_SW;         // warps per CTA (16: 4 per SM sub-partition, <= 128 registers)
-constexpr int STHREADS = 32 * SW;
-constexpr int STW = 32 * SW;              // plane words per tile (one per lane)
-constexpr int SLOAD = STW + 4;            // words per plane and stage: tile + halo (16-byte multiple)
-#ifndef COF_SINGLE_STAGES
-#define COF_SINGLE_STAGES 4
-#endif
-constexpr int SSTAGES = COF_SINGLE_STAGES;
+// Kernel geometry.  Two instantiations (measured on B200): few guide blocks
+// (<= 8: C1-C4) take two sites per lane per batch -- the per-site work (queueing, table
+// addresses) is amortised over more lookups -- and 20 warps; many blocks (C5) take one
+// site per lane and 28 warps, which hides the filter's dependency latency better and keeps
+// all 32 blocks of a 1000-guide plan in one launch's shared memory.
+template <int W, int R, int S>
+struct SCfg {
+    static constexpr int SW = W;                  // warps per CTA (one CTA per SM)
+    static constexpr int STHREADS = 32 * W;
+    static constexpr int STW = 32 * W;            // plane words per tile (one per lane)
+    static constexpr int SLOAD = STW + 4;         // words per plane and stage: tile + halo (16-byte multiple)
+    static constexpr int SSTAGES = S;             // TMA ring depth
+    static constexpr int SR = R;                  // sites per lane and batch
+    static constexpr uint32_t SQ = 64u * R;       // queued sites per warp (16-byte entries): two batches
+    static constexpr uint32_t SBATCH = 32u * R;
+    static constexpr uint32_t SVC = R == 1 ? 64u : 128u;   // survivor entries per warp (ring)
+    static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH, "ring");
+    static_assert(5 * SVC >= SQ, "the owner list shares the survivor ring's space");
+    static_assert(SVC >= 31 + 32 * SR, "a group of blocks appends at most 32 entries per site row");
+};
+using SCfgFew = SCfg<20, 2, 4>;
+using SCfgMany = SCfg<28, 1, 4>;
+constexpr uint32_t SFEW_BLOCKS = 8;       // guide blocks up to which SCfgFew runs
 constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
-#ifndef COF_SINGLE_R
-#define COF_SINGLE_R 2
-#endif
-constexpr int SR = COF_SINGLE_R;          // sites per lane and batch
-constexpr uint32_t SQ = 64u * SR;           // queued sites per warp (16-byte entries): two batches
-constexpr uint32_t SBATCH = 32 * SR;
-constexpr uint32_t SVC = SR == 1 ? 64u : 128u;   // survivor entries per warp (ring; shares the owner list's space)
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
 constexpr uint32_t S_END = 0xFFFFFFFFu;   // tile id: no more tiles
-static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH, "ring");
-static_assert(5 * SVC >= SQ, "the owner list shares the survivor ring's space");
-static_assert(SVC >= 31 + 32 * SR, "a group of blocks appends at most 32 entries per site row");
 
 struct SingleArgs {
     const uint32_t* lo;
@@ -157,8 +159,11 @@ __device__ __forceinline__ unsigned long long s_key(uint32_t pos, uint32_t stran
            (unsigned long long)mm;
 }
 
-template <int NP, int TC, bool CONCRETE>
-__global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_constant__ SingleArgs a) {
+template <int NP, int TC, bool CONCRETE, class CFG>
+__global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __grid_constant__ SingleArgs a) {
+    constexpr int SW = CFG::SW, STHREADS = CFG::STHREADS, STW = CFG::STW, SLOAD = CFG::SLOAD;
+    constexpr int SSTAGES = CFG::SSTAGES, SR = CFG::SR;
+    constexpr uint32_t SQ = CFG::SQ, SBATCH = CFG::SBATCH, SVC = CFG::SVC;
     extern __shared__ __align__(128) uint8_t smem[];
     // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
     //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
@@ -232,56 +237,66 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
     uint32_t head = 0, q_n = 0;           // warp-uniform site ring state
     unsigned long long cnt_f = 0, cnt_r = 0;
 
-    // Verify up to 32 survivor entries [sv_h, sv_h + n): lane i takes entry i -- one site
-    // (its queue slot) and the four 32-guide survivor masks of one group of blocks -- and the
-    // warp walks the set bits block by block in warp-uniform rounds (a round per bit of the
-    // fullest lane; most masks are empty or hold one bit): exact count from the guide's
-    // record, the round's hits appended with one atomic.
-    auto flush = [&](uint32_t sv_h, uint32_t n) {
-        uint32_t mk[4] = {0u, 0u, 0u, 0u}, g0 = 0, pos = 0, wl = 0, wh = 0, wn = 0, sd = 0;
-        if ((uint32_t)lane < n) {
+    // Verify the survivor entries [sv_h, sv_h + n), n <= 32 (one site and the four 32-guide
+    // survivor masks of one group of blocks each) in ONE warp-wide round: lane i takes the
+    // lowest survivor of entry i, counts its mismatches exactly from the guide's record and
+    // clears it; an entry with survivors left goes back to the tail of the ring (ballot
+    // append) for a later round.  No per-bit loop: every round verifies one survivor per
+    // active lane; the round's hits are appended with one atomic.  Returns
+    // the number of entries re-appended.
+    auto flush = [&](uint32_t sv_h, uint32_t n, uint32_t tail) -> uint32_t {
+        uint32_t m0 = 0, m1 = 0, m2 = 0, m3 = 0, x = 0;
+        bool have = (uint32_t)lane < n;
+        if (have) {
             const uint32_t e = (sv_h + lane) & (SVC - 1);
-            const uint32_t x = sv_x[e];
-#pragma unroll
-            for (int q = 0; q < 4; q++) mk[q] = sv_m[q * SVC + e];
+            x = sv_x[e];
+            m0 = sv_m[e]; m1 = sv_m[SVC + e]; m2 = sv_m[2 * SVC + e]; m3 = sv_m[3 * SVC + e];
+        }
+        bool hit = false;
+        uint32_t g = 0, mm = 0, pos = 0, sd = 0;
+        if (have) {
+            const uint32_t sel = m0 ? m0 : (m1 ? m1 : (m2 ? m2 : m3));
+            const uint32_t bi = m0 ? 0u : (m1 ? 32u : (m2 ? 64u : 96u));
+            const uint32_t low = sel & (0u - sel);
+            if (m0) m0 ^= low; else if (m1) m1 ^= low; else if (m2) m2 ^= low; else m3 ^= low;
+            g = (x >> 8) * 128u + bi + (uint32_t)(__ffs(low) - 1);    // launch-local guide
             const uint4 it = queue[x & (SQ - 1)];
-            pos = it.x; wl = it.y; wh = it.z; sd = it.w >> 31; wn = it.w & 0x7FFFFFFFu;
-            g0 = (x >> 8) * 128u;                                 // first guide of the group
-        }
-        const uint4* vr = sd ? vrec1 : s_vrec;
-#pragma unroll 1
-        for (int q = 0; q < 4; q++) {
-            uint32_t msk = q == 0 ? mk[0] : q == 1 ? mk[1] : q == 2 ? mk[2] : mk[3];
-            while (__any_sync(0xFFFFFFFFu, msk != 0u)) {
-                bool hit = false;
-                uint32_t g = 0, mm = 0;
-                if (msk) {
-                    g = g0 + 32u * q + (uint32_t)(__ffs(msk) - 1);   // launch-local guide
-                    msk &= msk - 1;
-                    const uint4 r0 = vr[g * VSTR];                    // {lo, hi, care, t}
-                    uint32_t mis;
-                    if constexpr (CONCRETE) {
-                        mis = ((wl ^ r0.x) | (wh ^ r0.y) | wn) & r0.z;
-                    } else {
-                        const uint4 oh = vr[g * VSTR + 1];            // one-hot {A, C, G, T}
-                        const uint32_t nn = ~wn;
-                        const uint32_t match = (oh.x & ~wl & ~wh & nn) | (oh.y & wl & ~wh & nn) |
-                                               (oh.z & ~wl & wh & nn) | (oh.w & wl & wh & nn);
-                        mis = r0.z & ~match;
-                    }
-                    mm = (uint32_t)__popc(mis);
-                    hit = mm <= r0.w;
-                }
-                const unsigned hm = __ballot_sync(0xFFFFFFFFu, hit);
-                if (hm) {
-                    const int leader = __ffs(hm) - 1;
-                    unsigned long long o = 0;
-                    if (lane == leader) o = atomicAdd(&a.counters[2], (unsigned long long)__popc(hm));
-                    o = __shfl_sync(0xFFFFFFFFu, o, leader) + (unsigned)__popc(hm & lanemask_lt());
-                    if (hit && o < a.cap) a.hits[o] = s_key(pos, sd, a.block_base * 32u + g, mm);
-                }
+            pos = it.x;
+            sd = it.w >> 31;
+            const uint32_t wl = it.y, wh = it.z, wn = it.w & 0x7FFFFFFFu;
+            const uint4* rec = (sd ? vrec1 : s_vrec) + g * VSTR;
+            const uint4 r0 = rec[0];                                  // {lo, hi, care, t}
+            uint32_t mis;
+            if constexpr (CONCRETE) {
+                mis = ((wl ^ r0.x) | (wh ^ r0.y) | wn) & r0.z;
+            } else {
+                const uint4 oh = rec[1];                              // one-hot {A, C, G, T}
+                const uint32_t nn = ~wn;
+                const uint32_t match = (oh.x & ~wl & ~wh & nn) | (oh.y & wl & ~wh & nn) |
+                                       (oh.z & ~wl & wh & nn) | (oh.w & wl & wh & nn);
+                mis = r0.z & ~match;
             }
+            mm = (uint32_t)__popc(mis);
+            hit = mm <= r0.w;
         }
+        const unsigned hm = __ballot_sync(0xFFFFFFFFu, hit);
+        if (hm) {
+            const int leader = __ffs(hm) - 1;
+            unsigned long long o = 0;
+            if (lane == leader) o = atomicAdd(&a.counters[2], (unsigned long long)__popc(hm));
+            o = __shfl_sync(0xFFFFFFFFu, o, leader) + (unsigned)__popc(hm & lanemask_lt());
+            if (hit && o < a.cap) a.hits[o] = s_key(pos, sd, a.block_base * 32u + g, mm);
+        }
+        // entries with survivors left -> back to the ring's tail (their slots were just read)
+        const bool more = (m0 | m1 | m2 | m3) != 0u;
+        const unsigned mb = __ballot_sync(0xFFFFFFFFu, more);
+        __syncwarp();
+        if (more) {
+            const uint32_t e = (tail + (uint32_t)__popc(mb & lanemask_lt())) & (SVC - 1);
+            sv_x[e] = x;
+            sv_m[e] = m0; sv_m[SVC + e] = m1; sv_m[2 * SVC + e] = m2; sv_m[3 * SVC + e] = m3;
+        }
+        return (uint32_t)__popc(mb);
     };
 
     // per-lane state of the tile being appended: its plane words and the PAM bits not yet queued
@@ -342,11 +357,14 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
 
                 }
                 __syncwarp();
-                while (sv_n >= 32 || (drain && sv_n > 0)) {   // (<= 31 + SR x 32 entries: SVC holds them)
+                // (at most 31 + SR x 32 entries are queued: SVC holds them; a round takes 32 and
+                // puts back at most 32, and every round verifies one survivor per entry taken)
+                while (sv_n >= 32 || (drain && sv_n > 0)) {
                     const uint32_t nf = min(sv_n, 32u);
-                    flush(sv_h, nf);
+                    const uint32_t back = flush(sv_h, nf, sv_h + sv_n);
                     sv_h = (sv_h + nf) & (SVC - 1);
-                    sv_n -= nf;
+                    sv_n = sv_n - nf + back;
+                    __syncwarp();
                 }
                 if (drain) break;
             }
@@ -408,7 +426,7 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
         }
         // ---------------- next tile: words -> registers, release the stage, PAM test
         const int st = (int)(k % SSTAGES);
-        mbar_wait_parity(&full[st], (k / SSTAGES) & 1u);
+        mbar_wait_parity_sleep(&full[st], (k / SSTAGES) & 1u);
         k++;
         const uint32_t tile = s_tile[st];
         if (tile == S_END) {
@@ -462,26 +480,8 @@ __global__ void __launch_bounds__(STHREADS, 1) cof_single_kernel(const __grid_co
 typedef void (*SingleFn)(SingleArgs);
 
 template <int NP, int TC, bool CONCRETE>
-static SingleFn single_fn_t() { return cof_single_kernel<NP, TC, CONCRETE>; }
-
-template <int NP>
-static SingleFn single_fn_np(int tc, bool concrete) {
-    if constexpr (NP == 10 || NP == 12) {
-        if (concrete) {
-            switch (tc) {
-                case 0: return single_fn_t<NP, 0, true>();
-                case 1: return single_fn_t<NP, 1, true>();
-                case 2: return single_fn_t<NP, 2, true>();
-                case 3: return single_fn_t<NP, 3, true>();
-                case 4: return single_fn_t<NP, 4, true>();
-                case 5: return single_fn_t<NP, 5, true>();
-                case 6: return single_fn_t<NP, 6, true>();
-                case 7: return single_fn_t<NP, 7, true>();
-                default: break;
-            }
-        }
-    }
-    return single_fn_t<NP, -1, false>();
+static SingleFn single_fn_t(bool few) {
+    return few ? cof_single_kernel<NP, TC, CONCRETE, SCfgFew> : cof_single_kernel<NP, TC, CONCRETE, SCfgMany>;
 }
 
 // The kernel variant a plan runs: uniform-threshold, concrete-letter specialisations for
@@ -491,42 +491,70 @@ static bool single_uses_concrete(uint32_t np, int tc, bool concrete) {
     return (np == 10 || np == 12) && concrete && tc >= 0 && tc <= 7;
 }
 
-static SingleFn single_fn(uint32_t np, int tc, bool concrete) {
+template <int NP>
+static SingleFn single_fn_np(int tc, bool concrete, bool few) {
+    if constexpr (NP == 10 || NP == 12) {
+        if (concrete) {
+            switch (tc) {
+                case 0: return single_fn_t<NP, 0, true>(few);
+                case 1: return single_fn_t<NP, 1, true>(few);
+                case 2: return single_fn_t<NP, 2, true>(few);
+                case 3: return single_fn_t<NP, 3, true>(few);
+                case 4: return single_fn_t<NP, 4, true>(few);
+                case 5: return single_fn_t<NP, 5, true>(few);
+                case 6: return single_fn_t<NP, 6, true>(few);
+                case 7: return single_fn_t<NP, 7, true>(few);
+                default: break;
+            }
+        }
+    }
+    return single_fn_t<NP, -1, false>(few);
+}
+
+static SingleFn single_fn(uint32_t np, int tc, bool concrete, bool few) {
     switch (np) {
-        case 1: return single_fn_np<1>(tc, concrete);
-        case 2: return single_fn_np<2>(tc, concrete);
-        case 3: return single_fn_np<3>(tc, concrete);
-        case 4: return single_fn_np<4>(tc, concrete);
-        case 5: return single_fn_np<5>(tc, concrete);
-        case 6: return single_fn_np<6>(tc, concrete);
-        case 7: return single_fn_np<7>(tc, concrete);
-        case 8: return single_fn_np<8>(tc, concrete);
-        case 9: return single_fn_np<9>(tc, concrete);
-        case 10: return single_fn_np<10>(tc, concrete);
-        case 11: return single_fn_np<11>(tc, concrete);
-        case 12: return single_fn_np<12>(tc, concrete);
-        case 13: return single_fn_np<13>(tc, concrete);
-        case 14: return single_fn_np<14>(tc, concrete);
-        case 15: return single_fn_np<15>(tc, concrete);
-        case 16: return single_fn_np<16>(tc, concrete);
+        case 1: return single_fn_np<1>(tc, concrete, few);
+        case 2: return single_fn_np<2>(tc, concrete, few);
+        case 3: return single_fn_np<3>(tc, concrete, few);
+        case 4: return single_fn_np<4>(tc, concrete, few);
+        case 5: return single_fn_np<5>(tc, concrete, few);
+        case 6: return single_fn_np<6>(tc, concrete, few);
+        case 7: return single_fn_np<7>(tc, concrete, few);
+        case 8: return single_fn_np<8>(tc, concrete, few);
+        case 9: return single_fn_np<9>(tc, concrete, few);
+        case 10: return single_fn_np<10>(tc, concrete, few);
+        case 11: return single_fn_np<11>(tc, concrete, few);
+        case 12: return single_fn_np<12>(tc, concrete, few);
+        case 13: return single_fn_np<13>(tc, concrete, few);
+        case 14: return single_fn_np<14>(tc, concrete, few);
+        case 15: return single_fn_np<15>(tc, concrete, few);
+        case 16: return single_fn_np<16>(tc, concrete, few);
         default: return nullptr;
     }
 }
 
-static size_t single_smem(uint32_t np, uint32_t nb, bool concrete) {
+struct SGeom {
+    int threads, stw, sload, stages;
+    uint32_t sq, svc, sw;
+};
+template <class C>
+static SGeom sgeom() { return {C::STHREADS, C::STW, C::SLOAD, C::SSTAGES, C::SQ, C::SVC, (uint32_t)C::SW}; }
+static SGeom single_geom(bool few) { return few ? sgeom<SCfgFew>() : sgeom<SCfgMany>(); }
+
+static size_t single_smem(const SGeom& g, uint32_t np, uint32_t nb, bool concrete) {
     const size_t fbw = filter_block_words(np);
     // (+ 64 bytes after the '+' filter tables and 64 after the '+' records: bank offsets)
     return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * (concrete ? 16 : 32) + 64 +
-           (size_t)SSTAGES * SPL * SLOAD * 4 + (size_t)SW * SQ * 16 + (size_t)SW * 5 * SVC * 4 +
-           2 * SSTAGES * 4 + SSTAGES * 8;
+           (size_t)g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * 5 * g.svc * 4 +
+           2 * g.stages * 4 + g.stages * 8;
 }
 
 static constexpr size_t SMEM_MAX = 227 * 1024;
 
 // Guide blocks per launch: as many as fit the shared-memory budget (a multiple of 4).
-static uint32_t single_blocks_per_launch(uint32_t np, bool concrete) {
+static uint32_t single_blocks_per_launch(const SGeom& g, uint32_t np, bool concrete) {
     uint32_t nb = SMAX_BLOCKS;
-    while (nb > 4 && single_smem(np, nb, concrete) > SMEM_MAX) nb -= 4;
+    while (nb > 4 && single_smem(g, np, nb, concrete) > SMEM_MAX) nb -= 4;
     return nb;
 }
 
@@ -561,6 +589,28 @@ bool single_supported(const cof_plan* plan, bool strict) {
     return tmax + 3 <= np;
 }
 
+struct SinglePlanInfo {
+    uint32_t np;
+    int ut;            // the uniform threshold, -1 if the guides' thresholds differ
+    bool concrete;     // the concrete-letter kernel runs
+    bool few;          // SCfgFew geometry
+    SGeom geom;
+    uint32_t bpl;      // guide blocks per launch
+};
+
+static SinglePlanInfo single_info(const cof_plan* plan) {
+    SinglePlanInfo I;
+    I.np = plan->pairs[0].n_pairs;
+    I.ut = (int)plan->max_mm[0];
+    for (uint32_t i = 1; i < plan->n_guides && I.ut >= 0; i++)
+        if (plan->max_mm[i] != plan->max_mm[0]) I.ut = -1;
+    I.concrete = single_uses_concrete(I.np, I.ut, !plan->any_degenerate);
+    I.few = plan->n_blocks <= SFEW_BLOCKS;
+    I.geom = single_geom(I.few);
+    I.bpl = single_blocks_per_launch(I.geom, I.np, I.concrete);
+    return I;
+}
+
 static std::mutex g_single_mu;
 
 cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, unsigned int* tickets,
@@ -570,16 +620,13 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     if (((uintptr_t)dev->lo | (uintptr_t)dev->hi | (uintptr_t)dev->nm | (uintptr_t)dev->vs) & 15)
         return set_error(COF_E_ARG, "single pass: planes must be 16-byte aligned");
     if (dev->n_segs && !dev->vs) return set_error(COF_E_ARG, "single pass: multi-segment chunk without vs plane");
+    const SinglePlanInfo I = single_info(plan);
+    const SGeom& G = I.geom;
     uint64_t limit = dev->n_bases >= L ? dev->n_bases - L + 1 : 0;
     if (!dev->n_segs && limit > dev->n_owned) limit = dev->n_owned;
-    const uint32_t n_tiles = (uint32_t)((limit + (uint64_t)STW * 32 - 1) / ((uint64_t)STW * 32));
-    const uint32_t np = plan->pairs[0].n_pairs;
-    int ut = (int)plan->max_mm[0];
-    for (uint32_t i = 1; i < plan->n_guides && ut >= 0; i++)
-        if (plan->max_mm[i] != plan->max_mm[0]) ut = -1;
-    const bool concrete = single_uses_concrete(np, ut, !plan->any_degenerate);
-    SingleFn fn = single_fn(np, ut, concrete);
-    if (!fn) return set_error(COF_E_STATE, "single pass: %u pairs", np);
+    const uint32_t n_tiles = (uint32_t)((limit + (uint64_t)G.stw * 32 - 1) / ((uint64_t)G.stw * 32));
+    SingleFn fn = single_fn(I.np, I.ut, I.concrete, I.few);
+    if (!fn) return set_error(COF_E_STATE, "single pass: %u pairs", I.np);
     int dev_id = 0;
     cudaGetDevice(&dev_id);
     int sms = 0;
@@ -611,18 +658,17 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     }
     A.contig = plan->pairs[0].contig && plan->pairs[1].contig && plan->pairs[0].n_cmp == plan->pairs[1].n_cmp;
     A.cmp_mask = plan->pairs[0].n_cmp >= 32 ? ~0u : ((1u << plan->pairs[0].n_cmp) - 1u);
-    const uint32_t bpl = single_blocks_per_launch(np, concrete);
-    const uint32_t fbw = filter_block_words(np);
+    const uint32_t fbw = filter_block_words(I.np);
     const uint32_t* pm = (const uint32_t*)(plan->image.data() + plan->lay.pmeta_fwd);
     {
         std::lock_guard<std::mutex> lk(g_single_mu);   // (per device state; cheap, set every call)
         cudaError_t e = cudaFuncSetAttribute((const void*)fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)single_smem(np, bpl, concrete));
+                                             (int)single_smem(G, I.np, I.bpl, I.concrete));
         if (e != cudaSuccess) return cuda_error(e, "single pass smem attribute");
     }
     uint32_t li = 0;
-    for (uint32_t bb = 0; bb < plan->n_blocks; bb += bpl, li++) {
-        const uint32_t nbl = std::min(bpl, plan->n_blocks - bb);
+    for (uint32_t bb = 0; bb < plan->n_blocks; bb += I.bpl, li++) {
+        const uint32_t nbl = std::min(I.bpl, plan->n_blocks - bb);
         // whole groups of 4 blocks: padding blocks (zero tables in the plan image) have no valid guide
         const uint32_t nb4 = (nbl + 3) & ~3u;
         A.n_blocks = nb4;
@@ -638,7 +684,7 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
         if (n_tiles == 0) continue;
         uint32_t grid = (uint32_t)sms;
         if (grid > n_tiles) grid = n_tiles;
-        fn<<<grid, STHREADS, single_smem(np, nb4, concrete), stream>>>(A);
+        fn<<<grid, G.threads, single_smem(G, I.np, nb4, I.concrete), stream>>>(A);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "cof_single_kernel launch");
         count_launches(1);
@@ -647,12 +693,8 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
 }
 
 uint32_t single_launches(const cof_plan* plan) {
-    int ut = (int)plan->max_mm[0];
-    for (uint32_t i = 1; i < plan->n_guides && ut >= 0; i++)
-        if (plan->max_mm[i] != plan->max_mm[0]) ut = -1;
-    const uint32_t np = plan->pairs[0].n_pairs;
-    const uint32_t bpl = single_blocks_per_launch(np, single_uses_concrete(np, ut, !plan->any_degenerate));
-    return (plan->n_blocks + bpl - 1) / bpl;
+    const SinglePlanInfo I = single_info(plan);
+    return (plan->n_blocks + I.bpl - 1) / I.bpl;
 }
 
 }  // namespace cof
