@@ -65,8 +65,27 @@ struct SCfg {
     static_assert(5 * SVC >= SQ, "the owner list shares the survivor ring's space");
     static_assert(SVC >= 31 + 32 * SR, "a group of blocks appends at most 32 entries per site row");
 };
-using SCfgFew = SCfg<20, 2, 4>;
-using SCfgMany = SCfg<28, 1, 4>;
+// (warps, sites per lane, ring stages); -DCOF_FEW_W=... etc. override for A/B builds
+#ifndef COF_FEW_W
+#define COF_FEW_W 20
+#endif
+#ifndef COF_FEW_R
+#define COF_FEW_R 2
+#endif
+#ifndef COF_FEW_S
+#define COF_FEW_S 8
+#endif
+#ifndef COF_MANY_W
+#define COF_MANY_W 28
+#endif
+#ifndef COF_MANY_R
+#define COF_MANY_R 1
+#endif
+#ifndef COF_MANY_S
+#define COF_MANY_S 4
+#endif
+using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S>;
+using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S>;
 constexpr uint32_t SFEW_BLOCKS = 8;       // guide blocks up to which SCfgFew runs
 constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
@@ -231,7 +250,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     uint4* queue = queues + warp * SQ;
     uint32_t* owner = owners + warp * 5 * SVC;           // append: (lane, bit) of queued sites
     uint32_t* sv_x = owner;                              // batch: survivor entries: slot | group << 8
-    uint32_t* sv_m = owner + SVC;                        //        and the group's 4 survivor masks
+    uint4* sv_m = reinterpret_cast<uint4*>(owner + SVC); //        and the group's 4 survivor masks (16 B)
     const uint32_t tb0 = smem_u32(s_ftab), tb1 = tb0 + nb * FBW * 4 + 64;
     const uint4* vrec1 = s_vrec + nb * 32 * VSTR + 4;
     uint32_t head = 0, q_n = 0;           // warp-uniform site ring state
@@ -250,7 +269,8 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         if (have) {
             const uint32_t e = (sv_h + lane) & (SVC - 1);
             x = sv_x[e];
-            m0 = sv_m[e]; m1 = sv_m[SVC + e]; m2 = sv_m[2 * SVC + e]; m3 = sv_m[3 * SVC + e];
+            const uint4 mv = sv_m[e];
+            m0 = mv.x; m1 = mv.y; m2 = mv.z; m3 = mv.w;
         }
         bool hit = false;
         uint32_t g = 0, mm = 0, pos = 0, sd = 0;
@@ -294,7 +314,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         if (more) {
             const uint32_t e = (tail + (uint32_t)__popc(mb & lanemask_lt())) & (SVC - 1);
             sv_x[e] = x;
-            sv_m[e] = m0; sv_m[SVC + e] = m1; sv_m[2 * SVC + e] = m2; sv_m[3 * SVC + e] = m3;
+            sv_m[e] = make_uint4(m0, m1, m2, m3);
         }
         return (uint32_t)__popc(mb);
     };
@@ -350,7 +370,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                         const uint32_t e = (sv_h + sv_n + (uint32_t)__popc(hb & lanemask_lt())) & (SVC - 1);
                         if (has) {
                             sv_x[e] = ((head + (uint32_t)r * 32 + lane) & (SQ - 1)) | ((b >> 2) << 8);
-                            sv_m[e] = p0; sv_m[SVC + e] = p1; sv_m[2 * SVC + e] = p2; sv_m[3 * SVC + e] = p3;
+                            sv_m[e] = make_uint4(p0, p1, p2, p3);
                         }
                         sv_n += (uint32_t)__popc(hb);
                     }
