@@ -54,9 +54,10 @@ template <int W, int R, int S>
 struct SCfg {
     static constexpr int SW = W;                  // warps per CTA (one CTA per SM)
     static constexpr int STHREADS = 32 * W;
-    static constexpr int STW = 32 * W;            // plane words per tile (one per lane)
+    static constexpr int STW = 32;                // plane words per warp tile (one per lane)
     static constexpr int SLOAD = STW + 4;         // words per plane and stage: tile + halo (16-byte multiple)
-    static constexpr int SSTAGES = S;             // TMA ring depth
+    static constexpr int SSTAGES = S;             // per-warp TMA ring depth
+    static constexpr uint32_t SGRAB = 4;          // warp tiles per ticket (4096 window starts)
     static constexpr int SR = R;                  // sites per lane and batch
     static constexpr uint32_t SQ = 64u * R;       // queued sites per warp (16-byte entries): two batches
     static constexpr uint32_t SBATCH = 32u * R;
@@ -73,7 +74,7 @@ struct SCfg {
 #define COF_FEW_R 2
 #endif
 #ifndef COF_FEW_S
-#define COF_FEW_S 8
+#define COF_FEW_S 4
 #endif
 #ifndef COF_MANY_W
 #define COF_MANY_W 28
@@ -82,7 +83,7 @@ struct SCfg {
 #define COF_MANY_R 1
 #endif
 #ifndef COF_MANY_S
-#define COF_MANY_S 4
+#define COF_MANY_S 3
 #endif
 using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S>;
 using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S>;
@@ -182,11 +183,12 @@ template <int NP, int TC, bool CONCRETE, class CFG>
 __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __grid_constant__ SingleArgs a) {
     constexpr int SW = CFG::SW, STHREADS = CFG::STHREADS, STW = CFG::STW, SLOAD = CFG::SLOAD;
     constexpr int SSTAGES = CFG::SSTAGES, SR = CFG::SR;
+    constexpr uint32_t SGRAB = CFG::SGRAB;
     constexpr uint32_t SQ = CFG::SQ, SBATCH = CFG::SBATCH, SVC = CFG::SVC;
     extern __shared__ __align__(128) uint8_t smem[];
     // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
     //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
-    //         [ring: SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
+    //         [per warp: TMA ring SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
     //         [per warp: append owner list (SQ words) / survivor ring (SVC x 5 words)]
     //         [tile ids, release counters][full mbarriers]
     constexpr uint32_t FBW = (NP * 25u + 15u) & ~15u;
@@ -195,17 +197,28 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     uint32_t* s_ftab = reinterpret_cast<uint32_t*>(smem);
     uint4* s_vrec = reinterpret_cast<uint4*>(smem + 2 * nb * FBW * 4 + 64);
     uint32_t* ring = reinterpret_cast<uint32_t*>(reinterpret_cast<uint8_t*>(s_vrec) + 2 * nb * 32 * VSTR * 16 + 64);
-    uint4* queues = reinterpret_cast<uint4*>(ring + SSTAGES * SPL * SLOAD);
+    uint4* queues = reinterpret_cast<uint4*>(ring + SW * SSTAGES * SPL * SLOAD);
     uint32_t* owners = reinterpret_cast<uint32_t*>(queues + SW * SQ);   // per warp: 5 x SVC words
-    uint32_t* s_tile = owners + SW * 5 * SVC;
-    uint32_t* s_rel = s_tile + SSTAGES;
-    uint64_t* full = reinterpret_cast<uint64_t*>(s_tile + 2 * SSTAGES);
+    uint32_t* s_tiles = owners + SW * 5 * SVC;                        // per warp: tile id of each stage
+    uint64_t* fulls = reinterpret_cast<uint64_t*>(s_tiles + ((SW * SSTAGES + 1) & ~1));
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const bool vsp = a.vs != nullptr;
-    // grab the next tile and stream it into stage st (or mark the stage as the end)
-    auto refill = [&](int st) {
-        const uint32_t tile = atomicAdd(a.ticket, 1u);
+    // Every warp streams its own warp tiles (32 plane words = 1024 window starts) through its
+    // own TMA ring: no warp waits for another one to release a stage (with a ring shared by
+    // the CTA, the warps' random per-tile work made them drift apart until the ring blocked
+    // the leaders).  Lane 0 grabs SGRAB consecutive warp tiles per global ticket.
+    uint32_t* wring = ring + warp * SSTAGES * SPL * SLOAD;
+    uint32_t* s_tile = s_tiles + warp * SSTAGES;
+    uint64_t* full = fulls + warp * SSTAGES;
+    uint32_t grab_base = 0, grab_left = 0;               // lane 0's current ticket
+    auto refill = [&](int st) {                           // (lane 0 only)
+        if (grab_left == 0) {
+            grab_base = atomicAdd(a.ticket, 1u) * SGRAB;
+            grab_left = SGRAB;
+        }
+        const uint32_t tile = grab_base++;
+        grab_left--;
         if (tile >= a.n_tiles) {
             s_tile[st] = S_END;
             mbar_arrive(&full[st]);
@@ -213,10 +226,10 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         }
         s_tile[st] = tile;
         const size_t w0 = (size_t)tile * STW;
-        // (a tile size that does not divide the planes' 512-word padding: the last tile's
-        // copy stops at the allocation; the words past it only feed invalid starts)
+        // (the last tile's copy stops at the planes' allocation; the words past it only feed
+        // invalid starts)
         const uint32_t nbytes = (uint32_t)min((uint64_t)SLOAD, a.words - w0) * 4u;
-        uint32_t* S = ring + st * SPL * SLOAD;
+        uint32_t* S = wring + st * SPL * SLOAD;
         fence_proxy_async_smem();
         mbar_arrive_expect_tx(&full[st], (vsp ? 4 : 3) * nbytes);
         bulk_g2s(S + 0 * SLOAD, a.lo + w0, nbytes, &full[st]);
@@ -237,15 +250,14 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             s_vrec[nv * VSTR + 4 + i] = __ldg(a.vrec[1] + 2 * g + h);
         }
     }
-    if (tid == 0) {
-        for (int s = 0; s < SSTAGES; s++) {
-            mbar_init(&full[s], 1);
-            s_rel[s] = 0;
-        }
+    if (lane == 0) {
+        for (int s = 0; s < SSTAGES; s++) mbar_init(&full[s], 1);
         fence_mbar_init();
-        for (int s = 0; s < SSTAGES; s++) refill(s);
     }
     __syncthreads();
+    if (lane == 0)
+        for (int s = 0; s < SSTAGES; s++) refill(s);
+    __syncwarp();
 
     uint4* queue = queues + warp * SQ;
     uint32_t* owner = owners + warp * 5 * SVC;           // append: (lane, bit) of queued sites
@@ -322,7 +334,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     // per-lane state of the tile being appended: its plane words and the PAM bits not yet queued
     uint32_t lo0 = 0, lo1 = 0, lo2 = 0, hi0 = 0, hi1 = 0, hi2 = 0, nm0 = 0, nm1 = 0, nm2 = 0;
     uint32_t pend0 = 0u, pend1 = 0u, pbase = 0;
-    const int w = warp * 32 + lane;
+    const int w = lane;                                   // this lane's word in the warp tile
     uint32_t k = 0;
     bool tiles_done = false;
     // One loop, one call site each for the batch comparison and the queue append (the
@@ -446,28 +458,25 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         }
         // ---------------- next tile: words -> registers, release the stage, PAM test
         const int st = (int)(k % SSTAGES);
+#ifdef COF_SINGLE_SPIN
+        mbar_wait_parity(&full[st], (k / SSTAGES) & 1u);
+#else
         mbar_wait_parity_sleep(&full[st], (k / SSTAGES) & 1u);
+#endif
         k++;
         const uint32_t tile = s_tile[st];
         if (tile == S_END) {
             tiles_done = true;
             continue;
         }
-        const uint32_t* S = ring + st * SPL * SLOAD;
+        const uint32_t* S = wring + st * SPL * SLOAD;
         lo0 = S[w]; lo1 = S[w + 1]; lo2 = S[w + 2];
         hi0 = S[SLOAD + w]; hi1 = S[SLOAD + w + 1]; hi2 = S[SLOAD + w + 2];
         nm0 = S[2 * SLOAD + w]; nm1 = S[2 * SLOAD + w + 1]; nm2 = S[2 * SLOAD + w + 2];
         uint32_t valid = vsp ? S[3 * SLOAD + w] : ~0u;
         __syncwarp();
-        if (lane == 0) {   // this warp is done with the stage; the last of the SW warps refills it
-            __threadfence_block();
-            if (atomicAdd(&s_rel[st], 1u) == SW - 1) {
-                s_rel[st] = 0;
-                __threadfence_block();
-                refill(st);
-            }
-        }
-        const uint64_t pw = ((uint64_t)tile * STW + (uint32_t)w) * 32u;   // first start of this word
+        if (lane == 0) refill(st);   // the warp has the stage in registers: stream its tile k + SSTAGES
+        const uint64_t pw = ((uint64_t)tile * STW + (uint32_t)lane) * 32u;   // first start of this word
         if (pw + 32 > a.limit) valid &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
         pend0 = pend1 = valid;
         for (uint32_t e = 0; e < a.ne; e++) {
@@ -481,7 +490,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             cnt_f += (unsigned)__popc(pend0);
             cnt_r += (unsigned)__popc(pend1);
         }
-        pbase = (uint32_t)(((uint64_t)tile * STW + (uint32_t)warp * 32u) * 32u);   // first start of lane 0's word
+        pbase = (uint32_t)((uint64_t)tile * STW * 32u);   // first start of lane 0's word
     }
     if (a.count_items) {
 #pragma unroll
@@ -565,8 +574,8 @@ static size_t single_smem(const SGeom& g, uint32_t np, uint32_t nb, bool concret
     const size_t fbw = filter_block_words(np);
     // (+ 64 bytes after the '+' filter tables and 64 after the '+' records: bank offsets)
     return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * (concrete ? 16 : 32) + 64 +
-           (size_t)g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * 5 * g.svc * 4 +
-           2 * g.stages * 4 + g.stages * 8;
+           (size_t)g.sw * g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * 5 * g.svc * 4 +
+           (size_t)((g.sw * g.stages + 1) & ~1) * 4 + (size_t)g.sw * g.stages * 8;
 }
 
 static constexpr size_t SMEM_MAX = 227 * 1024;

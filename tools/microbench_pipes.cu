@@ -1,7 +1,7 @@
 // Micro-benchmark of the integer pipes the comparer binds on (sm_100a).
 // Measures warp-instruction throughput of POPC, LOP3 and the comparer's inner-loop mix.
 // Output: one line per variant with ops/clk/SM, using the measured SM clock
-// (clock64 delta over the kernel, averaged over CTAs).
+// (CTA 0's clock64 delta over its own globaltimer delta: the SM clock while it ran).
 #include <cstdio>
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -22,7 +22,8 @@ __global__ void kern(const uint32_t* __restrict__ in, uint32_t* out, int iters, 
     for (int i = 0; i < 8; i++) r[i] = in[(threadIdx.x + i) & 255] + blockIdx.x;
     uint32_t g0 = in[300], g1 = in[301], nt = in[302];
     uint32_t acc = 0;
-    unsigned long long t0 = clock64();
+    unsigned long long t0 = clock64(), gt0;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt0));
     if (V == 0) {          // POPC throughput: popc on 8 independent values per iter, values perturbed by one LOP3 every 4 iters
         uint32_t s[8] = {0,0,0,0,0,0,0,0};
         for (int it = 0; it < iters; it++) {
@@ -67,8 +68,9 @@ __global__ void kern(const uint32_t* __restrict__ in, uint32_t* out, int iters, 
             if (o < 0) acc += 1;
         }
     }
-    unsigned long long t1 = clock64();
-    if (threadIdx.x == 0) atomicAdd(clk, t1 - t0);
+    unsigned long long t1 = clock64(), gt1;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt1));
+    if (threadIdx.x == 0 && blockIdx.x == 0) { clk[0] = t1 - t0; clk[1] = gt1 - gt0; }
     if (acc == 0x12345678u) out[0] = acc;
 }
 
@@ -76,7 +78,7 @@ int main() {
     int dev = 0; cudaDeviceProp prop; CK(cudaGetDeviceProperties(&prop, dev));
     int sms = prop.multiProcessorCount;
     uint32_t* in; uint32_t* out; unsigned long long* clk;
-    CK(cudaMalloc(&in, 4096)); CK(cudaMalloc(&out, 64)); CK(cudaMalloc(&clk, 8));
+    CK(cudaMalloc(&in, 4096)); CK(cudaMalloc(&out, 64)); CK(cudaMalloc(&clk, 16));
     uint32_t h[1024]; for (int i = 0; i < 1024; i++) h[i] = 0x9E3779B9u * (i + 1);
     h[302] = (uint32_t)-7;  // nt = -(t+1), t = 6
     CK(cudaMemcpy(in, h, 4096, cudaMemcpyHostToDevice));
@@ -84,7 +86,7 @@ int main() {
     for (int v = 0; v < 4; v++) {
         for (int rep = 0; rep < 2; rep++) {
             int iters = 20000, threads = 256, blocks = sms * 8;
-            CK(cudaMemset(clk, 0, 8));
+            CK(cudaMemset(clk, 0, 16));
             cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
             cudaEventRecord(a);
             if (v == 0) kern<0><<<blocks, threads>>>(in, out, iters, clk);
@@ -93,9 +95,8 @@ int main() {
             if (v == 3) kern<3><<<blocks, threads>>>(in, out, iters, clk);
             cudaEventRecord(b); CK(cudaEventSynchronize(b));
             float ms; cudaEventElapsedTime(&ms, a, b);
-            unsigned long long c; CK(cudaMemcpy(&c, clk, 8, cudaMemcpyDeviceToHost));
-            double avg_clk = (double)c / blocks;             // cycles per CTA
-            double mhz = avg_clk * (blocks / (double)(sms * 8)) / (ms * 1e3);  // CTAs run concurrently (8/SM)
+            unsigned long long c[2]; CK(cudaMemcpy(c, clk, 16, cudaMemcpyDeviceToHost));
+            double mhz = (double)c[0] / (double)c[1] * 1e3;   // cycles per ns of CTA 0 -> MHz
             double units = (double)blocks * threads * iters;  // loop iterations (per thread)
             double per_iter_ops = (v == 0) ? 8 : (v == 1) ? 16 : 8;  // popcs / lop3s / comparisons
             double rate = units * per_iter_ops / (ms * 1e-3);
