@@ -54,10 +54,9 @@ template <int W, int R, int S>
 struct SCfg {
     static constexpr int SW = W;                  // warps per CTA (one CTA per SM)
     static constexpr int STHREADS = 32 * W;
-    static constexpr int STW = 32;                // plane words per warp tile (one per lane)
+    static constexpr int STW = 32 * W;            // plane words per tile (one per lane)
     static constexpr int SLOAD = STW + 4;         // words per plane and stage: tile + halo (16-byte multiple)
-    static constexpr int SSTAGES = S;             // per-warp TMA ring depth
-    static constexpr uint32_t SGRAB = 4;          // warp tiles per ticket (4096 window starts)
+    static constexpr int SSTAGES = S;             // TMA ring depth
     static constexpr int SR = R;                  // sites per lane and batch
     static constexpr uint32_t SQ = 64u * R;       // queued sites per warp (16-byte entries): two batches
     static constexpr uint32_t SBATCH = 32u * R;
@@ -68,7 +67,7 @@ struct SCfg {
 };
 // (warps, sites per lane, ring stages); -DCOF_FEW_W=... etc. override for A/B builds
 #ifndef COF_FEW_W
-#define COF_FEW_W 20
+#define COF_FEW_W 24
 #endif
 #ifndef COF_FEW_R
 #define COF_FEW_R 2
@@ -83,7 +82,7 @@ struct SCfg {
 #define COF_MANY_R 1
 #endif
 #ifndef COF_MANY_S
-#define COF_MANY_S 3
+#define COF_MANY_S 4
 #endif
 using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S>;
 using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S>;
@@ -183,12 +182,11 @@ template <int NP, int TC, bool CONCRETE, class CFG>
 __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __grid_constant__ SingleArgs a) {
     constexpr int SW = CFG::SW, STHREADS = CFG::STHREADS, STW = CFG::STW, SLOAD = CFG::SLOAD;
     constexpr int SSTAGES = CFG::SSTAGES, SR = CFG::SR;
-    constexpr uint32_t SGRAB = CFG::SGRAB;
     constexpr uint32_t SQ = CFG::SQ, SBATCH = CFG::SBATCH, SVC = CFG::SVC;
     extern __shared__ __align__(128) uint8_t smem[];
     // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
     //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
-    //         [per warp: TMA ring SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
+    //         [ring: SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
     //         [per warp: append owner list (SQ words) / survivor ring (SVC x 5 words)]
     //         [tile ids, release counters][full mbarriers]
     constexpr uint32_t FBW = (NP * 25u + 15u) & ~15u;
@@ -197,28 +195,18 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     uint32_t* s_ftab = reinterpret_cast<uint32_t*>(smem);
     uint4* s_vrec = reinterpret_cast<uint4*>(smem + 2 * nb * FBW * 4 + 64);
     uint32_t* ring = reinterpret_cast<uint32_t*>(reinterpret_cast<uint8_t*>(s_vrec) + 2 * nb * 32 * VSTR * 16 + 64);
-    uint4* queues = reinterpret_cast<uint4*>(ring + SW * SSTAGES * SPL * SLOAD);
+    uint4* queues = reinterpret_cast<uint4*>(ring + SSTAGES * SPL * SLOAD);
     uint32_t* owners = reinterpret_cast<uint32_t*>(queues + SW * SQ);   // per warp: 5 x SVC words
-    uint32_t* s_tiles = owners + SW * 5 * SVC;                        // per warp: tile id of each stage
-    uint64_t* fulls = reinterpret_cast<uint64_t*>(s_tiles + ((SW * SSTAGES + 1) & ~1));
+    uint32_t* s_tile = owners + SW * 5 * SVC;
+    uint32_t* s_rel = s_tile + SSTAGES;
+    uint32_t* s_next = s_rel + SSTAGES;                              // next chunk to take (ring order)
+    uint64_t* full = reinterpret_cast<uint64_t*>(s_tile + 2 * SSTAGES + 2);
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const bool vsp = a.vs != nullptr;
-    // Every warp streams its own warp tiles (32 plane words = 1024 window starts) through its
-    // own TMA ring: no warp waits for another one to release a stage (with a ring shared by
-    // the CTA, the warps' random per-tile work made them drift apart until the ring blocked
-    // the leaders).  Lane 0 grabs SGRAB consecutive warp tiles per global ticket.
-    uint32_t* wring = ring + warp * SSTAGES * SPL * SLOAD;
-    uint32_t* s_tile = s_tiles + warp * SSTAGES;
-    uint64_t* full = fulls + warp * SSTAGES;
-    uint32_t grab_base = 0, grab_left = 0;               // lane 0's current ticket
-    auto refill = [&](int st) {                           // (lane 0 only)
-        if (grab_left == 0) {
-            grab_base = atomicAdd(a.ticket, 1u) * SGRAB;
-            grab_left = SGRAB;
-        }
-        const uint32_t tile = grab_base++;
-        grab_left--;
+    // grab the next tile and stream it into stage st (or mark the stage as the end)
+    auto refill = [&](int st) {
+        const uint32_t tile = atomicAdd(a.ticket, 1u);
         if (tile >= a.n_tiles) {
             s_tile[st] = S_END;
             mbar_arrive(&full[st]);
@@ -226,10 +214,10 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         }
         s_tile[st] = tile;
         const size_t w0 = (size_t)tile * STW;
-        // (the last tile's copy stops at the planes' allocation; the words past it only feed
-        // invalid starts)
+        // (a tile size that does not divide the planes' 512-word padding: the last tile's
+        // copy stops at the allocation; the words past it only feed invalid starts)
         const uint32_t nbytes = (uint32_t)min((uint64_t)SLOAD, a.words - w0) * 4u;
-        uint32_t* S = wring + st * SPL * SLOAD;
+        uint32_t* S = ring + st * SPL * SLOAD;
         fence_proxy_async_smem();
         mbar_arrive_expect_tx(&full[st], (vsp ? 4 : 3) * nbytes);
         bulk_g2s(S + 0 * SLOAD, a.lo + w0, nbytes, &full[st]);
@@ -250,14 +238,16 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             s_vrec[nv * VSTR + 4 + i] = __ldg(a.vrec[1] + 2 * g + h);
         }
     }
-    if (lane == 0) {
-        for (int s = 0; s < SSTAGES; s++) mbar_init(&full[s], 1);
+    if (tid == 0) {
+        for (int s = 0; s < SSTAGES; s++) {
+            mbar_init(&full[s], 1);
+            s_rel[s] = 0;
+        }
+        *s_next = 0;
         fence_mbar_init();
+        for (int s = 0; s < SSTAGES; s++) refill(s);
     }
     __syncthreads();
-    if (lane == 0)
-        for (int s = 0; s < SSTAGES; s++) refill(s);
-    __syncwarp();
 
     uint4* queue = queues + warp * SQ;
     uint32_t* owner = owners + warp * 5 * SVC;           // append: (lane, bit) of queued sites
@@ -334,8 +324,6 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     // per-lane state of the tile being appended: its plane words and the PAM bits not yet queued
     uint32_t lo0 = 0, lo1 = 0, lo2 = 0, hi0 = 0, hi1 = 0, hi2 = 0, nm0 = 0, nm1 = 0, nm2 = 0;
     uint32_t pend0 = 0u, pend1 = 0u, pbase = 0;
-    const int w = lane;                                   // this lane's word in the warp tile
-    uint32_t k = 0;
     bool tiles_done = false;
     // One loop, one call site each for the batch comparison and the queue append (the
     // kernel's code stays small): compare while a full batch is queued, else append the
@@ -407,14 +395,13 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         }
         if (tiles_done) break;
         if (__any_sync(0xFFFFFFFFu, (pend0 | pend1) != 0u)) {
-            // ---------------- append pending sites of one strand (all '+' first, then '-'):
-            // (1) each lane writes (lane, bit) of its sites into the warp's owner list (a short
-            // per-lane loop), (2) the warp builds the queue entries cooperatively, 32 per round:
-            // lane i takes owner i and shuffles the owner's strand-shifted words
-            const bool any0 = __any_sync(0xFFFFFFFFu, pend0 != 0u);
-            const uint32_t sdw = any0 ? 0u : 1u;          // warp-uniform strand of this append
-            uint32_t m = any0 ? pend0 : pend1;
-            const uint32_t c = (uint32_t)__popc(m);
+            // ---------------- append the pending sites of both strands:
+            // (1) each lane writes (lane, strand, bit) of its sites into the warp's owner list
+            // (a short count-bounded per-lane loop), (2) the warp builds the queue entries
+            // cooperatively, 32 per round: lane i takes owner i and shuffles the owner's words
+            // shifted to the site's strand offset p0 (one append per chunk of 32 words: for
+            // sparse PAMs such as Cas12a TTTV the per-append cost dominates)
+            const uint32_t c = (uint32_t)(__popc(pend0) + __popc(pend1));
             uint32_t x = c;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -424,59 +411,79 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             const uint32_t total = __shfl_sync(0xFFFFFFFFu, x, 31);
             const uint32_t take = min(SQ - q_n, total);
             const uint32_t first = x - c;
-            // this lane's sites with rank < take: a count-bounded loop (one test per site)
+            // this lane's sites with rank < take ('+' first): one test per site
             const int n_mine = (int)min(c, take > first ? take - first : 0u);
             uint32_t* ow = owner + first;
-            const uint32_t lane5 = (uint32_t)lane << 5;
+            const uint32_t lane6 = (uint32_t)lane << 6;
             for (int i = 0; i < n_mine; i++) {
+                const bool s0 = pend0 != 0u;
+                const uint32_t m = s0 ? pend0 : pend1;
                 const uint32_t low = m & (0u - m);
-                ow[i] = lane5 | (uint32_t)(__ffs(low) - 1);
-                m ^= low;
+                ow[i] = lane6 | (s0 ? 0u : 32u) | (uint32_t)(__ffs(low) - 1);
+                if (s0) pend0 ^= low; else pend1 ^= low;
             }
-            if (any0) pend0 = m; else pend1 = m;
             __syncwarp();
-            const uint32_t p0s = a.p0[sdw];
-            const uint32_t Al = __funnelshift_r(lo0, lo1, p0s), Bl = __funnelshift_r(lo1, lo2, p0s);
-            const uint32_t Ah = __funnelshift_r(hi0, hi1, p0s), Bh = __funnelshift_r(hi1, hi2, p0s);
-            const uint32_t An = __funnelshift_r(nm0, nm1, p0s), Bn = __funnelshift_r(nm1, nm2, p0s);
+            const uint32_t p0f = a.p0[0], p0r = a.p0[1];
+            const uint32_t Alf = __funnelshift_r(lo0, lo1, p0f), Blf = __funnelshift_r(lo1, lo2, p0f);
+            const uint32_t Ahf = __funnelshift_r(hi0, hi1, p0f), Bhf = __funnelshift_r(hi1, hi2, p0f);
+            const uint32_t Anf = __funnelshift_r(nm0, nm1, p0f), Bnf = __funnelshift_r(nm1, nm2, p0f);
+            const uint32_t Alr = __funnelshift_r(lo0, lo1, p0r), Blr = __funnelshift_r(lo1, lo2, p0r);
+            const uint32_t Ahr = __funnelshift_r(hi0, hi1, p0r), Bhr = __funnelshift_r(hi1, hi2, p0r);
+            const uint32_t Anr = __funnelshift_r(nm0, nm1, p0r), Bnr = __funnelshift_r(nm1, nm2, p0r);
             const uint32_t tail = head + q_n;
             for (uint32_t j0 = 0; j0 < take; j0 += 32) {
                 const uint32_t j = j0 + lane;
                 const uint32_t o = j < take ? owner[j] : 0u;
-                const int src = (int)(o >> 5), bit = (int)(o & 31u);
-                const uint32_t al = __shfl_sync(0xFFFFFFFFu, Al, src), bl = __shfl_sync(0xFFFFFFFFu, Bl, src);
-                const uint32_t ah = __shfl_sync(0xFFFFFFFFu, Ah, src), bh = __shfl_sync(0xFFFFFFFFu, Bh, src);
-                const uint32_t an = __shfl_sync(0xFFFFFFFFu, An, src), bn = __shfl_sync(0xFFFFFFFFu, Bn, src);
+                const int src = (int)(o >> 6), bit = (int)(o & 31u);
+                const bool rv = (o & 32u) != 0u;
+                const uint32_t alf = __shfl_sync(0xFFFFFFFFu, Alf, src), blf = __shfl_sync(0xFFFFFFFFu, Blf, src);
+                const uint32_t ahf = __shfl_sync(0xFFFFFFFFu, Ahf, src), bhf = __shfl_sync(0xFFFFFFFFu, Bhf, src);
+                const uint32_t anf = __shfl_sync(0xFFFFFFFFu, Anf, src), bnf = __shfl_sync(0xFFFFFFFFu, Bnf, src);
+                const uint32_t alr = __shfl_sync(0xFFFFFFFFu, Alr, src), blr = __shfl_sync(0xFFFFFFFFu, Blr, src);
+                const uint32_t ahr = __shfl_sync(0xFFFFFFFFu, Ahr, src), bhr = __shfl_sync(0xFFFFFFFFu, Bhr, src);
+                const uint32_t anr = __shfl_sync(0xFFFFFFFFu, Anr, src), bnr = __shfl_sync(0xFFFFFFFFu, Bnr, src);
                 if (j < take)
-                    queue[(tail + j) & (SQ - 1)] =
-                        make_uint4(pbase + 32u * (uint32_t)src + (uint32_t)bit, __funnelshift_r(al, bl, bit),
-                                   __funnelshift_r(ah, bh, bit), (__funnelshift_r(an, bn, bit) & 0x7FFFFFFFu) | (sdw << 31));
+                    queue[(tail + j) & (SQ - 1)] = make_uint4(
+                        pbase + 32u * (uint32_t)src + (uint32_t)bit,
+                        __funnelshift_r(rv ? alr : alf, rv ? blr : blf, bit),
+                        __funnelshift_r(rv ? ahr : ahf, rv ? bhr : bhf, bit),
+                        (__funnelshift_r(rv ? anr : anf, rv ? bnr : bnf, bit) & 0x7FFFFFFFu) | (rv ? 0x80000000u : 0u));
             }
             __syncwarp();
             q_n += take;
             continue;
         }
-        // ---------------- next tile: words -> registers, release the stage, PAM test
-        const int st = (int)(k % SSTAGES);
-#ifdef COF_SINGLE_SPIN
-        mbar_wait_parity(&full[st], (k / SSTAGES) & 1u);
-#else
-        mbar_wait_parity_sleep(&full[st], (k / SSTAGES) & 1u);
-#endif
-        k++;
+        // ---------------- next chunk of 32 plane words (any warp may take any chunk of the
+        // ring's tiles, in order: no fixed word ownership, so a warp that is ahead simply takes
+        // more chunks instead of waiting for the slowest warp to release the stage)
+        uint32_t c = 0;
+        if (lane == 0) c = atomicAdd(s_next, 1u);
+        c = __shfl_sync(0xFFFFFFFFu, c, 0);
+        const uint32_t kk = c / (uint32_t)SW, chunk = c % (uint32_t)SW;
+        const int st = (int)(kk % SSTAGES);
+        mbar_wait_parity_sleep(&full[st], (kk / SSTAGES) & 1u);
         const uint32_t tile = s_tile[st];
         if (tile == S_END) {
             tiles_done = true;
             continue;
         }
-        const uint32_t* S = wring + st * SPL * SLOAD;
+        const uint32_t* S = ring + st * SPL * SLOAD;
+        const int w = (int)chunk * 32 + lane;
         lo0 = S[w]; lo1 = S[w + 1]; lo2 = S[w + 2];
         hi0 = S[SLOAD + w]; hi1 = S[SLOAD + w + 1]; hi2 = S[SLOAD + w + 2];
         nm0 = S[2 * SLOAD + w]; nm1 = S[2 * SLOAD + w + 1]; nm2 = S[2 * SLOAD + w + 2];
         uint32_t valid = vsp ? S[3 * SLOAD + w] : ~0u;
         __syncwarp();
-        if (lane == 0) refill(st);   // the warp has the stage in registers: stream its tile k + SSTAGES
-        const uint64_t pw = ((uint64_t)tile * STW + (uint32_t)lane) * 32u;   // first start of this word
+        if (lane == 0) {   // the chunk is in registers; the last of the tile's SW chunks refills the stage
+            __threadfence_block();
+            if (atomicAdd(&s_rel[st], 1u) == SW - 1) {
+                s_rel[st] = 0;
+                __threadfence_block();
+                refill(st);
+            }
+        }
+        pbase = (uint32_t)(((uint64_t)tile * STW + chunk * 32u) * 32u);   // first start of lane 0's word
+        const uint64_t pw = (uint64_t)pbase + (uint32_t)lane * 32u;        // first start of this word
         if (pw + 32 > a.limit) valid &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
         pend0 = pend1 = valid;
         for (uint32_t e = 0; e < a.ne; e++) {
@@ -490,7 +497,6 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             cnt_f += (unsigned)__popc(pend0);
             cnt_r += (unsigned)__popc(pend1);
         }
-        pbase = (uint32_t)((uint64_t)tile * STW * 32u);   // first start of lane 0's word
     }
     if (a.count_items) {
 #pragma unroll
@@ -574,8 +580,8 @@ static size_t single_smem(const SGeom& g, uint32_t np, uint32_t nb, bool concret
     const size_t fbw = filter_block_words(np);
     // (+ 64 bytes after the '+' filter tables and 64 after the '+' records: bank offsets)
     return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * (concrete ? 16 : 32) + 64 +
-           (size_t)g.sw * g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * 5 * g.svc * 4 +
-           (size_t)((g.sw * g.stages + 1) & ~1) * 4 + (size_t)g.sw * g.stages * 8;
+           (size_t)g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * 5 * g.svc * 4 +
+           (2 * g.stages + 2) * 4 + g.stages * 8;
 }
 
 static constexpr size_t SMEM_MAX = 227 * 1024;
