@@ -108,6 +108,7 @@ struct SingleArgs {
     uint32_t n_blocks;                // guide blocks in this launch
     uint32_t block_base;              // first block of this launch (global guide = (base + b) * 32 + k)
     uint32_t count_items;             // count PAM sites (one launch per search does)
+    uint32_t merge;                   // sparse PAM: append both strands' sites at once
     uint32_t ne;                      // non-N pattern letters per strand
     uint32_t pj[2][32];               // their window offsets
     uint4 psel[2][32];                // their IUPAC sets as splat words {A, C, G, T}
@@ -395,13 +396,17 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         }
         if (tiles_done) break;
         if (__any_sync(0xFFFFFFFFu, (pend0 | pend1) != 0u)) {
-            // ---------------- append the pending sites of both strands:
-            // (1) each lane writes (lane, strand, bit) of its sites into the warp's owner list
-            // (a short count-bounded per-lane loop), (2) the warp builds the queue entries
-            // cooperatively, 32 per round: lane i takes owner i and shuffles the owner's words
-            // shifted to the site's strand offset p0 (one append per chunk of 32 words: for
-            // sparse PAMs such as Cas12a TTTV the per-append cost dominates)
-            const uint32_t c = (uint32_t)(__popc(pend0) + __popc(pend1));
+            // ---------------- append pending sites: (1) each lane writes (lane, strand, bit) of
+            // its sites into the warp's owner list (a short count-bounded per-lane loop), (2) the
+            // warp builds the queue entries cooperatively, 32 per round: lane i takes owner i and
+            // shuffles the owner's words shifted to the site's strand offset p0.  Sparse PAMs
+            // (a.merge: Cas12a TTTV) append both strands at once -- one append per chunk, the
+            // per-append cost dominates there; dense ones one strand at a time ('+' first), which
+            // halves the shuffles per site.
+            const bool merge = a.merge != 0u;
+            const bool any0 = __any_sync(0xFFFFFFFFu, pend0 != 0u);
+            const uint32_t mf = (merge || any0) ? pend0 : 0u, mr = (merge || !any0) ? pend1 : 0u;
+            const uint32_t c = (uint32_t)(__popc(mf) + __popc(mr));
             uint32_t x = c;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -416,38 +421,56 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             uint32_t* ow = owner + first;
             const uint32_t lane6 = (uint32_t)lane << 6;
             for (int i = 0; i < n_mine; i++) {
-                const bool s0 = pend0 != 0u;
+                const bool s0 = (pend0 & mf) != 0u;
                 const uint32_t m = s0 ? pend0 : pend1;
                 const uint32_t low = m & (0u - m);
                 ow[i] = lane6 | (s0 ? 0u : 32u) | (uint32_t)(__ffs(low) - 1);
                 if (s0) pend0 ^= low; else pend1 ^= low;
             }
             __syncwarp();
-            const uint32_t p0f = a.p0[0], p0r = a.p0[1];
+            const uint32_t tail = head + q_n;
+            // strand-shifted words: '+' in the f set, '-' in the r set (one-strand appends use
+            // only the set of their strand)
+            const uint32_t p0f = merge || any0 ? a.p0[0] : a.p0[1], p0r = a.p0[1];
             const uint32_t Alf = __funnelshift_r(lo0, lo1, p0f), Blf = __funnelshift_r(lo1, lo2, p0f);
             const uint32_t Ahf = __funnelshift_r(hi0, hi1, p0f), Bhf = __funnelshift_r(hi1, hi2, p0f);
             const uint32_t Anf = __funnelshift_r(nm0, nm1, p0f), Bnf = __funnelshift_r(nm1, nm2, p0f);
-            const uint32_t Alr = __funnelshift_r(lo0, lo1, p0r), Blr = __funnelshift_r(lo1, lo2, p0r);
-            const uint32_t Ahr = __funnelshift_r(hi0, hi1, p0r), Bhr = __funnelshift_r(hi1, hi2, p0r);
-            const uint32_t Anr = __funnelshift_r(nm0, nm1, p0r), Bnr = __funnelshift_r(nm1, nm2, p0r);
-            const uint32_t tail = head + q_n;
-            for (uint32_t j0 = 0; j0 < take; j0 += 32) {
-                const uint32_t j = j0 + lane;
-                const uint32_t o = j < take ? owner[j] : 0u;
-                const int src = (int)(o >> 6), bit = (int)(o & 31u);
-                const bool rv = (o & 32u) != 0u;
-                const uint32_t alf = __shfl_sync(0xFFFFFFFFu, Alf, src), blf = __shfl_sync(0xFFFFFFFFu, Blf, src);
-                const uint32_t ahf = __shfl_sync(0xFFFFFFFFu, Ahf, src), bhf = __shfl_sync(0xFFFFFFFFu, Bhf, src);
-                const uint32_t anf = __shfl_sync(0xFFFFFFFFu, Anf, src), bnf = __shfl_sync(0xFFFFFFFFu, Bnf, src);
-                const uint32_t alr = __shfl_sync(0xFFFFFFFFu, Alr, src), blr = __shfl_sync(0xFFFFFFFFu, Blr, src);
-                const uint32_t ahr = __shfl_sync(0xFFFFFFFFu, Ahr, src), bhr = __shfl_sync(0xFFFFFFFFu, Bhr, src);
-                const uint32_t anr = __shfl_sync(0xFFFFFFFFu, Anr, src), bnr = __shfl_sync(0xFFFFFFFFu, Bnr, src);
-                if (j < take)
-                    queue[(tail + j) & (SQ - 1)] = make_uint4(
-                        pbase + 32u * (uint32_t)src + (uint32_t)bit,
-                        __funnelshift_r(rv ? alr : alf, rv ? blr : blf, bit),
-                        __funnelshift_r(rv ? ahr : ahf, rv ? bhr : bhf, bit),
-                        (__funnelshift_r(rv ? anr : anf, rv ? bnr : bnf, bit) & 0x7FFFFFFFu) | (rv ? 0x80000000u : 0u));
+            if (merge) {
+                const uint32_t Alr = __funnelshift_r(lo0, lo1, p0r), Blr = __funnelshift_r(lo1, lo2, p0r);
+                const uint32_t Ahr = __funnelshift_r(hi0, hi1, p0r), Bhr = __funnelshift_r(hi1, hi2, p0r);
+                const uint32_t Anr = __funnelshift_r(nm0, nm1, p0r), Bnr = __funnelshift_r(nm1, nm2, p0r);
+                for (uint32_t j0 = 0; j0 < take; j0 += 32) {
+                    const uint32_t j = j0 + lane;
+                    const uint32_t o = j < take ? owner[j] : 0u;
+                    const int src = (int)(o >> 6), bit = (int)(o & 31u);
+                    const bool rv = (o & 32u) != 0u;
+                    const uint32_t alf = __shfl_sync(0xFFFFFFFFu, Alf, src), blf = __shfl_sync(0xFFFFFFFFu, Blf, src);
+                    const uint32_t ahf = __shfl_sync(0xFFFFFFFFu, Ahf, src), bhf = __shfl_sync(0xFFFFFFFFu, Bhf, src);
+                    const uint32_t anf = __shfl_sync(0xFFFFFFFFu, Anf, src), bnf = __shfl_sync(0xFFFFFFFFu, Bnf, src);
+                    const uint32_t alr = __shfl_sync(0xFFFFFFFFu, Alr, src), blr = __shfl_sync(0xFFFFFFFFu, Blr, src);
+                    const uint32_t ahr = __shfl_sync(0xFFFFFFFFu, Ahr, src), bhr = __shfl_sync(0xFFFFFFFFu, Bhr, src);
+                    const uint32_t anr = __shfl_sync(0xFFFFFFFFu, Anr, src), bnr = __shfl_sync(0xFFFFFFFFu, Bnr, src);
+                    if (j < take)
+                        queue[(tail + j) & (SQ - 1)] = make_uint4(
+                            pbase + 32u * (uint32_t)src + (uint32_t)bit,
+                            __funnelshift_r(rv ? alr : alf, rv ? blr : blf, bit),
+                            __funnelshift_r(rv ? ahr : ahf, rv ? bhr : bhf, bit),
+                            (__funnelshift_r(rv ? anr : anf, rv ? bnr : bnf, bit) & 0x7FFFFFFFu) | (rv ? 0x80000000u : 0u));
+                }
+            } else {
+                const uint32_t sbit = any0 ? 0u : 0x80000000u;
+                for (uint32_t j0 = 0; j0 < take; j0 += 32) {
+                    const uint32_t j = j0 + lane;
+                    const uint32_t o = j < take ? owner[j] : 0u;
+                    const int src = (int)(o >> 6), bit = (int)(o & 31u);
+                    const uint32_t al = __shfl_sync(0xFFFFFFFFu, Alf, src), bl = __shfl_sync(0xFFFFFFFFu, Blf, src);
+                    const uint32_t ah = __shfl_sync(0xFFFFFFFFu, Ahf, src), bh = __shfl_sync(0xFFFFFFFFu, Bhf, src);
+                    const uint32_t an = __shfl_sync(0xFFFFFFFFu, Anf, src), bn = __shfl_sync(0xFFFFFFFFu, Bnf, src);
+                    if (j < take)
+                        queue[(tail + j) & (SQ - 1)] =
+                            make_uint4(pbase + 32u * (uint32_t)src + (uint32_t)bit, __funnelshift_r(al, bl, bit),
+                                       __funnelshift_r(ah, bh, bit), (__funnelshift_r(an, bn, bit) & 0x7FFFFFFFu) | sbit);
+                }
             }
             __syncwarp();
             q_n += take;
@@ -690,6 +713,12 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
             A.j1[s][q] = q < pl.n_pairs ? pl.j1[q] - pl.p0 : 0u;
             A.j2[s][q] = q < pl.n_pairs && pl.j2[q] < 0xFE ? pl.j2[q] - pl.p0 : 0xFFu;
         }
+    }
+    {   // expected PAM sites per start and strand on a uniform genome: below 1/32 (about one per
+        // lane's word), one append per chunk for both strands pays (measured: Cas12a TTTV)
+        double d = 1.0;
+        for (uint32_t k = 0; k < plan->pam[0].n; k++) d *= __builtin_popcount(plan->pam[0].set[k]) / 4.0;
+        A.merge = d < 0.03 ? 1u : 0u;
     }
     A.contig = plan->pairs[0].contig && plan->pairs[1].contig && plan->pairs[0].n_cmp == plan->pairs[1].n_cmp;
     A.cmp_mask = plan->pairs[0].n_cmp >= 32 ? ~0u : ((1u << plan->pairs[0].n_cmp) - 1u);
