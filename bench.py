@@ -38,6 +38,7 @@ E2E_CHUNK_BASES = int(os.environ.get("COF_E2E_CHUNK_BASES", 250_000_000))  # e2e
 # e2e: chromosomes cut into pieces of <= this many window starts first (0 = whole chromosomes)
 E2E_PIECE_BASES = int(os.environ.get("COF_E2E_PIECE_BASES", 0))
 SHARD_PIECE_BASES = 16_000_000   # N > 1: chromosome pieces LPT-assigned to ranks
+RESIDENT_CHUNK_BASES = int(os.environ.get("COF_RESIDENT_CHUNK_BASES", 800_000_000))   # e2e_resident chunks
 
 
 def _peaks():
@@ -842,7 +843,12 @@ def measure_resident(wl, st, dev, args, genome_bases):
     caller's pinned buffer inside the timed region; wall clock."""
     import torch
     from paper_conf_socc_jinv23_b200 import search
-    rg = search.ResidentGenome(st.e2e_host, dev)
+    # a few large chunks (the genome is resident: no H2D to overlap, only the records' D2H,
+    # which overlaps the next chunk's kernels; fewer chunks = fewer per-chunk round trips)
+    pieces = [p for ch in st.chunks for p in ch.pieces]
+    host = search.HostGenome(wl.seqs, search.pack_pieces(pieces, RESIDENT_CHUNK_BASES))
+    rg = search.ResidentGenome(host, dev)
+    del host
     srch = search.Searcher(wl.cfg.pattern, wl.guides, wl.thresholds, device=dev)
     srch.reserve(max(ch.n_bases for ch in rg.chunks), max(st.caps))
     h0 = srch.search_resident(rg)
