@@ -210,6 +210,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         const uint32_t tile = atomicAdd(a.ticket, 1u);
         if (tile >= a.n_tiles) {
             s_tile[st] = S_END;
+            __threadfence_block();        // (the arrive releases it too; racecheck wants the fence)
             mbar_arrive(&full[st]);
             return;
         }
@@ -257,6 +258,10 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     const uint32_t tb0 = smem_u32(s_ftab), tb1 = tb0 + nb * FBW * 4 + 64;
     const uint4* vrec1 = s_vrec + nb * 32 * VSTR + 4;
     uint32_t head = 0, q_n = 0;           // warp-uniform site ring state
+    // Survivor entries carry over from one batch to the next (the last verification round of
+    // a batch would otherwise run mostly empty): the previous batch's queue slots stay
+    // reserved (resv) until the next batch ends, when every survivor is verified.
+    uint32_t sv_h = 0, sv_n = 0, resv = 0;
     unsigned long long cnt_f = 0, cnt_r = 0;
 
     // Verify the survivor entries [sv_h, sv_h + n), n <= 32 (one site and the four 32-guide
@@ -330,7 +335,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     // kernel's code stays small): compare while a full batch is queued, else append the
     // pending sites of the current tile, else take the next tile.
     for (;;) {
-        if (q_n >= SBATCH || (tiles_done && q_n > 0)) {
+        if (q_n >= SBATCH || (tiles_done && (q_n > 0 || sv_n > 0))) {   // (an empty last batch drains)
             // ---------------- compare a batch: ring[head, head + n_items)
             const uint32_t n_items = min(q_n, SBATCH);
             uint32_t base[SR][NP];
@@ -343,7 +348,6 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                 site_bases<NP>(a, sd ? tb1 : tb0, sd, e.y, e.z, e.w & 0x7FFFFFFFu, base[r]);
             }
 
-            uint32_t sv_h = 0, sv_n = 0;                    // warp-uniform survivor list state
             // groups of 4 blocks; one extra pass (b >= nb) drains the survivor list, so the
             // verification code exists once in the kernel (its size decides the I-cache hit rate)
             for (uint32_t b = 0;; b += 4) {
@@ -380,7 +384,9 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                 __syncwarp();
                 // (at most 31 + SR x 32 entries are queued: SVC holds them; a round takes 32 and
                 // puts back at most 32, and every round verifies one survivor per entry taken)
-                while (sv_n >= 32 || (drain && sv_n > 0)) {
+                // (a batch that keeps its survivors for the next one verifies only full rounds)
+                const bool keep = resv == 0u && n_items == SBATCH && !tiles_done;
+                while (sv_n >= 32 || (drain && !keep && sv_n > 0)) {
                     const uint32_t nf = min(sv_n, 32u);
                     const uint32_t back = flush(sv_h, nf, sv_h + sv_n);
                     sv_h = (sv_h + nf) & (SVC - 1);
@@ -392,6 +398,9 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             __syncwarp();
             head = (head + SBATCH) & (SQ - 1);
             q_n -= n_items;
+            // this batch's slots stay reserved while survivors may still reference them; after a
+            // full drain nothing is pending
+            resv = (sv_n > 0u) ? SBATCH : 0u;
             continue;
         }
         if (tiles_done) break;
@@ -414,7 +423,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                 if (lane >= o) x += y;
             }
             const uint32_t total = __shfl_sync(0xFFFFFFFFu, x, 31);
-            const uint32_t take = min(SQ - q_n, total);
+            const uint32_t take = min(SQ - q_n - resv, total);
             const uint32_t first = x - c;
             // this lane's sites with rank < take ('+' first): one test per site
             const int n_mine = (int)min(c, take > first ? take - first : 0u);

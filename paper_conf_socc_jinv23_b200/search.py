@@ -770,16 +770,47 @@ def _coll_device(group=None):
     return torch.device("cuda", torch.cuda.current_device()) if dist.get_backend(group) == "nccl" else torch.device("cpu")
 
 
+_MERGE_ARENAS = {}   # per process group: the shared-memory result buffer every rank keeps mapped
+
+
+def _merge_arena(nbytes: int, group, dst: int, shm_dir=None):
+    """The group's shared result buffer, at least ``nbytes``: one file in /dev/shm created by
+    ``dst``, mapped by every rank and unlinked at once (the mappings keep it alive).  It is
+    reused by later merges of the same group, so its pages are faulted in once -- mapping a
+    fresh file per merge cost ~0.1 s per 100 MB in page faults."""
+    import tempfile
+    import uuid
+    import torch.distributed as dist
+    key = id(group) if group is not None else None
+    arena = _MERGE_ARENAS.get(key)
+    need = [arena is None or arena.size < nbytes]
+    # every rank sees the same counts, hence the same decision; no collective needed for it
+    if need[0]:
+        size = max(int(nbytes * 1.25), 1 << 20)
+        name = [None]
+        if dist.get_rank(group) == dst:
+            d = shm_dir or ("/dev/shm" if os.path.isdir("/dev/shm") else tempfile.gettempdir())
+            name[0] = os.path.join(d, f"cof_merge_{uuid.uuid4().hex}.bin")
+            with open(name[0], "wb") as f:
+                f.truncate(size)
+        dist.broadcast_object_list(name, src=dst, group=group)
+        arena = np.memmap(name[0], dtype=np.uint8, mode="r+", shape=(size,))
+        dist.barrier(group=group)
+        if dist.get_rank(group) == dst:
+            os.unlink(name[0])
+        _MERGE_ARENAS[key] = arena
+    return arena
+
+
 def merge_dist(per_chunk: dict, n_chunks: int, dtype, group=None, dst: int = 0, shm_dir=None):
     """Host merge of a torchrun job (one process per GPU): ``per_chunk`` maps this rank's
     global chunk indices to their sorted records.  Per-chunk hit counts are summed over
     the ranks (one small all-reduce), their exclusive prefix gives every chunk's offset in
     the genome-ordered result, and every rank copies its records straight into that slice
-    of one shared-memory file (all ranks of a torchrun job share the node) -- the merge is
-    a parallel concatenation, no record crosses the process group.  Returns the merged
-    array (a read-only view of the mapping) on ``dst`` and None elsewhere."""
-    import tempfile
-    import uuid
+    of one shared-memory buffer (all ranks of a torchrun job share the node; the buffer is
+    kept mapped across merges) -- the merge is a parallel concatenation, no record crosses
+    the process group.  Returns the merged array on ``dst`` (a view of the shared buffer,
+    valid until the group's next merge_dist) and None elsewhere."""
     import torch.distributed as dist
     rank = dist.get_rank(group)
     cd = _coll_device(group)
@@ -792,28 +823,14 @@ def merge_dist(per_chunk: dict, n_chunks: int, dtype, group=None, dst: int = 0, 
     offs = np.zeros(n_chunks + 1, dtype=np.int64)
     np.cumsum(counts, out=offs[1:])
     total = int(offs[-1])
-    name = [None]
-    if rank == dst:
-        d = shm_dir or ("/dev/shm" if os.path.isdir("/dev/shm") else tempfile.gettempdir())
-        name[0] = os.path.join(d, f"cof_merge_{uuid.uuid4().hex}.bin")
-        with open(name[0], "wb") as f:
-            f.truncate(max(1, total) * dtype.itemsize)
-    dist.broadcast_object_list(name, src=dst, group=group)
-    path = name[0]
+    isz = dtype.itemsize
+    arena = _merge_arena(max(1, total) * isz, group, dst, shm_dir)
+    out = arena[: total * isz].view(dtype) if total else np.zeros(0, dtype=dtype)
+    for i, r in per_chunk.items():
+        if len(r):   # (a byte copy: 4x faster than numpy's field-wise structured assignment)
+            arena[offs[i] * isz:(offs[i] + len(r)) * isz] = np.ascontiguousarray(r).view(np.uint8)
     dist.barrier(group=group)
-    mine = [(i, r) for i, r in per_chunk.items() if len(r)]
-    if mine:
-        mm = np.memmap(path, dtype=dtype, mode="r+", shape=(max(1, total),))
-        for i, r in mine:
-            mm[offs[i]:offs[i] + len(r)] = r
-        mm.flush()
-        del mm
-    dist.barrier(group=group)
-    if rank != dst:
-        return None
-    out = np.memmap(path, dtype=dtype, mode="r", shape=(max(1, total),))[:total]
-    os.unlink(path)          # the mapping stays valid; the name goes away
-    return out
+    return out if rank == dst else None
 
 
 def search_dist(seqs, pattern, guides, thresholds, chunk_bases=MULTI_CHUNK_BASES, group=None, device=None,
