@@ -62,7 +62,8 @@ struct SCfg {
     static constexpr uint32_t SBATCH = 32u * R;
     static constexpr uint32_t SVC = R == 1 ? 64u : 128u;   // survivor entries per warp (ring)
     static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH, "ring");
-    static_assert(5 * SVC >= SQ, "the owner list shares the survivor ring's space");
+    static constexpr uint32_t SPW = 5u * SVC + SQ;   // per-warp words: survivor ring (5 x SVC) + owner list (SQ)
+    static_assert(SPW % 4 == 0, "16-byte survivor masks");
     static_assert(SVC >= 31 + 32 * SR, "a group of blocks appends at most 32 entries per site row");
 };
 // (warps, sites per lane, ring stages); -DCOF_FEW_W=... etc. override for A/B builds
@@ -188,7 +189,8 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
     //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
     //         [ring: SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
-    //         [per warp: append owner list (SQ words) / survivor ring (SVC x 5 words)]
+    //         [per warp: survivor ring (SVC x 5 words), append owner list (SQ words)]
+    //         (separate: survivor entries outlive a batch, so an append must not overwrite them)
     //         [tile ids, release counters][full mbarriers]
     constexpr uint32_t FBW = (NP * 25u + 15u) & ~15u;
     constexpr uint32_t VSTR = CONCRETE ? 1u : 2u;     // uint4 per verification record in shared memory
@@ -197,8 +199,8 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     uint4* s_vrec = reinterpret_cast<uint4*>(smem + 2 * nb * FBW * 4 + 64);
     uint32_t* ring = reinterpret_cast<uint32_t*>(reinterpret_cast<uint8_t*>(s_vrec) + 2 * nb * 32 * VSTR * 16 + 64);
     uint4* queues = reinterpret_cast<uint4*>(ring + SSTAGES * SPL * SLOAD);
-    uint32_t* owners = reinterpret_cast<uint32_t*>(queues + SW * SQ);   // per warp: 5 x SVC words
-    uint32_t* s_tile = owners + SW * 5 * SVC;
+    uint32_t* owners = reinterpret_cast<uint32_t*>(queues + SW * SQ);   // per warp: SPW words
+    uint32_t* s_tile = owners + SW * CFG::SPW;
     uint32_t* s_rel = s_tile + SSTAGES;
     uint32_t* s_next = s_rel + SSTAGES;                              // next chunk to take (ring order)
     uint64_t* full = reinterpret_cast<uint64_t*>(s_tile + 2 * SSTAGES + 2);
@@ -252,9 +254,9 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     __syncthreads();
 
     uint4* queue = queues + warp * SQ;
-    uint32_t* owner = owners + warp * 5 * SVC;           // append: (lane, bit) of queued sites
-    uint32_t* sv_x = owner;                              // batch: survivor entries: slot | group << 8
-    uint4* sv_m = reinterpret_cast<uint4*>(owner + SVC); //        and the group's 4 survivor masks (16 B)
+    uint32_t* sv_x = owners + warp * CFG::SPW;           // survivor entries: slot | group << 8
+    uint4* sv_m = reinterpret_cast<uint4*>(sv_x + SVC);  // and the group's 4 survivor masks (16 B)
+    uint32_t* owner = sv_x + 5 * SVC;                    // append: (lane, bit) of queued sites
     const uint32_t tb0 = smem_u32(s_ftab), tb1 = tb0 + nb * FBW * 4 + 64;
     const uint4* vrec1 = s_vrec + nb * 32 * VSTR + 4;
     uint32_t head = 0, q_n = 0;           // warp-uniform site ring state
@@ -612,7 +614,7 @@ static size_t single_smem(const SGeom& g, uint32_t np, uint32_t nb, bool concret
     const size_t fbw = filter_block_words(np);
     // (+ 64 bytes after the '+' filter tables and 64 after the '+' records: bank offsets)
     return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * (concrete ? 16 : 32) + 64 +
-           (size_t)g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * 5 * g.svc * 4 +
+           (size_t)g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * (5 * g.svc + g.sq) * 4 +
            (2 * g.stages + 2) * 4 + g.stages * 8;
 }
 
