@@ -50,7 +50,7 @@ namespace cof {
 // addresses) is amortised over more lookups -- and 20 warps; many blocks (C5) take one
 // site per lane and 28 warps, which hides the filter's dependency latency better and keeps
 // all 32 blocks of a 1000-guide plan in one launch's shared memory.
-template <int W, int R, int S>
+template <int W, int R, int S, int QB>
 struct SCfg {
     static constexpr int SW = W;                  // warps per CTA (one CTA per SM)
     static constexpr int STHREADS = 32 * W;
@@ -58,15 +58,15 @@ struct SCfg {
     static constexpr int SLOAD = STW + 4;         // words per plane and stage: tile + halo (16-byte multiple)
     static constexpr int SSTAGES = S;             // TMA ring depth
     static constexpr int SR = R;                  // sites per lane and batch
-    static constexpr uint32_t SQ = 64u * R;       // queued sites per warp (16-byte entries): two batches
+    static constexpr uint32_t SQ = 32u * R * QB;  // queued sites per warp (16-byte entries): QB batches
     static constexpr uint32_t SBATCH = 32u * R;
     static constexpr uint32_t SVC = R == 1 ? 64u : 128u;   // survivor entries per warp (ring)
-    static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH, "ring");
-    static constexpr uint32_t SPW = 5u * SVC + SQ;   // per-warp words: survivor ring (5 x SVC) + owner list (SQ)
+    static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH && (SQ & (SQ - 1)) == 0, "ring");
+    static constexpr uint32_t SPW = 5u * SVC;     // per-warp words of the survivor ring
     static_assert(SPW % 4 == 0, "16-byte survivor masks");
     static_assert(SVC >= 31 + 32 * SR, "a group of blocks appends at most 32 entries per site row");
 };
-// (warps, sites per lane, ring stages); -DCOF_FEW_W=... etc. override for A/B builds
+// (warps, sites per lane, ring stages, queue batches); -DCOF_FEW_W=... etc. override for A/B builds
 #ifndef COF_FEW_W
 #define COF_FEW_W 24
 #endif
@@ -75,6 +75,12 @@ struct SCfg {
 #endif
 #ifndef COF_FEW_S
 #define COF_FEW_S 4
+#endif
+#ifndef COF_FEW_Q
+#define COF_FEW_Q 4
+#endif
+#ifndef COF_MANY_Q
+#define COF_MANY_Q 2
 #endif
 #ifndef COF_MANY_W
 #define COF_MANY_W 28
@@ -85,8 +91,8 @@ struct SCfg {
 #ifndef COF_MANY_S
 #define COF_MANY_S 4
 #endif
-using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S>;
-using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S>;
+using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q>;
+using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S, COF_MANY_Q>;
 constexpr uint32_t SFEW_BLOCKS = 8;       // guide blocks up to which SCfgFew runs
 constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
@@ -109,7 +115,6 @@ struct SingleArgs {
     uint32_t n_blocks;                // guide blocks in this launch
     uint32_t block_base;              // first block of this launch (global guide = (base + b) * 32 + k)
     uint32_t count_items;             // count PAM sites (one launch per search does)
-    uint32_t merge;                   // sparse PAM: append both strands' sites at once
     uint32_t ne;                      // non-N pattern letters per strand
     uint32_t pj[2][32];               // their window offsets
     uint4 psel[2][32];                // their IUPAC sets as splat words {A, C, G, T}
@@ -189,8 +194,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
     //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
     //         [ring: SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
-    //         [per warp: survivor ring (SVC x 5 words), append owner list (SQ words)]
-    //         (separate: survivor entries outlive a batch, so an append must not overwrite them)
+    //         [per warp: survivor ring (SVC x 5 words)]
     //         [tile ids, release counters][full mbarriers]
     constexpr uint32_t FBW = (NP * 25u + 15u) & ~15u;
     constexpr uint32_t VSTR = CONCRETE ? 1u : 2u;     // uint4 per verification record in shared memory
@@ -199,8 +203,8 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     uint4* s_vrec = reinterpret_cast<uint4*>(smem + 2 * nb * FBW * 4 + 64);
     uint32_t* ring = reinterpret_cast<uint32_t*>(reinterpret_cast<uint8_t*>(s_vrec) + 2 * nb * 32 * VSTR * 16 + 64);
     uint4* queues = reinterpret_cast<uint4*>(ring + SSTAGES * SPL * SLOAD);
-    uint32_t* owners = reinterpret_cast<uint32_t*>(queues + SW * SQ);   // per warp: SPW words
-    uint32_t* s_tile = owners + SW * CFG::SPW;
+    uint32_t* survs = reinterpret_cast<uint32_t*>(queues + SW * SQ);    // per warp: SPW words
+    uint32_t* s_tile = survs + SW * CFG::SPW;
     uint32_t* s_rel = s_tile + SSTAGES;
     uint32_t* s_next = s_rel + SSTAGES;                              // next chunk to take (ring order)
     uint64_t* full = reinterpret_cast<uint64_t*>(s_tile + 2 * SSTAGES + 2);
@@ -254,9 +258,8 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     __syncthreads();
 
     uint4* queue = queues + warp * SQ;
-    uint32_t* sv_x = owners + warp * CFG::SPW;           // survivor entries: slot | group << 8
+    uint32_t* sv_x = survs + warp * CFG::SPW;            // survivor entries: slot | group << 8
     uint4* sv_m = reinterpret_cast<uint4*>(sv_x + SVC);  // and the group's 4 survivor masks (16 B)
-    uint32_t* owner = sv_x + 5 * SVC;                    // append: (lane, bit) of queued sites
     const uint32_t tb0 = smem_u32(s_ftab), tb1 = tb0 + nb * FBW * 4 + 64;
     const uint4* vrec1 = s_vrec + nb * 32 * VSTR + 4;
     uint32_t head = 0, q_n = 0;           // warp-uniform site ring state
@@ -368,11 +371,10 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                         p2 = filter_pass<NP, TC>(v, m + 16);
                         lds_filter<NP, 3 * FBW * 4>(base[r], boff, v);
                         p3 = filter_pass<NP, TC>(v, m + 24);
-                        const uint32_t ok = (uint32_t)r * 32u + lane < n_items ? ~0u : 0u;
-                        p0 &= ok; p1 &= ok; p2 &= ok; p3 &= ok;
                         // a site with a survivor in this group of 4 blocks -> one survivor
-                        // entry (ballot append; blocks past the plan have valid 0)
-                        const bool has = (p0 | p1 | p2 | p3) != 0u;
+                        // entry (ballot append; blocks past the plan have valid 0; a missing
+                        // site of a partial batch appends nothing)
+                        const bool has = (p0 | p1 | p2 | p3) != 0u && (uint32_t)r * 32u + lane < n_items;
                         const unsigned hb = __ballot_sync(0xFFFFFFFFu, has);
                         const uint32_t e = (sv_h + sv_n + (uint32_t)__popc(hb & lanemask_lt())) & (SVC - 1);
                         if (has) {
@@ -407,17 +409,13 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         }
         if (tiles_done) break;
         if (__any_sync(0xFFFFFFFFu, (pend0 | pend1) != 0u)) {
-            // ---------------- append pending sites: (1) each lane writes (lane, strand, bit) of
-            // its sites into the warp's owner list (a short count-bounded per-lane loop), (2) the
-            // warp builds the queue entries cooperatively, 32 per round: lane i takes owner i and
-            // shuffles the owner's words shifted to the site's strand offset p0.  Sparse PAMs
-            // (a.merge: Cas12a TTTV) append both strands at once -- one append per chunk, the
-            // per-append cost dominates there; dense ones one strand at a time ('+' first), which
-            // halves the shuffles per site.
-            const bool merge = a.merge != 0u;
-            const bool any0 = __any_sync(0xFFFFFFFFu, pend0 != 0u);
-            const uint32_t mf = (merge || any0) ? pend0 : 0u, mr = (merge || !any0) ? pend1 : 0u;
-            const uint32_t c = (uint32_t)(__popc(mf) + __popc(mr));
+            // ---------------- append pending sites: a warp scan ranks the lanes' sites ('+' before
+            // '-' within a lane), and every lane writes the queue entries of its own sites that fit
+            // (rank < take), each the site's three 32-base windows funnel-shifted out of the
+            // lane's registers at the strand's first compared offset p0 (bit 31 of the N window
+            // carries the strand).  The order of entries in the queue is immaterial (hits are
+            // sorted afterwards); a site that does not fit stays pending for the next append.
+            const uint32_t c0 = (uint32_t)__popc(pend0), c = c0 + (uint32_t)__popc(pend1);
             uint32_t x = c;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -427,61 +425,44 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             const uint32_t total = __shfl_sync(0xFFFFFFFFu, x, 31);
             const uint32_t take = min(SQ - q_n - resv, total);
             const uint32_t first = x - c;
-            // this lane's sites with rank < take ('+' first): one test per site
-            const int n_mine = (int)min(c, take > first ? take - first : 0u);
-            uint32_t* ow = owner + first;
-            const uint32_t lane6 = (uint32_t)lane << 6;
-            for (int i = 0; i < n_mine; i++) {
-                const bool s0 = (pend0 & mf) != 0u;
-                const uint32_t m = s0 ? pend0 : pend1;
-                const uint32_t low = m & (0u - m);
-                ow[i] = lane6 | (s0 ? 0u : 32u) | (uint32_t)(__ffs(low) - 1);
-                if (s0) pend0 ^= low; else pend1 ^= low;
+            const uint32_t n_mine = min(c, take > first ? take - first : 0u);
+            const uint32_t pw = pbase + (uint32_t)lane * 32u;     // first start of this lane's word
+            uint32_t slot = head + q_n + first;
+            const uint32_t nf = min(n_mine, c0);
+            if (nf) {
+                const uint32_t p0 = a.p0[0];
+                const uint32_t Al = __funnelshift_r(lo0, lo1, p0), Bl = __funnelshift_r(lo1, lo2, p0);
+                const uint32_t Ah = __funnelshift_r(hi0, hi1, p0), Bh = __funnelshift_r(hi1, hi2, p0);
+                const uint32_t An = __funnelshift_r(nm0, nm1, p0), Bn = __funnelshift_r(nm1, nm2, p0);
+                uint32_t m = pend0;
+                for (uint32_t i = 0; i < nf; i++) {
+                    const uint32_t low = m & (0u - m);
+                    const uint32_t bit = 31u - (uint32_t)__clz(low);
+                    m ^= low;
+                    queue[slot & (SQ - 1)] = make_uint4(pw + bit, __funnelshift_r(Al, Bl, bit),
+                                                        __funnelshift_r(Ah, Bh, bit),
+                                                        __funnelshift_r(An, Bn, bit) & 0x7FFFFFFFu);
+                    slot++;
+                }
+                pend0 = m;
             }
-            __syncwarp();
-            const uint32_t tail = head + q_n;
-            // strand-shifted words: '+' in the f set, '-' in the r set (one-strand appends use
-            // only the set of their strand)
-            const uint32_t p0f = merge || any0 ? a.p0[0] : a.p0[1], p0r = a.p0[1];
-            const uint32_t Alf = __funnelshift_r(lo0, lo1, p0f), Blf = __funnelshift_r(lo1, lo2, p0f);
-            const uint32_t Ahf = __funnelshift_r(hi0, hi1, p0f), Bhf = __funnelshift_r(hi1, hi2, p0f);
-            const uint32_t Anf = __funnelshift_r(nm0, nm1, p0f), Bnf = __funnelshift_r(nm1, nm2, p0f);
-            if (merge) {
-                const uint32_t Alr = __funnelshift_r(lo0, lo1, p0r), Blr = __funnelshift_r(lo1, lo2, p0r);
-                const uint32_t Ahr = __funnelshift_r(hi0, hi1, p0r), Bhr = __funnelshift_r(hi1, hi2, p0r);
-                const uint32_t Anr = __funnelshift_r(nm0, nm1, p0r), Bnr = __funnelshift_r(nm1, nm2, p0r);
-                for (uint32_t j0 = 0; j0 < take; j0 += 32) {
-                    const uint32_t j = j0 + lane;
-                    const uint32_t o = j < take ? owner[j] : 0u;
-                    const int src = (int)(o >> 6), bit = (int)(o & 31u);
-                    const bool rv = (o & 32u) != 0u;
-                    const uint32_t alf = __shfl_sync(0xFFFFFFFFu, Alf, src), blf = __shfl_sync(0xFFFFFFFFu, Blf, src);
-                    const uint32_t ahf = __shfl_sync(0xFFFFFFFFu, Ahf, src), bhf = __shfl_sync(0xFFFFFFFFu, Bhf, src);
-                    const uint32_t anf = __shfl_sync(0xFFFFFFFFu, Anf, src), bnf = __shfl_sync(0xFFFFFFFFu, Bnf, src);
-                    const uint32_t alr = __shfl_sync(0xFFFFFFFFu, Alr, src), blr = __shfl_sync(0xFFFFFFFFu, Blr, src);
-                    const uint32_t ahr = __shfl_sync(0xFFFFFFFFu, Ahr, src), bhr = __shfl_sync(0xFFFFFFFFu, Bhr, src);
-                    const uint32_t anr = __shfl_sync(0xFFFFFFFFu, Anr, src), bnr = __shfl_sync(0xFFFFFFFFu, Bnr, src);
-                    if (j < take)
-                        queue[(tail + j) & (SQ - 1)] = make_uint4(
-                            pbase + 32u * (uint32_t)src + (uint32_t)bit,
-                            __funnelshift_r(rv ? alr : alf, rv ? blr : blf, bit),
-                            __funnelshift_r(rv ? ahr : ahf, rv ? bhr : bhf, bit),
-                            (__funnelshift_r(rv ? anr : anf, rv ? bnr : bnf, bit) & 0x7FFFFFFFu) | (rv ? 0x80000000u : 0u));
+            const uint32_t nr = n_mine - nf;
+            if (nr) {
+                const uint32_t p0 = a.p0[1];
+                const uint32_t Al = __funnelshift_r(lo0, lo1, p0), Bl = __funnelshift_r(lo1, lo2, p0);
+                const uint32_t Ah = __funnelshift_r(hi0, hi1, p0), Bh = __funnelshift_r(hi1, hi2, p0);
+                const uint32_t An = __funnelshift_r(nm0, nm1, p0), Bn = __funnelshift_r(nm1, nm2, p0);
+                uint32_t m = pend1;
+                for (uint32_t i = 0; i < nr; i++) {
+                    const uint32_t low = m & (0u - m);
+                    const uint32_t bit = 31u - (uint32_t)__clz(low);
+                    m ^= low;
+                    queue[slot & (SQ - 1)] = make_uint4(pw + bit, __funnelshift_r(Al, Bl, bit),
+                                                        __funnelshift_r(Ah, Bh, bit),
+                                                        __funnelshift_r(An, Bn, bit) | 0x80000000u);
+                    slot++;
                 }
-            } else {
-                const uint32_t sbit = any0 ? 0u : 0x80000000u;
-                for (uint32_t j0 = 0; j0 < take; j0 += 32) {
-                    const uint32_t j = j0 + lane;
-                    const uint32_t o = j < take ? owner[j] : 0u;
-                    const int src = (int)(o >> 6), bit = (int)(o & 31u);
-                    const uint32_t al = __shfl_sync(0xFFFFFFFFu, Alf, src), bl = __shfl_sync(0xFFFFFFFFu, Blf, src);
-                    const uint32_t ah = __shfl_sync(0xFFFFFFFFu, Ahf, src), bh = __shfl_sync(0xFFFFFFFFu, Bhf, src);
-                    const uint32_t an = __shfl_sync(0xFFFFFFFFu, Anf, src), bn = __shfl_sync(0xFFFFFFFFu, Bnf, src);
-                    if (j < take)
-                        queue[(tail + j) & (SQ - 1)] =
-                            make_uint4(pbase + 32u * (uint32_t)src + (uint32_t)bit, __funnelshift_r(al, bl, bit),
-                                       __funnelshift_r(ah, bh, bit), (__funnelshift_r(an, bn, bit) & 0x7FFFFFFFu) | sbit);
-                }
+                pend1 = m;
             }
             __syncwarp();
             q_n += take;
@@ -614,7 +595,7 @@ static size_t single_smem(const SGeom& g, uint32_t np, uint32_t nb, bool concret
     const size_t fbw = filter_block_words(np);
     // (+ 64 bytes after the '+' filter tables and 64 after the '+' records: bank offsets)
     return 2 * nb * fbw * 4 + 64 + 2 * (size_t)nb * 32 * (concrete ? 16 : 32) + 64 +
-           (size_t)g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * (5 * g.svc + g.sq) * 4 +
+           (size_t)g.stages * SPL * g.sload * 4 + (size_t)g.sw * g.sq * 16 + (size_t)g.sw * 5 * g.svc * 4 +
            (2 * g.stages + 2) * 4 + g.stages * 8;
 }
 
@@ -674,7 +655,9 @@ static SinglePlanInfo single_info(const cof_plan* plan) {
     for (uint32_t i = 1; i < plan->n_guides && I.ut >= 0; i++)
         if (plan->max_mm[i] != plan->max_mm[0]) I.ut = -1;
     I.concrete = single_uses_concrete(I.np, I.ut, !plan->any_degenerate);
-    I.few = plan->n_blocks <= SFEW_BLOCKS;
+    // the few-blocks geometry when the plan's blocks fit one launch of it
+    I.few = plan->n_blocks <= SFEW_BLOCKS &&
+            single_smem(single_geom(true), I.np, (plan->n_blocks + 3) & ~3u, I.concrete) <= SMEM_MAX;
     I.geom = single_geom(I.few);
     I.bpl = single_blocks_per_launch(I.geom, I.np, I.concrete);
     return I;
@@ -724,12 +707,6 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
             A.j1[s][q] = q < pl.n_pairs ? pl.j1[q] - pl.p0 : 0u;
             A.j2[s][q] = q < pl.n_pairs && pl.j2[q] < 0xFE ? pl.j2[q] - pl.p0 : 0xFFu;
         }
-    }
-    {   // expected PAM sites per start and strand on a uniform genome: below 1/32 (about one per
-        // lane's word), one append per chunk for both strands pays (measured: Cas12a TTTV)
-        double d = 1.0;
-        for (uint32_t k = 0; k < plan->pam[0].n; k++) d *= __builtin_popcount(plan->pam[0].set[k]) / 4.0;
-        A.merge = d < 0.03 ? 1u : 0u;
     }
     A.contig = plan->pairs[0].contig && plan->pairs[1].contig && plan->pairs[0].n_cmp == plan->pairs[1].n_cmp;
     A.cmp_mask = plan->pairs[0].n_cmp >= 32 ? ~0u : ((1u << plan->pairs[0].n_cmp) - 1u);
