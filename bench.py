@@ -430,7 +430,7 @@ def main():
     ap.add_argument("--config", default="C5")
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--comparer", default="table", choices=["table", "popc", "mma"])
+    ap.add_argument("--comparer", default="table", choices=["table", "popc"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
@@ -546,32 +546,18 @@ def main():
     roof = comparer_roof(st.plan, n_sm, sm_max, args.comparer, st.path_name)
     cmp_rate = comps_mine * args.steps / (cmp_ms * 1e-3) if cmp_ms > 0 else 0.0
     n_cmp_launch = len(events)
-    if args.comparer == "mma":
-        # int8 tensor-core GEMM: algorithmic ops = 2 x items x guides x K (K = the encoded
-        # contraction length of the plan); peak = measured dense bf16 x 2 (nominal int8:bf16)
-        kpad = cof.cof_plan_mma_kpad(st.plan)
-        ops = 2.0 * comps_mine * kpad * args.steps
-        achieved = ops / (cmp_ms * 1e-3) / 1e12 if cmp_ms > 0 else 0.0
-        pk = 2.0 * float(peaks.get("bf16_tflops", 2250.0 / 2))
-        roofline = {"bound": "tensor", "kernel": "cof_comparer_mma", "achieved": achieved, "peak": pk,
-                    "unit": "TFLOP/s", "frac": achieved / pk, "traffic": traffic_for("cof_comparer_mma", st, cfgname),
-                    "peak_basis": f"int8 dense = 2 x measured bf16 dense ({peaks.get('bf16_tflops')} TFLOP/s); "
-                                  f"ops = 2 x items x guides x K={kpad} (int8 OPs)",
-                    "comparisons_per_s": cmp_rate, "alu_table_roof_comparisons_per_s": roof["peak"],
-                    "launches": n_cmp_launch, "share_of_step": cmp_ms_max / ms_total if ms_total else None}
-    else:
-        kname = {"single": "cof_single_kernel", "fused": "cof_comparer_fused"}.get(st.path_name,
-                                                                                  f"cof_comparer_{args.comparer}")
-        roofline = {"bound": "alu", "kernel": kname,
-                    "achieved": cmp_rate, "peak": roof["peak"], "unit": "comparisons/s",
-                    "frac": cmp_rate / roof["peak"] if roof["peak"] else None,
-                    "traffic": traffic_for("cof_single_kernel" if st.path_name == "single" else "cof_comparer",
-                                           st, cfgname),
-                    "peak_basis": roof["basis"], "launches": n_cmp_launch,
-                    "share_of_step": cmp_ms_max / ms_total if ms_total else None,
-                    # the same rate against SURVEY §8(d)'s roof (one POPC per comparison)
-                    "frac_popc_roof": cmp_rate / popc_roof(n_sm, sm_max),
-                    "popc_roof": popc_roof(n_sm, sm_max)}
+    kname = {"single": "cof_single_kernel", "fused": "cof_comparer_fused"}.get(st.path_name,
+                                                                              f"cof_comparer_{args.comparer}")
+    roofline = {"bound": "alu", "kernel": kname,
+                "achieved": cmp_rate, "peak": roof["peak"], "unit": "comparisons/s",
+                "frac": cmp_rate / roof["peak"] if roof["peak"] else None,
+                "traffic": traffic_for("cof_single_kernel" if st.path_name == "single" else "cof_comparer",
+                                       st, cfgname),
+                "peak_basis": roof["basis"], "launches": n_cmp_launch,
+                "share_of_step": cmp_ms_max / ms_total if ms_total else None,
+                # the same rate against SURVEY §8(d)'s roof (one POPC per comparison)
+                "frac_popc_roof": cmp_rate / popc_roof(n_sm, sm_max),
+                "popc_roof": popc_roof(n_sm, sm_max)}
 
     # finder roofline (HBM): algorithmic bytes of the search kernel per step
     plane_bytes = sum(cof.cof_plane_words(ch.n_bases) * 4 * (4 if ch.multi else 3) for ch in st.chunks)
@@ -734,7 +720,6 @@ def table_roof(plan, n_sm, sm_mhz, impl):
     clk = sm_mhz * 1e6
     if impl == "popc":
         return {"peak": popc_roof(n_sm, sm_mhz), "basis": "POPC pipe 16/clk/SM x SMs x max SM clock"}
-    # (mma: the table comparer's ALU roof is reported beside the tensor roofline)
     import importlib.util
     spec = importlib.util.spec_from_file_location(
         "gen_csa", os.path.join(ROOT, "paper_conf_socc_jinv23_b200", "csrc", "gen_csa.py"))

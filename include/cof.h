@@ -69,8 +69,8 @@ uint64_t cof_launch_count(void);
  *  out       receives a host-only, immutable plan (thread-safe to share read-only).
  * Errors: COF_E_ARG for a non-IUPAC letter (G18), guide length != L (G11), L>64, max_mm > L, a
  * guide with 64 compared (non-N) letters, n_guides == 0 or > 2^24, NULL pointers.  For
- * L > 32 the comparer is always the pair-table one (cof_set_comparer's popc / mma
- * variants need L <= 32).  The plan reverse-complements pattern and
+ * L > 32 the comparer is always the pair-table one (cof_set_comparer's popc variant
+ * needs L <= 32).  The plan reverse-complements pattern and
  * guides for the '-' strand and groups guides by compared-position mask. */
 typedef struct cof_plan cof_plan;
 cof_status cof_plan_create(const char *pattern, uint32_t n_guides, const char *const *guides,
@@ -223,15 +223,10 @@ cof_status cof_compare(const cof_plan *plan, void *plan_dev, const cof_chunk *de
                        uint64_t *hits, uint64_t hits_cap, uint64_t *n_hits, cof_stream s);
 
 /* Comparer implementation for cof_compare (process-wide): 0 = "popc" (POPC per
- * comparison), 1 = "table" (bit-sliced pair tables on the ALU, default), 2 = "mma" (the
- * comparison as an int8 GEMM on the tcgen05 tensor cores, comparer_mma.cu).  All three
- * return the same hits.  COF_E_ARG for another value.  (Env COF_COMPARER=popc|table|mma
- * sets the initial choice.)  The fused path (cof_find_compare) is the table comparer's. */
+ * comparison), 1 = "table" (bit-sliced pair tables on the ALU, default).  Both return the
+ * same hits.  COF_E_ARG for another value.  (Env COF_COMPARER=popc|table sets the initial
+ * choice.)  The fused path (cof_find_compare) is the table comparer's. */
 cof_status cof_set_comparer(int impl);
-/* Contraction length K in bytes per int8 row of the plan's "mma" comparer: three sign
- * bytes per position of the compared span (rounded to 4), two constant bytes and one byte
- * per N-correction class, padded to 32.  0 for a NULL plan. */
-uint32_t   cof_plan_mma_kpad(const cof_plan *plan);
 
 /* ------------------------------------------------------------------ fused find + compare
  * the search and compare kernels of P:L29 without the host hand-off and

@@ -40,6 +40,21 @@ def _digest(files):
     return h.hexdigest()
 
 
+def _local_includes(src, seen=None):
+    """Local headers (csrc/, include/) that ``src`` includes, transitively."""
+    import re
+    seen = set() if seen is None else seen
+    for name in re.findall(r'#include\s+"([^"]+)"', open(src).read()):
+        for d in (os.path.dirname(src), CSRC, INCLUDE):
+            path = os.path.join(d, name)
+            if os.path.exists(path):
+                if path not in seen:
+                    seen.add(path)
+                    _local_includes(path, seen)
+                break
+    return sorted(seen)
+
+
 def _generate():
     gen = os.path.join(CSRC, "gen_csa.py")
     out = os.path.join(CSRC, "csa_gen.cuh")
@@ -64,25 +79,36 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
     dflags = [f"-D{d}" for d in defines]
     objs = []
     procs = []
+    def compile_obj(src, cmd, obj):
+        # per-object stamp: the source, the local headers it includes (transitively) and the
+        # command; an unchanged object is not rebuilt
+        d = _digest([src, *_local_includes(src)]) + " ".join(cmd)
+        ostamp = obj + ".stamp"
+        if not force and os.path.exists(obj) and os.path.exists(ostamp) and open(ostamp).read() == d:
+            return
+        procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT), ostamp, d))
+
     for src in cu:
         obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fopenmp",
                "-Xptxas", "-v" if verbose else "-O3", *dflags, "-I", INCLUDE, "-c", src, "-o", obj]
-        procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
+        compile_obj(src, cmd, obj)
         objs.append(obj)
     for src in cpp:
         obj = os.path.join(build_dir, os.path.basename(src) + ".o")
         cmd = ["g++", "-O3", "-std=c++17", "-fPIC", "-fopenmp", "-Wall", *dflags, "-I", INCLUDE,
                "-I", os.path.join(CUDA, "include"), "-c", src, "-o", obj]
-        procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
+        compile_obj(src, cmd, obj)
         objs.append(obj)
-    for cmd, p in procs:
+    for cmd, p, ostamp, d in procs:
         out, _ = p.communicate()
         if p.returncode != 0:
             sys.stderr.write(out.decode(errors="replace"))
             raise RuntimeError("build failed: " + " ".join(cmd))
         if verbose and out:
             sys.stderr.write(out.decode(errors="replace"))
+        with open(ostamp, "w") as f:
+            f.write(d)
     tmp = lib + f".{os.getpid()}.tmp"
     cmd = ["g++", "-shared", "-fopenmp", "-o", tmp, *objs, "-L", os.path.join(CUDA, "lib64"),
            "-lcudart_static", "-ldl", "-lrt", "-lpthread", "-Wl,--no-undefined"]

@@ -107,7 +107,6 @@ def _load():
         "cof_find_compare": (I32, [P, P, P, P, P, U64, P, P]),
         "cof_find_masks": (I32, [P, P, P, P, P]),
         "cof_compare_masks": (I32, [P, P, P, P, P, U64, P, P]),
-        "cof_plan_mma_kpad": (U32, [P]),
         "cof_2bit_open": (I32, [ctypes.c_char_p, P]),
         "cof_2bit_close": (None, [P]),
         "cof_2bit_count": (U32, [P]),
@@ -137,7 +136,7 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_decorate_workspace_bytes", "cof_decorate", "cof_decorate64",
                        "cof_decorate_check", "cof_find_compare_supported",
                        "cof_find_compare_workspace_bytes", "cof_find_compare", "cof_find_masks",
-                       "cof_compare_masks", "cof_single_supported", "cof_search_single", "cof_plan_mma_kpad", "cof_set_comparer", "cof_2bit_open",
+                       "cof_compare_masks", "cof_single_supported", "cof_search_single", "cof_set_comparer", "cof_2bit_open",
                        "cof_2bit_close", "cof_2bit_count", "cof_2bit_name", "cof_2bit_length",
                        "cof_2bit_pack")]
 
@@ -439,15 +438,9 @@ def cof_merge(lists) -> np.ndarray:
     return out
 
 
-def cof_plan_mma_kpad(plan) -> int:
-    """Contraction length K (bytes per int8 row) of the plan's tensor-core comparer."""
-    return int(lib.cof_plan_mma_kpad(plan.handle))
-
-
 def cof_set_comparer(impl: str):
-    """'table' (bit-sliced pair tables, default), 'popc' (POPC per comparison) or 'mma'
-    (int8 tcgen05 tensor-core GEMM, comparer_mma.cu)."""
-    _check(lib.cof_set_comparer({"popc": 0, "table": 1, "mma": 2}[impl]))
+    """'table' (bit-sliced pair tables, default) or 'popc' (POPC per comparison)."""
+    _check(lib.cof_set_comparer({"popc": 0, "table": 1}[impl]))
 
 
 class Fasta:

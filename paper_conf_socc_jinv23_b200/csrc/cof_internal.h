@@ -79,27 +79,6 @@ struct PairLayout {
     uint32_t n_real;           // pairs before the padding
 };
 
-// Tensor-core comparer (comparer_mma.cu): the mismatch count of every (item, guide) pair
-// as an int8 GEMM.  A row (one item, site S in guide orientation) holds, for each position
-// r of the compared span, the three Hadamard signs u(S_r) in {+1,-1}^3 (0 for a genome N),
-// then two constant ones and, per N-class c, minus the number of genome Ns the site has
-// at the class's positions.  A B row (one guide) holds v_r = sum_{b in IUPAC set} u(b),
-// the threshold offset c_g split over two bytes, and the class weights |S_j|.  Then
-// D = A.B^T = 4 (t_g - mm), so a hit is D >= 0 and mm = t_g - D/4.
-struct MmaBatch {
-    uint32_t g0, ng;           // guides [g0, g0 + ng) of this launch
-    uint32_t nt, tn;           // nt N-tiles of tn columns (tn multiple of 32, <= 128)
-    size_t b_off;              // byte offset of the batch's B image inside the mma_b region
-};
-struct MmaPlan {
-    uint32_t j0, npos;         // compared span (forward orientation window offsets)
-    uint32_t pw;               // words per sign dimension = ceil(npos / 4)
-    uint32_t ks, kpad;         // K steps of 32 bytes; kpad = 32 * ks bytes per row
-    uint32_t nclass;           // N-correction classes
-    uint32_t cmask[32];        // class position masks (bit r = span position r)
-    std::vector<MmaBatch> batches;
-};
-
 // Device plan image layout (byte offsets from plan_dev; all 256-byte aligned)
 struct DevLayout {
     size_t counters;           // uint64[8]: n_fwd, n_rev, n_hits, ...
@@ -108,8 +87,6 @@ struct DevLayout {
     size_t ptab_fwd, ptab_rev;       // pair tables: uint2[n_blocks][n_pairs][25]
     size_t pmeta_fwd, pmeta_rev;     // per block: uint32[8] = {T0..T5 threshold planes, valid, 0}
     size_t onehot;                   // uint64[2][n_guides][5] decoration masks (see cof_plan::onehot)
-    size_t mma_b;                    // tensor-core comparer: int8 B images of all guide batches
-    size_t mma_thr;                  // uint8[n_guides]: min(t_g, #compared positions)
     size_t ftab_fwd, ftab_rev;       // single-pass filter tables: uint32[n_blocks][filter_block_words(np)]
     size_t vrec_fwd, vrec_rev;       // single-pass verification records: uint4[n_blocks * 32][2]
     size_t total;
@@ -130,7 +107,6 @@ struct cof_plan {
     uint32_t n_recs = 0;
     uint32_t n_blocks = 0;               // 32-guide blocks (pair-table comparer)
     cof::PairLayout pairs[2];
-    cof::MmaPlan mma;
     uint64_t union_care[2] = {0, 0};
     bool any_degenerate = false;
     cof::DevLayout lay;

@@ -817,21 +817,16 @@ static cof_status launch_popc(const CompareArgs& a, uint64_t tiles_hint, cudaStr
     return COF_OK;
 }
 
-static int g_impl = -1;   // 0 = popc, 1 = table (default), 2 = mma; COF_COMPARER=popc|table|mma overrides
+static int g_impl = -1;   // 0 = popc, 1 = table (default); COF_COMPARER=popc|table overrides
 
 static int comparer_impl() {
     if (g_impl < 0) {
         const char* e = getenv("COF_COMPARER");
-        g_impl = (e && e[0] == 'p') ? 0 : (e && e[0] == 'm') ? 2 : 1;
+        g_impl = (e && e[0] == 'p') ? 0 : 1;
     }
     return g_impl;
 }
 
-bool mma_supported(const cof_plan* plan);
-cof_status run_mma(const cof_plan* plan, uint8_t* pd, const uint32_t* lo, const uint32_t* hi, const uint32_t* nm,
-                   const uint32_t* items_fwd, uint64_t n_fwd, const uint32_t* items_rev, uint64_t n_rev,
-                   uint64_t items_cap, unsigned long long* hits, uint64_t cap, unsigned long long* counters,
-                   cudaStream_t stream);
 
 cof_status find_launch(const cof_plan* plan, void* plan_dev, const cof_chunk* dev, void* workspace,
                        uint32_t* items_fwd, uint32_t* items_rev, uint64_t items_cap, bool masks_only,
@@ -1024,9 +1019,6 @@ cof_status cof_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* de
         cof_status st;
         if (comparer_impl() == 0 && plan->L <= 32) {   // (v1 records are 32-bit windows)
             st = launch_popc(a, tiles_hint, stream);
-        } else if (comparer_impl() == 2 && mma_supported(plan)) {
-            st = run_mma(plan, pd, a.lo, a.hi, a.nm, items_fwd, n_fwd, items_rev, n_rev, a.items_cap, a.hits, a.cap,
-                         a.counters, stream);
         } else {
             st = run_table(plan, pd, a, stream);
         }
@@ -1045,10 +1037,10 @@ cof_status cof_compare(const cof_plan* plan, void* plan_dev, const cof_chunk* de
     return COF_OK;
 }
 
-// Select the comparer implementation at run time (0 = popc, 1 = table, 2 = mma).  Not part of the
+// Select the comparer implementation at run time (0 = popc, 1 = table).  Not part of the
 // stable ABI (declared here for tests / benchmarks).
 cof_status cof_set_comparer(int impl) {
-    if (impl < 0 || impl > 2) return set_error(COF_E_ARG, "cof_set_comparer: impl must be 0, 1 or 2");
+    if (impl < 0 || impl > 1) return set_error(COF_E_ARG, "cof_set_comparer: impl must be 0 or 1");
     g_impl = impl;
     return COF_OK;
 }

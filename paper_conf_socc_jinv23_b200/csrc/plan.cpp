@@ -192,49 +192,6 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     const uint32_t NPAIR = p->pairs[0].n_pairs;
     if (p->pairs[1].n_pairs != NPAIR) { delete p; return set_error(COF_E_STATE, "internal: pair count mismatch"); }
 
-    // ---- tensor-core comparer: span, N-classes, guide batches (see MmaPlan)
-    MmaPlan& mp = p->mma;
-    if (L <= 32) {   // the tensor-core comparer's span is one 32-bit word
-        const uint32_t uc = (uint32_t)p->union_care[0];
-        mp.j0 = uc ? (uint32_t)__builtin_ctz(uc) : 0u;
-        mp.npos = uc ? 32u - (uint32_t)__builtin_clz(uc) - mp.j0 : 1u;
-        mp.pw = (mp.npos + 3) / 4;
-        // positions grouped by their weight vector (w_r(g) = |S_r(g)|, 0 if not compared)
-        std::map<std::vector<uint8_t>, uint32_t> cls;
-        mp.nclass = 0;
-        memset(mp.cmask, 0, sizeof mp.cmask);
-        for (uint32_t r = 0; r < mp.npos; r++) {
-            std::vector<uint8_t> w(n_guides);
-            bool any = false;
-            for (uint32_t i = 0; i < n_guides; i++) {
-                uint8_t m = p->gmask[(size_t)i * L + mp.j0 + r];
-                w[i] = m == 15 ? 0 : (uint8_t)__builtin_popcount(m);
-                any |= w[i] != 0;
-            }
-            if (!any) continue;
-            auto it = cls.find(w);
-            uint32_t c;
-            if (it == cls.end()) { c = mp.nclass++; cls.emplace(std::move(w), c); } else c = it->second;
-            mp.cmask[c] |= 1u << r;
-        }
-        mp.ks = (12 * mp.pw + 2 + mp.nclass + 31) / 32;
-        mp.kpad = 32 * mp.ks;
-        // guides per launch: the B image of a batch stays resident in shared memory
-        // (smem: B + 4-stage A ring + 32 KB of epilogue hit buffers + thresholds <= 227 KB)
-        const uint32_t gmax = std::max<uint32_t>(128, ((186u * 1024u - 4u * 128u * mp.kpad) / (mp.kpad + 1)) / 128u * 128u);
-        size_t boff = 0;
-        for (uint32_t g0 = 0; g0 < n_guides; g0 += gmax) {
-            MmaBatch b;
-            b.g0 = g0;
-            b.ng = std::min(gmax, n_guides - g0);
-            b.nt = (b.ng + 127) / 128;
-            b.tn = ((b.ng + b.nt - 1) / b.nt + 31) / 32 * 32;
-            b.b_off = boff;
-            boff += (size_t)b.nt * b.tn * mp.kpad;
-            mp.batches.push_back(b);
-        }
-    }
-
     // ---- device image layout
     DevLayout& lay = p->lay;
     size_t off = 0;
@@ -250,10 +207,6 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
     lay.pmeta_fwd = off; off = align256(off + pmeta_bytes);
     lay.pmeta_rev = off; off = align256(off + pmeta_bytes);
     lay.onehot = off; off = align256(off + p->onehot.size() * 8);
-    size_t mma_b_bytes = 0;
-    for (const MmaBatch& b : mp.batches) mma_b_bytes += (size_t)b.nt * b.tn * mp.kpad;
-    lay.mma_b = off; off = align256(off + mma_b_bytes);
-    lay.mma_thr = off; off = align256(off + n_guides);
     // (rounded up to whole groups of 4 blocks: the single-pass kernel reads blocks four at a time)
     const size_t ftab_bytes = (size_t)((p->n_blocks + 3) & ~3u) * filter_block_words(NPAIR) * 4;
     lay.ftab_fwd = off; off = align256(off + ftab_bytes);
@@ -335,47 +288,6 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
             }
         }
     }
-    // tensor-core comparer B images: row n of a batch at byte (n/8)*8*kpad + (k/16)*128 +
-    // (n%8)*16 + k%16 (K-major "interleaved" canonical layout of tcgen05: 8x16-byte core
-    // matrices, LBO = 128 B between K-adjacent ones, SBO = 8*kpad between row groups)
-    {
-        static const int8_t U[4][3] = {{1, 1, 1}, {-1, 1, -1}, {1, -1, -1}, {-1, -1, 1}};   // A C G T
-        uint8_t* thr = img + lay.mma_thr;
-        for (const MmaBatch& b : mp.batches) {
-            int8_t* B = (int8_t*)(img + lay.mma_b + b.b_off);
-            auto at = [&](uint32_t n, uint32_t k) -> int8_t& {
-                return B[(size_t)(n / 8) * 8 * mp.kpad + (k / 16) * 128 + (n % 8) * 16 + (k % 16)];
-            };
-            for (uint32_t n = 0; n < b.nt * b.tn; n++) {
-                const uint32_t kc = 12 * mp.pw;
-                if (n >= b.ng) { at(n, kc) = -128; at(n, kc + 1) = -128; continue; }   // padding: never a hit
-                const uint32_t i = b.g0 + n;
-                int32_t ncmp = 0, sum_set = 0;
-                for (uint32_t r = 0; r < mp.npos; r++) {
-                    const uint8_t m = p->gmask[(size_t)i * L + mp.j0 + r];
-                    if (m == 15) continue;
-                    ncmp++;
-                    sum_set += __builtin_popcount(m);
-                    for (int d = 0; d < 3; d++) {
-                        int v = 0;
-                        for (int base = 0; base < 4; base++) if (m >> base & 1) v += U[base][d];
-                        at(n, 4 * mp.pw * d + r) = (int8_t)v;
-                    }
-                }
-                const int32_t teff = std::min<int32_t>(p->max_mm[i], ncmp);
-                thr[i] = (uint8_t)teff;
-                const int32_t c = -(4 * (ncmp - teff) - sum_set);      // in [-128, 128]
-                const int32_t c1 = c / 2, c2 = c - c1;
-                at(n, kc) = (int8_t)c1;
-                at(n, kc + 1) = (int8_t)c2;
-                for (uint32_t cl = 0; cl < mp.nclass; cl++) {
-                    const uint32_t r = (uint32_t)__builtin_ctz(mp.cmask[cl]);
-                    const uint8_t m = p->gmask[(size_t)i * L + mp.j0 + r];
-                    at(n, kc + 2 + cl) = (int8_t)(m == 15 ? 0 : __builtin_popcount(m));
-                }
-            }
-        }
-    }
     *out = p;
     return COF_OK;
 }
@@ -384,7 +296,6 @@ void cof_plan_destroy(cof_plan* p) { delete p; }
 uint32_t cof_plan_length(const cof_plan* p) { return p ? p->L : 0; }
 uint32_t cof_plan_n_guides(const cof_plan* p) { return p ? p->n_guides : 0; }
 size_t cof_plan_device_bytes(const cof_plan* p) { return p ? p->lay.total : 0; }
-uint32_t cof_plan_mma_kpad(const cof_plan* p) { return p ? p->mma.kpad : 0; }
 
 cof_status cof_plan_upload(const cof_plan* p, void* plan_dev, cof_stream s) {
     if (!p || !plan_dev) return set_error(COF_E_ARG, "cof_plan_upload: NULL argument");

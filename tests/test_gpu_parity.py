@@ -14,7 +14,7 @@ from paper_conf_socc_jinv23_b200 import cof, search, synth
 from tests import golden_io
 
 pytestmark = pytest.mark.gpu
-IMPLS = ["table", "popc", "mma"]
+IMPLS = ["table", "popc"]
 
 
 @pytest.fixture(autouse=True)
@@ -88,18 +88,6 @@ def test_configs_scaled(name, scale, chunk, pack):
                     fused=True) == exp
 
 
-@pytest.mark.parametrize("name,scale,chunk,pack", [("C2", 0.1, None, None), ("C3", 0.004, 1_000_003, None),
-                                                   ("C4", 0.004, 333_333, 0), ("C5", 0.002, None, 0)])
-def test_configs_scaled_mma(name, scale, chunk, pack):
-    """The tensor-core comparer on the configs' shapes (incl. Cas12a TTTV with 23 compared
-    positions: three K steps) against the oracle."""
-    w = synth.make_workload(name, scale=scale, n_guides=None if name != "C5" else 1000)
-    cfg = w.cfg
-    exp = ref_hits(w.seqs, cfg.pattern, w.guides, w.thresholds)
-    assert gpu_hits(w.seqs, cfg.pattern, w.guides, w.thresholds, chunk_bases=chunk, pack_bases=pack,
-                    impl="mma") == exp
-
-
 @pytest.mark.parametrize("shape", ["spcas9", "cas12a"])
 @pytest.mark.parametrize("n_guides", [1, 37, 512, 600])
 def test_uniform_threshold_paths(shape, n_guides):
@@ -138,7 +126,7 @@ def test_random_long(seed):
     offsets >= 32: the finder's three-word slices), guides whose compared span is either
     <= 32 or up to 63 (two-word comparer windows, padded pair tables), degenerate letters,
     genome N / lowercase; fused and two-call paths, one chunk and packed pieces; the popc
-    and mma selections fall back to the table comparer."""
+    selection falls back to the table comparer."""
     rng = np.random.default_rng(900 + seed)
     L = int(rng.integers(33, 65))
     pat = "".join(rng.choice(list("N" * 24 + "ACGTRYSWKMBDHV"), L))
@@ -163,7 +151,6 @@ def test_random_long(seed):
     assert gpu_hits(seqs, pat, guides, thr, fused=False) == exp
     assert gpu_hits(seqs, pat, guides, thr, fused=True, pack_bases=0) == exp
     assert gpu_hits(seqs, pat, guides, thr, impl="popc") == exp
-    assert gpu_hits(seqs, pat, guides, thr, impl="mma", fused=False) == exp
 
 
 @pytest.mark.parametrize("name,scale,n_guides", [("X1", 0.05, None), ("X2", 0.05, None), ("X1", 0.01, 300)])
@@ -312,11 +299,10 @@ def test_search_host_into_caller_buffer_and_chunk_pipeline(decorate):
     assert cof.hits_to_tuples(srch.search_host(packed, decorate=decorate)) == exp
 
 
-@pytest.mark.parametrize("impl", ["table", "mma"])
+@pytest.mark.parametrize("impl", ["table"])
 def test_many_guides_multiple_table_launches(impl):
     """> 4096 guides: the table comparer splits the guides into launches of 128 blocks
-    (thresholds in the parameter space) and tiles them through shared memory; the mma
-    comparer into guide batches whose B image fits shared memory."""
+    (thresholds in the parameter space) and tiles them through shared memory."""
     rng = np.random.default_rng(21)
     seq = synth.random_genome_text(rng, 30_000)
     n_g = 4096 + 300
