@@ -62,10 +62,13 @@ COF_HD uint32_t pair_entry(uint32_t np, uint32_t q, uint32_t b1, uint32_t b2) {
 }
 
 // Single-pass comparer filter table (single.cu): per strand and 32-guide block, per
-// position pair, 25 one-word entries (bit k = guide k's pair has >= 1 mismatch for that
-// base pair), indexed like pair_entry; blocks padded to a 64-byte multiple so the
-// 16 ACGT entries of a pair (64 bytes) can be addressed by OR-ing the pair nibble in.
-COF_HD uint32_t filter_block_words(uint32_t np) { return (np * 25u + 15u) & ~15u; }
+// position pair, the 16 ACGT one-word entries (bit k = guide k's pair has >= 1 mismatch
+// for that base pair), indexed like pair_entry's ACGT part: 64 bytes per pair, addressed by
+// OR-ing the pair nibble in.  No N entries: the filter reads a genome N as the A its
+// planes hold (lo = hi = 0), which can only hide mismatches, so the filter stays a
+// necessary condition and the exact verification counts the N.  Guides past the plan
+// (the last block's padding, padding blocks) have every bit set: they never survive.
+COF_HD uint32_t filter_block_words(uint32_t np) { return np * 16u; }
 
 // Bit-sliced pair-table comparer (v2): per strand, per 32-guide block, per position pair,
 // 25 entries (base pair combos incl. N) of {bit0, bit1} mismatch-count planes.

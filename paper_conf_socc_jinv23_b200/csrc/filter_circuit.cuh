@@ -60,12 +60,15 @@ COF_FC uint32_t filter_fail_fast(const uint32_t (&v)[NP], bool& done) {
 }
 
 // Filter: bit k of the result = guide k of the block survives (its number of pairs with a
-// mismatch is <= its threshold).  TC >= 0: one threshold for every guide of the launch.
+// mismatch is <= its threshold).  TC >= 0: one threshold for every guide of the launch,
+// TC < NP; guides past the plan need no mask there, their table bits are all set (count
+// NP > TC).  TC < 0: per-guide threshold planes m[0..5] and the valid-guide mask m[6].
 template <int NP, int TC>
 COF_FC uint32_t filter_pass(const uint32_t (&v)[NP], const uint32_t* __restrict__ m) {
+    static_assert(TC < NP, "a uniform threshold below the pair count");
     bool fast;
     const uint32_t ff = filter_fail_fast<NP, TC>(v, fast);
-    if (fast) return m[6] & ~ff;
+    if (fast) return ~ff;
     uint32_t c[5];
     nz_count<NP>(v, c);
     uint32_t bw;                       // borrow out of (t - count): set where count > t
@@ -73,6 +76,7 @@ COF_FC uint32_t filter_pass(const uint32_t (&v)[NP], const uint32_t* __restrict_
         bw = (TC & 1) ? 0u : c[0];
 #pragma unroll
         for (int w = 1; w < 5; w++) bw = ((TC >> w) & 1) ? (c[w] & bw) : (c[w] | bw);
+        return ~bw;
     } else {
         bw = c[0] & ~m[0];
 #pragma unroll

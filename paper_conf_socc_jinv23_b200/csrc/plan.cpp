@@ -260,11 +260,20 @@ cof_status cof_plan_create(const char* pattern, uint32_t n_guides, const char* c
                     size_t e = (size_t)b * NPAIR * 25 + pair_entry(NPAIR, q, b1, b2);
                     tab[e * 2 + 0] = w0;
                     tab[e * 2 + 1] = w1;
-                    // single-pass filter: the pair has at least one mismatch (count 1 or 2)
-                    uint32_t* ft = (uint32_t*)(img + (s == 0 ? lay.ftab_fwd : lay.ftab_rev));
-                    ft[(size_t)b * filter_block_words(NPAIR) + pair_entry(NPAIR, q, b1, b2)] = w0 | w1;
+                    // single-pass filter: the pair has at least one mismatch (count 1 or 2);
+                    // guides past the plan always "mismatch" (ACGT entries only)
+                    if (b1 < 4 && b2 < 4) {
+                        uint32_t* ft = (uint32_t*)(img + (s == 0 ? lay.ftab_fwd : lay.ftab_rev));
+                        const uint32_t nv = n_guides - b * 32 >= 32 ? 0u : ~0u << (n_guides - b * 32);
+                        ft[(size_t)b * filter_block_words(NPAIR) + pair_entry(NPAIR, q, b1, b2)] = w0 | w1 | nv;
+                    }
                 }
             }
+        }
+        {   // padding blocks of the last group of 4: no guide, every bit set
+            uint32_t* ft = (uint32_t*)(img + (s == 0 ? lay.ftab_fwd : lay.ftab_rev));
+            for (uint32_t b = p->n_blocks; b < ((p->n_blocks + 3) & ~3u); b++)
+                for (uint32_t w = 0; w < filter_block_words(NPAIR); w++) ft[(size_t)b * filter_block_words(NPAIR) + w] = ~0u;
         }
         // single-pass verification records, window offsets relative to p0 (compared spans
         // <= 32 only): {lo, hi, care, t} of the concrete letters and the one-hot {A, C, G, T}

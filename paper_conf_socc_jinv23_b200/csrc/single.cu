@@ -35,6 +35,7 @@
 //    rare verifications, against ~1.2 + 0.3 (64-bit lookups) for the exact pair-table sum.
 #include <algorithm>
 #include <mutex>
+#include <type_traits>
 
 #include <cuda_runtime.h>
 
@@ -50,7 +51,7 @@ namespace cof {
 // addresses) is amortised over more lookups -- and 20 warps; many blocks (C5) take one
 // site per lane and 28 warps, which hides the filter's dependency latency better and keeps
 // all 32 blocks of a 1000-guide plan in one launch's shared memory.
-template <int W, int R, int S, int QB>
+template <int W, int R, int S, int QB, int GUN>
 struct SCfg {
     static constexpr int SW = W;                  // warps per CTA (one CTA per SM)
     static constexpr int STHREADS = 32 * W;
@@ -60,11 +61,12 @@ struct SCfg {
     static constexpr int SR = R;                  // sites per lane and batch
     static constexpr uint32_t SQ = 32u * R * QB;  // queued sites per warp (16-byte entries): QB batches
     static constexpr uint32_t SBATCH = 32u * R;
-    static constexpr uint32_t SVC = R == 1 ? 64u : 128u;   // survivor entries per warp (ring)
+    static constexpr int GU = GUN;                // groups of 4 guide blocks per filter step
+    static constexpr uint32_t SVC = 32u * R * GU <= 32u ? 64u : 32u * R * GU <= 96u ? 128u : 256u;   // survivor ring
     static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH && (SQ & (SQ - 1)) == 0, "ring");
     static constexpr uint32_t SPW = 5u * SVC;     // per-warp words of the survivor ring
     static_assert(SPW % 4 == 0, "16-byte survivor masks");
-    static_assert(SVC >= 31 + 32 * SR, "a group of blocks appends at most 32 entries per site row");
+    static_assert(SVC >= 31 + 32 * SR * GU, "a group of blocks appends at most 32 entries per site row");
 };
 // (warps, sites per lane, ring stages, queue batches); -DCOF_FEW_W=... etc. override for A/B builds
 #ifndef COF_FEW_W
@@ -82,6 +84,12 @@ struct SCfg {
 #ifndef COF_MANY_Q
 #define COF_MANY_Q 2
 #endif
+#ifndef COF_FEW_G
+#define COF_FEW_G 1
+#endif
+#ifndef COF_MANY_G
+#define COF_MANY_G 2
+#endif
 #ifndef COF_MANY_W
 #define COF_MANY_W 28
 #endif
@@ -91,8 +99,8 @@ struct SCfg {
 #ifndef COF_MANY_S
 #define COF_MANY_S 4
 #endif
-using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q>;
-using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S, COF_MANY_Q>;
+using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q, COF_FEW_G>;
+using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S, COF_MANY_Q, COF_MANY_G>;
 constexpr uint32_t SFEW_BLOCKS = 8;       // guide blocks up to which SCfgFew runs
 constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
@@ -156,7 +164,7 @@ __device__ __forceinline__ void lds_filter(const uint32_t (&base)[NP], uint32_t 
 template <int NP>
 __device__ __forceinline__ void site_bases(const SingleArgs& a, uint32_t tbase, uint32_t sd, uint32_t wl,
                                            uint32_t wh, uint32_t wn, uint32_t (&base)[NP]) {
-    if (a.contig && (wn & a.cmp_mask) == 0) {
+    if (a.contig) {
         // pair q = window offsets (2q, 2q + 1): its 4-bit entry index lo(b1) | lo(b2) << 1 |
         // hi(b1) << 2 | hi(b2) << 3 is nibble q/2 of Y (even q) or Z (odd q)
         const uint32_t Y = (wl & 0x33333333u) | ((wh & 0x33333333u) << 2);
@@ -173,9 +181,10 @@ __device__ __forceinline__ void site_bases(const SingleArgs& a, uint32_t tbase, 
 #pragma unroll
     for (int q = 0; q < NP; q++) {
         const uint32_t j1 = a.j1[sd][q], j2 = a.j2[sd][q];
-        const uint32_t b1 = ((wn >> j1) & 1u) ? 4u : (((wl >> j1) & 1u) | (((wh >> j1) & 1u) << 1));
+        // (a genome N reads as the A of its planes: the filter tables have no N entries)
+        const uint32_t b1 = ((wl >> j1) & 1u) | (((wh >> j1) & 1u) << 1);
         uint32_t b2 = 0;
-        if (j2 < 32u) b2 = ((wn >> j2) & 1u) ? 4u : (((wl >> j2) & 1u) | (((wh >> j2) & 1u) << 1));
+        if (j2 < 32u) b2 = ((wl >> j2) & 1u) | (((wh >> j2) & 1u) << 1);
         base[q] = tbase + pair_entry(NP, (uint32_t)q, b1, b2) * 4u - (uint32_t)q * 64u;
     }
 }
@@ -190,13 +199,14 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     constexpr int SW = CFG::SW, STHREADS = CFG::STHREADS, STW = CFG::STW, SLOAD = CFG::SLOAD;
     constexpr int SSTAGES = CFG::SSTAGES, SR = CFG::SR;
     constexpr uint32_t SQ = CFG::SQ, SBATCH = CFG::SBATCH, SVC = CFG::SVC;
+    constexpr int GU = CFG::GU;
     extern __shared__ __align__(128) uint8_t smem[];
     // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
     //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
     //         [ring: SSTAGES x SPL x SLOAD words][site queues: SW x SQ x uint4]
     //         [per warp: survivor ring (SVC x 5 words)]
     //         [tile ids, release counters][full mbarriers]
-    constexpr uint32_t FBW = (NP * 25u + 15u) & ~15u;
+    constexpr uint32_t FBW = NP * 16u;
     constexpr uint32_t VSTR = CONCRETE ? 1u : 2u;     // uint4 per verification record in shared memory
     const uint32_t nb = a.n_blocks;
     uint32_t* s_ftab = reinterpret_cast<uint32_t*>(smem);
@@ -347,46 +357,55 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
 #pragma unroll
             for (int r = 0; r < SR; r++) {
                 const uint32_t i = (uint32_t)r * 32 + lane;
-                // a missing site gets an all-N window (every pair mismatches) and is masked below
-                const uint4 e = i < n_items ? queue[(head + i) & (SQ - 1)] : make_uint4(0u, 0u, 0u, 0x7FFFFFFFu);
+                // (a missing site of a partial batch appends no survivor)
+                const uint4 e = i < n_items ? queue[(head + i) & (SQ - 1)] : make_uint4(0u, 0u, 0u, 0u);
                 const uint32_t sd = e.w >> 31;
                 site_bases<NP>(a, sd ? tb1 : tb0, sd, e.y, e.z, e.w & 0x7FFFFFFFu, base[r]);
             }
 
-            // groups of 4 blocks; one extra pass (b >= nb) drains the survivor list, so the
-            // verification code exists once in the kernel (its size decides the I-cache hit rate)
-            for (uint32_t b = 0;; b += 4) {
+            // steps of GU groups of 4 blocks (immediate table offsets inside a step); one extra
+            // pass (b >= nb) drains the survivor list, so the verification code exists once in
+            // the kernel (its size decides the I-cache hit rate)
+            for (uint32_t b = 0;; b += 4 * GU) {
                 const bool drain = b >= nb;
                 if (!drain) {
-                    const uint32_t* m = a.meta[b];
                     const uint32_t boff = b * FBW * 4;
+                    // one group: blocks b + 4G .. b + 4G + 3
+                    auto group = [&](auto G) {
+                        constexpr uint32_t GO = (uint32_t)decltype(G)::value * 4u * FBW * 4u;
+                        const uint32_t bg = b + (uint32_t)decltype(G)::value * 4u;
+                        const uint32_t* m = a.meta[bg];     // (read by the generic kernel only)
 #pragma unroll
-                    for (int r = 0; r < SR; r++) {
-                        uint32_t v[NP], p0, p1, p2, p3;
-                        lds_filter<NP, 0 * FBW * 4>(base[r], boff, v);
-                        p0 = filter_pass<NP, TC>(v, m);
-                        lds_filter<NP, 1 * FBW * 4>(base[r], boff, v);
-                        p1 = filter_pass<NP, TC>(v, m + 8);
-                        lds_filter<NP, 2 * FBW * 4>(base[r], boff, v);
-                        p2 = filter_pass<NP, TC>(v, m + 16);
-                        lds_filter<NP, 3 * FBW * 4>(base[r], boff, v);
-                        p3 = filter_pass<NP, TC>(v, m + 24);
-                        // a site with a survivor in this group of 4 blocks -> one survivor
-                        // entry (ballot append; blocks past the plan have valid 0; a missing
-                        // site of a partial batch appends nothing)
-                        const bool has = (p0 | p1 | p2 | p3) != 0u && (uint32_t)r * 32u + lane < n_items;
-                        const unsigned hb = __ballot_sync(0xFFFFFFFFu, has);
-                        const uint32_t e = (sv_h + sv_n + (uint32_t)__popc(hb & lanemask_lt())) & (SVC - 1);
-                        if (has) {
-                            sv_x[e] = ((head + (uint32_t)r * 32 + lane) & (SQ - 1)) | ((b >> 2) << 8);
-                            sv_m[e] = make_uint4(p0, p1, p2, p3);
+                        for (int r = 0; r < SR; r++) {
+                            uint32_t v[NP], p0, p1, p2, p3;
+                            lds_filter<NP, GO + 0 * FBW * 4>(base[r], boff, v);
+                            p0 = filter_pass<NP, TC>(v, m);
+                            lds_filter<NP, GO + 1 * FBW * 4>(base[r], boff, v);
+                            p1 = filter_pass<NP, TC>(v, m + 8);
+                            lds_filter<NP, GO + 2 * FBW * 4>(base[r], boff, v);
+                            p2 = filter_pass<NP, TC>(v, m + 16);
+                            lds_filter<NP, GO + 3 * FBW * 4>(base[r], boff, v);
+                            p3 = filter_pass<NP, TC>(v, m + 24);
+                            // a site with a survivor in this group of 4 blocks -> one survivor
+                            // entry (ballot append; guides past the plan never survive; a
+                            // missing site of a partial batch appends nothing)
+                            const bool has = (p0 | p1 | p2 | p3) != 0u && (uint32_t)r * 32u + lane < n_items;
+                            const unsigned hb = __ballot_sync(0xFFFFFFFFu, has);
+                            const uint32_t e = (sv_h + sv_n + (uint32_t)__popc(hb & lanemask_lt())) & (SVC - 1);
+                            if (has) {
+                                sv_x[e] = ((head + (uint32_t)r * 32 + lane) & (SQ - 1)) | ((bg >> 2) << 8);
+                                sv_m[e] = make_uint4(p0, p1, p2, p3);
+                            }
+                            sv_n += (uint32_t)__popc(hb);
                         }
-                        sv_n += (uint32_t)__popc(hb);
+                    };
+                    group(std::integral_constant<int, 0>{});
+                    if constexpr (GU > 1) {
+                        if (b + 4 < nb) group(std::integral_constant<int, 1>{});
                     }
-
                 }
                 __syncwarp();
-                // (at most 31 + SR x 32 entries are queued: SVC holds them; a round takes 32 and
+                // (at most 31 + SR x GU x 32 entries are queued: SVC holds them; a round takes 32 and
                 // puts back at most 32, and every round verifies one survivor per entry taken)
                 // (a batch that keeps its survivors for the next one verifies only full rounds)
                 const bool keep = resv == 0u && n_items == SBATCH && !tiles_done;
