@@ -562,12 +562,14 @@ def main():
     # finder roofline (HBM): algorithmic bytes of the search kernel per step
     plane_bytes = sum(cof.cof_plane_words(ch.n_bases) * 4 * (4 if ch.multi else 3) for ch in st.chunks)
     words = sum(cof.cof_plane_words(ch.n_bases) for ch in st.chunks)
-    if st.path_name == "single":   # planes streamed once per launch by the single-pass kernel
-        n_launch = max(1, len(events) // max(1, args.steps))
-        find_bytes = plane_bytes * n_launch
-        find_basis = ("single pass: no separate search kernel; planes (+ valid-start plane) streamed once per "
-                      "launch by cof_single_kernel (PAM test fused into it) -- bytes / that kernel's time")
-        find_ms = cmp_ms
+    if st.path_name == "single":
+        # the single pass has no separate search kernel: the paper's search step (ordered PAM
+        # item lists, cof_find_pam -> cof_finder_kernel) is timed on its own, after the step
+        find_ms, n_items_sk = time_search_kernel(st, args.steps)
+        find_bytes = plane_bytes + 4 * n_items_sk
+        find_basis = ("search kernel alone (cof_find_pam: count pass, grid exchange, ordered item lists; the "
+                      "single pass fuses the PAM test into cof_single_kernel): planes (+ valid-start plane) read + "
+                      f"4 B per item written, timed {args.steps} times after the step's timed region")
     elif st.fused:      # planes (+ valid-start plane) read, {fwd, rev} masks written
         find_bytes = plane_bytes + words * 8
         find_basis = "planes read + 8 B of PAM masks per plane word written (fused path)"
@@ -576,11 +578,11 @@ def main():
         find_basis = "planes read + 4 B per item written (two-call path)"
     find_gbs = find_bytes * args.steps / (find_ms * 1e-3) / 1e9 if find_ms > 0 else 0.0
     hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
-    finder_roof = {"bound": "hbm", "kernel": "cof_single_kernel" if st.path_name == "single" else "cof_finder_kernel",
+    finder_roof = {"bound": "hbm", "kernel": "cof_finder_kernel",
                    "achieved": round(find_gbs, 1),
                    "peak": hbm_peak, "unit": "GB/s", "frac": find_gbs / hbm_peak,
                    "bytes_per_step": int(find_bytes), "basis": find_basis,
-                   "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_single_kernel" if st.path_name == "single" else "cof_finder_kernel", st, cfgname)}
+                   "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_finder_kernel", st, cfgname)}
 
     e2e = None
     resident = None
@@ -646,6 +648,34 @@ def main():
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def time_search_kernel(st, steps):
+    """The search kernel alone (cof_find_pam: ordered PAM item lists of every chunk) on the
+    resident planes, ``steps`` launches per chunk after one warm-up, CUDA events on the
+    launching stream.  Returns (ms per step, items per step)."""
+    import torch
+    from paper_conf_socc_jinv23_b200 import cof
+    s = st.stream
+    total_ms, n_items = 0.0, 0
+    for i in range(len(st.chunks)):
+        nf, nr = st.counts[i][0], st.counts[i][1]
+        cap = max(nf, nr) + 1024
+        items = torch.empty((2, cap), dtype=torch.int32, device=st.device)
+        ws = torch.empty(cof.cof_find_workspace_bytes(st.chunks[i].n_bases), dtype=torch.uint8, device=st.device)
+        got = cof.cof_find_pam(st.plan, st.plan_devs[i], st.d_chunks[i], ws, items[0], items[1], cap, s)
+        if tuple(got) != (nf, nr):
+            raise RuntimeError(f"search kernel counts {got} != the step's {(nf, nr)}")
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        for _ in range(steps):
+            cof.cof_find_pam(st.plan, st.plan_devs[i], st.d_chunks[i], ws, items[0], items[1], cap, s, sync=False)
+        e1.record(s)
+        torch.cuda.synchronize(st.device)
+        total_ms += e0.elapsed_time(e1)
+        n_items += nf + nr
+        del items, ws
+    return total_ms, n_items
 
 
 def traffic_for(kernel, st, cfgname):

@@ -21,6 +21,7 @@ BUILD = os.path.join(HERE, "_build")
 CUDA = os.environ.get("CUDA_HOME", "/usr/local/cuda")
 NVCC = os.path.join(CUDA, "bin", "nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+VARIANT_SOURCES = {"single.cu", "finder.cu"}   # the sources a variant build's -D defines apply to
 
 
 def _sources():
@@ -88,15 +89,26 @@ def build(force: bool = False, verbose: bool = False, defines=(), out: str | Non
             return
         procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT), ostamp, d))
 
+    # a variant build (defines) recompiles only the sources the defines are for (VARIANT_SOURCES)
+    # and shares every other object with the main build
+    os.makedirs(BUILD, exist_ok=True)
+
+    def where(src):
+        if defines and os.path.basename(src) not in VARIANT_SOURCES:
+            return BUILD, []
+        return build_dir, dflags
+
     for src in cu:
-        obj = os.path.join(build_dir, os.path.basename(src) + ".o")
+        bdir, df = where(src)
+        obj = os.path.join(bdir, os.path.basename(src) + ".o")
         cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-fopenmp",
-               "-Xptxas", "-v" if verbose else "-O3", *dflags, "-I", INCLUDE, "-c", src, "-o", obj]
+               "-Xptxas", "-v" if verbose else "-O3", *df, "-I", INCLUDE, "-c", src, "-o", obj]
         compile_obj(src, cmd, obj)
         objs.append(obj)
     for src in cpp:
-        obj = os.path.join(build_dir, os.path.basename(src) + ".o")
-        cmd = ["g++", "-O3", "-std=c++17", "-fPIC", "-fopenmp", "-Wall", *dflags, "-I", INCLUDE,
+        bdir, df = where(src)
+        obj = os.path.join(bdir, os.path.basename(src) + ".o")
+        cmd = ["g++", "-O3", "-std=c++17", "-fPIC", "-fopenmp", "-Wall", *df, "-I", INCLUDE,
                "-I", os.path.join(CUDA, "include"), "-c", src, "-o", obj]
         compile_obj(src, cmd, obj)
         objs.append(obj)

@@ -93,9 +93,10 @@ def test_finder_grid_exchange_next_to_a_busy_stream():
     import torch
     rng = np.random.default_rng(9)
     seq = synth.random_genome_text(rng, 3_000_000, b"ACGTN", p=[.24, .24, .24, .24, .04])
-    pat = "TTTV" + "N" * 23                       # sparse PAM: the warp-per-tile pass 2
+    pat = "TTTV" + "N" * 23                       # sparse PAM
     guides = ["NNNN" + "".join(rng.choice(list("ACGT"), 23)) for _ in range(4)]
     srch = search.Searcher(pat, guides, [5] * 4)
+    srch.fused = False            # the two-call path: item lists sized for cof_find_pam
     host = search.HostGenome([seq], search.plan_chunks([len(seq)], len(pat)))
     srch.reserve(host.chunks[0].n_bases, 1 << 16)
     dch = srch.device_chunk(host.chunks[0])

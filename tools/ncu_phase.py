@@ -18,7 +18,7 @@ MARKERS = [   # (marker substring, phase starting at that line)
     ("auto flush = [&]", "verify (flush)"),
     ("// per-lane state of the tile being appended", "other"),
     ("// ---------------- compare a batch", "batch start"),
-    ("for (uint32_t b = 0;; b += 4)", "filter loop + survivor append"),
+    ("for (uint32_t b = 0;; b += 4", "filter loop + survivor append"),
     ("__syncwarp();\n                // (at most", "survivor rounds mgmt"),
     ("head = (head + SBATCH) & (SQ - 1);", "other"),
     ("// ---------------- append pending sites", "append"),
