@@ -107,3 +107,21 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 #define COF_LOP3(d, a, b, c, lut) asm("lop3.b32 %0, %1, %2, %3, " #lut ";" : "=r"(d) : "r"(a), "r"(b), "r"(c))
 
 }  // namespace cof
+
+// Device-side invariant checks (a substitute for the CUDA sanitizers, which this pool does
+// not run): a build with -DCOF_CHECKS (python -m paper_conf_socc_jinv23_b200.build
+// -DCOF_CHECKS --out=...) traps on the first violated bound, so the parity tests run
+// against it fail loudly; the product build compiles them away.
+#ifdef COF_CHECKS
+#include <cstdio>
+#define COF_ASSERT(cond, what)                                                                  \
+    do {                                                                                        \
+        if (!(cond)) {                                                                          \
+            printf("COF_CHECKS: %s violated (%s:%d, block %d thread %d)\n", what, __FILE__,    \
+                   __LINE__, (int)blockIdx.x, (int)threadIdx.x);                                \
+            __trap();                                                                           \
+        }                                                                                       \
+    } while (0)
+#else
+#define COF_ASSERT(cond, what) ((void)0)
+#endif

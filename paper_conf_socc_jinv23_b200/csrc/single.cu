@@ -234,6 +234,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         const size_t w0 = (size_t)tile * STW;
         // (a tile size that does not divide the planes' 512-word padding: the last tile's
         // copy stops at the allocation; the words past it only feed invalid starts)
+        COF_ASSERT(w0 < a.words, "single: tile inside the planes");
         const uint32_t nbytes = (uint32_t)min((uint64_t)SLOAD, a.words - w0) * 4u;
         uint32_t* S = ring + st * SPL * SLOAD;
         fence_proxy_async_smem();
@@ -303,6 +304,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             const uint32_t low = sel & (0u - sel);
             if (m0) m0 ^= low; else if (m1) m1 ^= low; else if (m2) m2 ^= low; else m3 ^= low;
             g = (x >> 8) * 128u + bi + (uint32_t)(__ffs(low) - 1);    // launch-local guide
+            COF_ASSERT(g < a.n_blocks * 32u, "single: survivor guide inside the launch");
             const uint4 it = queue[x & (SQ - 1)];
             pos = it.x;
             sd = it.w >> 31;
@@ -397,6 +399,8 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                                 sv_m[e] = make_uint4(p0, p1, p2, p3);
                             }
                             sv_n += (uint32_t)__popc(hb);
+                            COF_ASSERT(sv_n <= SVC, "single: survivor ring capacity");
+                            COF_ASSERT(bg < SMAX_BLOCKS && bg < nb, "single: guide block index");
                         }
                     };
                     group(std::integral_constant<int, 0>{});
@@ -411,9 +415,11 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                 const bool keep = resv == 0u && n_items == SBATCH && !tiles_done;
                 while (sv_n >= 32 || (drain && !keep && sv_n > 0)) {
                     const uint32_t nf = min(sv_n, 32u);
+                    COF_ASSERT(nf <= 32 && sv_n <= SVC, "single: verification round size");
                     const uint32_t back = flush(sv_h, nf, sv_h + sv_n);
                     sv_h = (sv_h + nf) & (SVC - 1);
                     sv_n = sv_n - nf + back;
+                    COF_ASSERT(sv_n <= SVC && back <= nf, "single: survivors re-appended");
                     __syncwarp();
                 }
                 if (drain) break;
@@ -442,6 +448,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                 if (lane >= o) x += y;
             }
             const uint32_t total = __shfl_sync(0xFFFFFFFFu, x, 31);
+            COF_ASSERT(q_n + resv <= SQ, "single: site queue occupancy");
             const uint32_t take = min(SQ - q_n - resv, total);
             const uint32_t first = x - c;
             const uint32_t n_mine = min(c, take > first ? take - first : 0u);
@@ -485,6 +492,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             }
             __syncwarp();
             q_n += take;
+            COF_ASSERT(q_n + resv <= SQ, "single: site queue capacity");
             continue;
         }
         // ---------------- next chunk of 32 plane words (any warp may take any chunk of the
