@@ -284,6 +284,11 @@ cof_status cof_sort_hits(const cof_plan *plan, void *plan_dev, const cof_chunk *
 /* Device counters of plan_dev: out[0]=n_fwd, out[1]=n_rev, out[2]=n_hits (synchronizes). */
 cof_status cof_read_counts(const cof_plan *plan, const void *plan_dev, uint64_t out[3],
                            cof_stream s);
+/* The same three counters copied asynchronously on stream s into out_host (caller-owned,
+ * ideally pinned; valid once the stream reaches this point -- record an event after it).
+ * No synchronisation: lets a pipelined caller read chunk j's counts while chunk j+1 runs. */
+cof_status cof_counts_async(const cof_plan *plan, const void *plan_dev, uint64_t *out_host,
+                            cof_stream s);
 
 /* ------------------------------------------------------------------ collect (M10)
  * One output record: guide index, chromosome, 0-based '+'-strand chromosome

@@ -89,6 +89,7 @@ def _load():
         "cof_sort_workspace_bytes": (SZ, [U64]),
         "cof_sort_hits": (I32, [P, P, P, P, P, U64, U64, P, P]),
         "cof_read_counts": (I32, [P, P, P, P]),
+        "cof_counts_async": (I32, [P, P, P, P]),
         "cof_n_runs": (I32, [P, U64, P, U64, P]),
         "cof_load_chunk_runs": (I32, [P, P, U64, P, P]),
         "cof_load_chunk_runs_split": (I32, [P, P, U64, P, P, P]),
@@ -131,7 +132,7 @@ EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof
                        "cof_unpack", "cof_valid_starts", "cof_load_chunk", "cof_fasta_open", "cof_fasta_close",
                        "cof_fasta_count", "cof_fasta_name", "cof_fasta_length", "cof_fasta_pack",
                        "cof_find_workspace_bytes", "cof_find_pam", "cof_compare",
-                       "cof_sort_workspace_bytes", "cof_sort_hits", "cof_read_counts",
+                       "cof_sort_workspace_bytes", "cof_sort_hits", "cof_read_counts", "cof_counts_async",
                        "cof_n_runs", "cof_load_chunk_runs", "cof_load_chunk_runs_split", "cof_collect", "cof_collect64", "cof_merge", "cof_merge64",
                        "cof_decorate_workspace_bytes", "cof_decorate", "cof_decorate64",
                        "cof_decorate_check", "cof_find_compare_supported",
@@ -382,6 +383,12 @@ def cof_read_counts(plan, plan_dev, stream=None):
     out = (ctypes.c_uint64 * 3)()
     _check(lib.cof_read_counts(plan.handle, _ptr(plan_dev), ctypes.addressof(out), _stream(stream)))
     return int(out[0]), int(out[1]), int(out[2])
+
+
+def cof_counts_async(plan, plan_dev, out_host, stream=None):
+    """Async copy of the three device counters into ``out_host`` (a pinned uint64 tensor or
+    array of >= 3 elements) on ``stream``; read it after an event recorded behind it."""
+    _check(lib.cof_counts_async(plan.handle, _ptr(plan_dev), _ptr(out_host), _stream(stream)))
 
 
 def _collect_fn(plan):

@@ -186,6 +186,14 @@ cof_status cof_load_chunk(const cof_chunk* host, cof_chunk* dev, cof_stream s) {
     return COF_OK;
 }
 
+cof_status cof_counts_async(const cof_plan* plan, const void* plan_dev, uint64_t* out_host, cof_stream s) {
+    if (!plan || !plan_dev || !out_host) return set_error(COF_E_ARG, "cof_counts_async: NULL argument");
+    cudaError_t e = cudaMemcpyAsync(out_host, (const uint8_t*)plan_dev + plan->lay.counters, 3 * sizeof(uint64_t),
+                                    cudaMemcpyDeviceToHost, (cudaStream_t)s);
+    if (e != cudaSuccess) return cuda_error(e, "cof_counts_async");
+    return COF_OK;
+}
+
 cof_status cof_read_counts(const cof_plan* plan, const void* plan_dev, uint64_t out[3], cof_stream s) {
     if (!plan || !plan_dev || !out) return set_error(COF_E_ARG, "cof_read_counts: NULL argument");
     uint64_t tmp[3];

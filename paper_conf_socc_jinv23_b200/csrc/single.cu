@@ -51,7 +51,7 @@ namespace cof {
 // addresses) is amortised over more lookups -- and 20 warps; many blocks (C5) take one
 // site per lane and 28 warps, which hides the filter's dependency latency better and keeps
 // all 32 blocks of a 1000-guide plan in one launch's shared memory.
-template <int W, int R, int S, int QB, int GUN>
+template <int W, int R, int S, int QB, int GUN, int KBN>
 struct SCfg {
     static constexpr int SW = W;                  // warps per CTA (one CTA per SM)
     static constexpr int STHREADS = 32 * W;
@@ -62,6 +62,8 @@ struct SCfg {
     static constexpr uint32_t SQ = 32u * R * QB;  // queued sites per warp (16-byte entries): QB batches
     static constexpr uint32_t SBATCH = 32u * R;
     static constexpr int GU = GUN;                // groups of 4 guide blocks per filter step
+    static constexpr int KB = KBN;                // batches whose survivors may carry over
+    static_assert((KB + 1) * 32 * R <= 32 * R * QB, "carried batches leave room to append");
     static constexpr uint32_t SVC = 32u * R * GU <= 32u ? 64u : 32u * R * GU <= 96u ? 128u : 256u;   // survivor ring
     static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH && (SQ & (SQ - 1)) == 0, "ring");
     static constexpr uint32_t SPW = 5u * SVC;     // per-warp words of the survivor ring
@@ -90,6 +92,12 @@ struct SCfg {
 #ifndef COF_MANY_G
 #define COF_MANY_G 2
 #endif
+#ifndef COF_FEW_K
+#define COF_FEW_K 1
+#endif
+#ifndef COF_MANY_K
+#define COF_MANY_K 1
+#endif
 #ifndef COF_MANY_W
 #define COF_MANY_W 28
 #endif
@@ -99,8 +107,8 @@ struct SCfg {
 #ifndef COF_MANY_S
 #define COF_MANY_S 4
 #endif
-using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q, COF_FEW_G>;
-using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S, COF_MANY_Q, COF_MANY_G>;
+using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q, COF_FEW_G, COF_FEW_K>;
+using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S, COF_MANY_Q, COF_MANY_G, COF_MANY_K>;
 constexpr uint32_t SFEW_BLOCKS = 8;       // guide blocks up to which SCfgFew runs
 constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
@@ -274,9 +282,9 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     const uint32_t tb0 = smem_u32(s_ftab), tb1 = tb0 + nb * FBW * 4 + 64;
     const uint4* vrec1 = s_vrec + nb * 32 * VSTR + 4;
     uint32_t head = 0, q_n = 0;           // warp-uniform site ring state
-    // Survivor entries carry over from one batch to the next (the last verification round of
-    // a batch would otherwise run mostly empty): the previous batch's queue slots stay
-    // reserved (resv) until the next batch ends, when every survivor is verified.
+    // Survivor entries carry over from one batch to the next, up to KB batches (the last
+    // verification round of a batch would otherwise run mostly empty): those batches' queue
+    // slots stay reserved (resv) until a batch ends with a full drain.
     uint32_t sv_h = 0, sv_n = 0, resv = 0;
     unsigned long long cnt_f = 0, cnt_r = 0;
 
@@ -288,42 +296,43 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     // active lane; the round's hits are appended with one atomic.  Returns
     // the number of entries re-appended.
     auto flush = [&](uint32_t sv_h, uint32_t n, uint32_t tail) -> uint32_t {
-        uint32_t m0 = 0, m1 = 0, m2 = 0, m3 = 0, x = 0;
-        bool have = (uint32_t)lane < n;
-        if (have) {
-            const uint32_t e = (sv_h + lane) & (SVC - 1);
-            x = sv_x[e];
-            const uint4 mv = sv_m[e];
-            m0 = mv.x; m1 = mv.y; m2 = mv.z; m3 = mv.w;
+        // branch-free: every lane reads an entry slot of the ring (in bounds; stale for lanes
+        // >= n, whose masks are zeroed); the stored masks are the filter's FAIL masks (a set
+        // bit = no survivor), so the survivors are their complement
+        const bool have = (uint32_t)lane < n;
+        const uint32_t e = (sv_h + lane) & (SVC - 1);
+        const uint32_t x = sv_x[e];
+        const uint4 mv = sv_m[e];
+        const uint32_t keep = have ? ~0u : 0u;
+        uint32_t m0 = ~mv.x & keep, m1 = ~mv.y & keep, m2 = ~mv.z & keep, m3 = ~mv.w & keep;
+        const bool z0 = m0 == 0u, z1 = m1 == 0u, z2 = m2 == 0u;
+        const uint32_t sel = !z0 ? m0 : (!z1 ? m1 : (!z2 ? m2 : m3));
+        const uint32_t bi = !z0 ? 0u : (!z1 ? 32u : (!z2 ? 64u : 96u));
+        const uint32_t low = sel & (0u - sel);
+        m0 ^= !z0 ? low : 0u;
+        m1 ^= z0 && !z1 ? low : 0u;
+        m2 ^= z0 && z1 && !z2 ? low : 0u;
+        m3 ^= z0 && z1 && z2 ? low : 0u;
+        const bool any = sel != 0u;
+        const uint32_t g = any ? (x >> 8) * 128u + bi + (31u - (uint32_t)__clz(low)) : 0u;   // launch-local guide
+        COF_ASSERT(g < a.n_blocks * 32u, "single: survivor guide inside the launch");
+        const uint4 it = queue[x & (SQ - 1)];
+        const uint32_t pos = it.x, sd = it.w >> 31;
+        const uint32_t wl = it.y, wh = it.z, wn = it.w & 0x7FFFFFFFu;
+        const uint4* rec = (sd ? vrec1 : s_vrec) + g * VSTR;
+        const uint4 r0 = rec[0];                                      // {lo, hi, care, t}
+        uint32_t mis;
+        if constexpr (CONCRETE) {
+            mis = ((wl ^ r0.x) | (wh ^ r0.y) | wn) & r0.z;
+        } else {
+            const uint4 oh = rec[1];                                  // one-hot {A, C, G, T}
+            const uint32_t nn = ~wn;
+            const uint32_t match = (oh.x & ~wl & ~wh & nn) | (oh.y & wl & ~wh & nn) |
+                                   (oh.z & ~wl & wh & nn) | (oh.w & wl & wh & nn);
+            mis = r0.z & ~match;
         }
-        bool hit = false;
-        uint32_t g = 0, mm = 0, pos = 0, sd = 0;
-        if (have) {
-            const uint32_t sel = m0 ? m0 : (m1 ? m1 : (m2 ? m2 : m3));
-            const uint32_t bi = m0 ? 0u : (m1 ? 32u : (m2 ? 64u : 96u));
-            const uint32_t low = sel & (0u - sel);
-            if (m0) m0 ^= low; else if (m1) m1 ^= low; else if (m2) m2 ^= low; else m3 ^= low;
-            g = (x >> 8) * 128u + bi + (uint32_t)(__ffs(low) - 1);    // launch-local guide
-            COF_ASSERT(g < a.n_blocks * 32u, "single: survivor guide inside the launch");
-            const uint4 it = queue[x & (SQ - 1)];
-            pos = it.x;
-            sd = it.w >> 31;
-            const uint32_t wl = it.y, wh = it.z, wn = it.w & 0x7FFFFFFFu;
-            const uint4* rec = (sd ? vrec1 : s_vrec) + g * VSTR;
-            const uint4 r0 = rec[0];                                  // {lo, hi, care, t}
-            uint32_t mis;
-            if constexpr (CONCRETE) {
-                mis = ((wl ^ r0.x) | (wh ^ r0.y) | wn) & r0.z;
-            } else {
-                const uint4 oh = rec[1];                              // one-hot {A, C, G, T}
-                const uint32_t nn = ~wn;
-                const uint32_t match = (oh.x & ~wl & ~wh & nn) | (oh.y & wl & ~wh & nn) |
-                                       (oh.z & ~wl & wh & nn) | (oh.w & wl & wh & nn);
-                mis = r0.z & ~match;
-            }
-            mm = (uint32_t)__popc(mis);
-            hit = mm <= r0.w;
-        }
+        const uint32_t mm = (uint32_t)__popc(mis);
+        const bool hit = any && mm <= r0.w;
         const unsigned hm = __ballot_sync(0xFFFFFFFFu, hit);
         if (hm) {
             const int leader = __ffs(hm) - 1;
@@ -339,7 +348,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         if (more) {
             const uint32_t e = (tail + (uint32_t)__popc(mb & lanemask_lt())) & (SVC - 1);
             sv_x[e] = x;
-            sv_m[e] = make_uint4(m0, m1, m2, m3);
+            sv_m[e] = make_uint4(~m0, ~m1, ~m2, ~m3);
         }
         return (uint32_t)__popc(mb);
     };
@@ -396,7 +405,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                             const uint32_t e = (sv_h + sv_n + (uint32_t)__popc(hb & lanemask_lt())) & (SVC - 1);
                             if (has) {
                                 sv_x[e] = ((head + (uint32_t)r * 32 + lane) & (SQ - 1)) | ((bg >> 2) << 8);
-                                sv_m[e] = make_uint4(p0, p1, p2, p3);
+                                sv_m[e] = make_uint4(~p0, ~p1, ~p2, ~p3);   // fail masks (see flush)
                             }
                             sv_n += (uint32_t)__popc(hb);
                             COF_ASSERT(sv_n <= SVC, "single: survivor ring capacity");
@@ -412,7 +421,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
                 // (at most 31 + SR x GU x 32 entries are queued: SVC holds them; a round takes 32 and
                 // puts back at most 32, and every round verifies one survivor per entry taken)
                 // (a batch that keeps its survivors for the next one verifies only full rounds)
-                const bool keep = resv == 0u && n_items == SBATCH && !tiles_done;
+                const bool keep = resv < (uint32_t)CFG::KB * SBATCH && n_items == SBATCH && !tiles_done;
                 while (sv_n >= 32 || (drain && !keep && sv_n > 0)) {
                     const uint32_t nf = min(sv_n, 32u);
                     COF_ASSERT(nf <= 32 && sv_n <= SVC, "single: verification round size");
@@ -429,7 +438,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             q_n -= n_items;
             // this batch's slots stay reserved while survivors may still reference them; after a
             // full drain nothing is pending
-            resv = (sv_n > 0u) ? SBATCH : 0u;
+            resv = (sv_n > 0u) ? resv + SBATCH : 0u;
             continue;
         }
         if (tiles_done) break;

@@ -11,6 +11,7 @@ from __future__ import annotations
 
 import dataclasses
 import heapq
+import itertools
 import os
 
 import numpy as np
@@ -291,8 +292,13 @@ class ResidentGenome:
         return sum(d.numel() * 4 for d in self.d_planes)
 
 
-SPLIT_FILL = os.environ.get("COF_SPLIT_FILL", "0") == "1"   # measured slower end to end
-PLANE_BUFS = int(os.environ.get("COF_PLANE_BUFS", 2))   # device plane sets in the search_host pipeline (3 measured no faster)
+# search_host pipeline: the N / valid-start fills on the compute stream (on the
+# copy stream they queue behind the persistent kernel that holds every SM), three device
+# plane sets (the H2D runs two chunks ahead) and three record buffers (a chunk's hit count
+# is read two chunks late, so the host never idles the GPU)
+SPLIT_FILL = os.environ.get("COF_SPLIT_FILL", "1") == "1"
+PLANE_BUFS = int(os.environ.get("COF_PLANE_BUFS", 3))
+REC_BUFS = int(os.environ.get("COF_REC_BUFS", 3))
 if PLANE_BUFS < 2:
     # with one plane set chunk j+1's H2D would overwrite the planes chunk j is searched on
     raise ValueError(f"COF_PLANE_BUFS={PLANE_BUFS}: the search_host pipeline needs at least 2 device plane sets")
@@ -389,6 +395,29 @@ class Searcher:
                           self.d_sort_ws, s)
         return nf, nr, nh
 
+    def enqueue_device_chunk(self, dchunk: cof.cof_chunk, items_cap: int):
+        """find -> compare -> sort on the device with every count left on the device: no
+        host synchronisation (a capacity overflow shows in the device hit count, which the
+        caller reads later, cof_counts_async)."""
+        s = self.stream
+        ON = cof.COF_COUNT_ON_DEVICE
+        if not self.fused and self.d_items.shape[1] < items_cap:
+            self.d_items = torch.empty((2, items_cap), dtype=torch.int32, device=self.device)
+        if self.path == "single":
+            cof.cof_search_single(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_hits, self._hits_cap, s,
+                                  sync=False)
+        elif self.path == "fused":
+            cof.cof_find_masks(self.plan, self.plan_dev, dchunk, self.d_find_ws, s)
+            cof.cof_compare_masks(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_hits, self._hits_cap, s,
+                                  sync=False)
+        else:
+            cof.cof_find_pam(self.plan, self.plan_dev, dchunk, self.d_find_ws, self.d_items[0], self.d_items[1],
+                             items_cap, s, sync=False)
+            cof.cof_compare(self.plan, self.plan_dev, dchunk, self.d_items[0], ON, self.d_items[1], ON, self.d_hits,
+                            self._hits_cap, s, sync=False)
+        cof.cof_sort_hits(self.plan, self.plan_dev, dchunk, self.d_hits, self.d_tmp, self._hits_cap, ON,
+                          self.d_sort_ws, s)
+
     def search_host(self, host: HostGenome, indices=None, out=None, decorate="device", sink=None):
         """End-to-end over host-resident packed chunks.  Per chunk: H2D on a copy stream
         (double-buffered device planes, overlapping the previous chunk's kernels), find,
@@ -424,7 +453,7 @@ class Searcher:
             self.d2h_stream = torch.cuda.Stream(self.device)
         planes = [self.d_planes] + self.d_planes_more
         nb = len(planes)
-        rec_free = [None, None]
+        rec_free = [None] * REC_BUFS
         use_out = out is not None and sink is None
         ws_bytes = cof.cof_decorate_workspace_bytes(max_segs)
         ws = []                    # one decoration workspace (key-check flag) per chunk
@@ -461,55 +490,93 @@ class Searcher:
                     return dch
 
             dchs = [None] * nb
-            cur = next(it, None)
-            if cur is not None:
-                dchs[0] = load(0, cur, 0)
-            j = 0
-            while cur is not None:
-                i = cur
-                nxt = next(it, None)
-                k, kr = j % nb, j & 1
-                self.stream.wait_event(loaded[k])
-                if nxt is not None:
-                    if host.chunks[nxt].n_bases > self._cap_bases:
-                        raise ValueError(f"chunk {nxt} is larger than the chunks this call was sized for")
-                    dchs[(j + 1) % nb] = load(j + 1, nxt, (j + 1) % nb)
-                mark("dev0", j, self.stream)
-                _, _, nh = self.run_device_chunk(dchs[k], host.chunks[i].n_owned, counts=False)
-                if self.d_records is None or nh > self._rec_cap:
-                    self._reserve_records(nh)
-                recs = self.d_records[kr]
-                if rec_free[kr] is not None:         # the D2H of chunk j-2 from this buffer is done
-                    self.stream.wait_event(rec_free[kr])
-                ws.append(torch.empty(ws_bytes, dtype=torch.uint8, device=self.device))
-                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, nh, recs, ws[-1], self.stream,
-                                 cap=self._rec_cap)
-                mark("dev1", j, self.stream)
-                fr = torch.cuda.Event()
-                fr.record(self.stream)
-                freed[k] = fr
+            # Chunk j's kernels, sort and decoration run with every count on the device; its
+            # hit count reaches pinned host memory asynchronously and is read only after chunk
+            # j + 1 is queued, so the host never idles the GPU between chunks.  A count above
+            # the hit / record capacity restarts the call with larger buffers.
+            cnt_host = torch.zeros((REC_BUFS, 3), dtype=torch.int64, pin_memory=True)
+            consumed = []              # chunk indices taken from ``it`` (a restart replays them)
+            pending = []               # (chunk index, record buffer, event) awaiting their counts
+            need = 0
+
+            def finish(p):
+                nonlocal total, overflow, last_i, need
+                i_, kr_, ev_ = p
+                ev_.synchronize()
+                nh = int(cnt_host[kr_][2])
+                if nh > self._hits_cap or nh > self._rec_cap:
+                    need = max(need, nh)
+                    return
                 dst = None
                 if use_out and not overflow:
-                    if i > last_i and total + nh <= len(out):
+                    if i_ > last_i and total + nh <= len(out):
                         dst = out[total:total + nh]
                     else:
                         overflow = True
                 if dst is None:
                     dst = torch.empty(max(nh, 1) * self.hit_dtype.itemsize, dtype=torch.uint8,
                                       pin_memory=True).numpy().view(self.hit_dtype)[:nh]
-                if nh:   # D2H on its own stream: overlaps the next chunk's kernels (and H2D)
-                    self.d2h_stream.wait_event(fr)
+                if nh:   # D2H on its own stream: overlaps the next chunks' kernels (and H2D)
+                    self.d2h_stream.wait_event(ev_)
                     with torch.cuda.stream(self.d2h_stream):
-                        torch.from_numpy(dst.view(np.uint8)).copy_(recs[: nh * self.hit_dtype.itemsize],
+                        torch.from_numpy(dst.view(np.uint8)).copy_(self.d_records[kr_][: nh * self.hit_dtype.itemsize],
                                                                    non_blocking=True)
-                        ev = torch.cuda.Event()
-                        ev.record(self.d2h_stream)
-                    rec_free[kr] = ev
-                results.append((i, dst))
+                        e2 = torch.cuda.Event()
+                        e2.record(self.d2h_stream)
+                    rec_free[kr_] = e2
+                results.append((i_, dst))
                 total += nh
-                last_i = i
+                last_i = i_
+
+            if self.d_records is None:
+                self._reserve_records(self._hits_cap)
+            cur = next(it, None)
+            if cur is not None:
+                consumed.append(cur)
+                dchs[0] = load(0, cur, 0)
+            j = 0
+            while cur is not None:
+                i = cur
+                nxt = next(it, None)
+                if nxt is not None:
+                    consumed.append(nxt)
+                k, kr = j % nb, j % REC_BUFS
+                self.stream.wait_event(loaded[k])
+                if nxt is not None:
+                    if host.chunks[nxt].n_bases > self._cap_bases:
+                        raise ValueError(f"chunk {nxt} is larger than the chunks this call was sized for")
+                    dchs[(j + 1) % nb] = load(j + 1, nxt, (j + 1) % nb)
+                mark("dev0", j, self.stream)
+                self.enqueue_device_chunk(dchs[k], host.chunks[i].n_owned)
+                if rec_free[kr] is not None:         # the D2H of chunk j-2 from this buffer is done
+                    self.stream.wait_event(rec_free[kr])
+                ws.append(torch.empty(ws_bytes, dtype=torch.uint8, device=self.device))
+                cof.cof_decorate(self.plan, self.plan_dev, dchs[k], self.d_hits, cof.COF_COUNT_ON_DEVICE,
+                                 self.d_records[kr], ws[-1], self.stream, cap=min(self._rec_cap, self._hits_cap))
+                cof.cof_counts_async(self.plan, self.plan_dev, cnt_host[kr], self.stream)
+                mark("dev1", j, self.stream)
+                fr = torch.cuda.Event()
+                fr.record(self.stream)
+                freed[k] = fr
+                pending.append((i, kr, fr))
+                # finish every chunk that is done (its records' D2H starts at once), and block
+                # only when all record buffers are in flight
+                while pending and not need and (len(pending) >= REC_BUFS or pending[0][2].query()):
+                    finish(pending.pop(0))
+                if need:
+                    break
                 cur = nxt
                 j += 1
+            while pending and not need:
+                finish(pending.pop(0))
+            if need:   # a chunk's hits exceeded the buffers: grow them, replay every chunk taken
+                self.d2h_stream.synchronize()
+                self.stream.synchronize()
+                self.copy_stream.synchronize()
+                self.reserve(self._cap_bases, max(self._hits_cap, 2 * need + 1024))
+                self._reserve_records(2 * need)
+                return self.search_host(host, indices if listed else itertools.chain(consumed, it),
+                                        out=out, decorate=decorate, sink=sink)
             self.d2h_stream.synchronize()
             self.stream.synchronize()
             if trace:   # COF_TRACE=1: per-chunk H2D / device intervals in ms from the first mark
@@ -586,11 +653,12 @@ class Searcher:
         return merge_hit_lists(results, self.hit_dtype)
 
     def _reserve_records(self, n):
-        # two device record buffers: chunk j decorates into one while chunk j-1's D2H drains the other
+        # REC_BUFS device record buffers: chunk j decorates into one while the D2H of earlier
+        # chunks drains the others
         self.d2h_stream.synchronize() if hasattr(self, "d2h_stream") else None
         cap = int(n * 1.25 + 1024)
         self.d_records = [torch.empty(cap * self.hit_dtype.itemsize, dtype=torch.uint8, device=self.device)
-                          for _ in range(2)]
+                          for _ in range(REC_BUFS)]
         self._rec_cap = cap
 
     def _search_host_cpu_decorate(self, host: HostGenome, indices=None, out=None):
