@@ -560,10 +560,13 @@ class Searcher:
                 freed[k] = fr
                 pending.append((i, kr, fr))
                 # finish every chunk that is done (its records' D2H starts at once), and block
-                # only when all record buffers are in flight
-                while pending and not need and (len(pending) >= REC_BUFS or pending[0][2].query()):
+                # only when all record buffers are in flight -- or for the first chunk, whose
+                # count sizes the buffers before more chunks are queued on a guess
+                while pending and not need and (len(pending) >= REC_BUFS or j == 0 or pending[0][2].query()):
                     finish(pending.pop(0))
                 if need:
+                    # (scaled to the largest chunk: chunk sizes differ)
+                    need = int(need * max(1.0, max_bases / max(1, host.chunks[i].n_bases)))
                     break
                 cur = nxt
                 j += 1
@@ -609,43 +612,66 @@ class Searcher:
             self.d2h_stream = torch.cuda.Stream(self.device)
         ws_bytes = cof.cof_decorate_workspace_bytes(max((len(ch.pieces) for ch in rg.chunks), default=1))
         ws, results = [], []
-        rec_free = [None, None]
-        total, overflow = 0, False
+        rec_free = [None] * REC_BUFS
+        total, overflow, need = 0, False, 0
+        cnt_host = torch.zeros((REC_BUFS, 3), dtype=torch.int64, pin_memory=True)
+        pending = []
+        if self.d_records is None:
+            self._reserve_records(self._hits_cap)
+
+        def finish(p):   # as in search_host: the chunk is done, its count is in pinned memory
+            nonlocal total, overflow, need
+            kr_, ev_ = p
+            ev_.synchronize()
+            nh = int(cnt_host[kr_][2])
+            if nh > self._hits_cap or nh > self._rec_cap:
+                need = max(need, nh)
+                return
+            dst = None
+            if out is not None and not overflow:
+                if total + nh <= len(out):
+                    dst = out[total:total + nh]
+                else:
+                    overflow = True
+            if dst is None:
+                dst = torch.empty(max(nh, 1) * self.hit_dtype.itemsize, dtype=torch.uint8,
+                                  pin_memory=True).numpy().view(self.hit_dtype)[:nh]
+            if nh:
+                self.d2h_stream.wait_event(ev_)
+                with torch.cuda.stream(self.d2h_stream):
+                    torch.from_numpy(dst.view(np.uint8)).copy_(self.d_records[kr_][: nh * self.hit_dtype.itemsize],
+                                                               non_blocking=True)
+                    e2 = torch.cuda.Event()
+                    e2.record(self.d2h_stream)
+                rec_free[kr_] = e2
+            results.append(dst)
+            total += nh
+
         with torch.cuda.device(self.device):
             for j, (ch, dch) in enumerate(zip(rg.chunks, rg.d_chunks)):
-                kr = j & 1
-                _, _, nh = self.run_device_chunk(dch, ch.n_owned, counts=False)
-                if self.d_records is None or nh > self._rec_cap:
-                    self._reserve_records(nh)
-                recs = self.d_records[kr]
+                kr = j % REC_BUFS
+                self.enqueue_device_chunk(dch, ch.n_owned)
                 if rec_free[kr] is not None:
                     self.stream.wait_event(rec_free[kr])
                 ws.append(torch.empty(ws_bytes, dtype=torch.uint8, device=self.device))
-                cof.cof_decorate(self.plan, self.plan_dev, dch, self.d_hits, nh, recs, ws[-1], self.stream,
-                                 cap=self._rec_cap)
+                cof.cof_decorate(self.plan, self.plan_dev, dch, self.d_hits, cof.COF_COUNT_ON_DEVICE,
+                                 self.d_records[kr], ws[-1], self.stream, cap=min(self._rec_cap, self._hits_cap))
+                cof.cof_counts_async(self.plan, self.plan_dev, cnt_host[kr], self.stream)
                 fr = torch.cuda.Event()
                 fr.record(self.stream)
-                dst = None
-                if out is not None and not overflow:
-                    if total + nh <= len(out):
-                        dst = out[total:total + nh]
-                    else:
-                        overflow = True
-                if dst is None:
-                    dst = torch.empty(max(nh, 1) * self.hit_dtype.itemsize, dtype=torch.uint8,
-                                      pin_memory=True).numpy().view(self.hit_dtype)[:nh]
-                if nh:
-                    self.d2h_stream.wait_event(fr)
-                    with torch.cuda.stream(self.d2h_stream):
-                        torch.from_numpy(dst.view(np.uint8)).copy_(recs[: nh * self.hit_dtype.itemsize],
-                                                                   non_blocking=True)
-                        ev = torch.cuda.Event()
-                        ev.record(self.d2h_stream)
-                    rec_free[kr] = ev
-                results.append(dst)
-                total += nh
+                pending.append((kr, fr))
+                while pending and not need and (len(pending) >= REC_BUFS or pending[0][1].query()):
+                    finish(pending.pop(0))
+                if need:
+                    break
+            while pending and not need:
+                finish(pending.pop(0))
             self.d2h_stream.synchronize()
             self.stream.synchronize()
+            if need:   # grow the buffers and search again
+                self.reserve(self._cap_bases, max(self._hits_cap, 2 * need + 1024))
+                self._reserve_records(2 * need)
+                return self.search_resident(rg, out=out)
             for w in ws:
                 cof.cof_decorate_check(w, self.stream)
         if out is not None and not overflow:
