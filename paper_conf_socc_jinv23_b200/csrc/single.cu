@@ -93,7 +93,7 @@ struct SCfg {
 #define COF_MANY_G 2
 #endif
 #ifndef COF_FEW_K
-#define COF_FEW_K 1
+#define COF_FEW_K 3
 #endif
 #ifndef COF_MANY_K
 #define COF_MANY_K 1

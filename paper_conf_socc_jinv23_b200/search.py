@@ -883,7 +883,13 @@ def _merge_arena(nbytes: int, group, dst: int, shm_dir=None):
         size = max(int(nbytes * 1.25), 1 << 20)
         name = [None]
         if dist.get_rank(group) == dst:
-            d = shm_dir or ("/dev/shm" if os.path.isdir("/dev/shm") else tempfile.gettempdir())
+            d = shm_dir
+            if d is None:   # /dev/shm when it has room (a container's may be 64 MB), else the temp dir
+                d = tempfile.gettempdir()
+                if os.path.isdir("/dev/shm"):
+                    st = os.statvfs("/dev/shm")
+                    if st.f_bavail * st.f_frsize >= size + (64 << 20):
+                        d = "/dev/shm"
             name[0] = os.path.join(d, f"cof_merge_{uuid.uuid4().hex}.bin")
             with open(name[0], "wb") as f:
                 f.truncate(size)
