@@ -51,7 +51,7 @@ namespace cof {
 // addresses) is amortised over more lookups -- and 20 warps; many blocks (C5) take one
 // site per lane and 28 warps, which hides the filter's dependency latency better and keeps
 // all 32 blocks of a 1000-guide plan in one launch's shared memory.
-template <int W, int R, int S, int QB, int GUN, int KBN>
+template <int W, int R, int S, int QB, int GUN, int KBN, int WPLN>
 struct SCfg {
     static constexpr int SW = W;                  // warps per CTA (one CTA per SM)
     static constexpr int STHREADS = 32 * W;
@@ -63,6 +63,9 @@ struct SCfg {
     static constexpr uint32_t SBATCH = 32u * R;
     static constexpr int GU = GUN;                // groups of 4 guide blocks per filter step
     static constexpr int KB = KBN;                // batches whose survivors may carry over
+    static constexpr int WPL = WPLN;              // plane words per lane and chunk
+    static constexpr int CPT = W / WPLN;          // chunks per tile
+    static_assert(W % WPLN == 0, "whole chunks per tile");
     static_assert((KB + 1) * 32 * R <= 32 * R * QB, "carried batches leave room to append");
     static constexpr uint32_t SVC = 32u * R * GU <= 32u ? 64u : 32u * R * GU <= 96u ? 128u : 256u;   // survivor ring
     static_assert(SQ % SBATCH == 0 && SQ >= 2 * SBATCH && (SQ & (SQ - 1)) == 0, "ring");
@@ -107,8 +110,14 @@ struct SCfg {
 #ifndef COF_MANY_S
 #define COF_MANY_S 4
 #endif
-using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q, COF_FEW_G, COF_FEW_K>;
-using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S, COF_MANY_Q, COF_MANY_G, COF_MANY_K>;
+#ifndef COF_SPARSE_WPL
+#define COF_SPARSE_WPL 2
+#endif
+using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q, COF_FEW_G, COF_FEW_K, 1>;
+// few blocks and a sparse PAM (Cas12a TTTV): several plane words per lane and chunk, so the
+// per-chunk work (tile bookkeeping, the append's scan) is spread over more sites
+using SCfgSparse = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q, COF_FEW_G, COF_FEW_K, COF_SPARSE_WPL>;
+using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S, COF_MANY_Q, COF_MANY_G, COF_MANY_K, 1>;
 constexpr uint32_t SFEW_BLOCKS = 8;       // guide blocks up to which SCfgFew runs
 constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
@@ -208,6 +217,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     constexpr int SSTAGES = CFG::SSTAGES, SR = CFG::SR;
     constexpr uint32_t SQ = CFG::SQ, SBATCH = CFG::SBATCH, SVC = CFG::SVC;
     constexpr int GU = CFG::GU;
+    constexpr int WPL = CFG::WPL, CPT = CFG::CPT;
     extern __shared__ __align__(128) uint8_t smem[];
     // layout: [filter tables: '+' n_blocks x FBW words, 64 B, '-' likewise]
     //         [verification records: '+' n_blocks*32 x VS uint4, 64 B, '-' likewise]
@@ -354,8 +364,13 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
     };
 
     // per-lane state of the tile being appended: its plane words and the PAM bits not yet queued
-    uint32_t lo0 = 0, lo1 = 0, lo2 = 0, hi0 = 0, hi1 = 0, hi2 = 0, nm0 = 0, nm1 = 0, nm2 = 0;
-    uint32_t pend0 = 0u, pend1 = 0u, pbase = 0;
+    // (WPL consecutive plane words per lane and chunk: lo[q] .. lo[q + 2] hold word q's windows)
+    uint32_t lo[WPL + 2], hi[WPL + 2], nm[WPL + 2], pend[2][WPL];
+#pragma unroll
+    for (int q = 0; q < WPL + 2; q++) lo[q] = hi[q] = nm[q] = 0u;
+#pragma unroll
+    for (int q = 0; q < WPL; q++) pend[0][q] = pend[1][q] = 0u;
+    uint32_t pbase = 0;
     bool tiles_done = false;
     // One loop, one call site each for the batch comparison and the queue append (the
     // kernel's code stays small): compare while a full batch is queued, else append the
@@ -442,14 +457,23 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             continue;
         }
         if (tiles_done) break;
-        if (__any_sync(0xFFFFFFFFu, (pend0 | pend1) != 0u)) {
+        uint32_t anyp = 0u;
+#pragma unroll
+        for (int q = 0; q < WPL; q++) anyp |= pend[0][q] | pend[1][q];
+        if (__any_sync(0xFFFFFFFFu, anyp != 0u)) {
             // ---------------- append pending sites: a warp scan ranks the lanes' sites ('+' before
             // '-' within a lane), and every lane writes the queue entries of its own sites that fit
             // (rank < take), each the site's three 32-base windows funnel-shifted out of the
             // lane's registers at the strand's first compared offset p0 (bit 31 of the N window
             // carries the strand).  The order of entries in the queue is immaterial (hits are
             // sorted afterwards); a site that does not fit stays pending for the next append.
-            const uint32_t c0 = (uint32_t)__popc(pend0), c = c0 + (uint32_t)__popc(pend1);
+            uint32_t cs[2] = {0u, 0u};
+#pragma unroll
+            for (int q = 0; q < WPL; q++) {
+                cs[0] += (uint32_t)__popc(pend[0][q]);
+                cs[1] += (uint32_t)__popc(pend[1][q]);
+            }
+            const uint32_t c = cs[0] + cs[1];
             uint32_t x = c;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -460,44 +484,40 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             COF_ASSERT(q_n + resv <= SQ, "single: site queue occupancy");
             const uint32_t take = min(SQ - q_n - resv, total);
             const uint32_t first = x - c;
-            const uint32_t n_mine = min(c, take > first ? take - first : 0u);
-            const uint32_t pw = pbase + (uint32_t)lane * 32u;     // first start of this lane's word
+            uint32_t left = min(c, take > first ? take - first : 0u);   // this lane's sites that fit
+            const uint32_t pw = pbase + (uint32_t)lane * 32u * WPL;      // first start of this lane's words
             uint32_t slot = head + q_n + first;
-            const uint32_t nf = min(n_mine, c0);
-            if (nf) {
-                const uint32_t p0 = a.p0[0];
-                const uint32_t Al = __funnelshift_r(lo0, lo1, p0), Bl = __funnelshift_r(lo1, lo2, p0);
-                const uint32_t Ah = __funnelshift_r(hi0, hi1, p0), Bh = __funnelshift_r(hi1, hi2, p0);
-                const uint32_t An = __funnelshift_r(nm0, nm1, p0), Bn = __funnelshift_r(nm1, nm2, p0);
-                uint32_t m = pend0;
-                for (uint32_t i = 0; i < nf; i++) {
-                    const uint32_t low = m & (0u - m);
-                    const uint32_t bit = 31u - (uint32_t)__clz(low);
-                    m ^= low;
-                    queue[slot & (SQ - 1)] = make_uint4(pw + bit, __funnelshift_r(Al, Bl, bit),
-                                                        __funnelshift_r(Ah, Bh, bit),
-                                                        __funnelshift_r(An, Bn, bit) & 0x7FFFFFFFu);
-                    slot++;
+#pragma unroll
+            for (int sd = 0; sd < 2; sd++) {
+                const uint32_t ns = min(left, cs[sd]);
+                if (ns) {
+                    const uint32_t p0 = a.p0[sd];
+                    const uint32_t sbit = sd ? 0x80000000u : 0u;
+                    uint32_t L[WPL + 1], H[WPL + 1], N[WPL + 1];   // words shifted to the strand's offset p0
+#pragma unroll
+                    for (int q = 0; q <= WPL; q++) {
+                        L[q] = __funnelshift_r(lo[q], lo[q + 1], p0);
+                        H[q] = __funnelshift_r(hi[q], hi[q + 1], p0);
+                        N[q] = __funnelshift_r(nm[q], nm[q + 1], p0);
+                    }
+                    uint32_t todo = ns;
+#pragma unroll
+                    for (int q = 0; q < WPL; q++) {
+                        uint32_t m = pend[sd][q];
+                        while (todo && m) {
+                            const uint32_t low = m & (0u - m);
+                            const uint32_t bit = 31u - (uint32_t)__clz(low);
+                            m ^= low;
+                            todo--;
+                            queue[slot & (SQ - 1)] = make_uint4(pw + 32u * q + bit, __funnelshift_r(L[q], L[q + 1], bit),
+                                                                __funnelshift_r(H[q], H[q + 1], bit),
+                                                                (__funnelshift_r(N[q], N[q + 1], bit) & 0x7FFFFFFFu) | sbit);
+                            slot++;
+                        }
+                        pend[sd][q] = m;
+                    }
+                    left -= ns;
                 }
-                pend0 = m;
-            }
-            const uint32_t nr = n_mine - nf;
-            if (nr) {
-                const uint32_t p0 = a.p0[1];
-                const uint32_t Al = __funnelshift_r(lo0, lo1, p0), Bl = __funnelshift_r(lo1, lo2, p0);
-                const uint32_t Ah = __funnelshift_r(hi0, hi1, p0), Bh = __funnelshift_r(hi1, hi2, p0);
-                const uint32_t An = __funnelshift_r(nm0, nm1, p0), Bn = __funnelshift_r(nm1, nm2, p0);
-                uint32_t m = pend1;
-                for (uint32_t i = 0; i < nr; i++) {
-                    const uint32_t low = m & (0u - m);
-                    const uint32_t bit = 31u - (uint32_t)__clz(low);
-                    m ^= low;
-                    queue[slot & (SQ - 1)] = make_uint4(pw + bit, __funnelshift_r(Al, Bl, bit),
-                                                        __funnelshift_r(Ah, Bh, bit),
-                                                        __funnelshift_r(An, Bn, bit) | 0x80000000u);
-                    slot++;
-                }
-                pend1 = m;
             }
             __syncwarp();
             q_n += take;
@@ -510,7 +530,7 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
         uint32_t c = 0;
         if (lane == 0) c = atomicAdd(s_next, 1u);
         c = __shfl_sync(0xFFFFFFFFu, c, 0);
-        const uint32_t kk = c / (uint32_t)SW, chunk = c % (uint32_t)SW;
+        const uint32_t kk = c / (uint32_t)CPT, chunk = c % (uint32_t)CPT;
         const int st = (int)(kk % SSTAGES);
         mbar_wait_parity_sleep(&full[st], (kk / SSTAGES) & 1u);
         const uint32_t tile = s_tile[st];
@@ -519,34 +539,45 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             continue;
         }
         const uint32_t* S = ring + st * SPL * SLOAD;
-        const int w = (int)chunk * 32 + lane;
-        lo0 = S[w]; lo1 = S[w + 1]; lo2 = S[w + 2];
-        hi0 = S[SLOAD + w]; hi1 = S[SLOAD + w + 1]; hi2 = S[SLOAD + w + 2];
-        nm0 = S[2 * SLOAD + w]; nm1 = S[2 * SLOAD + w + 1]; nm2 = S[2 * SLOAD + w + 2];
-        uint32_t valid = vsp ? S[3 * SLOAD + w] : ~0u;
+        const int w = ((int)chunk * 32 + lane) * WPL;
+#pragma unroll
+        for (int q = 0; q < WPL + 2; q++) {
+            lo[q] = S[w + q];
+            hi[q] = S[SLOAD + w + q];
+            nm[q] = S[2 * SLOAD + w + q];
+        }
+        uint32_t valid[WPL];
+#pragma unroll
+        for (int q = 0; q < WPL; q++) valid[q] = vsp ? S[3 * SLOAD + w + q] : ~0u;
         __syncwarp();
-        if (lane == 0) {   // the chunk is in registers; the last of the tile's SW chunks refills the stage
+        if (lane == 0) {   // the chunk is in registers; the last of the tile's CPT chunks refills the stage
             __threadfence_block();
-            if (atomicAdd(&s_rel[st], 1u) == SW - 1) {
+            if (atomicAdd(&s_rel[st], 1u) == CPT - 1) {
                 s_rel[st] = 0;
                 __threadfence_block();
                 refill(st);
             }
         }
-        pbase = (uint32_t)(((uint64_t)tile * STW + chunk * 32u) * 32u);   // first start of lane 0's word
-        const uint64_t pw = (uint64_t)pbase + (uint32_t)lane * 32u;        // first start of this word
-        if (pw + 32 > a.limit) valid &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
-        pend0 = pend1 = valid;
-        for (uint32_t e = 0; e < a.ne; e++) {
-            const uint32_t j0 = a.pj[0][e], j1 = a.pj[1][e];
-            pend0 &= s_member(__funnelshift_r(lo0, lo1, j0), __funnelshift_r(hi0, hi1, j0),
-                              __funnelshift_r(nm0, nm1, j0), a.psel[0][e]);
-            pend1 &= s_member(__funnelshift_r(lo0, lo1, j1), __funnelshift_r(hi0, hi1, j1),
-                              __funnelshift_r(nm0, nm1, j1), a.psel[1][e]);
-        }
-        if (a.count_items) {
-            cnt_f += (unsigned)__popc(pend0);
-            cnt_r += (unsigned)__popc(pend1);
+        pbase = (uint32_t)(((uint64_t)tile * STW + chunk * 32u * WPL) * 32u);   // first start of lane 0's words
+#pragma unroll
+        for (int q = 0; q < WPL; q++) {
+            const uint64_t pw = (uint64_t)pbase + ((uint32_t)lane * WPL + q) * 32u;   // first start of word q
+            uint32_t v = valid[q];
+            if (pw + 32 > a.limit) v &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
+            uint32_t p0m = v, p1m = v;
+            for (uint32_t e = 0; e < a.ne; e++) {
+                const uint32_t j0 = a.pj[0][e], j1 = a.pj[1][e];
+                p0m &= s_member(__funnelshift_r(lo[q], lo[q + 1], j0), __funnelshift_r(hi[q], hi[q + 1], j0),
+                                __funnelshift_r(nm[q], nm[q + 1], j0), a.psel[0][e]);
+                p1m &= s_member(__funnelshift_r(lo[q], lo[q + 1], j1), __funnelshift_r(hi[q], hi[q + 1], j1),
+                                __funnelshift_r(nm[q], nm[q + 1], j1), a.psel[1][e]);
+            }
+            pend[0][q] = p0m;
+            pend[1][q] = p1m;
+            if (a.count_items) {
+                cnt_f += (unsigned)__popc(p0m);
+                cnt_r += (unsigned)__popc(p1m);
+            }
         }
     }
     if (a.count_items) {
@@ -566,8 +597,9 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
 typedef void (*SingleFn)(SingleArgs);
 
 template <int NP, int TC, bool CONCRETE>
-static SingleFn single_fn_t(bool few) {
-    return few ? cof_single_kernel<NP, TC, CONCRETE, SCfgFew> : cof_single_kernel<NP, TC, CONCRETE, SCfgMany>;
+static SingleFn single_fn_t(int geo) {   // 0: many blocks, 1: few, 2: few + sparse PAM
+    return geo == 1 ? cof_single_kernel<NP, TC, CONCRETE, SCfgFew>
+         : geo == 2 ? cof_single_kernel<NP, TC, CONCRETE, SCfgSparse> : cof_single_kernel<NP, TC, CONCRETE, SCfgMany>;
 }
 
 // The kernel variant a plan runs: uniform-threshold, concrete-letter specialisations for
@@ -578,43 +610,43 @@ static bool single_uses_concrete(uint32_t np, int tc, bool concrete) {
 }
 
 template <int NP>
-static SingleFn single_fn_np(int tc, bool concrete, bool few) {
+static SingleFn single_fn_np(int tc, bool concrete, int geo) {
     if constexpr (NP == 10 || NP == 12) {
         if (concrete) {
             switch (tc) {
-                case 0: return single_fn_t<NP, 0, true>(few);
-                case 1: return single_fn_t<NP, 1, true>(few);
-                case 2: return single_fn_t<NP, 2, true>(few);
-                case 3: return single_fn_t<NP, 3, true>(few);
-                case 4: return single_fn_t<NP, 4, true>(few);
-                case 5: return single_fn_t<NP, 5, true>(few);
-                case 6: return single_fn_t<NP, 6, true>(few);
-                case 7: return single_fn_t<NP, 7, true>(few);
+                case 0: return single_fn_t<NP, 0, true>(geo);
+                case 1: return single_fn_t<NP, 1, true>(geo);
+                case 2: return single_fn_t<NP, 2, true>(geo);
+                case 3: return single_fn_t<NP, 3, true>(geo);
+                case 4: return single_fn_t<NP, 4, true>(geo);
+                case 5: return single_fn_t<NP, 5, true>(geo);
+                case 6: return single_fn_t<NP, 6, true>(geo);
+                case 7: return single_fn_t<NP, 7, true>(geo);
                 default: break;
             }
         }
     }
-    return single_fn_t<NP, -1, false>(few);
+    return single_fn_t<NP, -1, false>(geo);
 }
 
-static SingleFn single_fn(uint32_t np, int tc, bool concrete, bool few) {
+static SingleFn single_fn(uint32_t np, int tc, bool concrete, int geo) {
     switch (np) {
-        case 1: return single_fn_np<1>(tc, concrete, few);
-        case 2: return single_fn_np<2>(tc, concrete, few);
-        case 3: return single_fn_np<3>(tc, concrete, few);
-        case 4: return single_fn_np<4>(tc, concrete, few);
-        case 5: return single_fn_np<5>(tc, concrete, few);
-        case 6: return single_fn_np<6>(tc, concrete, few);
-        case 7: return single_fn_np<7>(tc, concrete, few);
-        case 8: return single_fn_np<8>(tc, concrete, few);
-        case 9: return single_fn_np<9>(tc, concrete, few);
-        case 10: return single_fn_np<10>(tc, concrete, few);
-        case 11: return single_fn_np<11>(tc, concrete, few);
-        case 12: return single_fn_np<12>(tc, concrete, few);
-        case 13: return single_fn_np<13>(tc, concrete, few);
-        case 14: return single_fn_np<14>(tc, concrete, few);
-        case 15: return single_fn_np<15>(tc, concrete, few);
-        case 16: return single_fn_np<16>(tc, concrete, few);
+        case 1: return single_fn_np<1>(tc, concrete, geo);
+        case 2: return single_fn_np<2>(tc, concrete, geo);
+        case 3: return single_fn_np<3>(tc, concrete, geo);
+        case 4: return single_fn_np<4>(tc, concrete, geo);
+        case 5: return single_fn_np<5>(tc, concrete, geo);
+        case 6: return single_fn_np<6>(tc, concrete, geo);
+        case 7: return single_fn_np<7>(tc, concrete, geo);
+        case 8: return single_fn_np<8>(tc, concrete, geo);
+        case 9: return single_fn_np<9>(tc, concrete, geo);
+        case 10: return single_fn_np<10>(tc, concrete, geo);
+        case 11: return single_fn_np<11>(tc, concrete, geo);
+        case 12: return single_fn_np<12>(tc, concrete, geo);
+        case 13: return single_fn_np<13>(tc, concrete, geo);
+        case 14: return single_fn_np<14>(tc, concrete, geo);
+        case 15: return single_fn_np<15>(tc, concrete, geo);
+        case 16: return single_fn_np<16>(tc, concrete, geo);
         default: return nullptr;
     }
 }
@@ -625,7 +657,7 @@ struct SGeom {
 };
 template <class C>
 static SGeom sgeom() { return {C::STHREADS, C::STW, C::SLOAD, C::SSTAGES, C::SQ, C::SVC, (uint32_t)C::SW}; }
-static SGeom single_geom(bool few) { return few ? sgeom<SCfgFew>() : sgeom<SCfgMany>(); }
+static SGeom single_geom(int geo) { return geo == 1 ? sgeom<SCfgFew>() : geo == 2 ? sgeom<SCfgSparse>() : sgeom<SCfgMany>(); }
 
 static size_t single_smem(const SGeom& g, uint32_t np, uint32_t nb, bool concrete) {
     const size_t fbw = filter_block_words(np);
@@ -679,7 +711,7 @@ struct SinglePlanInfo {
     uint32_t np;
     int ut;            // the uniform threshold, -1 if the guides' thresholds differ
     bool concrete;     // the concrete-letter kernel runs
-    bool few;          // SCfgFew geometry
+    int geo;           // 0: SCfgMany, 1: SCfgFew, 2: SCfgSparse
     SGeom geom;
     uint32_t bpl;      // guide blocks per launch
 };
@@ -691,10 +723,21 @@ static SinglePlanInfo single_info(const cof_plan* plan) {
     for (uint32_t i = 1; i < plan->n_guides && I.ut >= 0; i++)
         if (plan->max_mm[i] != plan->max_mm[0]) I.ut = -1;
     I.concrete = single_uses_concrete(I.np, I.ut, !plan->any_degenerate);
-    // the few-blocks geometry when the plan's blocks fit one launch of it
-    I.few = plan->n_blocks <= SFEW_BLOCKS &&
-            single_smem(single_geom(true), I.np, (plan->n_blocks + 3) & ~3u, I.concrete) <= SMEM_MAX;
-    I.geom = single_geom(I.few);
+    // the few-blocks geometry when the plan's blocks fit one launch of it; its sparse variant
+    // when PAM sites are rarer than 0.03 per start and strand on a uniform genome (Cas12a
+    // TTTV: 0.012; NRG 0.125, NGG 0.0625)
+    const bool few = plan->n_blocks <= SFEW_BLOCKS &&
+                     single_smem(single_geom(1), I.np, (plan->n_blocks + 3) & ~3u, I.concrete) <= SMEM_MAX;
+    double d = 1.0;
+    for (uint32_t k = 0; k < plan->pam[0].n; k++) d *= __builtin_popcount(plan->pam[0].set[k]) / 4.0;
+    static int wpl_env = -2;
+    if (wpl_env == -2) {
+        const char* e = getenv("COF_SPARSE");   // 0: never the sparse geometry, 1: always (tests)
+        wpl_env = e ? atoi(e) : -1;
+    }
+    const bool sparse = wpl_env == 1 || (wpl_env != 0 && d < 0.03);
+    I.geo = few ? (sparse ? 2 : 1) : 0;
+    I.geom = single_geom(I.geo);
     I.bpl = single_blocks_per_launch(I.geom, I.np, I.concrete);
     return I;
 }
@@ -713,7 +756,7 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     uint64_t limit = dev->n_bases >= L ? dev->n_bases - L + 1 : 0;
     if (!dev->n_segs && limit > dev->n_owned) limit = dev->n_owned;
     const uint32_t n_tiles = (uint32_t)((limit + (uint64_t)G.stw * 32 - 1) / ((uint64_t)G.stw * 32));
-    SingleFn fn = single_fn(I.np, I.ut, I.concrete, I.few);
+    SingleFn fn = single_fn(I.np, I.ut, I.concrete, I.geo);
     if (!fn) return set_error(COF_E_STATE, "single pass: %u pairs", I.np);
     int dev_id = 0;
     cudaGetDevice(&dev_id);
