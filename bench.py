@@ -695,7 +695,7 @@ def traffic_for(kernel, st, cfgname):
 def popc_roof(n_sm, sm_mhz):
     """SURVEY §8(d)'s comparer roof: one POPC per comparison on the quarter-rate POPC pipe,
     16/clk/SM (measured 4.54e12 POPC/s = 15.6/clk/SM at 1965 MHz,
-    profiles/microbench_pipes_r1.txt)."""
+    profiles/microbench_pipes_r2.txt: 15.65/clk/SM at 1956 MHz)."""
     return 16.0 * n_sm * sm_mhz * 1e6
 
 
@@ -745,7 +745,7 @@ def table_roof(plan, n_sm, sm_mhz, impl):
     popc: 1 POPC per comparison, POPC = 16/clk/SM (measured, tools/microbench_pipes.cu).
     table: per item and 32-guide block, the minimal carry-save tree (FA/HA count from
     gen_csa for this plan's pair count) + 6-step borrow chain + 1 mask op, all LOP3 on
-    the 64/clk/SM ALU pipe (profiles/microbench_pipes_r1.txt); co-bound by shared memory: NP 64-bit lookups per item and
+    the 64/clk/SM ALU pipe (profiles/microbench_pipes_r2.txt); co-bound by shared memory: NP 64-bit lookups per item and
     block = 2*NP wavefronts per 32 items x 32 guides at 1 wavefront/clk/SM."""
     clk = sm_mhz * 1e6
     if impl == "popc":
@@ -771,7 +771,7 @@ def table_roof(plan, n_sm, sm_mhz, impl):
     alu_ops = 2 * fa + 2 * ha + 6 + 1
     # 64 LOP3/clk/SM: the ALU pipe issues one warp instruction per 2 cycles per SMSP
     # (B300_MICROARCH.md "Pipe rates"); measured 1.855e13 LOP3/s = 63.8/clk/SM at the
-    # 1965 MHz max clock (profiles/microbench_pipes_r1.txt; its own clock column is wrong)
+    # 1965 MHz max clock (profiles/microbench_pipes_r2.txt: 63.94 LOP3/clk/SM at a globaltimer-measured 1955 MHz)
     alu_rate = 64.0 * 32 / alu_ops           # comparisons / clk / SM
     lds_rate = 32.0 * 32 / (2 * npairs)      # comparisons / clk / SM
     per_clk = min(alu_rate, lds_rate)
