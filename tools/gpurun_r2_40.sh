@@ -1,4 +1,4 @@
-# round 2, call 40: checkpoint -- full GPU suite, full bench lines (all configs), C5 launch list,
+# round 2, call 40 (and 45): checkpoint -- full GPU suite, full bench lines (all configs), C5 launch list,
 # ncu --set full of the C5 single-pass kernel
 export PATH=/usr/local/cuda/bin:$PATH
 mkdir -p gpurun_out/r40
