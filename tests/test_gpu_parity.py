@@ -247,12 +247,15 @@ def test_sorted_keys_and_determinism():
 @pytest.mark.parametrize("name", ["C5", "C3", "C4"])
 def test_full_size_sampled(name):
     """C5 / C3 / C4 at full size on one GPU, in the bench's launch configuration (the whole
-    genome as one multi-segment chunk, device-resident planes, counts on device; fused
-    path for C5 and C3, two-call with the sparse-PAM finder pass 2 for C4); the oracle
-    recomputes sampled window ranges one by one."""
-    from bench import run_device_pipeline, prepare_workload   # same code the bench times
+    genome as one multi-segment chunk, device-resident planes, counts on device; the single
+    pass -- one launch, the sparse-PAM geometry for C4); the oracle recomputes sampled
+    window ranges one by one, every planted site is found with its exact count, and the
+    single pass's PAM-site counts equal the separate search kernel's (cof_find_pam)."""
+    from bench import run_device_pipeline, prepare_workload, time_search_kernel   # the bench's code
     wl, plan_obj = prepare_workload(name)
+    assert plan_obj.path_name == "single"
     res = run_device_pipeline(wl, plan_obj, collect=True)
+    time_search_kernel(plan_obj, 1)    # raises unless its item counts equal the step's
     rng = np.random.default_rng(77)
     cfg = wl.cfg
     n_samples = 0
