@@ -183,6 +183,29 @@ def prepare_workload(name: str, scale: float = 1.0, chunks=None, device=None, wl
     return wl, st
 
 
+GRAPH_STEP_MS = 1.0   # steps shorter than this (eager) are timed as CUDA-graph replays
+
+
+def capture_step(wl, st):
+    """One device step captured into a CUDA graph on a side stream (every call of the step
+    is asynchronous, counts stay on the device).  Returns (graph, kernels per step)."""
+    import torch
+    from paper_conf_socc_jinv23_b200 import cof
+    g = torch.cuda.CUDAGraph()
+    s0 = st.stream
+    cs = torch.cuda.Stream(st.device)
+    cs.wait_stream(s0)
+    n0 = cof.cof_launch_count()
+    try:
+        with torch.cuda.graph(g, stream=cs):
+            st.stream = torch.cuda.current_stream(st.device)
+            run_device_pipeline(wl, st)
+    finally:
+        st.stream = s0
+    s0.wait_stream(cs)
+    return g, cof.cof_launch_count() - n0
+
+
 def run_device_pipeline(wl, st, collect=False, events=None, fevents=None):
     """One step on the device: per chunk find -> compare -> sort, counts kept on the
     device (no host round trip between kernels).  ``events`` / ``fevents``: lists to append
@@ -506,21 +529,45 @@ def main():
     torch.cuda.synchronize(dev)
     barrier()
     torch.cuda.synchronize(dev)
+    # launch-bound steps (small genomes: the host's ~15 launches per step outlast the
+    # kernels) are captured once into a CUDA graph and replayed; long steps run eagerly
+    step_ms_est = (time.perf_counter() - t_w) * 1e3 / max(1, n_w)
+    graph, graph_note, graph_launches = None, None, 0
+    if step_ms_est < GRAPH_STEP_MS and os.environ.get("COF_GRAPH", "1") != "0":
+        try:
+            graph, graph_launches = capture_step(wl, st)
+            for _ in range(3):
+                graph.replay()
+            torch.cuda.synchronize(dev)
+        except Exception as e:   # (a capture the runtime refuses: eager steps)
+            graph, graph_note = None, f"eager (graph capture failed: {e})"
     events, fevents = [], []
     launches0 = cof.cof_launch_count()
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     t_start.record(st.stream)
     for _ in range(args.steps):
-        run_device_pipeline(wl, st, events=events, fevents=fevents)
+        if graph is not None:
+            graph.replay()
+        else:
+            run_device_pipeline(wl, st, events=events, fevents=fevents)
     t_end.record(st.stream)
     torch.cuda.synchronize(dev)
-    launches = cof.cof_launch_count() - launches0
+    launches = (cof.cof_launch_count() - launches0) if graph is None else graph_launches * args.steps
     clk = clocks.stop()
     barrier()
     ms_total = t_start.elapsed_time(t_end)
+    totals = step_counts(st)   # verifies capacities and every decorated key (graph replays too)
+    if graph is not None:
+        # the dominant kernel's own time cannot be bracketed inside a graph: K eager steps
+        # after the timed region, events around its launches
+        for _ in range(args.steps):
+            run_device_pipeline(wl, st, events=events, fevents=fevents)
+        torch.cuda.synchronize(dev)
+        step_counts(st)
+        graph_note = (f"CUDA graph of one step ({graph_launches} kernels) replayed K times in the timed region; "
+                      "kernel times from K eager steps after it")
     cmp_ms = sum(a.elapsed_time(b) for a, b in events)
     find_ms = sum(a.elapsed_time(b) for a, b in fevents)
-    totals = step_counts(st)   # verifies capacities
 
     # max over ranks
     t = torch.tensor([ms_total, cmp_ms, float(comps_mine), float(totals[2]), float(my_items)],
@@ -633,6 +680,7 @@ def main():
             "roofline": roofline,
             "finder_roofline": finder_roof,
             "gpu_launches": int(launches // args.steps) if args.steps else 0,
+            "step_launch": graph_note or "eager launches",
             "gpu_launches_timed_region": int(launches),
             "clocks": clk,
             "e2e": e2e,
