@@ -629,7 +629,8 @@ def main():
                    "achieved": round(find_gbs, 1),
                    "peak": hbm_peak, "unit": "GB/s", "frac": find_gbs / hbm_peak,
                    "bytes_per_step": int(find_bytes), "basis": find_basis,
-                   "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_finder_kernel", st, cfgname)}
+                   "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_finder_kernel", st, cfgname,
+                                          path="twocall" if st.path_name == "single" else None)}
 
     e2e = None
     resident = None
@@ -726,14 +727,14 @@ def time_search_kernel(st, steps):
     return total_ms, n_items
 
 
-def traffic_for(kernel, st, cfgname):
+def traffic_for(kernel, st, cfgname, path=None):
     """DRAM bytes per launch of ``kernel`` on THIS config and path from a committed ncu
     --set full capture (profiles/roofline_traffic.json, keyed "<config>:<kernel>_<path>"),
     or None when no capture of that config and path is committed."""
     try:
         with open(os.path.join(ROOT, "profiles", "roofline_traffic.json")) as f:
             d = json.load(f)
-        key = f"{cfgname}:{kernel}_{st.path_name}"
+        key = f"{cfgname}:{kernel}_{path or st.path_name}"
         e = d.get(key)
         return None if e is None else {"dram_bytes_per_launch": e["dram_bytes_per_launch"], "capture": e.get("capture")}
     except Exception:
