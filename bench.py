@@ -432,7 +432,7 @@ def main_bulge(args, cfgname):
     line = {"metric": "genome Gbases/s, bulge search (X + DNA<=%d + RNA<=%d)" % (dna, rna),
             "value": round(wl.total_bases / (ms * 1e-3) / 1e9, 4), "unit": "Gbases/s", "n_gpus": 1,
             "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": round(ms, 4),
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32 bit-planes",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32", "dtype_note": "2-bit bases in u32 bit-planes, bitwise integer arithmetic (exact)",
             "data": "synthetic (seeded hg38-shaped genome, synth.py)", "comparisons_per_s": comps / (ms * 1e-3),
             "hits_per_step": int(hits), "items_per_step": int(items),
             "config": {"workload": cfgname, "genome_bases": wl.total_bases, "guides": len(wl.guides),
@@ -593,13 +593,13 @@ def main():
     roof = comparer_roof(st.plan, n_sm, sm_max, args.comparer, st.path_name)
     cmp_rate = comps_mine * args.steps / (cmp_ms * 1e-3) if cmp_ms > 0 else 0.0
     n_cmp_launch = len(events)
+    traffic_k = traffic_for("cof_single_kernel" if st.path_name == "single" else "cof_comparer", st, cfgname)
     kname = {"single": "cof_single_kernel", "fused": "cof_comparer_fused"}.get(st.path_name,
                                                                               f"cof_comparer_{args.comparer}")
     roofline = {"bound": "alu", "kernel": kname,
                 "achieved": cmp_rate, "peak": roof["peak"], "unit": "comparisons/s",
                 "frac": cmp_rate / roof["peak"] if roof["peak"] else None,
-                "traffic": traffic_for("cof_single_kernel" if st.path_name == "single" else "cof_comparer",
-                                       st, cfgname),
+                "traffic": traffic_k[0], "traffic_capture": traffic_k[1],
                 "peak_basis": roof["basis"], "launches": n_cmp_launch,
                 "share_of_step": cmp_ms_max / ms_total if ms_total else None,
                 # the same rate against SURVEY §8(d)'s roof (one POPC per comparison)
@@ -625,12 +625,12 @@ def main():
         find_basis = "planes read + 4 B per item written (two-call path)"
     find_gbs = find_bytes * args.steps / (find_ms * 1e-3) / 1e9 if find_ms > 0 else 0.0
     hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
+    traffic_f = traffic_for("cof_finder_kernel", st, cfgname, path="twocall" if st.path_name == "single" else None)
     finder_roof = {"bound": "hbm", "kernel": "cof_finder_kernel",
                    "achieved": round(find_gbs, 1),
                    "peak": hbm_peak, "unit": "GB/s", "frac": find_gbs / hbm_peak,
                    "bytes_per_step": int(find_bytes), "basis": find_basis,
-                   "ms_per_step": find_ms / args.steps, "traffic": traffic_for("cof_finder_kernel", st, cfgname,
-                                          path="twocall" if st.path_name == "single" else None)}
+                   "ms_per_step": find_ms / args.steps, "traffic": traffic_f[0], "traffic_capture": traffic_f[1]}
 
     e2e = None
     resident = None
@@ -663,7 +663,7 @@ def main():
             "metric": metric, "value": round(gbases, 4), "unit": "Gbases/s", "n_gpus": world,
             "steps": args.steps, "warmup": max(args.warmup, 3), "warmup_steps_run": n_w,
             "ms_per_step": round(ms_step, 4),
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32 bit-planes",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32", "dtype_note": "2-bit bases in u32 bit-planes, bitwise integer arithmetic (exact)",
             "data": "synthetic (seeded hg38-shaped genome, synth.py)",
             "comparisons_per_s": comps_s, "hits_per_step": int(hits_all), "items_per_step": int(items_all),
             "config": {"workload": cfgname if not args.n_guides else f"{cfgname} with {args.n_guides} guides",
@@ -730,15 +730,15 @@ def time_search_kernel(st, steps):
 def traffic_for(kernel, st, cfgname, path=None):
     """DRAM bytes per launch of ``kernel`` on THIS config and path from a committed ncu
     --set full capture (profiles/roofline_traffic.json, keyed "<config>:<kernel>_<path>"),
-    or None when no capture of that config and path is committed."""
+    or None when no capture of that config and path is committed.  Returns (bytes, capture)."""
     try:
         with open(os.path.join(ROOT, "profiles", "roofline_traffic.json")) as f:
             d = json.load(f)
         key = f"{cfgname}:{kernel}_{path or st.path_name}"
         e = d.get(key)
-        return None if e is None else {"dram_bytes_per_launch": e["dram_bytes_per_launch"], "capture": e.get("capture")}
+        return (None, None) if e is None else (int(e["dram_bytes_per_launch"]), e.get("capture"))
     except Exception:
-        return None
+        return None, None
 
 
 def popc_roof(n_sm, sm_mhz):
