@@ -217,7 +217,9 @@ __device__ __forceinline__ unsigned long long s_key(uint32_t pos, uint32_t stran
            (unsigned long long)mm;
 }
 
-template <int NP, int TC, bool CONCRETE, class CFG>
+// NE: non-N PAM letters per strand when known at compile time (2: NRG / NGG, 4: TTTV), so the
+// PAM test is unrolled with constant parameter offsets; -1: any count (a loop).
+template <int NP, int TC, bool CONCRETE, class CFG, int NE = -1>
 __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __grid_constant__ SingleArgs a) {
     constexpr int SW = CFG::SW, STHREADS = CFG::STHREADS, STW = CFG::STW, SLOAD = CFG::SLOAD;
     constexpr int SSTAGES = CFG::SSTAGES, SR = CFG::SR;
@@ -571,7 +573,9 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
             uint32_t v = valid[q];
             if (pw + 32 > a.limit) v &= pw >= a.limit ? 0u : (1u << (uint32_t)(a.limit - pw)) - 1u;
             uint32_t p0m = v, p1m = v;
-            for (uint32_t e = 0; e < a.ne; e++) {
+            const uint32_t ne = NE >= 0 ? (uint32_t)NE : a.ne;
+#pragma unroll
+            for (uint32_t e = 0; e < (NE >= 0 ? (uint32_t)NE : ne); e++) {
                 const uint32_t j0 = a.pj[0][e], j1 = a.pj[1][e];
                 p0m &= s_member(__funnelshift_r(lo[q], lo[q + 1], j0), __funnelshift_r(hi[q], hi[q + 1], j0),
                                 __funnelshift_r(nm[q], nm[q + 1], j0), a.psel[0][e]);
@@ -602,10 +606,10 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
 // ============================================================================ host side
 typedef void (*SingleFn)(SingleArgs);
 
-template <int NP, int TC, bool CONCRETE>
+template <int NP, int TC, bool CONCRETE, int NE = -1>
 static SingleFn single_fn_t(int geo) {   // 0: many blocks, 1: few, 2: few + sparse PAM
-    return geo == 1 ? cof_single_kernel<NP, TC, CONCRETE, SCfgFew>
-         : geo == 2 ? cof_single_kernel<NP, TC, CONCRETE, SCfgSparse> : cof_single_kernel<NP, TC, CONCRETE, SCfgMany>;
+    return geo == 1 ? cof_single_kernel<NP, TC, CONCRETE, SCfgFew, NE>
+         : geo == 2 ? cof_single_kernel<NP, TC, CONCRETE, SCfgSparse, NE> : cof_single_kernel<NP, TC, CONCRETE, SCfgMany, NE>;
 }
 
 // The kernel variant a plan runs: uniform-threshold, concrete-letter specialisations for
@@ -616,9 +620,16 @@ static bool single_uses_concrete(uint32_t np, int tc, bool concrete) {
 }
 
 template <int NP>
-static SingleFn single_fn_np(int tc, bool concrete, int geo) {
+static SingleFn single_fn_np(int tc, bool concrete, int geo, uint32_t ne) {
     if constexpr (NP == 10 || NP == 12) {
         if (concrete) {
+            // the configs' shapes (t 4-6, 2 or 4 PAM letters) get the unrolled PAM test
+            if (ne == 2 && tc == 4) return single_fn_t<NP, 4, true, 2>(geo);
+            if (ne == 2 && tc == 5) return single_fn_t<NP, 5, true, 2>(geo);
+            if (ne == 2 && tc == 6) return single_fn_t<NP, 6, true, 2>(geo);
+            if (ne == 4 && tc == 4) return single_fn_t<NP, 4, true, 4>(geo);
+            if (ne == 4 && tc == 5) return single_fn_t<NP, 5, true, 4>(geo);
+            if (ne == 4 && tc == 6) return single_fn_t<NP, 6, true, 4>(geo);
             switch (tc) {
                 case 0: return single_fn_t<NP, 0, true>(geo);
                 case 1: return single_fn_t<NP, 1, true>(geo);
@@ -635,24 +646,24 @@ static SingleFn single_fn_np(int tc, bool concrete, int geo) {
     return single_fn_t<NP, -1, false>(geo);
 }
 
-static SingleFn single_fn(uint32_t np, int tc, bool concrete, int geo) {
+static SingleFn single_fn(uint32_t np, int tc, bool concrete, int geo, uint32_t ne) {
     switch (np) {
-        case 1: return single_fn_np<1>(tc, concrete, geo);
-        case 2: return single_fn_np<2>(tc, concrete, geo);
-        case 3: return single_fn_np<3>(tc, concrete, geo);
-        case 4: return single_fn_np<4>(tc, concrete, geo);
-        case 5: return single_fn_np<5>(tc, concrete, geo);
-        case 6: return single_fn_np<6>(tc, concrete, geo);
-        case 7: return single_fn_np<7>(tc, concrete, geo);
-        case 8: return single_fn_np<8>(tc, concrete, geo);
-        case 9: return single_fn_np<9>(tc, concrete, geo);
-        case 10: return single_fn_np<10>(tc, concrete, geo);
-        case 11: return single_fn_np<11>(tc, concrete, geo);
-        case 12: return single_fn_np<12>(tc, concrete, geo);
-        case 13: return single_fn_np<13>(tc, concrete, geo);
-        case 14: return single_fn_np<14>(tc, concrete, geo);
-        case 15: return single_fn_np<15>(tc, concrete, geo);
-        case 16: return single_fn_np<16>(tc, concrete, geo);
+        case 1: return single_fn_np<1>(tc, concrete, geo, ne);
+        case 2: return single_fn_np<2>(tc, concrete, geo, ne);
+        case 3: return single_fn_np<3>(tc, concrete, geo, ne);
+        case 4: return single_fn_np<4>(tc, concrete, geo, ne);
+        case 5: return single_fn_np<5>(tc, concrete, geo, ne);
+        case 6: return single_fn_np<6>(tc, concrete, geo, ne);
+        case 7: return single_fn_np<7>(tc, concrete, geo, ne);
+        case 8: return single_fn_np<8>(tc, concrete, geo, ne);
+        case 9: return single_fn_np<9>(tc, concrete, geo, ne);
+        case 10: return single_fn_np<10>(tc, concrete, geo, ne);
+        case 11: return single_fn_np<11>(tc, concrete, geo, ne);
+        case 12: return single_fn_np<12>(tc, concrete, geo, ne);
+        case 13: return single_fn_np<13>(tc, concrete, geo, ne);
+        case 14: return single_fn_np<14>(tc, concrete, geo, ne);
+        case 15: return single_fn_np<15>(tc, concrete, geo, ne);
+        case 16: return single_fn_np<16>(tc, concrete, geo, ne);
         default: return nullptr;
     }
 }
@@ -762,7 +773,7 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     uint64_t limit = dev->n_bases >= L ? dev->n_bases - L + 1 : 0;
     if (!dev->n_segs && limit > dev->n_owned) limit = dev->n_owned;
     const uint32_t n_tiles = (uint32_t)((limit + (uint64_t)G.stw * 32 - 1) / ((uint64_t)G.stw * 32));
-    SingleFn fn = single_fn(I.np, I.ut, I.concrete, I.geo);
+    SingleFn fn = single_fn(I.np, I.ut, I.concrete, I.geo, plan->pam[0].n);
     if (!fn) return set_error(COF_E_STATE, "single pass: %u pairs", I.np);
     int dev_id = 0;
     cudaGetDevice(&dev_id);
