@@ -282,7 +282,7 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
                         for (int w = 0; w < FWPT; w++) {
                             uint32_t mm = m[st][w];
                             while (mm) {
-                                const int b = __ffs(mm) - 1;
+                                const int b = 31 - __clz(mm & (0u - mm));   // (one FLO; __ffs is BREV + FLO)
                                 items[off++] = pbase + 32u * w + (uint32_t)b;
                                 mm &= mm - 1;
                             }
@@ -293,7 +293,7 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
                         for (int w = 0; w < FWPT; w++) {
                             uint32_t mm = m[st][w];
                             while (mm) {
-                                const int b = __ffs(mm) - 1;
+                                const int b = 31 - __clz(mm & (0u - mm));   // (one FLO; __ffs is BREV + FLO)
                                 if (rank >= r0 && rank < r0 + FSTAGE_ITEMS) items[rank - r0] = pbase + 32u * w + (uint32_t)b;
                                 rank++;
                                 mm &= mm - 1;
@@ -368,7 +368,7 @@ __global__ void __launch_bounds__(FT) cof_finder_kernel(const __grid_constant__ 
                     for (int w = 0; w < 2; w++) {
                         uint32_t mm = st == 0 ? (w ? m[j].z : m[j].x) : (w ? m[j].w : m[j].y);
                         while (mm) {
-                            const int b = __ffs(mm) - 1;
+                            const int b = 31 - __clz(mm & (0u - mm));   // (one FLO; __ffs is BREV + FLO)
                             if (o < a.cap) out[o] = pj + 32u * w + (uint32_t)b;
                             o++;
                             mm &= mm - 1;

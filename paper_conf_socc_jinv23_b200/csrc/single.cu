@@ -111,7 +111,7 @@ struct SCfg {
 #define COF_MANY_S 4
 #endif
 #ifndef COF_SPARSE_WPL
-#define COF_SPARSE_WPL 2
+#define COF_SPARSE_WPL 4
 #endif
 #ifndef COF_FEW_WPL
 #define COF_FEW_WPL 1
