@@ -33,3 +33,29 @@ def test_resident_genome_several_guide_sets():
     out = np.zeros(10**5, dtype=srch.hit_dtype)
     got = srch.search_resident(rg, out=out)
     assert cof.hits_to_tuples(got) == oracle.hits_to_tuples(oracle.search(w.seqs, *sets[0]))
+
+
+@pytest.mark.parametrize("path", ["single", "fused", "twocall"])
+def test_pipelines_restart_on_overflow(path):
+    """search_host and search_resident read each chunk's hit count only after later chunks
+    are queued; a count above the (deliberately tiny) buffers restarts the call with larger
+    ones.  The result must still equal the oracle's -- for a list of chunks, an iterator of
+    chunk indices (search_multi's shared queue: the chunks already taken are replayed) and
+    the resident genome."""
+    w = synth.make_workload("C3", scale=0.004, n_guides=60)
+    cfg = w.cfg
+    chunks = search.plan_chunks([len(s) for s in w.seqs], cfg.L, 2_000_003, 4_000_000)
+    host = search.HostGenome(w.seqs, chunks)
+    exp = oracle.hits_to_tuples(oracle.search(w.seqs, cfg.pattern, w.guides, w.thresholds))
+    assert len(exp) > 2000 and len(host.chunks) > 3
+
+    def fresh():
+        srch = search.Searcher(cfg.pattern, w.guides, w.thresholds)
+        srch.path = path if path != "fused" or cof.cof_find_compare_supported(srch.plan) else "twocall"
+        srch.reserve(max(ch.n_bases for ch in host.chunks), 64)    # far too small
+        return srch
+
+    assert cof.hits_to_tuples(fresh().search_host(host)) == exp
+    assert cof.hits_to_tuples(fresh().search_host(host, indices=iter(range(len(host.chunks))))) == exp
+    rg = search.ResidentGenome(host, "cuda")
+    assert cof.hits_to_tuples(fresh().search_resident(rg)) == exp
