@@ -496,6 +496,10 @@ def main():
         else:
             dist.init_process_group(backend)
     cof.cof_set_comparer(args.comparer)
+    if world > 1:   # torchrun sets OMP_NUM_THREADS=1: share the node's cores among the ranks instead
+        nthr = max(1, len(os.sched_getaffinity(0)) // int(os.environ.get("LOCAL_WORLD_SIZE", world)))
+        torch.set_num_threads(nthr)
+        cof.cof_set_host_threads(nthr)
     cfg = synth.config(cfgname, args.scale)
     L = cfg.L
     # N > 1: chromosomes cut into <= 16 Mbp pieces before the LPT assignment (max/ideal load

@@ -56,6 +56,10 @@ const char *cof_last_error(void);
 const char *cof_version(void);
 /* Number of CUDA kernels this library has launched in this process (monotone). */
 uint64_t cof_launch_count(void);
+/* Host threads of the library's OpenMP regions (packing, collection, merge); n <= 0 keeps
+ * the current setting.  (torchrun sets OMP_NUM_THREADS=1 for every rank; a multi-GPU
+ * caller shares the node's cores among its ranks instead.)  Returns the setting in force. */
+int cof_set_host_threads(int n);
 
 /* ------------------------------------------------------------------ plan (M1)
  * The input specification: a search pattern of length L (guide Ns + PAM, e.g.

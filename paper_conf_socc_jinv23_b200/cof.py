@@ -65,6 +65,7 @@ def _load():
     sig = {
         "cof_last_error": (ctypes.c_char_p, []),
         "cof_version": (ctypes.c_char_p, []),
+        "cof_set_host_threads": (I32, [I32]),
         "cof_launch_count": (U64, []),
         "cof_plan_create": (I32, [ctypes.c_char_p, U32, P, P, P]),
         "cof_plan_destroy": (None, [P]),
@@ -126,7 +127,7 @@ def _load():
 lib = _load()
 
 # names the header declares (checked by tests/test_abi_host.py)
-EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_launch_count", "cof_plan_create",
+EXPORTS = [n for n in ("cof_last_error", "cof_version", "cof_set_host_threads", "cof_launch_count", "cof_plan_create",
                        "cof_plan_destroy", "cof_plan_length", "cof_plan_n_guides",
                        "cof_plan_device_bytes", "cof_plan_upload", "cof_plane_words", "cof_pack",
                        "cof_unpack", "cof_valid_starts", "cof_load_chunk", "cof_fasta_open", "cof_fasta_close",
@@ -176,6 +177,11 @@ def cof_last_error() -> str:
 
 def cof_version() -> str:
     return lib.cof_version().decode()
+
+
+def cof_set_host_threads(n: int) -> int:
+    """Threads of the library's host OpenMP regions (n <= 0: unchanged); returns the setting."""
+    return int(lib.cof_set_host_threads(int(n)))
 
 
 def cof_launch_count() -> int:

@@ -98,6 +98,11 @@ extern "C" {
 
 const char* cof_last_error(void) { return g_err.c_str(); }
 const char* cof_version(void) { return "cof-b200 0.1 (sm_100a)"; }
+
+int cof_set_host_threads(int n) {
+    if (n > 0) omp_set_num_threads(n);
+    return omp_get_max_threads();
+}
 uint64_t cof_launch_count(void) { return g_launches.load(); }
 
 uint64_t cof_plane_words(uint64_t n_bases) {

@@ -927,8 +927,9 @@ def merge_dist(per_chunk: dict, n_chunks: int, dtype, group=None, dst: int = 0, 
     arena = _merge_arena(max(1, total) * isz, group, dst, shm_dir)
     out = arena[: total * isz].view(dtype) if total else np.zeros(0, dtype=dtype)
     for i, r in per_chunk.items():
-        if len(r):   # (a byte copy: 4x faster than numpy's field-wise structured assignment)
-            arena[offs[i] * isz:(offs[i] + len(r)) * isz] = np.ascontiguousarray(r).view(np.uint8)
+        if len(r):   # (a byte copy -- torch's is multi-threaded; numpy's field-wise one was 4x slower)
+            torch.from_numpy(arena[offs[i] * isz:(offs[i] + len(r)) * isz]).copy_(
+                torch.from_numpy(np.ascontiguousarray(r).view(np.uint8)))
     dist.barrier(group=group)
     return out if rank == dst else None
 
