@@ -636,6 +636,16 @@ def main():
                    "bytes_per_step": int(find_bytes), "basis": find_basis,
                    "ms_per_step": find_ms / args.steps, "traffic": traffic_f[0], "traffic_capture": traffic_f[1]}
 
+    masks_roof = None
+    if st.path_name == "single" and cof.cof_find_compare_supported(st.plan):
+        m_ms, m_bytes = time_masks_kernel(st, args.steps)
+        m_gbs = m_bytes * args.steps / (m_ms * 1e-3) / 1e9 if m_ms > 0 else 0.0
+        masks_roof = {"bound": "hbm", "kernel": "cof_finder_kernel (masks)", "achieved": round(m_gbs, 1),
+                      "peak": hbm_peak, "unit": "GB/s", "frac": m_gbs / hbm_peak, "bytes_per_step": int(m_bytes),
+                      "ms_per_step": m_ms / args.steps,
+                      "basis": "search kernel writing per-word PAM masks (cof_find_masks, the fused path's finder): "
+                               "planes (+ valid-start plane) read + 8 B of masks per plane word written; timed "
+                               f"{args.steps} times after the step's timed region"}
     e2e = None
     resident = None
     if not args.no_e2e:
@@ -684,6 +694,7 @@ def main():
                        "l2": "inputs larger than L2 (1.16 GB planes + item lists), no flush"},
             "roofline": roofline,
             "finder_roofline": finder_roof,
+            "finder_masks_roofline": masks_roof,
             "gpu_launches": int(launches // args.steps) if args.steps else 0,
             "step_launch": graph_note or "eager launches",
             "gpu_launches_timed_region": int(launches),
@@ -729,6 +740,30 @@ def time_search_kernel(st, steps):
         n_items += nf + nr
         del items, ws
     return total_ms, n_items
+
+
+def time_masks_kernel(st, steps):
+    """The search kernel in its masks form (cof_find_masks: per plane word {fwd, rev} PAM
+    masks, the fused path's finder) alone on the resident planes, ``steps`` launches per
+    chunk; returns (ms per step, algorithmic bytes per step: planes read + 8 B per word)."""
+    import torch
+    from paper_conf_socc_jinv23_b200 import cof
+    s = st.stream
+    total_ms, nbytes = 0.0, 0
+    for i, ch in enumerate(st.chunks):
+        ws = torch.empty(cof.cof_find_compare_workspace_bytes(ch.n_bases), dtype=torch.uint8, device=st.device)
+        cof.cof_find_masks(st.plan, st.plan_devs[i], st.d_chunks[i], ws, s)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        for _ in range(steps):
+            cof.cof_find_masks(st.plan, st.plan_devs[i], st.d_chunks[i], ws, s)
+        e1.record(s)
+        torch.cuda.synchronize(st.device)
+        total_ms += e0.elapsed_time(e1)
+        words = cof.cof_plane_words(ch.n_bases)
+        nbytes += words * 4 * (4 if ch.multi else 3) + words * 8
+        del ws
+    return total_ms, nbytes
 
 
 def traffic_for(kernel, st, cfgname, path=None):
