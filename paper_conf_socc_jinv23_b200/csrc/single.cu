@@ -147,6 +147,7 @@ struct SingleArgs {
     uint32_t block_base;              // first block of this launch (global guide = (base + b) * 32 + k)
     uint32_t count_items;             // count PAM sites (one launch per search does)
     uint32_t ne;                      // non-N pattern letters per strand
+    uint32_t pam_hi;                  // some PAM letter sits at window offset >= 32 (L > 32)
     uint32_t pj[2][32];               // their window offsets
     uint4 psel[2][32];                // their IUPAC sets as splat words {A, C, G, T}
     uint32_t p0[2];                   // first compared window offset per strand
@@ -577,10 +578,22 @@ __global__ void __launch_bounds__(CFG::STHREADS, 1) cof_single_kernel(const __gr
 #pragma unroll
             for (uint32_t e = 0; e < (NE >= 0 ? (uint32_t)NE : ne); e++) {
                 const uint32_t j0 = a.pj[0][e], j1 = a.pj[1][e];
-                p0m &= s_member(__funnelshift_r(lo[q], lo[q + 1], j0), __funnelshift_r(hi[q], hi[q + 1], j0),
-                                __funnelshift_r(nm[q], nm[q + 1], j0), a.psel[0][e]);
-                p1m &= s_member(__funnelshift_r(lo[q], lo[q + 1], j1), __funnelshift_r(hi[q], hi[q + 1], j1),
-                                __funnelshift_r(nm[q], nm[q + 1], j1), a.psel[1][e]);
+                if (NE >= 0 || !a.pam_hi) {   // (warp-uniform; the unrolled kernels never see L > 32 PAMs)
+                    p0m &= s_member(__funnelshift_r(lo[q], lo[q + 1], j0), __funnelshift_r(hi[q], hi[q + 1], j0),
+                                    __funnelshift_r(nm[q], nm[q + 1], j0), a.psel[0][e]);
+                    p1m &= s_member(__funnelshift_r(lo[q], lo[q + 1], j1), __funnelshift_r(hi[q], hi[q + 1], j1),
+                                    __funnelshift_r(nm[q], nm[q + 1], j1), a.psel[1][e]);
+                } else {           // L > 32: a letter at offset >= 32 reads the next word pair
+                    const int k0 = (int)(j0 >> 5), k1 = (int)(j1 >> 5);
+                    p0m &= s_member(__funnelshift_r(k0 ? lo[q + 1] : lo[q], k0 ? lo[q + 2] : lo[q + 1], j0),
+                                    __funnelshift_r(k0 ? hi[q + 1] : hi[q], k0 ? hi[q + 2] : hi[q + 1], j0),
+                                    __funnelshift_r(k0 ? nm[q + 1] : nm[q], k0 ? nm[q + 2] : nm[q + 1], j0),
+                                    a.psel[0][e]);
+                    p1m &= s_member(__funnelshift_r(k1 ? lo[q + 1] : lo[q], k1 ? lo[q + 2] : lo[q + 1], j1),
+                                    __funnelshift_r(k1 ? hi[q + 1] : hi[q], k1 ? hi[q + 2] : hi[q + 1], j1),
+                                    __funnelshift_r(k1 ? nm[q + 1] : nm[q], k1 ? nm[q + 2] : nm[q + 1], j1),
+                                    a.psel[1][e]);
+                }
             }
             pend[0][q] = p0m;
             pend[1][q] = p1m;
@@ -696,10 +709,11 @@ static uint32_t single_blocks_per_launch(const SGeom& g, uint32_t np, bool concr
 // The single-pass kernel handles one-word windows: every compared offset of both strands
 // within [p0, p0 + 31) (bit 31 of the queued N-window carries the strand), <= 16 pairs.
 static bool single_shape_ok(const cof_plan* plan) {
-    if (plan->L > 32) return false;
+    if (plan->L > 64) return false;
     for (int s = 0; s < 2; s++) {
         const PairLayout& pl = plan->pairs[s];
-        if (pl.wide || pl.n_pairs > 16) return false;
+        // (windows are taken at the strand's first compared offset p0 from a word pair)
+        if (pl.wide || pl.n_pairs > 16 || pl.p0 >= 32) return false;
         const uint64_t uc = plan->union_care[s];
         if (!uc) continue;
         const uint32_t span = 64u - (uint32_t)__builtin_clzll(uc) - pl.p0;
@@ -773,7 +787,11 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     uint64_t limit = dev->n_bases >= L ? dev->n_bases - L + 1 : 0;
     if (!dev->n_segs && limit > dev->n_owned) limit = dev->n_owned;
     const uint32_t n_tiles = (uint32_t)((limit + (uint64_t)G.stw * 32 - 1) / ((uint64_t)G.stw * 32));
-    SingleFn fn = single_fn(I.np, I.ut, I.concrete, I.geo, plan->pam[0].n);
+    // (the unrolled-PAM kernels assume every PAM letter within the first 32 window offsets)
+    bool pam_hi = false;
+    for (int s = 0; s < 2; s++)
+        for (uint32_t k = 0; k < plan->pam[s].n; k++) pam_hi |= plan->pam[s].j[k] >= 32;
+    SingleFn fn = single_fn(I.np, I.ut, I.concrete, I.geo, pam_hi ? 0u : plan->pam[0].n);
     if (!fn) return set_error(COF_E_STATE, "single pass: %u pairs", I.np);
     int dev_id = 0;
     cudaGetDevice(&dev_id);
@@ -789,6 +807,9 @@ cof_status run_single(const cof_plan* plan, uint8_t* pd, const cof_chunk* dev, u
     A.cap = hits_cap;
     A.counters = (unsigned long long*)(pd + plan->lay.counters);
     A.ne = plan->pam[0].n;
+    A.pam_hi = 0;
+    for (int s = 0; s < 2; s++)
+        for (uint32_t k = 0; k < plan->pam[s].n; k++) A.pam_hi |= plan->pam[s].j[k] >= 32 ? 1u : 0u;
     if (plan->pam[1].n != A.ne || A.ne > 32) return set_error(COF_E_STATE, "single pass: PAM letter counts");
     for (int s = 0; s < 2; s++) {
         for (uint32_t k = 0; k < A.ne; k++) {
