@@ -37,6 +37,7 @@ from paper_conf_socc_jinv23_b200 import synth  # noqa: E402
 E2E_CHUNK_BASES = int(os.environ.get("COF_E2E_CHUNK_BASES", 250_000_000))  # e2e: pieces packed into chunks of <= this
 # e2e: chromosomes cut into pieces of <= this many window starts first (0 = whole chromosomes)
 E2E_PIECE_BASES = int(os.environ.get("COF_E2E_PIECE_BASES", 0))
+E2E_FIRST_BASES = int(os.environ.get("COF_E2E_FIRST_BASES", 0))   # e2e: first chunk <= this (0: no limit)
 SHARD_PIECE_BASES = 16_000_000   # N > 1: chromosome pieces LPT-assigned to ranks
 RESIDENT_CHUNK_BASES = int(os.environ.get("COF_RESIDENT_CHUNK_BASES", 800_000_000))   # e2e_resident chunks
 
@@ -917,7 +918,9 @@ def measure_e2e(wl, st, dev, args, world, genome_bases, coll_dev=None):
     pieces = [p for ch in st.chunks for p in ch.pieces]
     if E2E_PIECE_BASES:
         pieces = search.split_pieces(pieces, E2E_PIECE_BASES, L)
-    chunks = search.pack_pieces(pieces, E2E_CHUNK_BASES)
+    if E2E_FIRST_BASES:   # a short first chunk: cut the first piece
+        pieces = search.split_pieces(pieces[:1], E2E_FIRST_BASES, L) + pieces[1:]
+    chunks = search.pack_pieces(pieces, E2E_CHUNK_BASES, E2E_FIRST_BASES)
     st.e2e_host = search.HostGenome(wl.seqs, chunks)
     srch = search.Searcher(wl.cfg.pattern, wl.guides, wl.thresholds, device=dev)
     srch.reserve(max(ch.n_bases for ch in chunks), max(st.caps))

@@ -144,11 +144,14 @@ def split_pieces(pieces, max_owned: int, L: int):
     return out
 
 
-def pack_pieces(pieces, pack_bases: int):
-    """Consecutive pieces -> multi-segment chunks of at most ``pack_bases`` bases (0: one)."""
+def pack_pieces(pieces, pack_bases: int, first_bases: int = 0):
+    """Consecutive pieces -> multi-segment chunks of at most ``pack_bases`` bases (0: one);
+    the first chunk at most ``first_bases`` if given (a short first chunk starts the
+    pipelined search sooner: its H2D is the only one nothing overlaps)."""
     out, cur, cur_bases = [], [], 0
     for p in pieces:
-        if cur and pack_bases and cur_bases + p.length > pack_bases:
+        limit = first_bases if (first_bases and not out) else pack_bases
+        if cur and limit and cur_bases + p.length > limit:
             out.append(Chunk(tuple(cur)))
             cur, cur_bases = [], 0
         cur.append(p)
