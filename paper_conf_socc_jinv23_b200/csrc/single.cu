@@ -87,7 +87,7 @@ struct SCfg {
 #define COF_FEW_Q 4
 #endif
 #ifndef COF_MANY_Q
-#define COF_MANY_Q 2
+#define COF_MANY_Q 4
 #endif
 #ifndef COF_FEW_G
 #define COF_FEW_G 1
@@ -99,7 +99,7 @@ struct SCfg {
 #define COF_FEW_K 3
 #endif
 #ifndef COF_MANY_K
-#define COF_MANY_K 1
+#define COF_MANY_K 2
 #endif
 #ifndef COF_MANY_W
 #define COF_MANY_W 28
@@ -108,7 +108,7 @@ struct SCfg {
 #define COF_MANY_R 1
 #endif
 #ifndef COF_MANY_S
-#define COF_MANY_S 4
+#define COF_MANY_S 2
 #endif
 #ifndef COF_SPARSE_WPL
 #define COF_SPARSE_WPL 4
