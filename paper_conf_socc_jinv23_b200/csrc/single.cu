@@ -99,7 +99,7 @@ struct SCfg {
 #define COF_FEW_K 3
 #endif
 #ifndef COF_MANY_K
-#define COF_MANY_K 2
+#define COF_MANY_K 3
 #endif
 #ifndef COF_MANY_W
 #define COF_MANY_W 28
