@@ -124,7 +124,10 @@ using SCfgFew = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q, COF_FEW_G, COF_
 // per-chunk work (tile bookkeeping, the append's scan) is spread over more sites
 using SCfgSparse = SCfg<COF_FEW_W, COF_FEW_R, COF_FEW_S, COF_FEW_Q, COF_FEW_G, COF_FEW_K, COF_SPARSE_WPL>;
 using SCfgMany = SCfg<COF_MANY_W, COF_MANY_R, COF_MANY_S, COF_MANY_Q, COF_MANY_G, COF_MANY_K, COF_MANY_WPL>;
-constexpr uint32_t SFEW_BLOCKS = 8;       // guide blocks up to which SCfgFew runs
+#ifndef COF_FEW_MAXB
+#define COF_FEW_MAXB 8
+#endif
+constexpr uint32_t SFEW_BLOCKS = COF_FEW_MAXB;   // guide blocks up to which SCfgFew runs
 constexpr int SPL = 4;                    // planes per stage: lo, hi, nm, vs
 constexpr uint32_t SMAX_BLOCKS = 64;      // guide blocks per launch (shared-memory tables)
 constexpr uint32_t S_END = 0xFFFFFFFFu;   // tile id: no more tiles
